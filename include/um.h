@@ -1,0 +1,173 @@
+/* um.h — C ABI of libum, a B200-native, discard-aware unified-memory paging layer.
+ *
+ * Method: "UVM Discard: Eliminating Redundant Memory Transfers for Accelerators"
+ * (Zhu et al., IISWC'22).  Citations "PAPER L<n>" are lines of its text
+ * (/root/reference/PAPER.md at build time); "A<n>"/"R<n>" are the readings listed in
+ * DESIGN.md §3 where the paper is silent.
+ *
+ * Model.  An arena of nblocks = arena_bytes / block_bytes virtual blocks (64 KiB or
+ * 2 MiB) is backed by nframes = budget_bytes / block_bytes GPU frames in HBM and by a
+ * pool of pinned, mapped host frames.  Every block is in one state:
+ *   U  never populated            H  valid on host              HD discarded, not on GPU
+ *   G  valid, mapped, in USED     GE eager-discarded (unmapped), in DISC
+ *   GL lazy-discarded (mapped, software dirty bit clear), in DISC
+ * GPU accesses ("faults") and prefetches to the GPU give a block a frame; when no frame
+ * is free a victim is reclaimed in the order discarded-FIFO, then used-LRU
+ * (PAPER L217-221).  Valid victims are written back (D2H); discarded ones are dropped
+ * (Fig. 2 (6)); a discarded-then-reclaimed block is zero-filled instead of
+ * migrated when it is used again (Fig. 2 (7)).
+ *
+ * Execution.  All planning (state tables, victim selection, work-list compaction) runs
+ * in sm_100a kernels on device-resident tables; data moves by a kernel-driven copy over
+ * mapped pinned host memory (or by the copy engines with UM_F_COPY_CE).  No CPU fallback.
+ *
+ * Conventions (all functions):
+ *  - Return um_status; UM_OK = 0.  No exceptions cross the ABI.
+ *  - Pointers are plain host pointers unless documented as device pointers.
+ *  - Streams are cudaStream_t values passed as void* (0 = legacy default stream).
+ *    Each op is stream-ordered like a CUDA memory op: it runs after
+ *    prior work on `stream`, and later work on `stream` sees its effects.  Ops of one
+ *    arena execute in call order on the arena's internal paging stream.
+ *  - Range errors (outside the arena, bad dst) return UM_EINVAL and enqueue nothing.
+ *    len == 0 is valid: it consumes one sequence number and moves nothing.
+ *  - A CUDA failure returns UM_ECUDA and is sticky: later calls return it too.
+ *  - One host thread per arena; a concurrent call returns UM_EBUSY.
+ *  - Every call that enqueues work consumes one sequence number per sub-op (A3).
+ */
+#ifndef UM_H
+#define UM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct um_arena um_arena; /* opaque; library-owned host bookkeeping */
+
+typedef enum {
+  UM_OK = 0,
+  UM_EINVAL = -1, /* bad argument / range; nothing enqueued                              */
+  UM_ENOMEM = -2, /* arena (um_alloc) or host-frame pool exhausted; sticky when on device */
+  UM_ECUDA = -3,  /* CUDA error; sticky                                                   */
+  UM_EBUSY = -4   /* concurrent call on the same arena                                   */
+} um_status;
+
+enum { UM_DST_GPU = 0, UM_DST_HOST = 1 };
+enum { UM_ACC_READ = 1u, UM_ACC_WRITE = 2u };
+enum { UM_ST_U = 0, UM_ST_H = 1, UM_ST_HD = 2, UM_ST_G = 3, UM_ST_GE = 4, UM_ST_GL = 5 };
+
+enum {
+  UM_F_DISCARD_OFF = 1u, /* "UVM-opt" baseline: discards are accepted no-ops */
+  UM_F_COPY_CE = 2u,     /* move data with cudaMemcpyAsync on side streams, not K4       */
+  UM_F_CHECK = 4u,       /* poison frames with 0xA5 at creation; extra validation       */
+  UM_F_APP_STAMP = 8u    /* harness: after each touch sub-op, write the content stamp of
+                            every UM_ACC_WRITE block (simulated application kernel)    */
+};
+
+/* One GPU access record of a batch (16 bytes).  Covers every block overlapping
+ * [off, off+len); kind = UM_ACC_READ | UM_ACC_WRITE.  len is u32 (< 4 GiB per record). */
+typedef struct {
+  uint64_t off;
+  uint32_t len;
+  uint32_t kind;
+} um_access;
+
+typedef struct {
+  int device;                 /* CUDA device ordinal                                       */
+  uint32_t block_bytes;       /* 65536 or 2097152 (any power of two >= 4096 is accepted)  */
+  uint64_t arena_bytes;       /* multiple of block_bytes; nblocks = arena/block < 2^32-1   */
+  uint64_t budget_bytes;      /* nframes = budget/block >= 1                               */
+  void *frames;               /* DEVICE, >= nframes*block_bytes, caller-owned              */
+  void *workspace;            /* DEVICE, >= um_workspace_size(), caller-owned              */
+  uint64_t workspace_bytes;
+  void *const *host_chunks;   /* HOST array of n_host_chunks pinned+mapped host pointers;
+                                 caller-owned, alive until destroy.  Together they form the
+                                 host-frame pool: n_host_chunks*host_chunk_bytes/block_bytes
+                                 frames (+1 block reserved as the zero page).  Contents need
+                                 not be zero: host frames are written before being read.   */
+  uint32_t n_host_chunks;
+  uint64_t host_chunk_bytes;  /* multiple of block_bytes                                   */
+  uint32_t flags;             /* UM_F_*                                                    */
+} um_config;
+
+/* Counters (int64, 16 slots).  Byte counters are multiples of block_bytes. */
+typedef struct {
+  int64_t h2d_bytes, d2h_bytes, zf_bytes, h2d_avoided_bytes, d2h_avoided_bytes,
+      faults, hits, remaps, unmaps, revalidations, refreshes, evictions, ops, subops;
+  int64_t pad[2];
+} um_stats;
+
+/* Bytes of device workspace the arena needs (state tables, rings, work lists). */
+um_status um_workspace_size(const um_config *cfg, uint64_t *bytes);
+
+/* Create an arena: all blocks start in U, all frames free.  Synchronizes. */
+um_status um_arena_create(const um_config *cfg, um_arena **out);
+
+/* Synchronize and free the library's host-side state (caller memory is not freed). */
+um_status um_arena_destroy(um_arena *a);
+
+/* Block-aligned bump allocation (layout rule: offset = previous end rounded up to
+ * block_bytes).  UM_ENOMEM if it does not fit.  No device work. */
+um_status um_alloc(um_arena *a, uint64_t bytes, uint64_t *off);
+
+/* cudaMemPrefetchAsync analogue (PAPER §2.1).  dst GPU: every block overlapping
+ * the range gets a frame (U/HD zero-filled, H migrated, G refreshed to MRU, GE
+ * re-mapped, GL revalidated = software dirty bit set); ops with more
+ * distinct blocks than frames are split into ascending sub-ops (A3).  dst HOST: G
+ * migrates back (D2H), GE/GL/HD/U become H with no transfer (A9). */
+um_status um_prefetch(um_arena *a, uint64_t off, uint64_t len, int dst, void *stream);
+
+/* UvmDiscard (PAPER §5.1): for blocks FULLY inside the range (PAPER L211,
+ * A4): G -> GE (unmap; appended to DISC), GL -> GE, H -> HD. */
+um_status um_discard(um_arena *a, uint64_t off, uint64_t len, void *stream);
+
+/* UvmDiscardLazy (PAPER §5.2): fully covered G -> GL (mapping kept, appended
+ * to DISC), H -> HD.  The caller MUST um_prefetch the range before reusing it (either
+ * destination, A17); an access without it does not revalidate (A8). */
+um_status um_discard_lazy(um_arena *a, uint64_t off, uint64_t len, void *stream);
+
+/* A batch of GPU accesses ("faults"): the distinct blocks of all
+ * records are serviced in ascending sub-ops of <= nframes blocks.  `acc` is read before
+ * return (the caller may reuse it). */
+um_status um_touch_batch(um_arena *a, const um_access *acc, uint32_t n, void *stream);
+
+/* Make >= bytes of frames free by the eviction policy (PAPER §5.5). */
+um_status um_evict(um_arena *a, uint64_t bytes, void *stream);
+
+/* Harness op (simulated CPU writes, Listing 6 "Generate data, labels" L330): every block
+ * overlapping the range must be host-resident (H); its host frame receives the content
+ * stamp of this op.  A block not in H sets a sticky device error (UM_EINVAL). */
+um_status um_host_write(um_arena *a, uint64_t off, uint64_t len, void *stream);
+
+/* DEVICE pointer to the block table map[nblocks] (u32 frame id, 0xffffffff = unmapped)
+ * that application kernels translate through: addr = frames + map[b]*block + off%block.
+ * G and GL blocks are mapped; U/H/HD/GE are not (an eager discard unmaps). */
+um_status um_block_table(um_arena *a, const uint32_t **dev_map);
+
+/* The arena's internal paging stream (work enqueued on it needs no event hand-off). */
+um_status um_stream(um_arena *a, void **stream);
+
+/* Synchronizes; copies the counters out. */
+um_status um_get_stats(um_arena *a, um_stats *out);
+
+/* Synchronizes; exports the observable result for parity: st[nblocks] (UM_ST_*),
+ * USED order (LRU first) and DISC order (FIFO head first) as block ids.  Buffers
+ * used_order/disc_order need room for nframes entries.  Any pointer may be NULL. */
+um_status um_dump(um_arena *a, uint8_t *st, uint32_t *used_order, uint32_t *n_used,
+                  uint32_t *disc_order, uint32_t *n_disc);
+
+/* Harness: synchronizes; content tag of every block (u64 per block): 0 = all-zero
+ * block, stamp s = block filled with the 16-byte pattern {s, ~s}, UINT64_MAX = anything
+ * else (corrupt).  Reads frames (G/GE/GL) or host frames (H; HD/U read as zero). */
+um_status um_content_tags(um_arena *a, uint64_t *tags);
+
+/* Harness: per-phase device timing of the last ops (ms), cumulative since reset. */
+um_status um_timing(um_arena *a, double *ms_plan, double *ms_xfer, int reset);
+
+const char *um_strerror(um_status s);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* UM_H */
