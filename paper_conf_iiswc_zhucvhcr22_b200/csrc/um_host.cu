@@ -1,0 +1,665 @@
+// Host runtime and C ABI of libum (include/um.h).
+//
+// The host side never inspects block states: it validates arguments, turns a batch of
+// accesses into sorted disjoint block intervals, splits GPU-destination ops into
+// sub-ops of <= nframes blocks (reading A3 of DESIGN.md), assigns sequence numbers,
+// stages the interval lists to the device and enqueues the kernel chain of
+// um_kernels.cu on the arena's paging stream.  All planning is on the device, so the
+// kernel-driven transfer path never round-trips to the host inside an op.
+#include "um_internal.h"
+
+#include <algorithm>
+#include <atomic>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <deque>
+#include <new>
+#include <vector>
+
+#include "../../include/um.h"
+
+#define UM_API extern "C" __attribute__((visibility("default")))
+
+using namespace um;
+
+namespace {
+
+constexpr uint64_t kAlign = 256;
+
+struct Layout {
+  uint64_t st, key, frame_of, map, hframe, pin, free_stack, hfree_stack;
+  uint64_t used[2], disc[2];
+  uint64_t need, needk, needhf, victim, vframe, vhf, vkind, d2h_frame, d2h_hf;
+  uint64_t tile_status, tags, ctl, hchunks, stage;
+  uint64_t stage_bytes, max_tiles, cap, total;
+};
+
+static uint64_t pow2_ceil(uint64_t x) {
+  uint64_t p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+static bool is_pow2(uint64_t x) { return x && !(x & (x - 1)); }
+
+static um_status check_cfg(const um_config* c) {
+  if (!c) return UM_EINVAL;
+  if (!is_pow2(c->block_bytes) || c->block_bytes < 4096) return UM_EINVAL;
+  if (c->arena_bytes == 0 || c->arena_bytes % c->block_bytes) return UM_EINVAL;
+  if (c->arena_bytes / c->block_bytes >= 0xffffffffull) return UM_EINVAL;
+  if (c->budget_bytes < c->block_bytes) return UM_EINVAL;
+  if (c->budget_bytes / c->block_bytes >= 0x7fffffffull) return UM_EINVAL;
+  if (c->host_chunk_bytes == 0 || c->host_chunk_bytes % c->block_bytes) return UM_EINVAL;
+  if (c->n_host_chunks == 0) return UM_EINVAL;
+  if ((uint64_t)c->n_host_chunks * (c->host_chunk_bytes / c->block_bytes) < 2) return UM_EINVAL;
+  return UM_OK;
+}
+
+static Layout make_layout(const um_config* c) {
+  Layout L{};
+  const uint64_t nb = c->arena_bytes / c->block_bytes;
+  const uint64_t nf = c->budget_bytes / c->block_bytes;
+  const uint64_t nh = (uint64_t)c->n_host_chunks * (c->host_chunk_bytes / c->block_bytes);
+  L.cap = pow2_ceil(std::max<uint64_t>(1024, 4 * nf));
+  L.max_tiles = (std::max(nb, L.cap) + kScanTile - 1) / kScanTile + 1;
+  L.stage_bytes = std::min<uint64_t>(64ull << 20, 12 * nb + (1 << 20));
+  uint64_t o = 0;
+  auto take = [&](uint64_t bytes) {
+    uint64_t r = o;
+    o += (bytes + kAlign - 1) / kAlign * kAlign;
+    return r;
+  };
+  L.st = take(nb);
+  L.key = take(4 * nb);
+  L.frame_of = take(4 * nb);
+  L.map = take(4 * nb);
+  L.hframe = take(4 * nb);
+  L.pin = take(4 * nb);
+  L.free_stack = take(4 * nf);
+  L.hfree_stack = take(4 * nh);
+  for (int i = 0; i < 2; ++i) L.used[i] = take(8 * L.cap);
+  for (int i = 0; i < 2; ++i) L.disc[i] = take(8 * L.cap);
+  L.need = take(4 * nf);
+  L.needk = take(nf);
+  L.needhf = take(4 * nf);
+  L.victim = take(4 * nf);
+  L.vframe = take(4 * nf);
+  L.vhf = take(4 * nf);
+  L.vkind = take(nf);
+  L.d2h_frame = take(4 * nf);
+  L.d2h_hf = take(4 * nf);
+  L.tile_status = take(8 * L.max_tiles);
+  L.tags = take(8 * nb);
+  L.ctl = take(sizeof(Ctl));
+  L.hchunks = take(8ull * c->n_host_chunks);
+  L.stage = take(L.stage_bytes);
+  L.total = o;
+  return L;
+}
+
+// Pinned host staging ring for interval lists, with events guarding in-flight copies.
+struct Stager {
+  uint8_t* host = nullptr;
+  uint8_t* dev = nullptr;
+  uint64_t cap = 0, pos = 0;
+  struct Fly { uint64_t lo, hi; cudaEvent_t ev; };
+  std::deque<Fly> fly;
+  std::vector<cudaEvent_t> pool;
+
+  cudaError_t init(uint8_t* d, uint64_t bytes) {
+    dev = d;
+    cap = bytes;
+    return cudaHostAlloc((void**)&host, bytes, cudaHostAllocDefault);
+  }
+  void destroy() {
+    for (auto& f : fly) cudaEventDestroy(f.ev);
+    for (auto e : pool) cudaEventDestroy(e);
+    fly.clear();
+    pool.clear();
+    if (host) cudaFreeHost(host);
+    host = nullptr;
+  }
+  // Reserve [off, off+bytes) of the ring; waits for copies still reading it.
+  cudaError_t reserve(uint64_t bytes, uint64_t* off) {
+    bytes = (bytes + 15) & ~15ull;
+    if (bytes > cap) return cudaErrorInvalidValue;
+    if (pos + bytes > cap) pos = 0;
+    uint64_t lo = pos, hi = pos + bytes;
+    while (!fly.empty()) {
+      Fly& f = fly.front();
+      bool overlap = f.lo < hi && lo < f.hi;
+      if (!overlap && cudaEventQuery(f.ev) != cudaSuccess) break;
+      cudaError_t e = cudaEventSynchronize(f.ev);
+      if (e) return e;
+      pool.push_back(f.ev);
+      fly.pop_front();
+    }
+    for (auto& f : fly)
+      if (f.lo < hi && lo < f.hi) {
+        cudaError_t e = cudaEventSynchronize(f.ev);
+        if (e) return e;
+      }
+    *off = lo;
+    pos = hi;
+    return cudaSuccess;
+  }
+  cudaError_t push(uint64_t off, uint64_t bytes, cudaStream_t s) {
+    cudaError_t e = cudaMemcpyAsync(dev + off, host + off, bytes, cudaMemcpyHostToDevice, s);
+    if (e) return e;
+    cudaEvent_t ev;
+    if (pool.empty()) {
+      e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+      if (e) return e;
+    } else {
+      ev = pool.back();
+      pool.pop_back();
+    }
+    e = cudaEventRecord(ev, s);
+    fly.push_back({off, off + bytes, ev});
+    return e;
+  }
+};
+
+struct Iv {
+  uint32_t lo, cnt;
+  uint8_t w;
+};
+
+}  // namespace
+
+struct um_arena {
+  um_config cfg{};
+  Layout L{};
+  Tables T{};
+  uint64_t* ring_buf[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};  // [ring][buffer]
+  int ring_cur[2] = {0, 0};
+  uint64_t ub[2] = {0, 0};  // upper bound of (tail - head) per ring
+  uint32_t B = 0, nblocks = 0, nframes = 0, nhframes = 0;
+  cudaStream_t ps = nullptr;
+  cudaEvent_t ev_in = nullptr, ev_out = nullptr;
+  uint32_t clock = 0;
+  uint64_t bump = 0;
+  int64_t ops = 0, subops = 0;
+  um_status sticky = UM_OK;
+  std::atomic<int> busy{0};
+  Stager stage;
+  Ctl* hctl = nullptr;  // pinned mirror for reads
+  std::vector<Iv> ivs;
+  std::vector<uint32_t> tmp_lo, tmp_pre;
+  std::vector<uint8_t> tmp_w;
+};
+
+namespace {
+
+struct Guard {
+  um_arena* a;
+  bool ok;
+  explicit Guard(um_arena* x) : a(x), ok(false) {
+    int z = 0;
+    ok = a && a->busy.compare_exchange_strong(z, 1);
+  }
+  ~Guard() {
+    if (ok) a->busy.store(0);
+  }
+};
+
+#define CK(x)                                         \
+  do {                                                \
+    cudaError_t e__ = (x);                            \
+    if (e__ != cudaSuccess) {                         \
+      a->sticky = UM_ECUDA;                           \
+      if (getenv("UM_DEBUG"))                         \
+        fprintf(stderr, "libum: %s at %s:%d\n", cudaGetErrorString(e__), __FILE__, __LINE__); \
+      return UM_ECUDA;                                \
+    }                                                 \
+  } while (0)
+
+#define ENTER(a)                           \
+  Guard g__(a);                            \
+  if (!a) return UM_EINVAL;                \
+  if (!g__.ok) return UM_EBUSY;            \
+  if (a->sticky != UM_OK) return a->sticky
+
+static um_status hand_in(um_arena* a, void* stream) {
+  cudaStream_t cs = (cudaStream_t)stream;
+  if (cs != a->ps) {
+    CK(cudaEventRecord(a->ev_in, cs));
+    CK(cudaStreamWaitEvent(a->ps, a->ev_in, 0));
+  }
+  return UM_OK;
+}
+
+static um_status hand_out(um_arena* a, void* stream) {
+  cudaStream_t cs = (cudaStream_t)stream;
+  if (cs != a->ps) {
+    CK(cudaEventRecord(a->ev_out, a->ps));
+    CK(cudaStreamWaitEvent(cs, a->ev_out, 0));
+  }
+  return UM_OK;
+}
+
+static void set_ring_ptrs(um_arena* a) {
+  a->T.used_ring = a->ring_buf[RING_USED][a->ring_cur[RING_USED]];
+  a->T.disc_ring = a->ring_buf[RING_DISC][a->ring_cur[RING_DISC]];
+}
+
+// K7 trigger: the host keeps an upper bound of each ring's occupancy (appends are
+// bounded by the op's block count; live entries never exceed nframes).
+static um_status ensure_ring_room(um_arena* a, int ring, uint64_t appends) {
+  if (a->ub[ring] + appends <= a->L.cap) {
+    a->ub[ring] += appends;
+    return UM_OK;
+  }
+  int nxt = a->ring_cur[ring] ^ 1;
+  CK(launch_ring_compact(a->T, ring, a->ring_buf[ring][nxt], a->L.cap, a->ps));
+  a->ring_cur[ring] = nxt;
+  set_ring_ptrs(a);
+  a->ub[ring] = std::min<uint64_t>(a->nframes, a->L.cap) + appends;
+  return UM_OK;
+}
+
+static bool range_ok(um_arena* a, uint64_t off, uint64_t len) {
+  return off <= a->cfg.arena_bytes && len <= a->cfg.arena_bytes - off;
+}
+
+// Sorted disjoint intervals with constant write flag from access records.
+static void build_intervals(um_arena* a, const um_access* acc, uint32_t n) {
+  struct Ev { uint64_t x; int dc, dw; };
+  std::vector<Ev> ev;
+  ev.reserve(2 * (size_t)n);
+  const uint64_t B = a->B;
+  for (uint32_t i = 0; i < n; ++i) {
+    if (!acc[i].len) continue;
+    uint64_t lo = acc[i].off / B, hi = (acc[i].off + acc[i].len - 1) / B + 1;
+    int w = (acc[i].kind & UM_ACC_WRITE) ? 1 : 0;
+    ev.push_back({lo, +1, w});
+    ev.push_back({hi, -1, -w});
+  }
+  std::sort(ev.begin(), ev.end(), [](const Ev& p, const Ev& q) { return p.x < q.x; });
+  a->ivs.clear();
+  int cov = 0, wr = 0;
+  for (size_t i = 0; i < ev.size();) {
+    uint64_t x = ev[i].x;
+    while (i < ev.size() && ev[i].x == x) {
+      cov += ev[i].dc;
+      wr += ev[i].dw;
+      ++i;
+    }
+    if (i < ev.size() && cov > 0) {
+      uint64_t nx = ev[i].x;
+      uint8_t w = wr > 0;
+      if (!a->ivs.empty() && (uint64_t)a->ivs.back().lo + a->ivs.back().cnt == x && a->ivs.back().w == w)
+        a->ivs.back().cnt += (uint32_t)(nx - x);
+      else
+        a->ivs.push_back({(uint32_t)x, (uint32_t)(nx - x), w});
+    }
+  }
+}
+
+// Enqueue the K1/K2 -> K3 -> K4/K5/K6 (-> K9) chain for every sub-op of a GPU op.
+static um_status run_gpu_op(um_arena* a, int touch) {
+  uint64_t total = 0;
+  bool anyw = false;
+  for (auto& v : a->ivs) {
+    total += v.cnt;
+    anyw |= v.w;
+  }
+  a->ops++;
+  if (total == 0) {
+    a->clock++;
+    a->subops++;
+    return UM_OK;
+  }
+  const uint32_t m = (uint32_t)a->ivs.size();
+  // stage lo[m], pre[m+1], w[m]
+  const uint64_t bytes_lo = 4ull * m, bytes_pre = 4ull * (m + 1), bytes_w = m;
+  const uint64_t o_lo = 0, o_pre = (bytes_lo + 15) & ~15ull, o_w = o_pre + ((bytes_pre + 15) & ~15ull);
+  const uint64_t bytes = o_w + bytes_w;
+  uint64_t off;
+  CK(a->stage.reserve(bytes, &off));
+  uint32_t* hlo = (uint32_t*)(a->stage.host + off + o_lo);
+  uint32_t* hpre = (uint32_t*)(a->stage.host + off + o_pre);
+  uint8_t* hw = a->stage.host + off + o_w;
+  uint32_t acc = 0;
+  for (uint32_t j = 0; j < m; ++j) {
+    hlo[j] = a->ivs[j].lo;
+    hpre[j] = acc;
+    hw[j] = a->ivs[j].w;
+    acc += a->ivs[j].cnt;
+  }
+  hpre[m] = acc;
+  CK(a->stage.push(off, (bytes + 15) & ~15ull, a->ps));
+  OpIv iv;
+  iv.lo = (const uint32_t*)(a->stage.dev + off + o_lo);
+  iv.pre = (const uint32_t*)(a->stage.dev + off + o_pre);
+  iv.wflag = a->stage.dev + off + o_w;
+  iv.m = m;
+  const uint32_t F = a->nframes;
+  for (uint64_t g0 = 0; g0 < total; g0 += F) {
+    const uint32_t n = (uint32_t)std::min<uint64_t>(F, total - g0);
+    const uint32_t seq = ++a->clock;
+    a->subops++;
+    um_status st = ensure_ring_room(a, RING_USED, n);
+    if (st) return st;
+    CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
+    CK(launch_victims(a->T, seq, 0, 0, a->ps));
+    CK(launch_service(a->T, SVC_SUBOP, seq, n, a->ps));
+    if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP))
+      CK(launch_app_stamp(a->T, iv, (uint32_t)g0, n, seq, a->ps));
+  }
+  return UM_OK;
+}
+
+}  // namespace
+
+// =====================================================================================
+// C ABI
+// =====================================================================================
+UM_API const char* um_strerror(um_status s) {
+  switch (s) {
+    case UM_OK: return "ok";
+    case UM_EINVAL: return "invalid argument";
+    case UM_ENOMEM: return "out of memory (arena or host-frame pool)";
+    case UM_ECUDA: return "CUDA error";
+    case UM_EBUSY: return "arena busy (concurrent call)";
+  }
+  return "unknown";
+}
+
+UM_API um_status um_workspace_size(const um_config* cfg, uint64_t* bytes) {
+  if (check_cfg(cfg) || !bytes) return UM_EINVAL;
+  *bytes = make_layout(cfg).total;
+  return UM_OK;
+}
+
+UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
+  if (check_cfg(cfg) || !out || !cfg->frames || !cfg->workspace || !cfg->host_chunks) return UM_EINVAL;
+  Layout L = make_layout(cfg);
+  if (cfg->workspace_bytes < L.total) return UM_EINVAL;
+  if (cfg->flags & UM_F_COPY_CE) return UM_EINVAL;  // copy-engine path: not in this build
+  um_arena* a = new (std::nothrow) um_arena();
+  if (!a) return UM_ENOMEM;
+  a->cfg = *cfg;
+  a->L = L;
+  a->B = cfg->block_bytes;
+  a->nblocks = (uint32_t)(cfg->arena_bytes / cfg->block_bytes);
+  a->nframes = (uint32_t)(cfg->budget_bytes / cfg->block_bytes);
+  const uint32_t hpc = (uint32_t)(cfg->host_chunk_bytes / cfg->block_bytes);
+  a->nhframes = cfg->n_host_chunks * hpc;
+  auto fail = [&](cudaError_t e) {
+    if (getenv("UM_DEBUG")) fprintf(stderr, "libum create: %s\n", cudaGetErrorString(e));
+    a->stage.destroy();
+    delete a;
+    return UM_ECUDA;
+  };
+  cudaError_t e;
+  if ((e = cudaSetDevice(cfg->device))) return fail(e);
+  if ((e = setup_kernels())) return fail(e);
+  char* ws = (char*)cfg->workspace;
+  Tables& T = a->T;
+  T.st = (uint8_t*)(ws + L.st);
+  T.key = (uint32_t*)(ws + L.key);
+  T.frame_of = (uint32_t*)(ws + L.frame_of);
+  T.map = (uint32_t*)(ws + L.map);
+  T.hframe = (uint32_t*)(ws + L.hframe);
+  T.pin = (uint32_t*)(ws + L.pin);
+  T.free_stack = (uint32_t*)(ws + L.free_stack);
+  T.hfree_stack = (uint32_t*)(ws + L.hfree_stack);
+  for (int i = 0; i < 2; ++i) {
+    a->ring_buf[RING_USED][i] = (uint64_t*)(ws + L.used[i]);
+    a->ring_buf[RING_DISC][i] = (uint64_t*)(ws + L.disc[i]);
+  }
+  T.cap_mask = L.cap - 1;
+  T.need = (uint32_t*)(ws + L.need);
+  T.needk = (uint8_t*)(ws + L.needk);
+  T.needhf = (uint32_t*)(ws + L.needhf);
+  T.victim = (uint32_t*)(ws + L.victim);
+  T.vframe = (uint32_t*)(ws + L.vframe);
+  T.vhf = (uint32_t*)(ws + L.vhf);
+  T.vkind = (uint8_t*)(ws + L.vkind);
+  T.d2h_frame = (uint32_t*)(ws + L.d2h_frame);
+  T.d2h_hf = (uint32_t*)(ws + L.d2h_hf);
+  T.tile_status = (unsigned long long*)(ws + L.tile_status);
+  T.tags = (uint64_t*)(ws + L.tags);
+  T.ctl = (Ctl*)(ws + L.ctl);
+  T.frames = (char*)cfg->frames;
+  T.hpc = hpc;
+  T.B = a->B;
+  T.nblocks = a->nblocks;
+  T.nframes = a->nframes;
+  T.nhframes = a->nhframes;
+  T.zero_hf = a->nhframes - 1;  // last host frame: the shared zero page
+  set_ring_ptrs(a);
+  // host chunk table (device pointers of the mapped pinned chunks)
+  std::vector<char*> hc(cfg->n_host_chunks);
+  for (uint32_t i = 0; i < cfg->n_host_chunks; ++i) {
+    void* dp = nullptr;
+    if (cudaHostGetDevicePointer(&dp, cfg->host_chunks[i], 0) != cudaSuccess) {
+      cudaGetLastError();
+      dp = cfg->host_chunks[i];  // UVA: the host pointer is the device pointer
+    }
+    hc[i] = (char*)dp;
+  }
+  char** dhc = (char**)(ws + L.hchunks);
+  T.hchunks = dhc;
+  // zero page
+  {
+    uint32_t z = T.zero_hf;
+    memset((char*)cfg->host_chunks[z / hpc] + (size_t)(z % hpc) * a->B, 0, a->B);
+  }
+  if ((e = cudaStreamCreateWithFlags(&a->ps, cudaStreamNonBlocking))) return fail(e);
+  if ((e = cudaEventCreateWithFlags(&a->ev_in, cudaEventDisableTiming))) return fail(e);
+  if ((e = cudaEventCreateWithFlags(&a->ev_out, cudaEventDisableTiming))) return fail(e);
+  if ((e = cudaHostAlloc((void**)&a->hctl, sizeof(Ctl), cudaHostAllocDefault))) return fail(e);
+  if ((e = a->stage.init((uint8_t*)(ws + L.stage), L.stage_bytes))) return fail(e);
+  if ((e = cudaMemcpyAsync(dhc, hc.data(), 8ull * cfg->n_host_chunks, cudaMemcpyHostToDevice, a->ps))) return fail(e);
+  if ((e = cudaMemsetAsync(T.tile_status, 0, 8 * L.max_tiles, a->ps))) return fail(e);
+  if ((e = launch_init(T, (int)(a->nhframes - 1), a->ps))) return fail(e);
+  if (cfg->flags & UM_F_CHECK)
+    if ((e = launch_poison(T, a->ps))) return fail(e);
+  if ((e = cudaStreamSynchronize(a->ps))) return fail(e);
+  *out = a;
+  return UM_OK;
+}
+
+UM_API um_status um_arena_destroy(um_arena* a) {
+  if (!a) return UM_EINVAL;
+  if (a->ps) cudaStreamSynchronize(a->ps);
+  a->stage.destroy();
+  if (a->hctl) cudaFreeHost(a->hctl);
+  if (a->ev_in) cudaEventDestroy(a->ev_in);
+  if (a->ev_out) cudaEventDestroy(a->ev_out);
+  if (a->ps) cudaStreamDestroy(a->ps);
+  delete a;
+  return UM_OK;
+}
+
+UM_API um_status um_alloc(um_arena* a, uint64_t bytes, uint64_t* off) {
+  ENTER(a);
+  if (!off) return UM_EINVAL;
+  uint64_t r = (bytes + a->B - 1) / a->B * a->B;
+  if (a->bump + r > a->cfg.arena_bytes || r < bytes) return UM_ENOMEM;
+  *off = a->bump;
+  a->bump += r;
+  return UM_OK;
+}
+
+UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, void* stream) {
+  ENTER(a);
+  if (n && !acc) return UM_EINVAL;
+  for (uint32_t i = 0; i < n; ++i)
+    if (!range_ok(a, acc[i].off, acc[i].len)) return UM_EINVAL;
+  build_intervals(a, acc, n);
+  um_status s = hand_in(a, stream);
+  if (s) return s;
+  s = run_gpu_op(a, 1);
+  if (s) return s;
+  return hand_out(a, stream);
+}
+
+UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, void* stream) {
+  ENTER(a);
+  if (!range_ok(a, off, len) || (dst != UM_DST_GPU && dst != UM_DST_HOST)) return UM_EINVAL;
+  um_status s = hand_in(a, stream);
+  if (s) return s;
+  if (dst == UM_DST_GPU) {
+    a->ivs.clear();
+    if (len) {
+      uint64_t lo = off / a->B, hi = (off + len - 1) / a->B + 1;
+      a->ivs.push_back({(uint32_t)lo, (uint32_t)(hi - lo), 0});
+    }
+    s = run_gpu_op(a, 0);
+    if (s) return s;
+  } else {
+    a->ops++;
+    a->subops++;
+    const uint32_t seq = ++a->clock;
+    if (len) {
+      uint32_t lo = (uint32_t)(off / a->B), hi = (uint32_t)((off + len - 1) / a->B + 1);
+      CK(launch_directive(a->T, DIR_PREFETCH_HOST, lo, hi - lo, seq, 0, a->ps));
+      CK(launch_service(a->T, SVC_D2H_ONLY, seq, std::min<uint32_t>(hi - lo, a->nframes), a->ps));
+    }
+  }
+  return hand_out(a, stream);
+}
+
+static um_status discard_common(um_arena* a, uint64_t off, uint64_t len, void* stream, int kind) {
+  ENTER(a);
+  if (!range_ok(a, off, len)) return UM_EINVAL;
+  um_status s = hand_in(a, stream);
+  if (s) return s;
+  a->ops++;
+  a->subops++;
+  const uint32_t seq = ++a->clock;
+  const uint64_t lo = (off + a->B - 1) / a->B, hi = (off + len) / a->B;  // fully covered blocks
+  if (hi > lo && !(a->cfg.flags & UM_F_DISCARD_OFF)) {
+    const uint32_t n = (uint32_t)(hi - lo);
+    s = ensure_ring_room(a, RING_DISC, std::min<uint32_t>(n, a->nframes));
+    if (s) return s;
+    CK(launch_directive(a->T, kind, (uint32_t)lo, n, seq, 0, a->ps));
+  }
+  return hand_out(a, stream);
+}
+
+UM_API um_status um_discard(um_arena* a, uint64_t off, uint64_t len, void* stream) {
+  return discard_common(a, off, len, stream, DIR_DISCARD);
+}
+
+UM_API um_status um_discard_lazy(um_arena* a, uint64_t off, uint64_t len, void* stream) {
+  return discard_common(a, off, len, stream, DIR_DISCARD_LAZY);
+}
+
+UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
+  ENTER(a);
+  um_status s = hand_in(a, stream);
+  if (s) return s;
+  a->ops++;
+  a->subops++;
+  const uint32_t seq = ++a->clock;
+  uint64_t want = (bytes + a->B - 1) / a->B;
+  if (want > a->nframes) want = a->nframes;
+  if (want) {
+    CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->ps));
+    CK(launch_service(a->T, SVC_D2H_ONLY, seq, (uint32_t)want, a->ps));
+  }
+  return hand_out(a, stream);
+}
+
+UM_API um_status um_host_write(um_arena* a, uint64_t off, uint64_t len, void* stream) {
+  ENTER(a);
+  if (!range_ok(a, off, len)) return UM_EINVAL;
+  um_status s = hand_in(a, stream);
+  if (s) return s;
+  a->ops++;
+  a->subops++;
+  const uint32_t seq = ++a->clock;
+  if (len) {
+    uint32_t lo = (uint32_t)(off / a->B), hi = (uint32_t)((off + len - 1) / a->B + 1);
+    CK(launch_host_write(a->T, lo, hi - lo, seq, a->ps));
+  }
+  return hand_out(a, stream);
+}
+
+UM_API um_status um_block_table(um_arena* a, const uint32_t** dev_map) {
+  if (!a || !dev_map) return UM_EINVAL;
+  *dev_map = a->T.map;
+  return UM_OK;
+}
+
+UM_API um_status um_stream(um_arena* a, void** stream) {
+  if (!a || !stream) return UM_EINVAL;
+  *stream = (void*)a->ps;
+  return UM_OK;
+}
+
+static um_status sync_ctl(um_arena* a) {
+  CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaStreamSynchronize(a->ps));
+  if (a->hctl->err == 1u) a->sticky = UM_EINVAL;
+  if (a->hctl->err == 2u) a->sticky = UM_ENOMEM;
+  return a->sticky;
+}
+
+UM_API um_status um_get_stats(um_arena* a, um_stats* out) {
+  ENTER(a);
+  if (!out) return UM_EINVAL;
+  um_status s = sync_ctl(a);
+  int64_t v[16];
+  for (int i = 0; i < 16; ++i) v[i] = a->hctl->stats[i];
+  v[S_OPS] = a->ops;
+  v[S_SUBOPS] = a->subops;
+  memcpy(out, v, sizeof(um_stats));
+  return s;
+}
+
+UM_API um_status um_dump(um_arena* a, uint8_t* st, uint32_t* used_order, uint32_t* n_used, uint32_t* disc_order,
+                         uint32_t* n_disc) {
+  ENTER(a);
+  um_status s = sync_ctl(a);
+  if (s) return s;
+  std::vector<uint8_t> hst(a->nblocks);
+  std::vector<uint32_t> hkey(a->nblocks);
+  CK(cudaMemcpy(hst.data(), a->T.st, a->nblocks, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(hkey.data(), a->T.key, 4ull * a->nblocks, cudaMemcpyDeviceToHost));
+  if (st) memcpy(st, hst.data(), a->nblocks);
+  std::vector<uint64_t> ring(a->L.cap);
+  for (int r = 0; r < 2; ++r) {
+    uint32_t* outp = r == RING_USED ? used_order : disc_order;
+    uint32_t* outn = r == RING_USED ? n_used : n_disc;
+    if (!outp && !outn) continue;
+    CK(cudaMemcpy(ring.data(), r == RING_USED ? a->T.used_ring : a->T.disc_ring, 8 * a->L.cap, cudaMemcpyDeviceToHost));
+    unsigned long long head = r == RING_USED ? a->hctl->used_head : a->hctl->disc_head;
+    unsigned long long tail = r == RING_USED ? a->hctl->used_tail : a->hctl->disc_tail;
+    uint32_t cnt = 0;
+    for (unsigned long long p = head; p < tail; ++p) {
+      uint64_t e = ring[p & (a->L.cap - 1)];
+      uint32_t b = (uint32_t)e, k = (uint32_t)(e >> 32);
+      uint8_t x = hst[b];
+      bool live = (r == RING_USED ? x == ST_G : (x == ST_GE || x == ST_GL)) && hkey[b] == k;
+      if (live) {
+        if (outp && cnt < a->nframes) outp[cnt] = b;
+        ++cnt;
+      }
+    }
+    if (outn) *outn = cnt;
+  }
+  return UM_OK;
+}
+
+UM_API um_status um_content_tags(um_arena* a, uint64_t* tags) {
+  ENTER(a);
+  if (!tags) return UM_EINVAL;
+  CK(launch_tags(a->T, a->ps));
+  CK(cudaMemcpyAsync(tags, a->T.tags, 8ull * a->nblocks, cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaStreamSynchronize(a->ps));
+  return UM_OK;
+}
+
+UM_API um_status um_timing(um_arena* a, double* ms_plan, double* ms_xfer, int reset) {
+  if (!a) return UM_EINVAL;
+  (void)reset;
+  if (ms_plan) *ms_plan = 0;
+  if (ms_xfer) *ms_xfer = 0;
+  return UM_OK;
+}

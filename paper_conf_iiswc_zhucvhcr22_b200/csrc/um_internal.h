@@ -1,0 +1,108 @@
+// Internal layout shared by the host runtime (um_host.cu) and the kernels
+// (um_kernels.cu).  Not part of the ABI.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#define UM_NONE 0xffffffffu
+
+namespace um {
+
+// Block states (same values as UM_ST_* in include/um.h).
+enum : uint8_t { ST_U = 0, ST_H = 1, ST_HD = 2, ST_G = 3, ST_GE = 4, ST_GL = 5 };
+
+// Stats slots (order of um_stats).
+enum {
+  S_H2D = 0, S_D2H, S_ZF, S_H2D_AV, S_D2H_AV, S_FAULTS, S_HITS, S_REMAPS, S_UNMAPS,
+  S_REVAL, S_REFRESH, S_EVICT, S_OPS, S_SUBOPS, S_N = 16
+};
+
+// Device control block: ring cursors, free-stack tops, the current sub-op's plan
+// sizes, counters and the self-cleaning scan state.
+struct Ctl {
+  unsigned long long used_head, used_tail, disc_head, disc_tail;
+  int free_top;          // free GPU frames: free_stack[0, free_top)
+  int hfree_top;         // free host frames: hfree_stack[0, hfree_top)
+  unsigned int n_need;   // current sub-op: blocks needing a frame (need list length)
+  unsigned int n_rekey;  // current sub-op: USED appends staged at used_tail
+  unsigned int f0;       // free_top when the sub-op's victims were chosen
+  unsigned int n_vict;   // victims chosen
+  unsigned int n_d2h;    // D2H-only work-list length (prefetch HOST / evict)
+  unsigned int err;      // sticky device error (0 or -um_status)
+  unsigned int scan_ticket, scan_done;  // decoupled look-back tile ticket / completion
+  unsigned int app_units;               // unused scratch
+  unsigned int pad[3];
+  long long stats[S_N];
+};
+
+// Everything a kernel needs, passed by value.
+struct Tables {
+  uint8_t* st;          // [nblocks] state
+  uint32_t* key;        // [nblocks] ukey / dkey (seq)
+  uint32_t* frame_of;   // [nblocks] GPU frame (G/GE/GL) or NONE
+  uint32_t* map;        // [nblocks] app-visible table: frame if mapped (G/GL) else NONE
+  uint32_t* hframe;     // [nblocks] host frame holding the block's data (H only) or NONE
+  uint32_t* pin;        // [nblocks] seq of the sub-op that pinned the block
+  uint32_t* free_stack; // [nframes]
+  uint32_t* hfree_stack;// [nhframes]
+  uint64_t* used_ring;  // [cap] (key<<32)|block, current buffer
+  uint64_t* disc_ring;  // [cap]
+  uint64_t cap_mask;
+  uint32_t* need;       // [nframes] blocks needing a frame, ascending
+  uint8_t* needk;       // [nframes] their state at classification
+  uint32_t* needhf;     // [nframes] their host frame at classification (H) or NONE
+  uint32_t* victim;     // [nframes] victims, in eviction order
+  uint32_t* vframe;     // [nframes] victim's frame
+  uint32_t* vhf;        // [nframes] host frame receiving a G victim's write-back, else NONE
+  uint8_t* vkind;       // [nframes] victim's state when chosen
+  uint32_t* d2h_frame;  // [nframes] D2H-only list (prefetch HOST, evict)
+  uint32_t* d2h_hf;     // [nframes]
+  unsigned long long* tile_status;  // [max tiles] decoupled look-back
+  uint64_t* tags;       // [nblocks] content tags (harness)
+  Ctl* ctl;
+  char* frames;             // device, nframes * B
+  char* const* hchunks;     // device array of host-chunk device pointers
+  uint32_t hpc;             // host frames per chunk
+  uint32_t B;               // block bytes
+  uint32_t nblocks, nframes, nhframes;
+  uint32_t zero_hf;         // host frame id of the zero page (never allocated)
+};
+
+// A GPU-destination op's distinct blocks as sorted disjoint intervals.  Interval j
+// covers blocks [lo[j], lo[j] + pre[j+1] - pre[j]); pre[] is the op-global exclusive
+// prefix of block counts; wflag[j] = the interval holds UM_ACC_WRITE blocks.
+struct OpIv {
+  const uint32_t* lo;
+  const uint32_t* pre;
+  const uint8_t* wflag;
+  uint32_t m;
+};
+
+constexpr int kScanTPB = 256;
+constexpr int kScanIPT = 4;
+constexpr int kScanTile = kScanTPB * kScanIPT;
+constexpr int kVictTPB = 1024;
+constexpr int kVictIPT = 4;
+constexpr int kXferStages = 4;
+constexpr uint32_t kXferChunk = 16384;
+
+enum SvcMode { SVC_SUBOP = 0, SVC_D2H_ONLY = 1 };
+enum DirKind { DIR_DISCARD = 0, DIR_DISCARD_LAZY = 1, DIR_PREFETCH_HOST = 2 };
+enum RingId { RING_USED = 0, RING_DISC = 1 };
+
+// Launch wrappers (um_kernels.cu).  All enqueue on `s`; none synchronizes.
+cudaError_t setup_kernels();
+cudaError_t launch_init(const Tables& T, int nhframes_alloc, cudaStream_t s);
+cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
+                            cudaStream_t s);
+cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, cudaStream_t s);
+cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max_items, cudaStream_t s);
+cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, cudaStream_t s);
+cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
+                             int discard_off, cudaStream_t s);
+cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64_t cap_bound, cudaStream_t s);
+cudaError_t launch_host_write(const Tables& T, uint32_t lo, uint32_t n, uint32_t seq, cudaStream_t s);
+cudaError_t launch_tags(const Tables& T, cudaStream_t s);
+cudaError_t launch_poison(const Tables& T, cudaStream_t s);
+
+}  // namespace um

@@ -1,0 +1,923 @@
+// sm_100a kernels of libum: the state/directive kernels (K1/K2 classify + ordered
+// compaction, K3 victim selection, K6 commit, K7 ring compaction, K8 directives), the
+// TMA-staged transfer engine over mapped pinned host memory with zero-fill (K4/K5),
+// and harness kernels (application stamp writes, content tags, host writes).
+//
+// Paper: "UVM Discard" (Zhu et al., IISWC'22).  PAPER L<n> = line of its text.
+// Design: DESIGN.md §4 (data layout) and §5 (kernels).  No tensor cores: nothing here
+// is a contraction.  Everything is integer/byte movement.
+#include "um_internal.h"
+
+#include <cstdio>
+
+namespace um {
+
+#define FULL 0xffffffffu
+
+__constant__ int c_dummy;
+
+// ------------------------------------------------------------------------------------
+// small helpers
+// ------------------------------------------------------------------------------------
+__device__ __forceinline__ char* hptr(const Tables& T, uint32_t hf) {
+  return T.hchunks[hf / T.hpc] + (size_t)(hf % T.hpc) * T.B;
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// Largest j in [0, m) with pre[j] <= g (pre strictly increasing, pre[0] = 0).
+__device__ __forceinline__ uint32_t iv_find(const OpIv& iv, uint32_t g) {
+  uint32_t lo = 0, hi = iv.m;  // answer in [lo, hi)
+  while (hi - lo > 1) {
+    uint32_t mid = (lo + hi) >> 1;
+    if (iv.pre[mid] <= g) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ void stat_add(const Tables& T, int slot, long long v) {
+  if (v) atomicAdd((unsigned long long*)&T.ctl->stats[slot], (unsigned long long)v);
+}
+
+// Exclusive block scan of a 64-bit value (two packed 31-bit counts add without carry).
+template <int TPB>
+__device__ __forceinline__ unsigned long long block_excl_scan(unsigned long long v, unsigned long long& total,
+                                                              unsigned long long* sm) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  unsigned long long x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    unsigned long long y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) sm[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    unsigned long long t = lane < TPB / 32 ? sm[lane] : 0ull;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      unsigned long long y = __shfl_up_sync(FULL, t, o);
+      if (lane >= o) t += y;
+    }
+    if (lane < TPB / 32) sm[lane] = t;
+  }
+  __syncthreads();
+  unsigned long long pre = (w ? sm[w - 1] : 0ull) + x - v;
+  total = sm[TPB / 32 - 1];
+  __syncthreads();
+  return pre;
+}
+
+// Decoupled look-back (single pass, tiles ordered by a ticket so predecessors always
+// run): returns the exclusive prefix of this tile.  Status word = flag(2b) | value(62b).
+__device__ unsigned long long lookback(const Tables& T, uint32_t tile, unsigned long long agg) {
+  volatile unsigned long long* st = T.tile_status;
+  const unsigned long long FA = 1ull << 62, FP = 2ull << 62, M = FA - 1;
+  if (tile == 0) {
+    st[0] = FP | agg;
+    __threadfence();
+    return 0ull;
+  }
+  st[tile] = FA | agg;
+  __threadfence();
+  unsigned long long excl = 0;
+  int p = (int)tile - 1;
+  while (true) {
+    unsigned long long v;
+    do { v = st[p]; } while ((v >> 62) == 0);
+    excl += v & M;
+    if ((v >> 62) == 2) break;
+    --p;
+  }
+  st[tile] = FP | (excl + agg);
+  __threadfence();
+  return excl;
+}
+
+// Called by every thread at the end of a scanning CTA: the last CTA to finish clears
+// the tile statuses and the ticket, so the next scanning launch starts clean.
+__device__ void scan_finish(const Tables& T, uint32_t ntiles) {
+  __shared__ int s_last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    unsigned int d = atomicAdd(&T.ctl->scan_done, 1u);
+    s_last = (d == ntiles - 1);
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    for (uint32_t i = threadIdx.x; i < ntiles; i += blockDim.x) T.tile_status[i] = 0ull;
+    if (threadIdx.x == 0) {
+      T.ctl->scan_done = 0;
+      T.ctl->scan_ticket = 0;
+    }
+    __threadfence();
+  }
+}
+
+__device__ __forceinline__ uint32_t take_ticket(const Tables& T) {
+  __shared__ uint32_t s_tile;
+  if (threadIdx.x == 0) s_tile = atomicAdd(&T.ctl->scan_ticket, 1u);
+  __syncthreads();
+  return s_tile;
+}
+
+__device__ __forceinline__ unsigned long long pack2(uint32_t a, uint32_t b) {
+  return (unsigned long long)a | ((unsigned long long)b << 31);
+}
+__device__ __forceinline__ uint32_t unpackA(unsigned long long v) { return (uint32_t)(v & 0x7fffffffull); }
+__device__ __forceinline__ uint32_t unpackB(unsigned long long v) { return (uint32_t)((v >> 31) & 0x7fffffffull); }
+
+// Sum of per-thread class counts over the CTA, then one atomic per class.
+template <int NC>
+__device__ __forceinline__ void block_counts_to(const Tables& T, uint32_t (&c)[NC], uint32_t* sm /*[NC]*/,
+                                                const int (&slots)[NC], const long long (&mul)[NC]) {
+  if (threadIdx.x < NC) sm[threadIdx.x] = 0;
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < NC; ++i) {
+    uint32_t v = __reduce_add_sync(FULL, c[i]);
+    if ((threadIdx.x & 31) == 0 && v) atomicAdd(&sm[i], v);
+  }
+  __syncthreads();
+  if (threadIdx.x < NC && slots[threadIdx.x] >= 0) stat_add(T, slots[threadIdx.x], (long long)sm[threadIdx.x] * mul[threadIdx.x]);
+}
+
+// ------------------------------------------------------------------------------------
+// init / poison
+// ------------------------------------------------------------------------------------
+__global__ void k_init(Tables T, int nh) {
+  size_t tid = blockIdx.x * (size_t)blockDim.x + threadIdx.x, str = (size_t)gridDim.x * blockDim.x;
+  for (size_t i = tid; i < T.nblocks; i += str) {
+    T.st[i] = ST_U;
+    T.key[i] = 0;
+    T.frame_of[i] = UM_NONE;
+    T.map[i] = UM_NONE;
+    T.hframe[i] = UM_NONE;
+    T.pin[i] = 0;
+  }
+  for (size_t i = tid; i < T.nframes; i += str) T.free_stack[i] = T.nframes - 1 - (uint32_t)i;
+  for (size_t i = tid; i < (size_t)nh; i += str) T.hfree_stack[i] = (uint32_t)(nh - 1 - i);
+  if (tid == 0) {
+    Ctl* c = T.ctl;
+    c->used_head = c->used_tail = c->disc_head = c->disc_tail = 0;
+    c->free_top = (int)T.nframes;
+    c->hfree_top = nh;
+    c->n_need = c->n_rekey = c->f0 = c->n_vict = c->n_d2h = c->err = 0;
+    c->scan_ticket = c->scan_done = c->app_units = 0;
+    for (int i = 0; i < S_N; ++i) c->stats[i] = 0;
+  }
+}
+
+__global__ void k_poison(char* p, size_t bytes) {
+  size_t n = bytes / 16;
+  uint4 v = make_uint4(0xA5A5A5A5u, 0xA5A5A5A5u, 0xA5A5A5A5u, 0xA5A5A5A5u);
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+    reinterpret_cast<uint4*>(p)[i] = v;
+}
+
+// ------------------------------------------------------------------------------------
+// K1+K2: classify a GPU-destination sub-op and compact its work lists in ascending
+// block order (warp ballot/popc-free: per-thread counts + block scan + decoupled
+// look-back).  Transitions that need no frame are committed here (refresh, revive
+// GE->G with re-map, revalidate GL->G: PAPER L217, L229, L190); blocks that need a
+// frame (U/H/HD) are listed for K3/K4.  Every rekeyed block is appended to USED at
+// used_tail + rank with key = seq, in ascending block order.
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
+                                                       int touch) {
+  __shared__ unsigned long long s_scan[kScanTPB / 32];
+  __shared__ unsigned long long s_excl;
+  __shared__ unsigned long long s_tail0;
+  __shared__ uint32_t s_cnt[6];
+  if (threadIdx.x == 0) s_tail0 = T.ctl->used_tail;
+  const uint32_t tile = take_ticket(T);
+  const uint32_t ntiles = n ? (n + kScanTile - 1) / kScanTile : 1;
+  const uint32_t first = tile * kScanTile + threadIdx.x * kScanIPT;
+
+  uint32_t b[kScanIPT];
+  uint8_t s[kScanIPT];
+  uint32_t cN = 0, cR = 0;
+  uint32_t cls[6] = {0, 0, 0, 0, 0, 0};
+  unsigned needm = 0, rekm = 0;
+  if (first < n) {
+    uint32_t j = iv_find(iv, g0 + first);
+#pragma unroll
+    for (int k = 0; k < kScanIPT; ++k) {
+      uint32_t idx = first + k;
+      if (idx < n) {
+        uint32_t g = g0 + idx;
+        while (g >= iv.pre[j + 1]) ++j;
+        uint32_t bb = iv.lo[j] + (g - iv.pre[j]);
+        uint8_t ss = T.st[bb];
+        T.pin[bb] = seq;
+        b[k] = bb;
+        s[k] = ss;
+        bool nd = ss <= ST_HD;
+        bool rk = touch ? (nd || ss == ST_GE) : true;
+        needm |= (unsigned)nd << k;
+        rekm |= (unsigned)rk << k;
+        cN += nd;
+        cR += rk;
+        cls[ss]++;
+      }
+    }
+  }
+  unsigned long long tot;
+  unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cN, cR), tot, s_scan);
+  if (threadIdx.x == 0) s_excl = lookback(T, tile, tot);
+  __syncthreads();
+  const unsigned long long base = s_excl + pre;
+  uint32_t pN = unpackA(base), pR = unpackB(base);
+  const unsigned long long tail0 = s_tail0;
+  if (first < n) {
+#pragma unroll
+    for (int k = 0; k < kScanIPT; ++k) {
+      if (first + k >= n) break;
+      const uint32_t bb = b[k];
+      const uint8_t ss = s[k];
+      const bool nd = (needm >> k) & 1, rk = (rekm >> k) & 1;
+      if (nd) {
+        T.need[pN] = bb;
+        T.needk[pN] = ss;
+        T.needhf[pN] = (ss == ST_H) ? T.hframe[bb] : UM_NONE;
+        ++pN;
+      }
+      if (rk) {
+        T.used_ring[(tail0 + pR) & T.cap_mask] = ((unsigned long long)seq << 32) | bb;
+        ++pR;
+        if (!nd) {
+          T.key[bb] = seq;
+          if (ss == ST_GE) {        // revive: re-map the frame kept since the discard
+            T.st[bb] = ST_G;
+            T.map[bb] = T.frame_of[bb];
+          } else if (ss == ST_GL) { // revalidate: mapping was kept (lazy)
+            T.st[bb] = ST_G;
+          }
+        }
+      }
+    }
+  }
+  // counters
+  {
+    const long long B = T.B;
+    // classes: U H HD G GE GL
+    uint32_t c6[6] = {cls[0], cls[1], cls[2], cls[3], cls[4], cls[5]};
+    if (touch) {
+      // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE ; h2d: H ; zf: U+HD ; h2d_av: HD
+      uint32_t v[6] = {c6[0] + c6[1] + c6[2] + c6[4], c6[3] + c6[5], c6[4], c6[1], c6[0] + c6[2], c6[2]};
+      const int slots[6] = {S_FAULTS, S_HITS, S_REMAPS, S_H2D, S_ZF, S_H2D_AV};
+      const long long mul[6] = {1, 1, 1, B, B, B};
+      block_counts_to<6>(T, v, s_cnt, slots, mul);
+    } else {
+      uint32_t v[6] = {c6[3], c6[4], c6[5], c6[1], c6[0] + c6[2], c6[2]};
+      const int slots[6] = {S_REFRESH, S_REMAPS, S_REVAL, S_H2D, S_ZF, S_H2D_AV};
+      const long long mul[6] = {1, 1, 1, B, B, B};
+      block_counts_to<6>(T, v, s_cnt, slots, mul);
+    }
+  }
+  if (tile == ntiles - 1 && threadIdx.x == 0) {
+    unsigned long long all = s_excl + tot;
+    T.ctl->n_need = unpackA(all);
+    T.ctl->n_rekey = unpackB(all);
+  }
+  scan_finish(T, ntiles);
+}
+
+// ------------------------------------------------------------------------------------
+// K3: victim selection + reclaim (PAPER §5.5: free -> (unused, empty) ->
+// discarded FIFO -> used LRU; §5.3: discarded victims need no transfer; A10:
+// valid victims are written back).  One CTA scans each ring from its head in windows,
+// ranks live & unpinned entries with a block scan and takes the first k; the head
+// advances over the maximal prefix of dead or consumed entries.
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, int evict_mode, uint32_t want) {
+  __shared__ unsigned long long s_scan[kVictTPB / 32];
+  __shared__ unsigned long long s_minkeep;
+  __shared__ uint32_t s_cnt[4];
+  Ctl* c = T.ctl;
+  const int f0 = c->free_top;
+  const uint32_t nn = evict_mode ? 0u : c->n_need;
+  uint32_t k;
+  if (evict_mode) k = want > (uint32_t)f0 ? want - (uint32_t)f0 : 0u;
+  else k = nn > (uint32_t)f0 ? nn - (uint32_t)f0 : 0u;
+  uint32_t found = 0;
+  const uint32_t W = kVictTPB * kVictIPT;
+  for (int r = 0; r < 2; ++r) {
+    const int ring = r == 0 ? RING_DISC : RING_USED;
+    uint64_t* R = ring == RING_DISC ? T.disc_ring : T.used_ring;
+    unsigned long long* headp = ring == RING_DISC ? &c->disc_head : &c->used_head;
+    const unsigned long long head = *headp;
+    const unsigned long long tail = ring == RING_DISC ? c->disc_tail : c->used_tail;
+    unsigned long long pos = head, newhead = head;
+    bool blocked = false;
+    while (found < k && pos < tail) {
+      const uint32_t w = (uint32_t)min((unsigned long long)W, tail - pos);
+      const uint32_t first = threadIdx.x * kVictIPT;
+      uint32_t bb[kVictIPT];
+      unsigned candm = 0, livem = 0;
+      uint32_t cc = 0;
+#pragma unroll
+      for (int q = 0; q < kVictIPT; ++q) {
+        bb[q] = 0;
+        if (first + q < w) {
+          unsigned long long e = R[(pos + first + q) & T.cap_mask];
+          uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
+          uint8_t ss = T.st[blk];
+          bool live = (ring == RING_USED ? ss == ST_G : (ss == ST_GE || ss == ST_GL)) && T.key[blk] == kk;
+          bool cand = live && T.pin[blk] != seq;
+          bb[q] = blk;
+          livem |= (unsigned)live << q;
+          candm |= (unsigned)cand << q;
+          cc += cand;
+        }
+      }
+      unsigned long long tot;
+      uint32_t rank = (uint32_t)block_excl_scan<kVictTPB>(cc, tot, s_scan);
+      if (threadIdx.x == 0) s_minkeep = ~0ull;
+      __syncthreads();
+      unsigned long long mykeep = ~0ull;
+#pragma unroll
+      for (int q = 0; q < kVictIPT; ++q) {
+        bool sel = false;
+        if ((candm >> q) & 1) {
+          uint32_t rr = found + rank++;
+          if (rr < k) {
+            T.victim[rr] = bb[q];
+            sel = true;
+          }
+        }
+        if (((livem >> q) & 1) && !sel && mykeep == ~0ull) mykeep = pos + first + q;
+      }
+      if (mykeep != ~0ull) atomicMin(&s_minkeep, mykeep);
+      __syncthreads();
+      if (!blocked) {
+        if (s_minkeep != ~0ull) {
+          newhead = s_minkeep;
+          blocked = true;
+        } else {
+          newhead = pos + w;
+        }
+      }
+      found = (uint32_t)min((unsigned long long)k, found + tot);
+      pos += w;
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) *headp = newhead;
+  }
+  __syncthreads();
+  // Reclaim the victims.  G victims are written back (host frames are assigned in
+  // victim order from the host free stack); GE/GL victims are dropped.
+  const int htop = c->hfree_top;
+  uint32_t gbase = 0;
+  uint32_t nGL = 0;
+  for (uint32_t base = 0; base < found; base += kVictTPB) {
+    const uint32_t j = base + threadIdx.x;
+    uint32_t v = 0, fr = UM_NONE;
+    uint8_t ss = 0;
+    uint32_t isG = 0;
+    if (j < found) {
+      v = T.victim[j];
+      ss = T.st[v];
+      fr = T.frame_of[v];
+      isG = ss == ST_G;
+    }
+    unsigned long long tot;
+    uint32_t gr = (uint32_t)block_excl_scan<kVictTPB>(isG, tot, s_scan) + gbase;
+    if (j < found) {
+      uint32_t hf = UM_NONE;
+      if (isG) {
+        int idx = htop - 1 - (int)gr;
+        if (idx >= 0) hf = T.hfree_stack[idx];
+        else atomicExch(&c->err, 2u);  // host-frame pool exhausted -> UM_ENOMEM
+      }
+      T.vframe[j] = fr;
+      T.vkind[j] = ss;
+      T.vhf[j] = hf;
+      T.st[v] = isG ? ST_H : ST_HD;
+      T.map[v] = UM_NONE;
+      T.frame_of[v] = UM_NONE;
+      T.hframe[v] = hf;
+      nGL += ss == ST_GL;
+      if (evict_mode) {
+        T.free_stack[f0 + j] = fr;
+        if (isG) {
+          T.d2h_frame[gr] = fr;
+          T.d2h_hf[gr] = hf;
+        }
+      }
+    }
+    gbase += (uint32_t)tot;
+  }
+  {
+    uint32_t v[4] = {threadIdx.x == 0 ? found : 0u, threadIdx.x == 0 ? gbase : 0u,
+                     threadIdx.x == 0 ? found - gbase : 0u, nGL};
+    const int slots[4] = {S_EVICT, S_D2H, S_D2H_AV, S_UNMAPS};
+    const long long mul[4] = {1, (long long)T.B, (long long)T.B, 1};
+    block_counts_to<4>(T, v, s_cnt, slots, mul);
+  }
+  if (threadIdx.x == 0) {
+    c->hfree_top = htop - (int)gbase;
+    if (evict_mode) {
+      c->free_top = f0 + (int)found;
+      c->n_d2h = gbase;
+    } else {
+      c->f0 = (uint32_t)f0;
+      c->n_vict = found;
+      c->free_top = f0 - (int)min((uint32_t)f0, nn);
+      c->used_tail += c->n_rekey;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// K4/K5/K6: the transfer engine.  One elected thread per CTA drives a kXferStages-deep
+// ring of TMA bulk copies (cp.async.bulk, mbarrier complete_tx) through shared memory.
+// Work unit = one kXferChunk slice of one frame.  Fused swap per unit: the victim's
+// bytes (HBM) and the new owner's bytes (mapped pinned host memory) are loaded into
+// smem together; only after both loads land are the stores issued (victim -> host,
+// new -> HBM), so the write-after-read hazard on the frame is resolved inside the
+// unit and both PCIe directions stay busy.  Blocks needing zeros get a bulk store of a
+// zeroed smem tile instead (zero-fill, PAPER L200 / Fig. 2 (7)).  Metadata of a newly
+// resident block is committed by the CTA that handles its first chunk.
+// ------------------------------------------------------------------------------------
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t cnt) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(cnt));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(sdst)),
+               "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void* gdst, const void* ssrc, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(smem_u32(ssrc)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+struct Unit {
+  char* frame;        // frame chunk (HBM)
+  char* d2h_dst;      // host chunk receiving the old content, or null
+  const char* h2d_src;// host chunk with the new content, or null
+  bool zf;            // zero-fill the frame chunk
+};
+
+__global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t seq) {
+  extern __shared__ __align__(128) char smem[];
+  __shared__ __align__(8) uint64_t bar[kXferStages];
+  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
+  const uint32_t cpb = T.B / CH;
+  char* zero = smem;
+  char* stA = smem + CH;                      // S stages of CH (victim/old bytes)
+  char* stB = smem + CH + kXferStages * CH;   // S stages of CH (new bytes)
+  for (uint32_t i = threadIdx.x * 16; i < CH; i += 32 * 16) *reinterpret_cast<uint4*>(zero + i) = make_uint4(0, 0, 0, 0);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  __syncwarp();
+  Ctl* c = T.ctl;
+  if (threadIdx.x == 0) {
+    const uint32_t n_items = mode == SVC_SUBOP ? c->n_need : c->n_d2h;
+    const uint32_t f0 = c->f0;
+    const uint32_t nfu = min(f0, n_items);
+    const unsigned long long units = (unsigned long long)n_items * cpb;
+    const unsigned long long mine =
+        units > blockIdx.x ? (units - blockIdx.x + gridDim.x - 1) / gridDim.x : 0ull;
+    for (int s = 0; s < kXferStages; ++s) mbar_init(&bar[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+
+    auto make = [&](unsigned long long t) -> Unit {
+      unsigned long long u = blockIdx.x + t * gridDim.x;
+      uint32_t i = (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
+      size_t coff = (size_t)ch * CH;
+      Unit x;
+      if (mode == SVC_SUBOP) {
+        uint32_t bb = T.need[i];
+        uint8_t kd = T.needk[i];
+        uint32_t hf = T.needhf[i];
+        uint32_t fr;
+        x.d2h_dst = nullptr;
+        if (i < nfu) {
+          fr = T.free_stack[f0 - 1 - i];
+        } else {
+          uint32_t j = i - f0;
+          fr = T.vframe[j];
+          if (T.vkind[j] == ST_G && T.vhf[j] != UM_NONE) x.d2h_dst = hptr(T, T.vhf[j]) + coff;
+        }
+        x.frame = T.frames + (size_t)fr * T.B + coff;
+        if (kd == ST_H) {
+          x.h2d_src = hptr(T, hf != UM_NONE ? hf : T.zero_hf) + coff;
+          x.zf = false;
+        } else {
+          x.h2d_src = nullptr;
+          x.zf = true;
+        }
+        if (ch == 0) {  // K6 commit of the newly resident block
+          T.st[bb] = ST_G;
+          T.key[bb] = seq;
+          T.frame_of[bb] = fr;
+          T.map[bb] = fr;
+          if (kd == ST_H && hf != UM_NONE) {
+            T.hframe[bb] = UM_NONE;
+            int idx = atomicAdd(&c->hfree_top, 1);
+            T.hfree_stack[idx] = hf;
+          }
+        }
+      } else {
+        uint32_t fr = T.d2h_frame[i], hf = T.d2h_hf[i];
+        x.frame = T.frames + (size_t)fr * T.B + coff;
+        x.d2h_dst = hf != UM_NONE ? hptr(T, hf) + coff : nullptr;
+        x.h2d_src = nullptr;
+        x.zf = false;
+      }
+      return x;
+    };
+    Unit U[kXferStages];
+    auto issue_loads = [&](int s, const Unit& x) {
+      uint32_t bytes = (x.d2h_dst ? CH : 0u) + (x.h2d_src ? CH : 0u);
+      mbar_expect_tx(&bar[s], bytes);
+      if (x.d2h_dst) bulk_g2s(stA + s * CH, x.frame, CH, &bar[s]);
+      if (x.h2d_src) bulk_g2s(stB + s * CH, x.h2d_src, CH, &bar[s]);
+    };
+    for (unsigned long long t = 0; t < mine && t < (unsigned long long)kXferStages; ++t) {
+      U[t] = make(t);
+      issue_loads((int)t, U[t]);
+    }
+    for (unsigned long long t = 0; t < mine; ++t) {
+      const int s = (int)(t % kXferStages);
+      mbar_wait(&bar[s], (uint32_t)((t / kXferStages) & 1));
+      const Unit& x = U[s];
+      if (x.d2h_dst) bulk_s2g(x.d2h_dst, stA + s * CH, CH);
+      if (x.h2d_src) bulk_s2g(x.frame, stB + s * CH, CH);
+      else if (x.zf) bulk_s2g(x.frame, zero, CH);
+      bulk_commit();
+      if (t >= 1 && t - 1 + kXferStages < mine) {
+        bulk_wait_read1();
+        const int sp = (int)((t - 1) % kXferStages);
+        U[sp] = make(t - 1 + kXferStages);
+        issue_loads(sp, U[sp]);
+      }
+    }
+    bulk_wait_all();
+    if (mode == SVC_D2H_ONLY) {
+      __threadfence();
+      unsigned int d = atomicAdd(&c->app_units, 1u);
+      if (d == gridDim.x - 1) {
+        c->n_d2h = 0;
+        c->app_units = 0;
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// Harness "application kernel": after a touch sub-op is serviced, every block with a
+// UM_ACC_WRITE access receives the content stamp s = (seq << 32) | block as the
+// 16-byte pattern {s, ~s}, written through its frame (G or GL blocks are mapped).
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq) {
+  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
+  const uint32_t cpb = T.B / CH;
+  const unsigned long long units = (unsigned long long)n * cpb;
+  for (unsigned long long u = blockIdx.x; u < units; u += gridDim.x) {
+    uint32_t i = (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
+    uint32_t g = g0 + i;
+    uint32_t j = iv_find(iv, g);
+    if (!iv.wflag[j]) continue;
+    uint32_t bb = iv.lo[j] + (g - iv.pre[j]);
+    uint32_t fr = T.frame_of[bb];
+    if (fr == UM_NONE) continue;
+    unsigned long long sv = ((unsigned long long)seq << 32) | bb;
+    uint4 pat = make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32));
+    uint4* dst = reinterpret_cast<uint4*>(T.frames + (size_t)fr * T.B + (size_t)ch * CH);
+    for (uint32_t t = threadIdx.x; t < CH / 16; t += blockDim.x) dst[t] = pat;
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// K8: directives over a contiguous block range (discard: fully covered blocks only,
+// PAPER L211; prefetch HOST: every overlapping block).
+//   discard      G -> GE (unmap, DISC append), GL -> GE, H -> HD
+//   discard_lazy G -> GL (DISC append, mapping kept), H -> HD
+//   prefetch HOST G -> H (D2H), GE/GL -> H (no transfer), HD/U -> H
+// DISC appends are ranked in ascending block order (block scan + look-back).
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
+                                                        int discard_off) {
+  __shared__ unsigned long long s_scan[kScanTPB / 32];
+  __shared__ unsigned long long s_excl;
+  __shared__ unsigned long long s_tail0;
+  __shared__ uint32_t s_cnt[6];
+  if (threadIdx.x == 0) s_tail0 = T.ctl->disc_tail;
+  const uint32_t tile = take_ticket(T);
+  const uint32_t ntiles = n ? (n + kScanTile - 1) / kScanTile : 1;
+  const uint32_t first = tile * kScanTile + threadIdx.x * kScanIPT;
+  uint32_t cA = 0;
+  uint8_t s[kScanIPT];
+#pragma unroll
+  for (int k = 0; k < kScanIPT; ++k) {
+    s[k] = 0xff;
+    if (first + k < n) {
+      s[k] = T.st[lo + first + k];
+      cA += (!discard_off && kind != DIR_PREFETCH_HOST && s[k] == ST_G);
+    }
+  }
+  unsigned long long tot;
+  unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cA, 0), tot, s_scan);
+  if (threadIdx.x == 0) s_excl = lookback(T, tile, tot);
+  __syncthreads();
+  uint32_t pA = unpackA(s_excl + pre);
+  const unsigned long long tail0 = s_tail0;
+  // counters: unmaps, d2h, d2h_av
+  uint32_t nUnmap = 0, nD2H = 0, nAv = 0;
+  if (!discard_off || kind == DIR_PREFETCH_HOST) {
+#pragma unroll
+    for (int k = 0; k < kScanIPT; ++k) {
+      if (first + k >= n) break;
+      const uint32_t bb = lo + first + k;
+      const uint8_t ss = s[k];
+      if (kind == DIR_DISCARD || kind == DIR_DISCARD_LAZY) {
+        if (ss == ST_G) {
+          T.st[bb] = kind == DIR_DISCARD ? ST_GE : ST_GL;
+          T.key[bb] = seq;
+          T.disc_ring[(tail0 + pA) & T.cap_mask] = ((unsigned long long)seq << 32) | bb;
+          ++pA;
+          if (kind == DIR_DISCARD) {
+            T.map[bb] = UM_NONE;
+            ++nUnmap;
+          }
+        } else if (ss == ST_GL && kind == DIR_DISCARD) {
+          T.st[bb] = ST_GE;
+          T.map[bb] = UM_NONE;
+          ++nUnmap;
+        } else if (ss == ST_H) {
+          T.st[bb] = ST_HD;
+          uint32_t hf = T.hframe[bb];
+          if (hf != UM_NONE) {  // the host copy is released (reading R1)
+            T.hframe[bb] = UM_NONE;
+            int idx = atomicAdd(&T.ctl->hfree_top, 1);
+            T.hfree_stack[idx] = hf;
+          }
+        }
+      } else {  // prefetch to HOST
+        if (ss == ST_G || ss == ST_GE || ss == ST_GL) {
+          uint32_t fr = T.frame_of[bb];
+          if (ss == ST_G) {
+            int idx = atomicSub(&T.ctl->hfree_top, 1) - 1;
+            uint32_t hf = UM_NONE;
+            if (idx >= 0) hf = T.hfree_stack[idx];
+            else atomicExch(&T.ctl->err, 2u);
+            uint32_t q = atomicAdd(&T.ctl->n_d2h, 1u);
+            T.d2h_frame[q] = fr;
+            T.d2h_hf[q] = hf;
+            T.hframe[bb] = hf;
+            ++nD2H;
+          } else {
+            ++nAv;
+            if (ss == ST_GL) ++nUnmap;
+          }
+          int fi = atomicAdd(&T.ctl->free_top, 1);
+          T.free_stack[fi] = fr;
+          T.frame_of[bb] = UM_NONE;
+          T.map[bb] = UM_NONE;
+        }
+        if (ss != ST_H) T.st[bb] = ST_H;
+      }
+    }
+  }
+  {
+    uint32_t v[3] = {nUnmap, nD2H, nAv};
+    const int slots[3] = {S_UNMAPS, S_D2H, S_D2H_AV};
+    const long long mul[3] = {1, (long long)T.B, (long long)T.B};
+    block_counts_to<3>(T, v, s_cnt, slots, mul);
+  }
+  if (tile == ntiles - 1 && threadIdx.x == 0) T.ctl->disc_tail = tail0 + unpackA(s_excl + tot);
+  scan_finish(T, ntiles);
+}
+
+// ------------------------------------------------------------------------------------
+// K7: stable compaction of a ring's live entries [head, tail) into `dst` at [0, cnt).
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(kScanTPB) k_ring_compact(Tables T, int ring, uint64_t* dst) {
+  __shared__ unsigned long long s_scan[kScanTPB / 32];
+  __shared__ unsigned long long s_excl, s_head, s_n;
+  Ctl* c = T.ctl;
+  if (threadIdx.x == 0) {
+    s_head = ring == RING_USED ? c->used_head : c->disc_head;
+    unsigned long long tl = ring == RING_USED ? c->used_tail : c->disc_tail;
+    s_n = tl - s_head;
+  }
+  const uint32_t tile = take_ticket(T);
+  const uint32_t ntiles = gridDim.x;
+  const uint64_t* R = ring == RING_USED ? T.used_ring : T.disc_ring;
+  const unsigned long long n = s_n, head = s_head;
+  const unsigned long long first = (unsigned long long)tile * kScanTile + threadIdx.x * kScanIPT;
+  unsigned long long e[kScanIPT];
+  unsigned livem = 0;
+  uint32_t cnt = 0;
+#pragma unroll
+  for (int k = 0; k < kScanIPT; ++k) {
+    e[k] = 0;
+    if (first + k < n) {
+      e[k] = R[(head + first + k) & T.cap_mask];
+      uint32_t blk = (uint32_t)e[k], kk = (uint32_t)(e[k] >> 32);
+      uint8_t ss = T.st[blk];
+      bool live = (ring == RING_USED ? ss == ST_G : (ss == ST_GE || ss == ST_GL)) && T.key[blk] == kk;
+      livem |= (unsigned)live << k;
+      cnt += live;
+    }
+  }
+  unsigned long long tot;
+  unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cnt, 0), tot, s_scan);
+  if (threadIdx.x == 0) s_excl = lookback(T, tile, tot);
+  __syncthreads();
+  uint32_t p = unpackA(s_excl + pre);
+#pragma unroll
+  for (int k = 0; k < kScanIPT; ++k)
+    if ((livem >> k) & 1) dst[p++] = e[k];
+  if (tile == ntiles - 1 && threadIdx.x == 0) {
+    unsigned long long total = unpackA(s_excl + tot);
+    if (ring == RING_USED) { c->used_head = 0; c->used_tail = total; }
+    else { c->disc_head = 0; c->disc_tail = total; }
+  }
+  scan_finish(T, ntiles);
+}
+
+// ------------------------------------------------------------------------------------
+// Harness: host writes (Listing 6 "Generate data, labels").
+// ------------------------------------------------------------------------------------
+__global__ void k_hw_alloc(Tables T, uint32_t lo, uint32_t n) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    uint32_t bb = lo + i;
+    if (T.st[bb] != ST_H) {
+      atomicExch(&T.ctl->err, 1u);
+      continue;
+    }
+    if (T.hframe[bb] == UM_NONE) {
+      int idx = atomicSub(&T.ctl->hfree_top, 1) - 1;
+      if (idx >= 0) T.hframe[bb] = T.hfree_stack[idx];
+      else atomicExch(&T.ctl->err, 2u);
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_hw_fill(Tables T, uint32_t lo, uint32_t n, uint32_t seq) {
+  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
+  const uint32_t cpb = T.B / CH;
+  const unsigned long long units = (unsigned long long)n * cpb;
+  for (unsigned long long u = blockIdx.x; u < units; u += gridDim.x) {
+    uint32_t bb = lo + (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
+    uint32_t hf = T.hframe[bb];
+    if (hf == UM_NONE || T.st[bb] != ST_H) continue;
+    unsigned long long sv = ((unsigned long long)seq << 32) | bb;
+    uint4 pat = make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32));
+    uint4* dst = reinterpret_cast<uint4*>(hptr(T, hf) + (size_t)ch * CH);
+    for (uint32_t t = threadIdx.x; t < CH / 16; t += blockDim.x) dst[t] = pat;
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// Harness: content tag of every block (0 = zeros, s = uniform {s,~s}, ~0 = corrupt).
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_tags(Tables T) {
+  __shared__ int s_ok, s_zero;
+  for (uint32_t bb = blockIdx.x; bb < T.nblocks; bb += gridDim.x) {
+    uint8_t ss = T.st[bb];
+    const uint4* src = nullptr;
+    if (ss == ST_G || ss == ST_GE || ss == ST_GL) {
+      uint32_t fr = T.frame_of[bb];
+      if (fr != UM_NONE) src = reinterpret_cast<const uint4*>(T.frames + (size_t)fr * T.B);
+    } else if (ss == ST_H) {
+      uint32_t hf = T.hframe[bb];
+      if (hf != UM_NONE) src = reinterpret_cast<const uint4*>(hptr(T, hf));
+    }
+    if (!src) {
+      if (threadIdx.x == 0) T.tags[bb] = (ss == ST_G || ss == ST_GE || ss == ST_GL) ? ~0ull : 0ull;
+      continue;
+    }
+    uint4 v0 = src[0];
+    bool ok = true;
+    for (uint32_t t = threadIdx.x; t < T.B / 16; t += blockDim.x) {
+      uint4 v = src[t];
+      ok &= (v.x == v0.x) & (v.y == v0.y) & (v.z == v0.z) & (v.w == v0.w);
+    }
+    ok = __syncthreads_and(ok);
+    if (threadIdx.x == 0) {
+      unsigned long long s = (unsigned long long)v0.x | ((unsigned long long)v0.y << 32);
+      unsigned long long ns = (unsigned long long)v0.z | ((unsigned long long)v0.w << 32);
+      unsigned long long tag;
+      if (!ok) tag = ~0ull;
+      else if (s == 0 && ns == 0) tag = 0;
+      else if (ns == ~s && s != 0) tag = s;
+      else tag = ~0ull;
+      T.tags[bb] = tag;
+    }
+    __syncthreads();
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// launch wrappers
+// ------------------------------------------------------------------------------------
+static int g_nsm = 0;
+
+cudaError_t setup_kernels() {
+  int dev;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e) return e;
+  e = cudaDeviceGetAttribute(&g_nsm, cudaDevAttrMultiProcessorCount, dev);
+  if (e) return e;
+  int smem = (int)(kXferChunk * (1 + 2 * kXferStages));
+  return cudaFuncSetAttribute(k_service, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+}
+
+static inline unsigned ceil_div(unsigned long long a, unsigned long long b) { return (unsigned)((a + b - 1) / b); }
+
+cudaError_t launch_init(const Tables& T, int nh, cudaStream_t s) {
+  k_init<<<g_nsm * 4, 256, 0, s>>>(T, nh);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_poison(const Tables& T, cudaStream_t s) {
+  k_poison<<<g_nsm * 4, 512, 0, s>>>(T.frames, (size_t)T.nframes * T.B);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
+                            cudaStream_t s) {
+  unsigned nt = n ? ceil_div(n, kScanTile) : 1;
+  k_classify<<<nt, kScanTPB, 0, s>>>(T, iv, g0, n, seq, touch);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, cudaStream_t s) {
+  k_victims<<<1, kVictTPB, 0, s>>>(T, seq, evict_mode, want);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max_items, cudaStream_t s) {
+  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
+  unsigned long long units = (unsigned long long)max_items * (T.B / CH);
+  unsigned grid = (unsigned)(units < (unsigned long long)g_nsm ? units : (unsigned long long)g_nsm);
+  if (grid == 0) grid = 1;
+  size_t smem = (size_t)CH * (1 + 2 * kXferStages);
+  k_service<<<grid, 32, smem, s>>>(T, mode, seq);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, cudaStream_t s) {
+  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
+  unsigned long long units = (unsigned long long)n * (T.B / CH);
+  unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
+  if (!grid) return cudaSuccess;
+  k_app_stamp<<<grid, 256, 0, s>>>(T, iv, g0, n, seq);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq, int discard_off,
+                             cudaStream_t s) {
+  unsigned nt = n ? ceil_div(n, kScanTile) : 1;
+  k_directive<<<nt, kScanTPB, 0, s>>>(T, kind, lo, n, seq, discard_off);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64_t cap_bound, cudaStream_t s) {
+  unsigned nt = ceil_div(cap_bound ? cap_bound : 1, kScanTile);
+  k_ring_compact<<<nt, kScanTPB, 0, s>>>(T, ring, dst);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_host_write(const Tables& T, uint32_t lo, uint32_t n, uint32_t seq, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  k_hw_alloc<<<ceil_div(n, 256), 256, 0, s>>>(T, lo, n);
+  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
+  unsigned long long units = (unsigned long long)n * (T.B / CH);
+  unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
+  k_hw_fill<<<grid, 256, 0, s>>>(T, lo, n, seq);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tags(const Tables& T, cudaStream_t s) {
+  unsigned grid = T.nblocks < (uint32_t)g_nsm * 16 ? T.nblocks : (unsigned)g_nsm * 16;
+  if (!grid) grid = 1;
+  k_tags<<<grid, 256, 0, s>>>(T);
+  return cudaGetLastError();
+}
+
+}  // namespace um

@@ -1,0 +1,233 @@
+"""Thin ctypes binding of libum (include/um.h): same names, argument marshalling only.
+
+Every step of the paging path runs in libum's sm_100a kernels; this module only
+converts Python values to C arguments.  It raises loudly if libum.so is missing —
+there is no CPU fallback.  PyTorch is used only to allocate device memory, pinned
+host memory and streams (the `Arena` helper at the bottom).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libum.so")
+
+UM_OK, UM_EINVAL, UM_ENOMEM, UM_ECUDA, UM_EBUSY = 0, -1, -2, -3, -4
+UM_DST_GPU, UM_DST_HOST = 0, 1
+UM_ACC_READ, UM_ACC_WRITE = 1, 2
+UM_ST_U, UM_ST_H, UM_ST_HD, UM_ST_G, UM_ST_GE, UM_ST_GL = range(6)
+ST_NAMES = ("U", "H", "HD", "G", "GE", "GL")
+UM_F_DISCARD_OFF, UM_F_COPY_CE, UM_F_CHECK, UM_F_APP_STAMP = 1, 2, 4, 8
+UM_NONE = 0xFFFFFFFF
+
+
+class um_access(C.Structure):
+    _fields_ = [("off", C.c_uint64), ("len", C.c_uint32), ("kind", C.c_uint32)]
+
+
+class um_config(C.Structure):
+    _fields_ = [("device", C.c_int), ("block_bytes", C.c_uint32), ("arena_bytes", C.c_uint64),
+                ("budget_bytes", C.c_uint64), ("frames", C.c_void_p), ("workspace", C.c_void_p),
+                ("workspace_bytes", C.c_uint64), ("host_chunks", C.POINTER(C.c_void_p)),
+                ("n_host_chunks", C.c_uint32), ("host_chunk_bytes", C.c_uint64), ("flags", C.c_uint32)]
+
+
+STAT_FIELDS = ("h2d_bytes", "d2h_bytes", "zf_bytes", "h2d_avoided_bytes", "d2h_avoided_bytes", "faults",
+               "hits", "remaps", "unmaps", "revalidations", "refreshes", "evictions", "ops", "subops")
+
+
+class um_stats(C.Structure):
+    _fields_ = [(n, C.c_int64) for n in STAT_FIELDS] + [("pad", C.c_int64 * 2)]
+
+    def as_dict(self):
+        return {n: int(getattr(self, n)) for n in STAT_FIELDS}
+
+
+class UmError(RuntimeError):
+    def __init__(self, fn, status):
+        super().__init__(f"{fn} failed: {status} ({um_strerror(status)})")
+        self.status = status
+
+
+_lib = None
+
+
+def lib():
+    """Load libum.so (raises if it was not built — no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} missing: run `python -m paper_conf_iiswc_zhucvhcr22_b200.build`")
+        L = C.CDLL(LIB_PATH)
+        P, U64, U32, I = C.c_void_p, C.c_uint64, C.c_uint32, C.c_int
+        sig = {
+            "um_workspace_size": [C.POINTER(um_config), C.POINTER(U64)],
+            "um_arena_create": [C.POINTER(um_config), C.POINTER(P)],
+            "um_arena_destroy": [P],
+            "um_alloc": [P, U64, C.POINTER(U64)],
+            "um_prefetch": [P, U64, U64, I, P],
+            "um_discard": [P, U64, U64, P],
+            "um_discard_lazy": [P, U64, U64, P],
+            "um_touch_batch": [P, P, U32, P],
+            "um_evict": [P, U64, P],
+            "um_host_write": [P, U64, U64, P],
+            "um_block_table": [P, C.POINTER(P)],
+            "um_stream": [P, C.POINTER(P)],
+            "um_get_stats": [P, C.POINTER(um_stats)],
+            "um_dump": [P, P, P, C.POINTER(U32), P, C.POINTER(U32)],
+            "um_content_tags": [P, P],
+            "um_timing": [P, C.POINTER(C.c_double), C.POINTER(C.c_double), I],
+        }
+        for name, args in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = C.c_int
+        L.um_strerror.argtypes = [C.c_int]
+        L.um_strerror.restype = C.c_char_p
+        _lib = L
+    return _lib
+
+
+EXPORTS = ("um_workspace_size", "um_arena_create", "um_arena_destroy", "um_alloc", "um_prefetch", "um_discard",
+           "um_discard_lazy", "um_touch_batch", "um_evict", "um_host_write", "um_block_table", "um_stream",
+           "um_get_stats", "um_dump", "um_content_tags", "um_timing", "um_strerror")
+
+
+def _ck(fn, st):
+    if st != UM_OK:
+        raise UmError(fn, st)
+
+
+def um_strerror(status: int) -> str:
+    return lib().um_strerror(status).decode()
+
+
+def um_workspace_size(cfg: um_config) -> int:
+    out = C.c_uint64()
+    _ck("um_workspace_size", lib().um_workspace_size(C.byref(cfg), C.byref(out)))
+    return out.value
+
+
+def um_arena_create(cfg: um_config) -> int:
+    out = C.c_void_p()
+    _ck("um_arena_create", lib().um_arena_create(C.byref(cfg), C.byref(out)))
+    return out.value
+
+
+def um_arena_destroy(a) -> None:
+    _ck("um_arena_destroy", lib().um_arena_destroy(a))
+
+
+def um_alloc(a, nbytes: int) -> int:
+    off = C.c_uint64()
+    _ck("um_alloc", lib().um_alloc(a, nbytes, C.byref(off)))
+    return off.value
+
+
+def um_prefetch(a, off: int, ln: int, dst: int, stream=None) -> None:
+    _ck("um_prefetch", lib().um_prefetch(a, off, ln, dst, stream))
+
+
+def um_discard(a, off: int, ln: int, stream=None) -> None:
+    _ck("um_discard", lib().um_discard(a, off, ln, stream))
+
+
+def um_discard_lazy(a, off: int, ln: int, stream=None) -> None:
+    _ck("um_discard_lazy", lib().um_discard_lazy(a, off, ln, stream))
+
+
+def um_touch_batch(a, acc: np.ndarray, stream=None) -> None:
+    """acc: numpy array with the 16-byte um_access layout (tracegen.ACC_DTYPE)."""
+    acc = np.ascontiguousarray(acc)
+    assert acc.dtype.itemsize == 16
+    _ck("um_touch_batch", lib().um_touch_batch(a, acc.ctypes.data if len(acc) else None, len(acc), stream))
+
+
+def um_evict(a, nbytes: int, stream=None) -> None:
+    _ck("um_evict", lib().um_evict(a, nbytes, stream))
+
+
+def um_host_write(a, off: int, ln: int, stream=None) -> None:
+    _ck("um_host_write", lib().um_host_write(a, off, ln, stream))
+
+
+def um_block_table(a) -> int:
+    p = C.c_void_p()
+    _ck("um_block_table", lib().um_block_table(a, C.byref(p)))
+    return p.value
+
+
+def um_stream(a) -> int:
+    p = C.c_void_p()
+    _ck("um_stream", lib().um_stream(a, C.byref(p)))
+    return p.value
+
+
+def um_get_stats(a) -> dict:
+    s = um_stats()
+    _ck("um_get_stats", lib().um_get_stats(a, C.byref(s)))
+    return s.as_dict()
+
+
+def um_dump(a, nblocks: int, nframes: int) -> dict:
+    st = np.zeros(nblocks, np.uint8)
+    used = np.zeros(max(1, nframes), np.uint32)
+    disc = np.zeros(max(1, nframes), np.uint32)
+    nu, nd = C.c_uint32(), C.c_uint32()
+    _ck("um_dump", lib().um_dump(a, st.ctypes.data, used.ctypes.data, C.byref(nu), disc.ctypes.data, C.byref(nd)))
+    return {"st": st, "used_order": used[:nu.value].tolist(), "disc_order": disc[:nd.value].tolist()}
+
+
+def um_content_tags(a, nblocks: int) -> np.ndarray:
+    t = np.zeros(nblocks, np.uint64)
+    _ck("um_content_tags", lib().um_content_tags(a, t.ctypes.data))
+    return t
+
+
+# -------------------------------------------------------------------------------------
+# Arena: allocates the caller-owned memory with torch (frames + workspace in HBM,
+# host-frame pool in pinned host memory) and creates the libum arena.
+# -------------------------------------------------------------------------------------
+class Arena:
+    def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, flags: int = 0,
+                 host_pool_bytes: int | None = None, host_chunk_bytes: int | None = None, device: int = 0):
+        import torch
+        self.torch = torch
+        self.B = block_bytes
+        self.nblocks = arena_bytes // block_bytes
+        self.nframes = budget_bytes // block_bytes
+        if host_pool_bytes is None:
+            host_pool_bytes = arena_bytes          # every block can be host-resident
+        host_pool_bytes += block_bytes             # + the zero page
+        if host_chunk_bytes is None:
+            host_chunk_bytes = min(1 << 30, max(block_bytes, 1 << (host_pool_bytes - 1).bit_length()))
+        nch = -(-host_pool_bytes // host_chunk_bytes)
+        dev = torch.device("cuda", device)
+        self.frames = torch.empty(self.nframes * block_bytes, dtype=torch.uint8, device=dev)
+        self.host_chunks = [torch.empty(host_chunk_bytes, dtype=torch.uint8, pin_memory=True) for _ in range(nch)]
+        self._hc = (C.c_void_p * nch)(*[t.data_ptr() for t in self.host_chunks])
+        cfg = um_config(device=device, block_bytes=block_bytes, arena_bytes=arena_bytes,
+                        budget_bytes=budget_bytes, frames=self.frames.data_ptr(), workspace=None,
+                        workspace_bytes=0, host_chunks=C.cast(self._hc, C.POINTER(C.c_void_p)),
+                        n_host_chunks=nch, host_chunk_bytes=host_chunk_bytes, flags=flags)
+        ws = um_workspace_size(cfg)
+        self.workspace = torch.empty(ws, dtype=torch.uint8, device=dev)
+        cfg.workspace = self.workspace.data_ptr()
+        cfg.workspace_bytes = ws
+        self.cfg = cfg
+        self.handle = um_arena_create(cfg)
+        self.stream_ptr = um_stream(self.handle)
+
+    def close(self):
+        if self.handle:
+            um_arena_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,173 @@
+"""Parity of the CUDA path (libum.so, called through the C ABI) with the CPU oracle:
+per-block final state, USED/DISC order, every counter and every block's content tag
+must match bit-exactly.  Run with `pytest -m gpu` on a B200."""
+import numpy as np
+import pytest
+
+import tracegen as tg
+from oracle.sim import replay as oracle_replay
+import scenarios as scn
+
+pytestmark = pytest.mark.gpu
+
+SCEN = scn.load()
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_iiswc_zhucvhcr22_b200 import build
+    build.build()
+
+
+def _gpu(trace, mode, **kw):
+    from paper_conf_iiswc_zhucvhcr22_b200 import harness
+    return harness.run_trace(trace, mode, **kw)
+
+
+def assert_parity(trace, mode, g=None):
+    g = g if g is not None else _gpu(trace, mode)
+    o = oracle_replay(trace, mode).dump()
+    st_g = np.asarray(g["st"])
+    st_o = np.asarray(o["st"])
+    bad = np.nonzero(st_g != st_o)[0]
+    assert len(bad) == 0, f"state mismatch at blocks {bad[:10]}: gpu {st_g[bad[:10]]} oracle {st_o[bad[:10]]}"
+    assert g["stats"] == o["stats"], {k: (g["stats"][k], o["stats"][k]) for k in o["stats"] if g["stats"][k] != o["stats"][k]}
+    assert g["used_order"] == o["used_order"]
+    assert g["disc_order"] == o["disc_order"]
+    ct_g = np.asarray(g["contents"], dtype=np.uint64)
+    ct_o = np.asarray(o["contents"], dtype=np.uint64)
+    badc = np.nonzero(ct_g != ct_o)[0]
+    assert len(badc) == 0, f"content mismatch at {badc[:10]}: gpu {[hex(x) for x in ct_g[badc[:5]]]} oracle {[hex(x) for x in ct_o[badc[:5]]]}"
+    return g, o
+
+
+@pytest.mark.parametrize("name", sorted(SCEN))
+def test_scenarios(name):
+    sc = SCEN[name]
+    trace, mode = scn.build(sc)
+    g, _ = assert_parity(trace, mode)
+    for k, v in sc["expect"]["stats"].items():
+        assert g["stats"][k] == v, k
+    assert [scn.ST[x] for x in sc["expect"]["st"]] == list(g["st"])
+    assert list(g["contents"]) == scn.expected_contents(sc)
+
+
+@pytest.mark.parametrize("seed", range(12))
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_small_random(seed, mode):
+    rng = np.random.default_rng(seed)
+    nb, nf = int(rng.integers(2, 24)), int(rng.integers(1, 6))
+    t = tg.gen_small(seed, nblocks=nb, nframes=nf, n_ops=300, max_ranges=4, max_blocks=6)
+    assert_parity(t, mode)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_c1(seed, mode):
+    """C1 tiny (BASELINE.json configs[0]): 64 MiB arena, 16 MiB budget, 64 KiB blocks, 10k ops."""
+    assert_parity(tg.gen_c1(seed), mode)
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_c2_ci(mode):
+    """C2 streaming at CI size: F = 2048 frames of 2 MiB (4 GiB), buffer 8 GiB, c = 512, P = 2;
+    also pins the closed form."""
+    F, c, P, B = 2048, 512, 2, 2 << 20
+    t = tg.gen_c2(F, c, P, block_bytes=B)
+    g, _ = assert_parity(t, mode)
+    s = g["stats"]
+    if mode == "base":
+        assert (s["h2d_bytes"], s["d2h_bytes"], s["zf_bytes"]) == (2 * (P - 1) * F * B, (2 * P - 1) * F * B, 2 * F * B)
+    else:
+        assert (s["h2d_bytes"], s["d2h_bytes"], s["zf_bytes"]) == (0, 0, 2 * P * F * B)
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_c3_small(mode):
+    """C3 (Listing 6) with a VGG-shaped profile scaled down: 2 iterations, 64 KiB blocks."""
+    t = tg.gen_c3(block_bytes=64 << 10, budget_bytes=192 << 20, iterations=2, workspace_bytes=4 << 20,
+                  layers=tg.scale_layers(tg.VGG16, 1.0 / 512, 1.0 / 64), batch=8)
+    assert t.arena_bytes > t.budget_bytes
+    assert_parity(t, mode)
+
+
+def test_split_large_op():
+    """One touch covering 4x the frame budget (ascending sub-ops, A3) and a prefetch of
+    the whole arena; ragged tails across many scan tiles."""
+    B = 64 << 10
+    tb = tg.TraceBuilder(B, 9000 * B, 2100 * B)
+    tb.touch([(0, 9000 * B - 100, tg.ACC_WRITE), (5 * B + 7, 3 * B, tg.ACC_READ)])
+    tb.discard(100 * B, 4000 * B, lazy_ok=True)
+    tb.prefetch(0, 9000 * B, tg.DST_GPU)
+    tb.touch([(B * 8000, 900 * B, tg.ACC_WRITE)])
+    tb.evict(1500 * B)
+    tb.prefetch(0, 3000 * B, tg.DST_HOST)
+    t = tb.build()
+    for mode in ("base", "eager", "lazy"):
+        assert_parity(t, mode)
+
+
+def test_edge_cases_and_errors():
+    from paper_conf_iiswc_zhucvhcr22_b200 import harness, um
+    B = 4096
+    tb = tg.TraceBuilder(B, 8 * B, 3 * B)
+    tb.touch([])                              # empty batch: consumes a seq
+    tb.prefetch(0, 0, tg.DST_GPU)             # len 0
+    tb.discard(B + 1, B)                      # covers no full block
+    tb.evict(0)
+    tb.touch([(0, 8 * B, tg.ACC_WRITE)])
+    tb.evict(100 * B)                         # more than resident: evict everything
+    tb.prefetch(7 * B, B, tg.DST_HOST)
+    t = tb.build()
+    assert_parity(t, "eager")
+    a = harness.make_arena(t, "eager")
+    try:
+        with pytest.raises(um.UmError) as e:
+            um.um_prefetch(a.handle, 7 * B, 2 * B, um.UM_DST_GPU)
+        assert e.value.status == um.UM_EINVAL
+        with pytest.raises(um.UmError):
+            um.um_prefetch(a.handle, 0, B, 5)
+        with pytest.raises(um.UmError):
+            um.um_touch_batch(a.handle, np.array([(0, B, 1), (8 * B, 1, 1)], dtype=tg.ACC_DTYPE))
+        with pytest.raises(um.UmError):
+            um.um_alloc(a.handle, 9 * B)
+        assert um.um_get_stats(a.handle)["ops"] == 0     # rejected calls enqueue nothing
+    finally:
+        a.close()
+
+
+class _CAI:
+    def __init__(self, ptr, n, typestr="<u4"):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3}
+
+
+def test_block_table_maps_resident_blocks():
+    """D1: map[b] is the frame while G/GL, NONE otherwise (an eager discard unmaps, PAPER
+    L176; a lazy discard keeps the mapping, L186); an app kernel can translate through it."""
+    import torch
+    from paper_conf_iiswc_zhucvhcr22_b200 import harness, um
+    B = 64 << 10
+    tb = tg.TraceBuilder(B, 16 * B, 8 * B)
+    tb.touch([(0, 8 * B, tg.ACC_WRITE)])
+    tb.discard(0, 2 * B)
+    tb.discard(2 * B, 2 * B, lazy_ok=True)
+    t = tb.build()
+    a = harness.make_arena(t, "lazy")
+    try:
+        harness.issue(a, t, "lazy")
+        st = um.um_dump(a.handle, a.nblocks, a.nframes)["st"]
+        m = torch.as_tensor(_CAI(um.um_block_table(a.handle), a.nblocks, "<i4"), device="cuda").cpu().numpy()
+        m = m.astype(np.int64) & 0xFFFFFFFF
+        assert [um.ST_NAMES[x] for x in st[:8]] == ["GE", "GE", "GL", "GL", "G", "G", "G", "G"]
+        assert (m[:2] == um.UM_NONE).all() and (m[2:8] != um.UM_NONE).all() and (m[8:] == um.UM_NONE).all()
+        assert len(set(m[2:8].tolist())) == 6
+        # translate block 5 through the table and read its stamp pattern from the frame
+        fr = int(m[5])
+        blk = a.frames[fr * B:(fr + 1) * B].view(torch.int64).cpu().numpy()
+        s = (1 << 32) | 5
+        assert blk[0] == s and blk[1] == ~s
+    finally:
+        a.close()
