@@ -61,8 +61,10 @@ enum {
   UM_F_DISCARD_OFF = 1u, /* "UVM-opt" baseline: discards are accepted no-ops */
   UM_F_COPY_CE = 2u,     /* move data with cudaMemcpyAsync on side streams, not K4       */
   UM_F_CHECK = 4u,       /* poison frames with 0xA5 at creation; extra validation       */
-  UM_F_APP_STAMP = 8u    /* harness: after each touch sub-op, write the content stamp of
+  UM_F_APP_STAMP = 8u,   /* harness: after each touch sub-op, write the content stamp of
                             every UM_ACC_WRITE block (simulated application kernel)    */
+  UM_F_TIMING = 16u      /* record CUDA events around the planning and transfer kernels
+                            of every op (read with um_timing)                          */
 };
 
 /* One GPU access record of a batch (16 bytes).  Covers every block overlapping
@@ -162,8 +164,13 @@ um_status um_dump(um_arena *a, uint8_t *st, uint32_t *used_order, uint32_t *n_us
  * else (corrupt).  Reads frames (G/GE/GL) or host frames (H; HD/U read as zero). */
 um_status um_content_tags(um_arena *a, uint64_t *tags);
 
-/* Harness: per-phase device timing of the last ops (ms), cumulative since reset. */
-um_status um_timing(um_arena *a, double *ms_plan, double *ms_xfer, int reset);
+/* Synchronizes.  Device time (ms) spent since the last reset in planning kernels
+ * (classify, victim selection, directives, ring compaction) and in the transfer engine
+ * (fused swap / write-back / zero-fill kernel), summed per launch from CUDA events
+ * (needs UM_F_TIMING, else 0), the number of transfer-kernel launches, and the number of
+ * libum kernel launches enqueued.  reset != 0 clears all four afterwards. */
+um_status um_timing(um_arena *a, double *ms_plan, double *ms_xfer, uint64_t *xfer_launches,
+                    uint64_t *launches, int reset);
 
 const char *um_strerror(um_status s);
 

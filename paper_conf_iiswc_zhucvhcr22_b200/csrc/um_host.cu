@@ -186,6 +186,12 @@ struct um_arena {
   Stager stage;
   Ctl* hctl = nullptr;  // pinned mirror for reads
   std::vector<Iv> ivs;
+  // UM_F_TIMING: event pairs around planning / transfer launches
+  struct Span { cudaEvent_t a, b; int xfer; };
+  std::vector<Span> spans;
+  std::vector<cudaEvent_t> evpool;
+  double ms_plan = 0, ms_xfer = 0;
+  uint64_t n_xfer = 0, n_launch = 0;
   std::vector<uint32_t> tmp_lo, tmp_pre;
   std::vector<uint8_t> tmp_w;
 };
@@ -244,6 +250,31 @@ static void set_ring_ptrs(um_arena* a) {
   a->T.disc_ring = a->ring_buf[RING_DISC][a->ring_cur[RING_DISC]];
 }
 
+static cudaEvent_t tev(um_arena* a) {
+  if (!a->evpool.empty()) {
+    cudaEvent_t e = a->evpool.back();
+    a->evpool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+// Open / close a timed span on the paging stream (no-ops without UM_F_TIMING).
+static cudaEvent_t span_open(um_arena* a) {
+  if (!(a->cfg.flags & UM_F_TIMING)) return nullptr;
+  cudaEvent_t e = tev(a);
+  cudaEventRecord(e, a->ps);
+  return e;
+}
+static void span_close(um_arena* a, cudaEvent_t open, int xfer) {
+  if (!open) return;
+  cudaEvent_t e = tev(a);
+  cudaEventRecord(e, a->ps);
+  a->spans.push_back({open, e, xfer});
+}
+
 // K7 trigger: the host keeps an upper bound of each ring's occupancy (appends are
 // bounded by the op's block count; live entries never exceed nframes).
 static um_status ensure_ring_room(um_arena* a, int ring, uint64_t appends) {
@@ -252,7 +283,10 @@ static um_status ensure_ring_room(um_arena* a, int ring, uint64_t appends) {
     return UM_OK;
   }
   int nxt = a->ring_cur[ring] ^ 1;
+  cudaEvent_t sp = span_open(a);
   CK(launch_ring_compact(a->T, ring, a->ring_buf[ring][nxt], a->L.cap, a->ps));
+  span_close(a, sp, 0);
+  a->n_launch++;
   a->ring_cur[ring] = nxt;
   set_ring_ptrs(a);
   a->ub[ring] = std::min<uint64_t>(a->nframes, a->L.cap) + appends;
@@ -342,11 +376,19 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     a->subops++;
     um_status st = ensure_ring_room(a, RING_USED, n);
     if (st) return st;
+    cudaEvent_t sp = span_open(a);
     CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
     CK(launch_victims(a->T, seq, 0, 0, a->ps));
+    span_close(a, sp, 0);
+    sp = span_open(a);
     CK(launch_service(a->T, SVC_SUBOP, seq, n, a->ps));
-    if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP))
+    span_close(a, sp, 1);
+    a->n_launch += 3;
+    a->n_xfer++;
+    if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP)) {
       CK(launch_app_stamp(a->T, iv, (uint32_t)g0, n, seq, a->ps));
+      a->n_launch++;
+    }
   }
   return UM_OK;
 }
@@ -467,6 +509,8 @@ UM_API um_status um_arena_destroy(um_arena* a) {
   if (!a) return UM_EINVAL;
   if (a->ps) cudaStreamSynchronize(a->ps);
   a->stage.destroy();
+  for (auto& sp : a->spans) { cudaEventDestroy(sp.a); cudaEventDestroy(sp.b); }
+  for (auto e : a->evpool) cudaEventDestroy(e);
   if (a->hctl) cudaFreeHost(a->hctl);
   if (a->ev_in) cudaEventDestroy(a->ev_in);
   if (a->ev_out) cudaEventDestroy(a->ev_out);
@@ -517,8 +561,14 @@ UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, v
     const uint32_t seq = ++a->clock;
     if (len) {
       uint32_t lo = (uint32_t)(off / a->B), hi = (uint32_t)((off + len - 1) / a->B + 1);
+      cudaEvent_t sp = span_open(a);
       CK(launch_directive(a->T, DIR_PREFETCH_HOST, lo, hi - lo, seq, 0, a->ps));
+      span_close(a, sp, 0);
+      sp = span_open(a);
       CK(launch_service(a->T, SVC_D2H_ONLY, seq, std::min<uint32_t>(hi - lo, a->nframes), a->ps));
+      span_close(a, sp, 1);
+      a->n_launch += 2;
+      a->n_xfer++;
     }
   }
   return hand_out(a, stream);
@@ -537,7 +587,10 @@ static um_status discard_common(um_arena* a, uint64_t off, uint64_t len, void* s
     const uint32_t n = (uint32_t)(hi - lo);
     s = ensure_ring_room(a, RING_DISC, std::min<uint32_t>(n, a->nframes));
     if (s) return s;
+    cudaEvent_t sp = span_open(a);
     CK(launch_directive(a->T, kind, (uint32_t)lo, n, seq, 0, a->ps));
+    span_close(a, sp, 0);
+    a->n_launch++;
   }
   return hand_out(a, stream);
 }
@@ -560,8 +613,14 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
   uint64_t want = (bytes + a->B - 1) / a->B;
   if (want > a->nframes) want = a->nframes;
   if (want) {
+    cudaEvent_t sp = span_open(a);
     CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->ps));
+    span_close(a, sp, 0);
+    sp = span_open(a);
     CK(launch_service(a->T, SVC_D2H_ONLY, seq, (uint32_t)want, a->ps));
+    span_close(a, sp, 1);
+    a->n_launch += 2;
+    a->n_xfer++;
   }
   return hand_out(a, stream);
 }
@@ -577,6 +636,7 @@ UM_API um_status um_host_write(um_arena* a, uint64_t off, uint64_t len, void* st
   if (len) {
     uint32_t lo = (uint32_t)(off / a->B), hi = (uint32_t)((off + len - 1) / a->B + 1);
     CK(launch_host_write(a->T, lo, hi - lo, seq, a->ps));
+    a->n_launch += 2;
   }
   return hand_out(a, stream);
 }
@@ -656,10 +716,25 @@ UM_API um_status um_content_tags(um_arena* a, uint64_t* tags) {
   return UM_OK;
 }
 
-UM_API um_status um_timing(um_arena* a, double* ms_plan, double* ms_xfer, int reset) {
-  if (!a) return UM_EINVAL;
-  (void)reset;
-  if (ms_plan) *ms_plan = 0;
-  if (ms_xfer) *ms_xfer = 0;
+UM_API um_status um_timing(um_arena* a, double* ms_plan, double* ms_xfer, uint64_t* xfer_launches,
+                           uint64_t* launches, int reset) {
+  ENTER(a);
+  CK(cudaStreamSynchronize(a->ps));
+  for (auto& sp : a->spans) {
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, sp.a, sp.b));
+    (sp.xfer ? a->ms_xfer : a->ms_plan) += ms;
+    a->evpool.push_back(sp.a);
+    a->evpool.push_back(sp.b);
+  }
+  a->spans.clear();
+  if (ms_plan) *ms_plan = a->ms_plan;
+  if (ms_xfer) *ms_xfer = a->ms_xfer;
+  if (xfer_launches) *xfer_launches = a->n_xfer;
+  if (launches) *launches = a->n_launch;
+  if (reset) {
+    a->ms_plan = a->ms_xfer = 0;
+    a->n_xfer = a->n_launch = 0;
+  }
   return UM_OK;
 }

@@ -369,28 +369,37 @@ __global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, in
     if (threadIdx.x == 0) *headp = newhead;
   }
   __syncthreads();
-  // Reclaim the victims.  G victims are written back (host frames are assigned in
-  // victim order from the host free stack); GE/GL victims are dropped.
+  // Reclaim the victims.  G victims are written back (A10).  In a GPU sub-op victim j's
+  // frame goes to need item f0 + j; when that item migrates in from a host frame, the
+  // fused swap exchanges the two (the victim's bytes land in the host frame the new
+  // block's bytes leave), so no host frame is allocated for it.  Other G victims take
+  // host frames from the free stack in victim order.
   const int htop = c->hfree_top;
-  uint32_t gbase = 0;
+  uint32_t gbase = 0, abase = 0;
   uint32_t nGL = 0;
   for (uint32_t base = 0; base < found; base += kVictTPB) {
     const uint32_t j = base + threadIdx.x;
-    uint32_t v = 0, fr = UM_NONE;
+    uint32_t v = 0, fr = UM_NONE, swap_hf = UM_NONE;
     uint8_t ss = 0;
-    uint32_t isG = 0;
+    uint32_t isG = 0, needA = 0;
     if (j < found) {
       v = T.victim[j];
       ss = T.st[v];
       fr = T.frame_of[v];
       isG = ss == ST_G;
+      if (isG && !evict_mode) {
+        const uint32_t i = (uint32_t)f0 + j;
+        if (T.needk[i] == ST_H) swap_hf = T.needhf[i];
+      }
+      needA = isG && swap_hf == UM_NONE;
     }
-    unsigned long long tot;
+    unsigned long long tot, totA;
     uint32_t gr = (uint32_t)block_excl_scan<kVictTPB>(isG, tot, s_scan) + gbase;
+    uint32_t ar = (uint32_t)block_excl_scan<kVictTPB>(needA, totA, s_scan) + abase;
     if (j < found) {
-      uint32_t hf = UM_NONE;
-      if (isG) {
-        int idx = htop - 1 - (int)gr;
+      uint32_t hf = swap_hf;
+      if (needA) {
+        int idx = htop - 1 - (int)ar;
         if (idx >= 0) hf = T.hfree_stack[idx];
         else atomicExch(&c->err, 2u);  // host-frame pool exhausted -> UM_ENOMEM
       }
@@ -411,6 +420,7 @@ __global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, in
       }
     }
     gbase += (uint32_t)tot;
+    abase += (uint32_t)totA;
   }
   {
     uint32_t v[4] = {threadIdx.x == 0 ? found : 0u, threadIdx.x == 0 ? gbase : 0u,
@@ -420,7 +430,7 @@ __global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, in
     block_counts_to<4>(T, v, s_cnt, slots, mul);
   }
   if (threadIdx.x == 0) {
-    c->hfree_top = htop - (int)gbase;
+    c->hfree_top = max(0, htop - (int)abase);
     if (evict_mode) {
       c->free_top = f0 + (int)found;
       c->n_d2h = gbase;
@@ -512,13 +522,17 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
         uint8_t kd = T.needk[i];
         uint32_t hf = T.needhf[i];
         uint32_t fr;
+        bool swapped = false;
         x.d2h_dst = nullptr;
         if (i < nfu) {
           fr = T.free_stack[f0 - 1 - i];
         } else {
           uint32_t j = i - f0;
           fr = T.vframe[j];
-          if (T.vkind[j] == ST_G && T.vhf[j] != UM_NONE) x.d2h_dst = hptr(T, T.vhf[j]) + coff;
+          if (T.vkind[j] == ST_G && T.vhf[j] != UM_NONE) {
+            x.d2h_dst = hptr(T, T.vhf[j]) + coff;
+            swapped = T.vhf[j] == hf;   // host frame handed over to the victim
+          }
         }
         x.frame = T.frames + (size_t)fr * T.B + coff;
         if (kd == ST_H) {
@@ -535,8 +549,10 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
           T.map[bb] = fr;
           if (kd == ST_H && hf != UM_NONE) {
             T.hframe[bb] = UM_NONE;
-            int idx = atomicAdd(&c->hfree_top, 1);
-            T.hfree_stack[idx] = hf;
+            if (!swapped) {
+              int idx = atomicAdd(&c->hfree_top, 1);
+              T.hfree_stack[idx] = hf;
+            }
           }
         }
       } else {
@@ -681,8 +697,12 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
           if (ss == ST_G) {
             int idx = atomicSub(&T.ctl->hfree_top, 1) - 1;
             uint32_t hf = UM_NONE;
-            if (idx >= 0) hf = T.hfree_stack[idx];
-            else atomicExch(&T.ctl->err, 2u);
+            if (idx >= 0) {
+              hf = T.hfree_stack[idx];
+            } else {
+              atomicAdd(&T.ctl->hfree_top, 1);
+              atomicExch(&T.ctl->err, 2u);
+            }
             uint32_t q = atomicAdd(&T.ctl->n_d2h, 1u);
             T.d2h_frame[q] = fr;
             T.d2h_hf[q] = hf;
@@ -771,8 +791,12 @@ __global__ void k_hw_alloc(Tables T, uint32_t lo, uint32_t n) {
     }
     if (T.hframe[bb] == UM_NONE) {
       int idx = atomicSub(&T.ctl->hfree_top, 1) - 1;
-      if (idx >= 0) T.hframe[bb] = T.hfree_stack[idx];
-      else atomicExch(&T.ctl->err, 2u);
+      if (idx >= 0) {
+        T.hframe[bb] = T.hfree_stack[idx];
+      } else {
+        atomicAdd(&T.ctl->hfree_top, 1);
+        atomicExch(&T.ctl->err, 2u);
+      }
     }
   }
 }

@@ -19,9 +19,9 @@ def mode_flags(mode: str) -> int:
 
 
 def make_arena(trace, mode: str, *, flags: int = um.UM_F_APP_STAMP | um.UM_F_CHECK, host_pool_bytes=None,
-               device: int = 0) -> um.Arena:
+               device: int = 0, mem=None) -> um.Arena:
     return um.Arena(trace.block_bytes, trace.arena_bytes, trace.budget_bytes, flags=flags | mode_flags(mode),
-                    host_pool_bytes=host_pool_bytes, device=device)
+                    host_pool_bytes=host_pool_bytes, device=device, mem=mem)
 
 
 def alloc_buffers(arena: um.Arena, trace) -> None:
@@ -29,6 +29,13 @@ def alloc_buffers(arena: um.Arena, trace) -> None:
         got = um.um_alloc(arena.handle, nbytes)
         if got != off:
             raise AssertionError(f"um_alloc({name}) = {got}, trace expects {off}")
+
+
+def iteration_bounds(trace) -> list:
+    """Op index ranges of the iterations of a periodic trace (C3)."""
+    it = int(trace.meta.get("iterations", 1))
+    per = len(trace.ops) // it
+    return [(i * per, (i + 1) * per) for i in range(it)]
 
 
 def issue(arena: um.Arena, trace, mode: str, start: int = 0, stop: int | None = None, stream=None) -> None:

@@ -20,7 +20,7 @@ UM_DST_GPU, UM_DST_HOST = 0, 1
 UM_ACC_READ, UM_ACC_WRITE = 1, 2
 UM_ST_U, UM_ST_H, UM_ST_HD, UM_ST_G, UM_ST_GE, UM_ST_GL = range(6)
 ST_NAMES = ("U", "H", "HD", "G", "GE", "GL")
-UM_F_DISCARD_OFF, UM_F_COPY_CE, UM_F_CHECK, UM_F_APP_STAMP = 1, 2, 4, 8
+UM_F_DISCARD_OFF, UM_F_COPY_CE, UM_F_CHECK, UM_F_APP_STAMP, UM_F_TIMING = 1, 2, 4, 8, 16
 UM_NONE = 0xFFFFFFFF
 
 
@@ -79,7 +79,7 @@ def lib():
             "um_get_stats": [P, C.POINTER(um_stats)],
             "um_dump": [P, P, P, C.POINTER(U32), P, C.POINTER(U32)],
             "um_content_tags": [P, P],
-            "um_timing": [P, C.POINTER(C.c_double), C.POINTER(C.c_double), I],
+            "um_timing": [P, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(U64), C.POINTER(U64), I],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -187,38 +187,76 @@ def um_content_tags(a, nblocks: int) -> np.ndarray:
     return t
 
 
+def um_timing(a, reset: bool = False) -> dict:
+    p, x = C.c_double(), C.c_double()
+    nx, nl = C.c_uint64(), C.c_uint64()
+    _ck("um_timing", lib().um_timing(a, C.byref(p), C.byref(x), C.byref(nx), C.byref(nl), int(reset)))
+    return {"ms_plan": p.value, "ms_xfer": x.value, "xfer_launches": nx.value, "launches": nl.value}
+
+
 # -------------------------------------------------------------------------------------
 # Arena: allocates the caller-owned memory with torch (frames + workspace in HBM,
 # host-frame pool in pinned host memory) and creates the libum arena.
 # -------------------------------------------------------------------------------------
-class Arena:
-    def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, flags: int = 0,
-                 host_pool_bytes: int | None = None, host_chunk_bytes: int | None = None, device: int = 0):
+class Memory:
+    """Caller-owned memory for an arena, allocated once with torch and reusable by
+    several arenas in sequence: frames (HBM), workspace (HBM), host-frame pool
+    (pinned host memory in chunks of <= 1 GiB, allocated from `threads` threads)."""
+
+    def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, host_pool_bytes=None,
+                 host_chunk_bytes=None, device: int = 0, threads: int = 1):
         import torch
-        self.torch = torch
         self.B = block_bytes
-        self.nblocks = arena_bytes // block_bytes
         self.nframes = budget_bytes // block_bytes
         if host_pool_bytes is None:
             host_pool_bytes = arena_bytes          # every block can be host-resident
         host_pool_bytes += block_bytes             # + the zero page
         if host_chunk_bytes is None:
             host_chunk_bytes = min(1 << 30, max(block_bytes, 1 << (host_pool_bytes - 1).bit_length()))
+        self.host_chunk_bytes = host_chunk_bytes
         nch = -(-host_pool_bytes // host_chunk_bytes)
+        self.device = device
         dev = torch.device("cuda", device)
         self.frames = torch.empty(self.nframes * block_bytes, dtype=torch.uint8, device=dev)
-        self.host_chunks = [torch.empty(host_chunk_bytes, dtype=torch.uint8, pin_memory=True) for _ in range(nch)]
+        mk = lambda _: torch.empty(host_chunk_bytes, dtype=torch.uint8, pin_memory=True)
+        if threads > 1 and nch > 1:
+            from concurrent.futures import ThreadPoolExecutor
+            with ThreadPoolExecutor(threads) as ex:
+                self.host_chunks = list(ex.map(mk, range(nch)))
+        else:
+            self.host_chunks = [mk(i) for i in range(nch)]
         self._hc = (C.c_void_p * nch)(*[t.data_ptr() for t in self.host_chunks])
-        cfg = um_config(device=device, block_bytes=block_bytes, arena_bytes=arena_bytes,
-                        budget_bytes=budget_bytes, frames=self.frames.data_ptr(), workspace=None,
-                        workspace_bytes=0, host_chunks=C.cast(self._hc, C.POINTER(C.c_void_p)),
-                        n_host_chunks=nch, host_chunk_bytes=host_chunk_bytes, flags=flags)
-        ws = um_workspace_size(cfg)
+        probe = um_config(device=device, block_bytes=block_bytes, arena_bytes=arena_bytes,
+                          budget_bytes=budget_bytes, frames=self.frames.data_ptr(), workspace=None,
+                          workspace_bytes=0, host_chunks=C.cast(self._hc, C.POINTER(C.c_void_p)),
+                          n_host_chunks=nch, host_chunk_bytes=host_chunk_bytes, flags=0)
+        ws = um_workspace_size(probe)
         self.workspace = torch.empty(ws, dtype=torch.uint8, device=dev)
-        cfg.workspace = self.workspace.data_ptr()
-        cfg.workspace_bytes = ws
-        self.cfg = cfg
-        self.handle = um_arena_create(cfg)
+        self.nch = nch
+
+    def config(self, arena_bytes: int, budget_bytes: int, flags: int) -> um_config:
+        return um_config(device=self.device, block_bytes=self.B, arena_bytes=arena_bytes,
+                         budget_bytes=budget_bytes, frames=self.frames.data_ptr(),
+                         workspace=self.workspace.data_ptr(), workspace_bytes=self.workspace.numel(),
+                         host_chunks=C.cast(self._hc, C.POINTER(C.c_void_p)), n_host_chunks=self.nch,
+                         host_chunk_bytes=self.host_chunk_bytes, flags=flags)
+
+
+class Arena:
+    """A libum arena over `Memory` (allocated here unless `mem` is given)."""
+
+    def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, flags: int = 0,
+                 host_pool_bytes: int | None = None, host_chunk_bytes: int | None = None, device: int = 0,
+                 mem: Memory | None = None):
+        self.B = block_bytes
+        self.nblocks = arena_bytes // block_bytes
+        self.nframes = budget_bytes // block_bytes
+        self.mem = mem if mem is not None else Memory(block_bytes, arena_bytes, budget_bytes,
+                                                      host_pool_bytes=host_pool_bytes,
+                                                      host_chunk_bytes=host_chunk_bytes, device=device)
+        self.frames = self.mem.frames
+        self.cfg = self.mem.config(arena_bytes, budget_bytes, flags)
+        self.handle = um_arena_create(self.cfg)
         self.stream_ptr = um_stream(self.handle)
 
     def close(self):

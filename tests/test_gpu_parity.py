@@ -171,3 +171,15 @@ def test_block_table_maps_resident_blocks():
         assert blk[0] == s and blk[1] == ~s
     finally:
         a.close()
+
+
+@pytest.mark.parametrize("mode", ["base", "eager"])
+def test_c3_small_tight_host_pool(mode):
+    """Host-frame pool sized to the host-resident set (R1/NEXT-4): arena - budget + 2
+    blocks.  The fused swap hands the migrating block's host frame to the victim, so the
+    pool never needs more than the oracle's max |H| (+ frames freed later in the op)."""
+    t = tg.gen_c3(block_bytes=64 << 10, budget_bytes=192 << 20, iterations=2, workspace_bytes=4 << 20,
+                  layers=tg.scale_layers(tg.VGG16, 1.0 / 512, 1.0 / 64), batch=8)
+    pool = t.arena_bytes - t.budget_bytes + 2 * t.block_bytes
+    g = _gpu(t, mode, host_pool_bytes=pool)
+    assert_parity(t, mode, g)
