@@ -46,6 +46,8 @@ def parse():
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--no-discard-bench", action="store_true")
     p.add_argument("--pin-threads", type=int, default=8)
+    p.add_argument("--no-compare", action="store_true")
+    p.add_argument("--no-state-bench", action="store_true")
     return p.parse_args()
 
 
@@ -235,10 +237,58 @@ def discard_bench(torch, um, reps=20):
     return out
 
 
+def state_bench(torch, um, mem, budget, arena_bytes, seed=0):
+    """State-kernel microbench (SURVEY §8(d) last row): C3-64K-sized tables (64 KiB blocks
+    over the same 170 GiB of frames / 255 GiB arena), one touch_batch of 2^21 distinct
+    uniformly random blocks, then one 2^21-block discard.  Planning kernels timed apart
+    from the zero-fill (um_timing); algorithmic bytes per block as in DESIGN.md §5."""
+    import numpy as np
+    import tracegen as tg
+    B = 64 * 1024
+    nb = arena_bytes // B
+    n = 1 << 21
+    cfg = mem.config(arena_bytes, budget, um.UM_F_TIMING)
+    cfg.block_bytes = B
+    ws_bytes = um.um_workspace_size(cfg)
+    ws = torch.empty(ws_bytes, dtype=torch.uint8, device=mem.frames.device)
+    cfg.workspace, cfg.workspace_bytes = ws.data_ptr(), ws_bytes
+    h = um.um_arena_create(cfg)
+    try:
+        rng = np.random.default_rng(seed)
+        blocks = np.sort(rng.choice(nb, size=n, replace=False))
+        acc = np.zeros(n, dtype=tg.ACC_DTYPE)
+        acc["off"] = blocks.astype(np.uint64) * B
+        acc["len"] = B
+        acc["kind"] = tg.ACC_READ
+        um.um_timing(h, reset=True)
+        um.um_touch_batch(h, acc)
+        t_touch = um.um_timing(h, reset=True)
+        um.um_discard(h, 0, n * B)
+        t_disc = um.um_timing(h, reset=True)
+        st = um.um_get_stats(h)
+        assert st["zf_bytes"] == n * B
+        g_in = int(np.count_nonzero(blocks < n))        # G blocks inside the discarded range
+        # bytes per block: classify 1 st + 4 pin + 8 ring + 9 need list + 4 hframe + 8 intervals;
+        # victims: none needed (frames free).  directive: 1 st rd; G: 1 st + 4 key + 4 map + 8 DISC
+        cls_bytes = n * (1 + 4 + 8 + 9 + 4 + 8)
+        dir_bytes = n * 1 + g_in * (1 + 4 + 4 + 8)
+        peak = 6548.5
+        def rl(name, by, ms):
+            a = by / (ms / 1e3) / 1e9 if ms else None
+            return {"kernel": name, "bound": "hbm", "achieved": a, "peak": peak, "unit": "GB/s",
+                    "frac": a / peak if a else None, "algorithmic_bytes": by, "ms": ms, "blocks": n}
+        return {"touch_2^21_random": rl("k_classify+k_victims", cls_bytes, t_touch["ms_plan"]),
+                "discard_2^21": rl("k_directive", dir_bytes, t_disc["ms_plan"]),
+                "zero_fill_gbs": (n * B) / (t_touch["ms_xfer"] / 1e3) / 1e9 if t_touch["ms_xfer"] else None,
+                "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, read+write)", "nblocks": nb}
+    finally:
+        um.um_arena_destroy(h)
+        del ws
+
+
 def _barrier(torch):
-    import torch.distributed as dist
-    if dist.is_available() and dist.is_initialized():
-        dist.barrier()
+    from paper_conf_iiswc_zhucvhcr22_b200.dist import barrier
+    barrier()
     torch.cuda.synchronize()
 
 
@@ -265,6 +315,19 @@ def cpu_oracle_baseline(trace, W, budget_s=20.0):
     return {"value": n / dt, "unit": "iter/s", "cores": 1, "kind": "oracle",
             "sample": f"C3 eager iterations 2..{n + 1} of the bench trace (iteration 1 replayed untimed)",
             "s_per_iter": dt / n}
+
+
+def _paths(auto, k4, link):
+    def one(r):
+        if not r:
+            return None
+        sp = r["stats_per_iter"]
+        lb = sp["h2d_bytes"] + sp["d2h_bytes"]
+        ach = lb * len(r["iter_ms_each"]) / (r["timing"]["ms_xfer"] / 1e3) / 1e9 if r["timing"]["ms_xfer"] else None
+        t_ideal = sp["h2d_bytes"] / (link["h2d_gbs"] * 1e9) + sp["d2h_bytes"] / (link["d2h_gbs"] * 1e9)
+        pk = lb / t_ideal / 1e9 if t_ideal else None
+        return {"iter_ms": r["iter_ms"], "achieved_gbs": ach, "frac_of_link": (ach / pk) if (ach and pk) else None}
+    return {"auto (K4-CE >= 16 MiB)": one(auto), "k4_tma_kernel_only": one(k4)}
 
 
 def build_trace(args, budget, with_host_data, iterations):
@@ -307,21 +370,19 @@ def main_ours(args):
     clocks = Clocks(dev.index)
     for mode in args.modes.split(","):
         res[mode] = run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=clocks if mode == "eager" else None)
+    # the TMA kernel path (K4) on the same step, for comparison with the auto path
+    k4 = run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=um.UM_F_COPY_KERNEL) \
+        if not args.no_compare else None
+    state = state_bench(torch, um, mem, budget, arena_bytes) if not args.no_state_bench else None
     e2e_s = None
     if not args.no_e2e:
         e2e_s = run_e2e(torch, um, harness, mem, trace, 1, min(K, 3))
 
     head = res.get("eager") or next(iter(res.values()))
     t_iter_ms = head["iter_ms"]
-    # max over ranks
-    if ws > 1:
-        import torch.distributed as dist
-        t = torch.tensor([t_iter_ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        t_iter_ms = float(t.item())
-        sv = torch.tensor([head["stats_per_iter"][k] for k in sorted(head["stats_per_iter"])], device=dev,
-                          dtype=torch.float64)
-        dist.all_reduce(sv)   # the one collective of the path: stats all-reduce (north_star)
+    # max over ranks; the run's only collective: counters all-reduce (north_star)
+    from paper_conf_iiswc_zhucvhcr22_b200.dist import reduce_run
+    stats_all, t_iter_ms = reduce_run(head["stats_per_iter"], t_iter_ms, device=dev)
     if rank != 0:
         return
     spi = head["stats_per_iter"]
@@ -361,7 +422,8 @@ def main_ours(args):
         "serviced_gbs": (link_bytes + spi["zf_bytes"]) / (t_iter_ms / 1e3) / 1e9,
         "discard_us_per_gb": ({"eager": disc[-1]["eager"]["us_per_gb"], "lazy": disc[-1]["lazy"]["us_per_gb"],
                                "sweep": disc} if disc else None),
-        "roofline": {"kernel": "k_service (TMA fused-swap transfer + zero-fill)", "bound": "host_link",
+        "roofline": {"kernel": "transfer engine: K4-CE (copy engines, device-made plan) for sub-ops >= 16 MiB, K4 TMA kernel below",
+                     "bound": "host_link",
                      "achieved": achieved, "peak": peak_eff, "unit": "GB/s",
                      "frac": (achieved / peak_eff) if achieved else None, "traffic": None,
                      "frac_vs_duplex": (achieved / link["duplex_gbs"]) if achieved else None,
@@ -369,8 +431,11 @@ def main_ours(args):
                      "algorithmic_bytes_per_launch": link_bytes_per_launch, "ms_per_launch": xfer_ms_per_launch,
                      "launches_per_iter": tm["xfer_launches"] / K, "xfer_share_of_step": tm["ms_xfer"] / (t_iter_ms * K)},
         "link_peak": link,
+        "transfer_paths": _paths(res.get("eager"), k4, link),
+        "roofline_state": state,
         "clocks": head["clocks"],
         "gpu_launches": tm["launches"],
+        "stats_per_iter_all_ranks": stats_all,
         "setup_s": {"pin_and_alloc": t_alloc},
     })
     if e2e_s is not None:

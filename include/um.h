@@ -18,8 +18,10 @@
  * migrated when it is used again (Fig. 2 (7)).
  *
  * Execution.  All planning (state tables, victim selection, work-list compaction) runs
- * in sm_100a kernels on device-resident tables; data moves by a kernel-driven copy over
- * mapped pinned host memory (or by the copy engines with UM_F_COPY_CE).  No CPU fallback.
+ * in sm_100a kernels on device-resident tables; data moves by a kernel-driven TMA copy
+ * over mapped pinned host memory (K4, no host round trip) or, for large sub-ops, by the
+ * copy engines from the device-made plan (K4-CE, one host sync per sub-op).  No CPU
+ * fallback: the host never computes a state, a victim or a transfer list.
  *
  * Conventions (all functions):
  *  - Return um_status; UM_OK = 0.  No exceptions cross the ABI.
@@ -59,12 +61,15 @@ enum { UM_ST_U = 0, UM_ST_H = 1, UM_ST_HD = 2, UM_ST_G = 3, UM_ST_GE = 4, UM_ST_
 
 enum {
   UM_F_DISCARD_OFF = 1u, /* "UVM-opt" baseline: discards are accepted no-ops */
-  UM_F_COPY_CE = 2u,     /* move data with cudaMemcpyAsync on side streams, not K4       */
+  UM_F_COPY_CE = 2u,     /* always move data with the copy engines (K4-CE: device plan,
+                            one host sync per sub-op, cudaMemcpyBatchAsync on 2 streams)  */
   UM_F_CHECK = 4u,       /* poison frames with 0xA5 at creation; extra validation       */
   UM_F_APP_STAMP = 8u,   /* harness: after each touch sub-op, write the content stamp of
                             every UM_ACC_WRITE block (simulated application kernel)    */
-  UM_F_TIMING = 16u      /* record CUDA events around the planning and transfer kernels
+  UM_F_TIMING = 16u,     /* record CUDA events around the planning and transfer kernels
                             of every op (read with um_timing)                          */
+  UM_F_COPY_KERNEL = 32u /* always move data with the TMA kernel (K4).  Default (neither
+                            flag): sub-ops moving >= 16 MiB use K4-CE, smaller ones K4  */
 };
 
 /* One GPU access record of a batch (16 bytes).  Covers every block overlapping

@@ -31,8 +31,8 @@ struct Layout {
   uint64_t st, key, frame_of, map, hframe, pin, free_stack, hfree_stack;
   uint64_t used[2], disc[2];
   uint64_t need, needk, needhf, victim, vframe, vhf, vkind, d2h_frame, d2h_hf;
-  uint64_t tile_status, tags, ctl, hchunks, stage;
-  uint64_t stage_bytes, max_tiles, cap, total;
+  uint64_t tile_status, tile_cnt, tags, ctl, hchunks, stage, xitems, bounce;
+  uint64_t stage_bytes, max_tiles, cap, total, ce_group, bounce_bytes;
 };
 
 static uint64_t pow2_ceil(uint64_t x) {
@@ -90,10 +90,17 @@ static Layout make_layout(const um_config* c) {
   L.d2h_frame = take(4 * nf);
   L.d2h_hf = take(4 * nf);
   L.tile_status = take(8 * L.max_tiles);
+  L.tile_cnt = take(32 * L.max_tiles);
   L.tags = take(8 * nb);
   L.ctl = take(sizeof(Ctl));
   L.hchunks = take(8ull * c->n_host_chunks);
   L.stage = take(L.stage_bytes);
+  L.xitems = take(sizeof(XItem) * nf);
+  // K4-CE: groups of ce_group items alternate between two copy streams; fused swaps
+  // bounce the victim's bytes through HBM (one slot per item per stream)
+  L.ce_group = std::max<uint64_t>(1, std::min<uint64_t>(1024, (64ull << 20) / c->block_bytes));
+  L.bounce_bytes = 2 * L.ce_group * c->block_bytes;
+  L.bounce = take(L.bounce_bytes);
   L.total = o;
   return L;
 }
@@ -192,8 +199,15 @@ struct um_arena {
   std::vector<cudaEvent_t> evpool;
   double ms_plan = 0, ms_xfer = 0;
   uint64_t n_xfer = 0, n_launch = 0;
-  std::vector<uint32_t> tmp_lo, tmp_pre;
-  std::vector<uint8_t> tmp_w;
+  // K4-CE path
+  cudaStream_t cs[2] = {nullptr, nullptr};
+  cudaEvent_t ev_cs[2] = {nullptr, nullptr};
+  XItem* hitems = nullptr;              // pinned mirror of xitems
+  uint32_t* hd2h = nullptr;             // pinned mirror of d2h_frame / d2h_hf
+  std::vector<char*> hhost;             // host chunk pointers
+  char* bounce = nullptr;
+  uint64_t ce_min_bytes = 16ull << 20;  // auto mode: sub-ops moving >= this use the copy engines
+  uint64_t n_ce = 0;
 };
 
 namespace {
@@ -331,6 +345,134 @@ static void build_intervals(um_arena* a, const um_access* acc, uint32_t n) {
   }
 }
 
+static bool use_ce(um_arena* a, uint64_t n) {
+  if (a->cfg.flags & UM_F_COPY_CE) return true;
+  if (a->cfg.flags & UM_F_COPY_KERNEL) return false;
+  return n * a->B >= a->ce_min_bytes;
+}
+
+static inline char* hframe_ptr(um_arena* a, uint32_t h) {
+  return a->hhost[h / a->T.hpc] + (size_t)(h % a->T.hpc) * a->B;
+}
+static inline char* frame_ptr(um_arena* a, uint32_t f) { return a->T.frames + (size_t)f * a->B; }
+
+// A copy list with run coalescing (adjacent items whose source and destination are
+// both contiguous AND inside the same host chunk allocation become one copy — a copy
+// may not span two pinned allocations even if they happen to be adjacent), issued as
+// one cudaMemcpyBatchAsync.
+struct CopyList {
+  std::vector<void*> dst, src;
+  std::vector<size_t> size;
+  std::vector<uint32_t> seg;
+  void clear() { dst.clear(); src.clear(); size.clear(); seg.clear(); }
+  void add(void* d, const void* s_, size_t n, uint32_t chunk) {
+    if (!dst.empty() && seg.back() == chunk && (char*)dst.back() + size.back() == (char*)d &&
+        (const char*)src.back() + size.back() == (const char*)s_) {
+      size.back() += n;
+      return;
+    }
+    dst.push_back(d);
+    src.push_back(const_cast<void*>(s_));
+    size.push_back(n);
+    seg.push_back(chunk);
+  }
+  cudaError_t issue(cudaStream_t st) {
+    if (dst.empty()) return cudaSuccess;
+    if (dst.size() == 1) return cudaMemcpyAsync(dst[0], src[0], size[0], cudaMemcpyDefault, st);
+    cudaMemcpyAttributes attr{};
+    attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+    attr.flags = cudaMemcpyFlagPreferOverlapWithCompute;
+    size_t aidx = 0, fail = 0;
+    cudaError_t e = cudaMemcpyBatchAsync(dst.data(), src.data(), size.data(), dst.size(), &attr, &aidx, 1, &fail, st);
+    if (e == cudaSuccess) return e;
+    cudaGetLastError();
+    if (getenv("UM_DEBUG")) {
+      fprintf(stderr, "libum: cudaMemcpyBatchAsync(%zu copies) failed: %s (fail idx %zu); falling back\n", dst.size(),
+              cudaGetErrorString(e), fail);
+      for (size_t i = 0; i < dst.size() && i < 4; ++i) {
+        cudaPointerAttributes pa{}, pb{};
+        cudaPointerGetAttributes(&pa, dst[i]);
+        cudaPointerGetAttributes(&pb, src[i]);
+        cudaGetLastError();
+        fprintf(stderr, "  [%zu] dst %p (type %d) src %p (type %d) size %zu\n", i, dst[i], (int)pa.type, src[i],
+                (int)pb.type, size[i]);
+      }
+    }
+    for (size_t i = 0; i < dst.size(); ++i) {
+      e = cudaMemcpyAsync(dst[i], src[i], size[i], cudaMemcpyDefault, st);
+      if (e) return e;
+    }
+    return cudaSuccess;
+  }
+};
+
+// K4-CE: the plan is on the device (K1-K3 + K6 in k_plan_commit); one host sync reads
+// it, then groups of items alternate between two copy-engine streams:
+//   D2D victim->bounce (fused swaps) ; D2H write-backs ; H2D migrations ; zero-fill
+//   kernel ; D2H bounce->host (fused swaps).
+// Stream order gives every frame its write-after-read order; alternating streams keep
+// both PCIe directions busy.  The paging stream waits for both copy streams.
+static um_status ce_subop(um_arena* a, uint32_t seq, uint32_t n) {
+  CK(launch_plan_commit(a->T, seq, n, a->ps));
+  CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaMemcpyAsync(a->hitems, a->T.xitems, sizeof(XItem) * n, cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaStreamSynchronize(a->ps));
+  const uint32_t nn = std::min<uint32_t>(a->hctl->n_need, n);
+  const uint64_t G = a->L.ce_group, B = a->B;
+  CopyList d2d, wb, h2d, sw;
+  for (uint32_t g0 = 0, gi = 0; g0 < nn; g0 += (uint32_t)G, ++gi) {
+    const uint32_t g1 = (uint32_t)std::min<uint64_t>(nn, g0 + G);
+    cudaStream_t st = a->cs[gi & 1];
+    char* bnc = a->bounce + (gi & 1) * G * B;
+    d2d.clear(); wb.clear(); h2d.clear(); sw.clear();
+    bool anyzf = false;
+    uint32_t k = 0;
+    for (uint32_t i = g0; i < g1; ++i) {
+      const XItem& x = a->hitems[i];
+      char* fr = frame_ptr(a, x.fr);
+      if (x.flags & XI_SWAP) {
+        d2d.add(bnc + (size_t)k * B, fr, B, UM_NONE);
+        sw.add(hframe_ptr(a, x.dst_hf), bnc + (size_t)k * B, B, x.dst_hf / a->T.hpc);
+        ++k;
+      } else if (x.flags & XI_D2H) {
+        wb.add(hframe_ptr(a, x.dst_hf), fr, B, x.dst_hf / a->T.hpc);
+      }
+      if (x.flags & XI_H2D) h2d.add(fr, hframe_ptr(a, x.src_hf), B, x.src_hf / a->T.hpc);
+      anyzf |= (x.flags & XI_ZF) != 0;
+    }
+    CK(d2d.issue(st));
+    CK(wb.issue(st));
+    CK(h2d.issue(st));
+    if (anyzf) CK(launch_zero_items(a->T, g0, g1, st));
+    CK(sw.issue(st));
+  }
+  for (int i = 0; i < 2; ++i) {
+    CK(cudaEventRecord(a->ev_cs[i], a->cs[i]));
+    CK(cudaStreamWaitEvent(a->ps, a->ev_cs[i], 0));
+  }
+  a->n_ce++;
+  return UM_OK;
+}
+
+// D2H-only list (prefetch HOST, evict) through the copy engines.
+static um_status ce_d2h_only(um_arena* a, uint32_t nmax) {
+  CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaMemcpyAsync(a->hd2h, a->T.d2h_frame, 4ull * nmax, cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaMemcpyAsync(a->hd2h + a->nframes, a->T.d2h_hf, 4ull * nmax, cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaMemsetAsync(&a->T.ctl->n_d2h, 0, sizeof(unsigned int), a->ps));
+  CK(cudaStreamSynchronize(a->ps));
+  const uint32_t nd = std::min<uint32_t>(a->hctl->n_d2h, nmax);
+  CopyList wb;
+  for (uint32_t i = 0; i < nd; ++i)
+    if (a->hd2h[a->nframes + i] != UM_NONE)
+      wb.add(hframe_ptr(a, a->hd2h[a->nframes + i]), frame_ptr(a, a->hd2h[i]), a->B, a->hd2h[a->nframes + i] / a->T.hpc);
+  CK(wb.issue(a->cs[0]));
+  CK(cudaEventRecord(a->ev_cs[0], a->cs[0]));
+  CK(cudaStreamWaitEvent(a->ps, a->ev_cs[0], 0));
+  a->n_ce++;
+  return UM_OK;
+}
+
 // Enqueue the K1/K2 -> K3 -> K4/K5/K6 (-> K9) chain for every sub-op of a GPU op.
 static um_status run_gpu_op(um_arena* a, int touch) {
   uint64_t total = 0;
@@ -380,10 +522,18 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
     CK(launch_victims(a->T, seq, 0, 0, a->ps));
     span_close(a, sp, 0);
-    sp = span_open(a);
-    CK(launch_service(a->T, SVC_SUBOP, seq, n, a->ps));
-    span_close(a, sp, 1);
-    a->n_launch += 3;
+    if (use_ce(a, n)) {
+      sp = span_open(a);
+      um_status st = ce_subop(a, seq, n);
+      if (st) return st;
+      span_close(a, sp, 1);
+      a->n_launch += 4;
+    } else {
+      sp = span_open(a);
+      CK(launch_service(a->T, SVC_SUBOP, seq, n, a->ps));
+      span_close(a, sp, 1);
+      a->n_launch += 3;
+    }
     a->n_xfer++;
     if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP)) {
       CK(launch_app_stamp(a->T, iv, (uint32_t)g0, n, seq, a->ps));
@@ -419,7 +569,7 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   if (check_cfg(cfg) || !out || !cfg->frames || !cfg->workspace || !cfg->host_chunks) return UM_EINVAL;
   Layout L = make_layout(cfg);
   if (cfg->workspace_bytes < L.total) return UM_EINVAL;
-  if (cfg->flags & UM_F_COPY_CE) return UM_EINVAL;  // copy-engine path: not in this build
+  if ((cfg->flags & UM_F_COPY_CE) && (cfg->flags & UM_F_COPY_KERNEL)) return UM_EINVAL;
   um_arena* a = new (std::nothrow) um_arena();
   if (!a) return UM_ENOMEM;
   a->cfg = *cfg;
@@ -463,8 +613,11 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   T.d2h_frame = (uint32_t*)(ws + L.d2h_frame);
   T.d2h_hf = (uint32_t*)(ws + L.d2h_hf);
   T.tile_status = (unsigned long long*)(ws + L.tile_status);
+  T.tile_cnt = (uint32_t*)(ws + L.tile_cnt);
   T.tags = (uint64_t*)(ws + L.tags);
   T.ctl = (Ctl*)(ws + L.ctl);
+  T.xitems = (XItem*)(ws + L.xitems);
+  a->bounce = ws + L.bounce;
   T.frames = (char*)cfg->frames;
   T.hpc = hpc;
   T.B = a->B;
@@ -494,6 +647,14 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   if ((e = cudaEventCreateWithFlags(&a->ev_in, cudaEventDisableTiming))) return fail(e);
   if ((e = cudaEventCreateWithFlags(&a->ev_out, cudaEventDisableTiming))) return fail(e);
   if ((e = cudaHostAlloc((void**)&a->hctl, sizeof(Ctl), cudaHostAllocDefault))) return fail(e);
+  if ((e = cudaHostAlloc((void**)&a->hitems, sizeof(XItem) * a->nframes, cudaHostAllocDefault))) return fail(e);
+  if ((e = cudaHostAlloc((void**)&a->hd2h, 8ull * a->nframes, cudaHostAllocDefault))) return fail(e);
+  for (int i = 0; i < 2; ++i) {
+    if ((e = cudaStreamCreateWithFlags(&a->cs[i], cudaStreamNonBlocking))) return fail(e);
+    if ((e = cudaEventCreateWithFlags(&a->ev_cs[i], cudaEventDisableTiming))) return fail(e);
+  }
+  for (uint32_t i = 0; i < cfg->n_host_chunks; ++i) a->hhost.push_back((char*)cfg->host_chunks[i]);
+  if (const char* v = getenv("UM_CE_MIN_BYTES")) a->ce_min_bytes = strtoull(v, nullptr, 10);
   if ((e = a->stage.init((uint8_t*)(ws + L.stage), L.stage_bytes))) return fail(e);
   if ((e = cudaMemcpyAsync(dhc, hc.data(), 8ull * cfg->n_host_chunks, cudaMemcpyHostToDevice, a->ps))) return fail(e);
   if ((e = cudaMemsetAsync(T.tile_status, 0, 8 * L.max_tiles, a->ps))) return fail(e);
@@ -512,6 +673,12 @@ UM_API um_status um_arena_destroy(um_arena* a) {
   for (auto& sp : a->spans) { cudaEventDestroy(sp.a); cudaEventDestroy(sp.b); }
   for (auto e : a->evpool) cudaEventDestroy(e);
   if (a->hctl) cudaFreeHost(a->hctl);
+  if (a->hitems) cudaFreeHost(a->hitems);
+  if (a->hd2h) cudaFreeHost(a->hd2h);
+  for (int i = 0; i < 2; ++i) {
+    if (a->ev_cs[i]) cudaEventDestroy(a->ev_cs[i]);
+    if (a->cs[i]) cudaStreamDestroy(a->cs[i]);
+  }
   if (a->ev_in) cudaEventDestroy(a->ev_in);
   if (a->ev_out) cudaEventDestroy(a->ev_out);
   if (a->ps) cudaStreamDestroy(a->ps);
@@ -564,8 +731,14 @@ UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, v
       cudaEvent_t sp = span_open(a);
       CK(launch_directive(a->T, DIR_PREFETCH_HOST, lo, hi - lo, seq, 0, a->ps));
       span_close(a, sp, 0);
+      const uint32_t nmax = std::min<uint32_t>(hi - lo, a->nframes);
       sp = span_open(a);
-      CK(launch_service(a->T, SVC_D2H_ONLY, seq, std::min<uint32_t>(hi - lo, a->nframes), a->ps));
+      if (use_ce(a, nmax)) {
+        s = ce_d2h_only(a, nmax);
+        if (s) return s;
+      } else {
+        CK(launch_service(a->T, SVC_D2H_ONLY, seq, nmax, a->ps));
+      }
       span_close(a, sp, 1);
       a->n_launch += 2;
       a->n_xfer++;
@@ -617,7 +790,12 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
     CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->ps));
     span_close(a, sp, 0);
     sp = span_open(a);
-    CK(launch_service(a->T, SVC_D2H_ONLY, seq, (uint32_t)want, a->ps));
+    if (use_ce(a, want)) {
+      s = ce_d2h_only(a, (uint32_t)want);
+      if (s) return s;
+    } else {
+      CK(launch_service(a->T, SVC_D2H_ONLY, seq, (uint32_t)want, a->ps));
+    }
     span_close(a, sp, 1);
     a->n_launch += 2;
     a->n_xfer++;

@@ -35,6 +35,15 @@ struct Ctl {
   long long stats[S_N];
 };
 
+// One need item's transfer plan (K4-CE path exports these to the host).
+struct XItem {
+  uint32_t fr;      // destination GPU frame
+  uint32_t src_hf;  // host frame to migrate from (XI_H2D), else NONE
+  uint32_t dst_hf;  // host frame receiving the victim's write-back (XI_D2H), else NONE
+  uint32_t flags;
+};
+enum { XI_H2D = 1u, XI_ZF = 2u, XI_D2H = 4u, XI_SWAP = 8u };
+
 // Everything a kernel needs, passed by value.
 struct Tables {
   uint8_t* st;          // [nblocks] state
@@ -58,7 +67,9 @@ struct Tables {
   uint32_t* d2h_frame;  // [nframes] D2H-only list (prefetch HOST, evict)
   uint32_t* d2h_hf;     // [nframes]
   unsigned long long* tile_status;  // [max tiles] decoupled look-back
+  uint32_t* tile_cnt;   // [max tiles * 8] per-tile counter partials
   uint64_t* tags;       // [nblocks] content tags (harness)
+  XItem* xitems;        // [nframes] exported plan of the current sub-op (K4-CE path)
   Ctl* ctl;
   char* frames;             // device, nframes * B
   char* const* hchunks;     // device array of host-chunk device pointers
@@ -103,6 +114,8 @@ cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n,
 cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64_t cap_bound, cudaStream_t s);
 cudaError_t launch_host_write(const Tables& T, uint32_t lo, uint32_t n, uint32_t seq, cudaStream_t s);
 cudaError_t launch_tags(const Tables& T, cudaStream_t s);
+cudaError_t launch_plan_commit(const Tables& T, uint32_t seq, uint32_t max_items, cudaStream_t s);
+cudaError_t launch_zero_items(const Tables& T, uint32_t i0, uint32_t i1, cudaStream_t s);
 cudaError_t launch_poison(const Tables& T, cudaStream_t s);
 
 }  // namespace um

@@ -146,6 +146,56 @@ __device__ __forceinline__ void block_counts_to(const Tables& T, uint32_t (&c)[N
   if (threadIdx.x < NC && slots[threadIdx.x] >= 0) stat_add(T, slots[threadIdx.x], (long long)sm[threadIdx.x] * mul[threadIdx.x]);
 }
 
+// Multi-CTA scans do not add their counters with same-address atomics (thousands of
+// CTAs serialise on one L2 atomic unit): each tile stores its block-reduced counts and
+// the last CTA of the launch (scan_finish) sums them and adds once per counter.
+template <int NC>
+__device__ __forceinline__ void tile_counts(const Tables& T, uint32_t tile, uint32_t (&c)[NC], uint32_t* sm) {
+  if (threadIdx.x < NC) sm[threadIdx.x] = 0;
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < NC; ++i) {
+    uint32_t v = __reduce_add_sync(FULL, c[i]);
+    if ((threadIdx.x & 31) == 0 && v) atomicAdd(&sm[i], v);
+  }
+  __syncthreads();
+  if (threadIdx.x < NC) {
+    T.tile_cnt[tile * 8 + threadIdx.x] = sm[threadIdx.x];
+    __threadfence();
+  }
+}
+
+template <int NC>
+__device__ void scan_finish(const Tables& T, uint32_t ntiles, const int (&slots)[NC], const long long (&mul)[NC]) {
+  __shared__ int s_last2;
+  __shared__ unsigned long long s_sum[NC];
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    unsigned int d = atomicAdd(&T.ctl->scan_done, 1u);
+    s_last2 = (d == ntiles - 1);
+  }
+  if (threadIdx.x < NC) s_sum[threadIdx.x] = 0;
+  __syncthreads();
+  if (s_last2) {
+    __threadfence();
+    for (int k = 0; k < NC; ++k) {
+      unsigned long long acc = 0;
+      for (uint32_t t = threadIdx.x; t < ntiles; t += blockDim.x) acc += ((volatile uint32_t*)T.tile_cnt)[t * 8 + k];
+      for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
+      if ((threadIdx.x & 31) == 0 && acc) atomicAdd(&s_sum[k], acc);
+    }
+    for (uint32_t i = threadIdx.x; i < ntiles; i += blockDim.x) T.tile_status[i] = 0ull;
+    __syncthreads();
+    if (threadIdx.x < NC && slots[threadIdx.x] >= 0) stat_add(T, slots[threadIdx.x], (long long)s_sum[threadIdx.x] * mul[threadIdx.x]);
+    if (threadIdx.x == 0) {
+      T.ctl->scan_done = 0;
+      T.ctl->scan_ticket = 0;
+    }
+    __threadfence();
+  }
+}
+
 // ------------------------------------------------------------------------------------
 // init / poison
 // ------------------------------------------------------------------------------------
@@ -261,30 +311,30 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
       }
     }
   }
-  // counters
-  {
-    const long long B = T.B;
-    // classes: U H HD G GE GL
-    uint32_t c6[6] = {cls[0], cls[1], cls[2], cls[3], cls[4], cls[5]};
-    if (touch) {
-      // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE ; h2d: H ; zf: U+HD ; h2d_av: HD
-      uint32_t v[6] = {c6[0] + c6[1] + c6[2] + c6[4], c6[3] + c6[5], c6[4], c6[1], c6[0] + c6[2], c6[2]};
-      const int slots[6] = {S_FAULTS, S_HITS, S_REMAPS, S_H2D, S_ZF, S_H2D_AV};
-      const long long mul[6] = {1, 1, 1, B, B, B};
-      block_counts_to<6>(T, v, s_cnt, slots, mul);
-    } else {
-      uint32_t v[6] = {c6[3], c6[4], c6[5], c6[1], c6[0] + c6[2], c6[2]};
-      const int slots[6] = {S_REFRESH, S_REMAPS, S_REVAL, S_H2D, S_ZF, S_H2D_AV};
-      const long long mul[6] = {1, 1, 1, B, B, B};
-      block_counts_to<6>(T, v, s_cnt, slots, mul);
-    }
+  // counters (classes: U H HD G GE GL)
+  const long long B = T.B;
+  if (touch) {
+    // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE ; h2d: H ; zf: U+HD ; h2d_av: HD
+    uint32_t v[6] = {cls[0] + cls[1] + cls[2] + cls[4], cls[3] + cls[5], cls[4], cls[1], cls[0] + cls[2], cls[2]};
+    tile_counts<6>(T, tile, v, s_cnt);
+  } else {
+    uint32_t v[6] = {cls[3], cls[4], cls[5], cls[1], cls[0] + cls[2], cls[2]};
+    tile_counts<6>(T, tile, v, s_cnt);
   }
   if (tile == ntiles - 1 && threadIdx.x == 0) {
     unsigned long long all = s_excl + tot;
     T.ctl->n_need = unpackA(all);
     T.ctl->n_rekey = unpackB(all);
   }
-  scan_finish(T, ntiles);
+  if (touch) {
+    const int slots[6] = {S_FAULTS, S_HITS, S_REMAPS, S_H2D, S_ZF, S_H2D_AV};
+    const long long mul[6] = {1, 1, 1, B, B, B};
+    scan_finish<6>(T, ntiles, slots, mul);
+  } else {
+    const int slots[6] = {S_REFRESH, S_REMAPS, S_REVAL, S_H2D, S_ZF, S_H2D_AV};
+    const long long mul[6] = {1, 1, 1, B, B, B};
+    scan_finish<6>(T, ntiles, slots, mul);
+  }
 }
 
 // ------------------------------------------------------------------------------------
@@ -483,11 +533,61 @@ __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.comm
 __device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
+// The plan of need item i of the current sub-op (K6 decides it from K3's output):
+// destination frame (free stack first, then victim frames in victim order), the
+// victim's write-back destination, the newcomer's source host frame, zero-fill, and
+// whether the newcomer's host frame was handed to the victim (fused swap, R5).
+__device__ __forceinline__ XItem item_plan(const Tables& T, uint32_t i, uint32_t f0, uint32_t nfu) {
+  XItem x;
+  const uint8_t kd = T.needk[i];
+  const uint32_t hf = T.needhf[i];
+  x.flags = 0;
+  x.dst_hf = UM_NONE;
+  if (i < nfu) {
+    x.fr = T.free_stack[f0 - 1 - i];
+  } else {
+    const uint32_t j = i - f0;
+    x.fr = T.vframe[j];
+    if (T.vkind[j] == ST_G && T.vhf[j] != UM_NONE) {
+      x.dst_hf = T.vhf[j];
+      x.flags |= XI_D2H;
+      if (x.dst_hf == hf) x.flags |= XI_SWAP;
+    }
+  }
+  if (kd == ST_H) {
+    x.src_hf = hf != UM_NONE ? hf : T.zero_hf;
+    x.flags |= XI_H2D;
+  } else {
+    x.src_hf = UM_NONE;
+    x.flags |= XI_ZF;
+  }
+  return x;
+}
+
+// K6 commit of need item i: the block becomes G in its frame; a host frame it leaves
+// is recycled unless it was handed to the victim.
+__device__ __forceinline__ void item_commit(const Tables& T, uint32_t i, const XItem& x, uint32_t seq) {
+  const uint32_t bb = T.need[i];
+  T.st[bb] = ST_G;
+  T.key[bb] = seq;
+  T.frame_of[bb] = x.fr;
+  T.map[bb] = x.fr;
+  const uint32_t hf = T.needhf[i];
+  if (T.needk[i] == ST_H && hf != UM_NONE) {
+    T.hframe[bb] = UM_NONE;
+    if (!(x.flags & XI_SWAP)) {
+      int idx = atomicAdd(&T.ctl->hfree_top, 1);
+      T.hfree_stack[idx] = hf;
+    }
+  }
+}
+
 struct Unit {
   char* frame;        // frame chunk (HBM)
   char* d2h_dst;      // host chunk receiving the old content, or null
   const char* h2d_src;// host chunk with the new content, or null
   bool zf;            // zero-fill the frame chunk
+  __device__ bool pure_zf() const { return zf && !d2h_dst; }
 };
 
 __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t seq) {
@@ -506,55 +606,33 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
     const uint32_t n_items = mode == SVC_SUBOP ? c->n_need : c->n_d2h;
     const uint32_t f0 = c->f0;
     const uint32_t nfu = min(f0, n_items);
+    // each CTA takes a contiguous range of units, so consecutive units mostly share an
+    // item and its plan is looked up once (the lookups are dependent global loads)
     const unsigned long long units = (unsigned long long)n_items * cpb;
-    const unsigned long long mine =
-        units > blockIdx.x ? (units - blockIdx.x + gridDim.x - 1) / gridDim.x : 0ull;
+    const unsigned long long ubeg = units * blockIdx.x / gridDim.x;
+    const unsigned long long mine = units * (blockIdx.x + 1) / gridDim.x - ubeg;
     for (int s = 0; s < kXferStages; ++s) mbar_init(&bar[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 
-    auto make = [&](unsigned long long t) -> Unit {
-      unsigned long long u = blockIdx.x + t * gridDim.x;
+    uint32_t cached_i = UM_NONE;
+    XItem cached;
+    // phase 1 commits pure zero-fill items, phase 2 all others (each exactly once)
+    auto make = [&](unsigned long long t, int phase) -> Unit {
+      unsigned long long u = ubeg + t;
       uint32_t i = (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
       size_t coff = (size_t)ch * CH;
       Unit x;
       if (mode == SVC_SUBOP) {
-        uint32_t bb = T.need[i];
-        uint8_t kd = T.needk[i];
-        uint32_t hf = T.needhf[i];
-        uint32_t fr;
-        bool swapped = false;
-        x.d2h_dst = nullptr;
-        if (i < nfu) {
-          fr = T.free_stack[f0 - 1 - i];
-        } else {
-          uint32_t j = i - f0;
-          fr = T.vframe[j];
-          if (T.vkind[j] == ST_G && T.vhf[j] != UM_NONE) {
-            x.d2h_dst = hptr(T, T.vhf[j]) + coff;
-            swapped = T.vhf[j] == hf;   // host frame handed over to the victim
-          }
+        if (i != cached_i) {
+          cached = item_plan(T, i, f0, nfu);
+          cached_i = i;
         }
-        x.frame = T.frames + (size_t)fr * T.B + coff;
-        if (kd == ST_H) {
-          x.h2d_src = hptr(T, hf != UM_NONE ? hf : T.zero_hf) + coff;
-          x.zf = false;
-        } else {
-          x.h2d_src = nullptr;
-          x.zf = true;
-        }
-        if (ch == 0) {  // K6 commit of the newly resident block
-          T.st[bb] = ST_G;
-          T.key[bb] = seq;
-          T.frame_of[bb] = fr;
-          T.map[bb] = fr;
-          if (kd == ST_H && hf != UM_NONE) {
-            T.hframe[bb] = UM_NONE;
-            if (!swapped) {
-              int idx = atomicAdd(&c->hfree_top, 1);
-              T.hfree_stack[idx] = hf;
-            }
-          }
-        }
+        const XItem& p = cached;
+        x.frame = T.frames + (size_t)p.fr * T.B + coff;
+        x.d2h_dst = (p.flags & XI_D2H) ? hptr(T, p.dst_hf) + coff : nullptr;
+        x.h2d_src = (p.flags & XI_H2D) ? hptr(T, p.src_hf) + coff : nullptr;
+        x.zf = (p.flags & XI_ZF) != 0;
+        if (ch == 0 && (x.pure_zf() ? 1 : 2) == phase) item_commit(T, i, p, seq);
       } else {
         uint32_t fr = T.d2h_frame[i], hf = T.d2h_hf[i];
         x.frame = T.frames + (size_t)fr * T.B + coff;
@@ -564,6 +642,26 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
       }
       return x;
     };
+    // Phase 1: zero-fill units need no load: bulk-store the zeroed tile right away.
+    if (mode == SVC_SUBOP) {
+      uint32_t issued = 0;
+      for (unsigned long long t = 0; t < mine; ++t) {
+        Unit x = make(t, 1);
+        if (!x.pure_zf()) continue;
+        bulk_s2g(x.frame, zero, CH);
+        if ((++issued & 31) == 0) bulk_commit();
+      }
+      bulk_commit();
+    }
+    // Phase 2: transfer units through the S-stage TMA ring.
+    unsigned long long tn = 0;
+    auto next_xfer = [&](Unit& x) -> bool {
+      while (tn < mine) {
+        x = make(tn++, 2);
+        if (!x.pure_zf()) return true;
+      }
+      return false;
+    };
     Unit U[kXferStages];
     auto issue_loads = [&](int s, const Unit& x) {
       uint32_t bytes = (x.d2h_dst ? CH : 0u) + (x.h2d_src ? CH : 0u);
@@ -571,23 +669,29 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
       if (x.d2h_dst) bulk_g2s(stA + s * CH, x.frame, CH, &bar[s]);
       if (x.h2d_src) bulk_g2s(stB + s * CH, x.h2d_src, CH, &bar[s]);
     };
-    for (unsigned long long t = 0; t < mine && t < (unsigned long long)kXferStages; ++t) {
-      U[t] = make(t);
-      issue_loads((int)t, U[t]);
+    unsigned long long loaded = 0;
+    for (int s = 0; s < kXferStages; ++s) {
+      if (!next_xfer(U[s])) break;
+      issue_loads(s, U[s]);
+      ++loaded;
     }
-    for (unsigned long long t = 0; t < mine; ++t) {
-      const int s = (int)(t % kXferStages);
-      mbar_wait(&bar[s], (uint32_t)((t / kXferStages) & 1));
+    for (unsigned long long k = 0; k < loaded; ++k) {
+      const int s = (int)(k % kXferStages);
+      mbar_wait(&bar[s], (uint32_t)((k / kXferStages) & 1));
       const Unit& x = U[s];
       if (x.d2h_dst) bulk_s2g(x.d2h_dst, stA + s * CH, CH);
       if (x.h2d_src) bulk_s2g(x.frame, stB + s * CH, CH);
       else if (x.zf) bulk_s2g(x.frame, zero, CH);
       bulk_commit();
-      if (t >= 1 && t - 1 + kXferStages < mine) {
-        bulk_wait_read1();
-        const int sp = (int)((t - 1) % kXferStages);
-        U[sp] = make(t - 1 + kXferStages);
-        issue_loads(sp, U[sp]);
+      if (k >= 1 && loaded == k - 1 + kXferStages) {
+        const int sp = (int)((k - 1) % kXferStages);
+        Unit y;
+        if (next_xfer(y)) {
+          bulk_wait_read1();
+          U[sp] = y;
+          issue_loads(sp, U[sp]);
+          ++loaded;
+        }
       }
     }
     bulk_wait_all();
@@ -603,26 +707,80 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
 }
 
 // ------------------------------------------------------------------------------------
+// K4-CE support: K6 plans + commits every need item on the device and exports the plan
+// (XItem records) for the host to turn into copy-engine batches; zero-fill of the
+// items that need it runs as a kernel on the copy streams.
+// ------------------------------------------------------------------------------------
+__global__ void k_plan_commit(Tables T, uint32_t seq) {
+  const uint32_t n = T.ctl->n_need, f0 = T.ctl->f0, nfu = min(f0, n);
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    XItem x = item_plan(T, i, f0, nfu);
+    T.xitems[i] = x;
+    item_commit(T, i, x, seq);
+  }
+}
+
+// HBM fills are done in segments of kFillSeg bytes: the segment's metadata is looked up
+// once (thread 0 -> smem) and 256 threads then stream 16-byte stores, 8 per thread in
+// flight, so the per-segment lookup latency is amortised over 256 KiB of writes.
+constexpr uint32_t kFillSeg = 256u << 10;
+
+__device__ __forceinline__ void fill_segment(uint4* dst, uint32_t n16, uint4 v) {
+  uint32_t t = threadIdx.x;
+  for (; t + 7 * 256 < n16; t += 8 * 256) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) dst[t + k * 256] = v;
+  }
+  for (; t < n16; t += 256) dst[t] = v;
+}
+
+__global__ void __launch_bounds__(256) k_zero_items(Tables T, uint32_t i0, uint32_t i1) {
+  __shared__ char* s_dst;
+  const uint32_t SEG = T.B < kFillSeg ? T.B : kFillSeg;
+  const uint32_t spb = T.B / SEG;
+  const unsigned long long units = (unsigned long long)(i1 - i0) * spb;
+  for (unsigned long long u = blockIdx.x; u < units; u += gridDim.x) {
+    if (threadIdx.x == 0) {
+      const XItem x = T.xitems[i0 + (uint32_t)(u / spb)];
+      s_dst = (x.flags & XI_ZF) ? T.frames + (size_t)x.fr * T.B + (size_t)(u % spb) * SEG : nullptr;
+    }
+    __syncthreads();
+    char* d = s_dst;
+    __syncthreads();
+    if (d) fill_segment(reinterpret_cast<uint4*>(d), SEG / 16, make_uint4(0, 0, 0, 0));
+  }
+}
+
+// ------------------------------------------------------------------------------------
 // Harness "application kernel": after a touch sub-op is serviced, every block with a
 // UM_ACC_WRITE access receives the content stamp s = (seq << 32) | block as the
 // 16-byte pattern {s, ~s}, written through its frame (G or GL blocks are mapped).
 // ------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq) {
-  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
-  const uint32_t cpb = T.B / CH;
-  const unsigned long long units = (unsigned long long)n * cpb;
+  __shared__ char* s_dst;
+  __shared__ uint32_t s_blk;
+  const uint32_t SEG = T.B < kFillSeg ? T.B : kFillSeg;
+  const uint32_t spb = T.B / SEG;
+  const unsigned long long units = (unsigned long long)n * spb;
   for (unsigned long long u = blockIdx.x; u < units; u += gridDim.x) {
-    uint32_t i = (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
-    uint32_t g = g0 + i;
-    uint32_t j = iv_find(iv, g);
-    if (!iv.wflag[j]) continue;
-    uint32_t bb = iv.lo[j] + (g - iv.pre[j]);
-    uint32_t fr = T.frame_of[bb];
-    if (fr == UM_NONE) continue;
-    unsigned long long sv = ((unsigned long long)seq << 32) | bb;
-    uint4 pat = make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32));
-    uint4* dst = reinterpret_cast<uint4*>(T.frames + (size_t)fr * T.B + (size_t)ch * CH);
-    for (uint32_t t = threadIdx.x; t < CH / 16; t += blockDim.x) dst[t] = pat;
+    if (threadIdx.x == 0) {
+      uint32_t g = g0 + (uint32_t)(u / spb);
+      uint32_t j = iv_find(iv, g);
+      char* d = nullptr;
+      uint32_t bb = iv.lo[j] + (g - iv.pre[j]);
+      if (iv.wflag[j]) {
+        uint32_t fr = T.frame_of[bb];
+        if (fr != UM_NONE) d = T.frames + (size_t)fr * T.B + (size_t)(u % spb) * SEG;
+      }
+      s_dst = d;
+      s_blk = bb;
+    }
+    __syncthreads();
+    char* d = s_dst;
+    const unsigned long long sv = ((unsigned long long)seq << 32) | s_blk;
+    __syncthreads();
+    if (d) fill_segment(reinterpret_cast<uint4*>(d), SEG / 16,
+                        make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32)));
   }
 }
 
@@ -723,12 +881,12 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
   }
   {
     uint32_t v[3] = {nUnmap, nD2H, nAv};
-    const int slots[3] = {S_UNMAPS, S_D2H, S_D2H_AV};
-    const long long mul[3] = {1, (long long)T.B, (long long)T.B};
-    block_counts_to<3>(T, v, s_cnt, slots, mul);
+    tile_counts<3>(T, tile, v, s_cnt);
   }
   if (tile == ntiles - 1 && threadIdx.x == 0) T.ctl->disc_tail = tail0 + unpackA(s_excl + tot);
-  scan_finish(T, ntiles);
+  const int slots[3] = {S_UNMAPS, S_D2H, S_D2H_AV};
+  const long long mul[3] = {1, (long long)T.B, (long long)T.B};
+  scan_finish<3>(T, ntiles, slots, mul);
 }
 
 // ------------------------------------------------------------------------------------
@@ -906,8 +1064,8 @@ cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max
 }
 
 cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, cudaStream_t s) {
-  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
-  unsigned long long units = (unsigned long long)n * (T.B / CH);
+  const uint32_t SEG = T.B < kFillSeg ? T.B : kFillSeg;
+  unsigned long long units = (unsigned long long)n * (T.B / SEG);
   unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
   if (!grid) return cudaSuccess;
   k_app_stamp<<<grid, 256, 0, s>>>(T, iv, g0, n, seq);
@@ -934,6 +1092,21 @@ cudaError_t launch_host_write(const Tables& T, uint32_t lo, uint32_t n, uint32_t
   unsigned long long units = (unsigned long long)n * (T.B / CH);
   unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
   k_hw_fill<<<grid, 256, 0, s>>>(T, lo, n, seq);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_plan_commit(const Tables& T, uint32_t seq, uint32_t max_items, cudaStream_t s) {
+  unsigned grid = ceil_div(max_items ? max_items : 1, 256);
+  k_plan_commit<<<grid, 256, 0, s>>>(T, seq);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_zero_items(const Tables& T, uint32_t i0, uint32_t i1, cudaStream_t s) {
+  const uint32_t SEG = T.B < kFillSeg ? T.B : kFillSeg;
+  unsigned long long units = (unsigned long long)(i1 - i0) * (T.B / SEG);
+  unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
+  if (!grid) return cudaSuccess;
+  k_zero_items<<<grid, 256, 0, s>>>(T, i0, i1);
   return cudaGetLastError();
 }
 

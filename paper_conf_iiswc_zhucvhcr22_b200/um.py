@@ -20,7 +20,7 @@ UM_DST_GPU, UM_DST_HOST = 0, 1
 UM_ACC_READ, UM_ACC_WRITE = 1, 2
 UM_ST_U, UM_ST_H, UM_ST_HD, UM_ST_G, UM_ST_GE, UM_ST_GL = range(6)
 ST_NAMES = ("U", "H", "HD", "G", "GE", "GL")
-UM_F_DISCARD_OFF, UM_F_COPY_CE, UM_F_CHECK, UM_F_APP_STAMP, UM_F_TIMING = 1, 2, 4, 8, 16
+UM_F_DISCARD_OFF, UM_F_COPY_CE, UM_F_CHECK, UM_F_APP_STAMP, UM_F_TIMING, UM_F_COPY_KERNEL = 1, 2, 4, 8, 16, 32
 UM_NONE = 0xFFFFFFFF
 
 

@@ -22,9 +22,13 @@ def _cuda():
     build.build()
 
 
-def _gpu(trace, mode, **kw):
-    from paper_conf_iiswc_zhucvhcr22_b200 import harness
-    return harness.run_trace(trace, mode, **kw)
+COPY_FLAGS = {"auto": 0, "kernel": 32, "ce": 2}   # UM_F_COPY_KERNEL / UM_F_COPY_CE
+
+
+def _gpu(trace, mode, copy="auto", **kw):
+    from paper_conf_iiswc_zhucvhcr22_b200 import harness, um
+    flags = um.UM_F_APP_STAMP | um.UM_F_CHECK | COPY_FLAGS[copy]
+    return harness.run_trace(trace, mode, flags=flags, **kw)
 
 
 def assert_parity(trace, mode, g=None):
@@ -72,12 +76,20 @@ def test_c1(seed, mode):
 
 
 @pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_c1_copy_engine_path(mode):
+    """The same C1 trace with every transfer through K4-CE (device plan, copy engines)."""
+    t = tg.gen_c1(3).slice_ops(0, 4000)
+    assert_parity(t, mode, _gpu(t, mode, copy="ce"))
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
 def test_c2_ci(mode):
     """C2 streaming at CI size: F = 2048 frames of 2 MiB (4 GiB), buffer 8 GiB, c = 512, P = 2;
     also pins the closed form."""
     F, c, P, B = 2048, 512, 2, 2 << 20
     t = tg.gen_c2(F, c, P, block_bytes=B)
     g, _ = assert_parity(t, mode)
+    assert_parity(t, mode, _gpu(t, mode, copy="kernel"))
     s = g["stats"]
     if mode == "base":
         assert (s["h2d_bytes"], s["d2h_bytes"], s["zf_bytes"]) == (2 * (P - 1) * F * B, (2 * P - 1) * F * B, 2 * F * B)
@@ -91,7 +103,8 @@ def test_c3_small(mode):
     t = tg.gen_c3(block_bytes=64 << 10, budget_bytes=192 << 20, iterations=2, workspace_bytes=4 << 20,
                   layers=tg.scale_layers(tg.VGG16, 1.0 / 512, 1.0 / 64), batch=8)
     assert t.arena_bytes > t.budget_bytes
-    assert_parity(t, mode)
+    for copy in ("auto", "kernel", "ce"):
+        assert_parity(t, mode, _gpu(t, mode, copy=copy))
 
 
 def test_split_large_op():
@@ -107,7 +120,8 @@ def test_split_large_op():
     tb.prefetch(0, 3000 * B, tg.DST_HOST)
     t = tb.build()
     for mode in ("base", "eager", "lazy"):
-        assert_parity(t, mode)
+        for copy in ("kernel", "ce"):
+            assert_parity(t, mode, _gpu(t, mode, copy=copy))
 
 
 def test_edge_cases_and_errors():
@@ -181,5 +195,5 @@ def test_c3_small_tight_host_pool(mode):
     t = tg.gen_c3(block_bytes=64 << 10, budget_bytes=192 << 20, iterations=2, workspace_bytes=4 << 20,
                   layers=tg.scale_layers(tg.VGG16, 1.0 / 512, 1.0 / 64), batch=8)
     pool = t.arena_bytes - t.budget_bytes + 2 * t.block_bytes
-    g = _gpu(t, mode, host_pool_bytes=pool)
-    assert_parity(t, mode, g)
+    for copy in ("kernel", "ce"):
+        assert_parity(t, mode, _gpu(t, mode, copy=copy, host_pool_bytes=pool))
