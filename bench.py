@@ -52,6 +52,16 @@ def parse():
 
 
 # ------------------------------------------------------------------------------ env
+def _mem_available():
+    try:
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemAvailable:"):
+                return int(line.split()[1]) * 1024
+    except OSError:
+        pass
+    return None
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     return int(os.environ.get("RANK", "0")), int(os.environ.get("LOCAL_RANK", "0")), ws
@@ -237,6 +247,31 @@ def discard_bench(torch, um, reps=20):
     return out
 
 
+def c1_rate(torch, um, harness):
+    """C1 tiny trace (BASELINE.json configs[0]; 10k ops, 64 KiB blocks): ops/s through
+    the public API (host wall clock, synchronised at the end) — the small-op,
+    launch-latency regime.  Planning and transfers stay on the device (kernel path)."""
+    import tracegen as tg
+    t = tg.gen_c1(0)
+    arena = harness.make_arena(t, "eager", flags=um.UM_F_APP_STAMP)
+    try:
+        harness.issue(arena, t, "eager", 0, 500)            # warm-up
+        um.um_get_stats(arena.handle)
+        ps = torch.cuda.ExternalStream(arena.stream_ptr)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        w0 = time.perf_counter()
+        e0.record(ps)
+        harness.issue(arena, t, "eager", 500, len(t))
+        e1.record(ps)
+        e1.synchronize()
+        wall = time.perf_counter() - w0
+        n = len(t) - 500
+        return {"ops": n, "ops_per_s": n / wall, "us_per_op_wall": wall / n * 1e6,
+                "us_per_op_device": e0.elapsed_time(e1) * 1e3 / n}
+    finally:
+        arena.close()
+
+
 def state_bench(torch, um, mem, budget, arena_bytes, seed=0):
     """State-kernel microbench (SURVEY §8(d) last row): C3-64K-sized tables (64 KiB blocks
     over the same 170 GiB of frames / 255 GiB arena), one touch_batch of 2^21 distinct
@@ -353,11 +388,19 @@ def main_ours(args):
 
     link = measure_link_peak(torch, dev)
     disc = None if args.no_discard_bench else discard_bench(torch, um)
+    c1 = None if args.no_discard_bench else c1_rate(torch, um, harness)
 
     torch.cuda.empty_cache()
     free, total = torch.cuda.mem_get_info(dev)
     B = args.block
     budget = min(int(args.budget_gib * GiB), free - 5 * GiB) // B * B
+    # host RAM guard: every local rank pins a pool of (arena - budget) + 2 GiB
+    lws = int(os.environ.get("LOCAL_WORLD_SIZE", str(ws)))
+    avail = _mem_available()
+    if avail:
+        fit = int((0.85 * avail / lws - 2 * GiB) / max(args.oversub - 1.0, 1e-9))
+        if fit < budget:
+            budget = max(B, fit // B * B)
     arena_bytes = int(budget * args.oversub) // B * B
     host_pool = arena_bytes - budget + 2 * GiB
     trace = build_trace(args, budget, True, W + K)
@@ -409,7 +452,7 @@ def main_ours(args):
         "config": {"workload": "C3 DNN activation trace, 1.5x oversubscription", "block_bytes": B_,
                    "budget_bytes": budget, "arena_bytes": arena_bytes, "batch": trace.meta["batch"],
                    "layers": trace.meta["layers"], "ops_per_iter": trace.meta["ops_per_iter"],
-                   "host_pool_bytes": host_pool, "parallelism": f"independent arenas x{ws}",
+                   "host_pool_bytes": host_pool, "budget_requested_bytes": int(args.budget_gib * GiB), "parallelism": f"independent arenas x{ws}",
                    "l2": "working set 255 GiB >> 126 MB L2 (no flush needed)",
                    "headline_mode": "eager (UvmDiscard)"},
         "iter_ms": {m: r["iter_ms"] for m, r in res.items()},
@@ -433,6 +476,7 @@ def main_ours(args):
         "link_peak": link,
         "transfer_paths": _paths(res.get("eager"), k4, link),
         "roofline_state": state,
+        "c1_directives": c1,
         "clocks": head["clocks"],
         "gpu_launches": tm["launches"],
         "stats_per_iter_all_ranks": stats_all,

@@ -197,3 +197,13 @@ def test_c3_small_tight_host_pool(mode):
     pool = t.arena_bytes - t.budget_bytes + 2 * t.block_bytes
     for copy in ("kernel", "ce"):
         assert_parity(t, mode, _gpu(t, mode, copy=copy, host_pool_bytes=pool))
+
+
+@pytest.mark.parametrize("ov", [0.8, 2, 4])
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_next3_radix_hashjoin(ov, mode):
+    MiB = 1 << 20
+    B = 64 * 1024
+    for t in (tg.gen_radix(block_bytes=B, budget_bytes=int(64 * MiB / ov) // B * B, data_bytes=32 * MiB),
+              tg.gen_hashjoin(block_bytes=B, budget_bytes=int(72 * MiB / ov) // B * B, table_bytes=8 * MiB)):
+        assert_parity(t, mode)

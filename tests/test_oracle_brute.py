@@ -495,3 +495,25 @@ def test_host_release_changes_only_discarded_contents():
             for x in range(t.nblocks):
                 if not dc[x]:
                     assert a["contents"][x] == b["contents"][x]
+
+
+@pytest.mark.parametrize("ov", [0.8, 2, 3, 4])
+def test_next3_radix_hashjoin_invariants(ov):
+    """NEXT-3 workloads (radix sort §7.3, hash join §7.4): lazy_ok discards are valid;
+    eager and lazy move identical bytes (vi); without pressure discard changes no
+    transfer (v; the equal <100 % columns of Tables 6 and 8); under pressure discard
+    never increases H2D+D2H."""
+    MiB = 1 << 20
+    B = 64 * 1024
+    traces = [tg.gen_radix(block_bytes=B, budget_bytes=int(64 * MiB / ov) // B * B, data_bytes=32 * MiB),
+              tg.gen_hashjoin(block_bytes=B, budget_bytes=int(72 * MiB / ov) // B * B, table_bytes=8 * MiB)]
+    for t in traces:
+        assert tg.check_lazy_ok(t) == []
+        s = {m: replay(t, m).stats for m in ("base", "eager", "lazy")}
+        for k in ("h2d_bytes", "d2h_bytes", "zf_bytes"):
+            assert s["eager"][k] == s["lazy"][k]
+        mv = {m: s[m]["h2d_bytes"] + s[m]["d2h_bytes"] for m in s}
+        if ov < 1:
+            assert mv["eager"] == mv["base"]
+        else:
+            assert mv["eager"] <= mv["base"]
