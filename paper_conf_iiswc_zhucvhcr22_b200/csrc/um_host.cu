@@ -520,7 +520,10 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     if (st) return st;
     cudaEvent_t sp = span_open(a);
     CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
-    CK(launch_victims(a->T, seq, 0, 0, a->ps));
+    if (n > kVictWideMin)
+      CK(launch_victims_wide(a->T, seq, 0, 0, a->ub[RING_DISC] + a->ub[RING_USED], n, a->ps));
+    else
+      CK(launch_victims(a->T, seq, 0, 0, a->ps));
     span_close(a, sp, 0);
     if (use_ce(a, n)) {
       sp = span_open(a);
@@ -787,7 +790,10 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
   if (want > a->nframes) want = a->nframes;
   if (want) {
     cudaEvent_t sp = span_open(a);
-    CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->ps));
+    if (want > kVictWideMin)
+      CK(launch_victims_wide(a->T, seq, 1, (uint32_t)want, a->ub[RING_DISC] + a->ub[RING_USED], (uint32_t)want, a->ps));
+    else
+      CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->ps));
     span_close(a, sp, 0);
     sp = span_open(a);
     if (use_ce(a, want)) {

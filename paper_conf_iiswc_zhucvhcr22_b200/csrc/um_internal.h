@@ -30,8 +30,11 @@ struct Ctl {
   unsigned int n_d2h;    // D2H-only work-list length (prefetch HOST / evict)
   unsigned int err;      // sticky device error (0 or -um_status)
   unsigned int scan_ticket, scan_done;  // decoupled look-back tile ticket / completion
-  unsigned int app_units;               // unused scratch
-  unsigned int pad[3];
+  unsigned int app_units;               // D2H-only service completion counter
+  unsigned int vict_done;               // wide victim apply completion counter
+  unsigned int pad[2];
+  unsigned long long minkeep[2];        // wide victim scan: first kept ring position
+  unsigned int k_want;                  // wide victim scan: victims wanted
   long long stats[S_N];
 };
 
@@ -89,8 +92,8 @@ struct OpIv {
   uint32_t m;
 };
 
-constexpr int kScanTPB = 256;
-constexpr int kScanIPT = 4;
+constexpr int kScanTPB = 512;
+constexpr int kScanIPT = 8;
 constexpr int kScanTile = kScanTPB * kScanIPT;
 constexpr int kVictTPB = 1024;
 constexpr int kVictIPT = 4;
@@ -107,6 +110,10 @@ cudaError_t launch_init(const Tables& T, int nhframes_alloc, cudaStream_t s);
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
                             cudaStream_t s);
 cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, cudaStream_t s);
+// multi-CTA victim selection for large sub-ops (scan bound = max ring entries to scan)
+cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, uint32_t want,
+                                uint64_t scan_bound, uint32_t max_victims, cudaStream_t s);
+constexpr uint32_t kVictWideMin = 8192;
 cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max_items, cudaStream_t s);
 cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, cudaStream_t s);
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq,

@@ -96,6 +96,42 @@ __device__ unsigned long long lookback(const Tables& T, uint32_t tile, unsigned 
   return excl;
 }
 
+// Warp-parallel decoupled look-back (called by all 32 lanes of warp 0): each round
+// inspects 32 predecessors at once; the closest one holding an inclusive prefix ends the
+// walk.  Returns the tile's exclusive prefix.
+__device__ unsigned long long lookback_warp(const Tables& T, uint32_t tile, unsigned long long agg) {
+  volatile unsigned long long* st = T.tile_status;
+  const unsigned long long FA = 1ull << 62, FP = 2ull << 62, M = FA - 1;
+  const int lane = threadIdx.x & 31;
+  if (tile == 0) {
+    if (lane == 0) st[0] = FP | agg;
+    __threadfence();
+    return 0ull;
+  }
+  if (lane == 0) st[tile] = FA | agg;
+  __threadfence();
+  unsigned long long excl = 0;
+  long long p = (long long)tile - 1;
+  while (true) {
+    const long long idx = p - lane;
+    unsigned long long v = FP;  // before tile 0: an inclusive prefix of 0
+    if (idx >= 0) {
+      do { v = st[idx]; } while ((v >> 62) == 0);
+    }
+    const unsigned pm = __ballot_sync(FULL, (v >> 62) == 2);
+    const int stop = pm ? __ffs(pm) - 1 : 31;
+    unsigned long long x = lane <= stop ? (v & M) : 0ull;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(FULL, x, o);
+    excl += x;
+    if (pm) break;
+    p -= 32;
+  }
+  if (lane == 0) st[tile] = FP | (excl + agg);
+  __threadfence();
+  return excl;
+}
+
 // Called by every thread at the end of a scanning CTA: the last CTA to finish clears
 // the tile statuses and the ticket, so the next scanning launch starts clean.
 __device__ void scan_finish(const Tables& T, uint32_t ntiles) {
@@ -217,7 +253,9 @@ __global__ void k_init(Tables T, int nh) {
     c->free_top = (int)T.nframes;
     c->hfree_top = nh;
     c->n_need = c->n_rekey = c->f0 = c->n_vict = c->n_d2h = c->err = 0;
-    c->scan_ticket = c->scan_done = c->app_units = 0;
+    c->scan_ticket = c->scan_done = c->app_units = c->vict_done = 0;
+    c->minkeep[0] = c->minkeep[1] = ~0ull;
+    c->k_want = 0;
     for (int i = 0; i < S_N; ++i) c->stats[i] = 0;
   }
 }
@@ -243,10 +281,31 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
   __shared__ unsigned long long s_excl;
   __shared__ unsigned long long s_tail0;
   __shared__ uint32_t s_cnt[6];
+  // the tile's slice of the interval list (<= kScanTile intervals), staged in smem so
+  // each thread's interval search runs in shared memory
+  __shared__ uint32_t s_lo[kScanTile], s_pre[kScanTile + 1];
+  __shared__ uint32_t s_j0, s_m;
   if (threadIdx.x == 0) s_tail0 = T.ctl->used_tail;
   const uint32_t tile = take_ticket(T);
   const uint32_t ntiles = n ? (n + kScanTile - 1) / kScanTile : 1;
-  const uint32_t first = tile * kScanTile + threadIdx.x * kScanIPT;
+  const uint32_t tbase = tile * kScanTile;
+  const uint32_t first = tbase + threadIdx.x * kScanIPT;
+  if (threadIdx.x == 0 && tbase < n) {
+    const uint32_t ja = iv_find(iv, g0 + tbase);
+    const uint32_t jb = iv_find(iv, g0 + min(n, tbase + kScanTile) - 1);
+    s_j0 = ja;
+    s_m = jb - ja + 1;
+  }
+  __syncthreads();
+  if (tbase < n) {
+    const uint32_t j0 = s_j0, m = s_m;
+    for (uint32_t q = threadIdx.x; q < m; q += blockDim.x) {
+      s_lo[q] = iv.lo[j0 + q];
+      s_pre[q] = iv.pre[j0 + q];
+    }
+    if (threadIdx.x == 0) s_pre[m] = iv.pre[j0 + m];
+  }
+  __syncthreads();
 
   uint32_t b[kScanIPT];
   uint8_t s[kScanIPT];
@@ -254,14 +313,22 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
   uint32_t cls[6] = {0, 0, 0, 0, 0, 0};
   unsigned needm = 0, rekm = 0;
   if (first < n) {
-    uint32_t j = iv_find(iv, g0 + first);
+    uint32_t lo = 0, hi = s_m;  // largest j with s_pre[j] <= g
+    {
+      const uint32_t g = g0 + first;
+      while (hi - lo > 1) {
+        uint32_t mid = (lo + hi) >> 1;
+        if (s_pre[mid] <= g) lo = mid; else hi = mid;
+      }
+    }
+    uint32_t j = lo;
 #pragma unroll
     for (int k = 0; k < kScanIPT; ++k) {
       uint32_t idx = first + k;
       if (idx < n) {
         uint32_t g = g0 + idx;
-        while (g >= iv.pre[j + 1]) ++j;
-        uint32_t bb = iv.lo[j] + (g - iv.pre[j]);
+        while (g >= s_pre[j + 1]) ++j;
+        uint32_t bb = s_lo[j] + (g - s_pre[j]);
         uint8_t ss = T.st[bb];
         T.pin[bb] = seq;
         b[k] = bb;
@@ -278,7 +345,10 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
   }
   unsigned long long tot;
   unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cN, cR), tot, s_scan);
-  if (threadIdx.x == 0) s_excl = lookback(T, tile, tot);
+  if (threadIdx.x < 32) {
+    unsigned long long e = lookback_warp(T, tile, tot);
+    if (threadIdx.x == 0) s_excl = e;
+  }
   __syncthreads();
   const unsigned long long base = s_excl + pre;
   uint32_t pN = unpackA(base), pR = unpackB(base);
@@ -487,6 +557,170 @@ __global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, in
     } else {
       c->f0 = (uint32_t)f0;
       c->n_vict = found;
+      c->free_top = f0 - (int)min((uint32_t)f0, nn);
+      c->used_tail += c->n_rekey;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------
+// K3 (wide): the same victim rule for large sub-ops, over all SMs.  Pass 1 scans the
+// concatenation DISC[head,tail) ++ USED[head,tail) in tiles: candidates (live, not
+// pinned) are ranked with a block scan + decoupled look-back, rank < k are the victims
+// (exactly the first k in queue order), and the first kept position of each ring is
+// found with atomicMin.  Pass 2 reclaims the victims in parallel (host frames for
+// write-backs come from the free stack by atomic pop; ids are not observable).
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want) {
+  __shared__ unsigned long long s_scan[kScanTPB / 32];
+  __shared__ unsigned long long s_excl, s_dh, s_ld, s_uh, s_lu, s_mk[2];
+  __shared__ uint32_t s_k;
+  Ctl* c = T.ctl;
+  if (threadIdx.x == 0) {
+    s_dh = c->disc_head;
+    s_ld = c->disc_tail - c->disc_head;
+    s_uh = c->used_head;
+    s_lu = c->used_tail - c->used_head;
+    const uint32_t f0 = (uint32_t)c->free_top;
+    const uint32_t nn = evict_mode ? want : c->n_need;
+    s_k = nn > f0 ? nn - f0 : 0u;
+    s_mk[0] = s_mk[1] = ~0ull;
+  }
+  const uint32_t tile = take_ticket(T);
+  const uint32_t ntiles = gridDim.x;
+  const unsigned long long L = s_ld + s_lu;
+  const uint32_t k = s_k;
+  const unsigned long long first = (unsigned long long)tile * kScanTile + threadIdx.x * kScanIPT;
+  uint32_t bb[kScanIPT];
+  unsigned candm = 0, livem = 0;
+  uint32_t cc = 0;
+#pragma unroll
+  for (int q = 0; q < kScanIPT; ++q) {
+    bb[q] = 0;
+    const unsigned long long idx = first + q;
+    if (k && idx < L) {
+      const bool disc = idx < s_ld;
+      const unsigned long long pos = disc ? s_dh + idx : s_uh + (idx - s_ld);
+      const unsigned long long e = (disc ? T.disc_ring : T.used_ring)[pos & T.cap_mask];
+      const uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
+      const uint8_t ss = T.st[blk];
+      const bool live = (disc ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) && T.key[blk] == kk;
+      const bool cand = live && T.pin[blk] != seq;
+      bb[q] = blk;
+      livem |= (unsigned)live << q;
+      candm |= (unsigned)cand << q;
+      cc += cand;
+    }
+  }
+  unsigned long long tot;
+  unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cc, 0), tot, s_scan);
+  if (threadIdx.x < 32) {
+    unsigned long long e = lookback_warp(T, tile, tot);
+    if (threadIdx.x == 0) s_excl = e;
+  }
+  __syncthreads();
+  uint32_t r = unpackA(s_excl + pre);
+  unsigned long long mk0 = ~0ull, mk1 = ~0ull;
+#pragma unroll
+  for (int q = 0; q < kScanIPT; ++q) {
+    bool sel = false;
+    if ((candm >> q) & 1) {
+      if (r < k) {
+        T.victim[r] = bb[q];
+        sel = true;
+      }
+      ++r;
+    }
+    if (((livem >> q) & 1) && !sel) {
+      const unsigned long long idx = first + q;
+      if (idx < s_ld) mk0 = min(mk0, s_dh + idx);
+      else mk1 = min(mk1, s_uh + (idx - s_ld));
+    }
+  }
+  if (mk0 != ~0ull) atomicMin(&s_mk[0], mk0);
+  if (mk1 != ~0ull) atomicMin(&s_mk[1], mk1);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    if (s_mk[0] != ~0ull) atomicMin(&c->minkeep[0], s_mk[0]);
+    if (s_mk[1] != ~0ull) atomicMin(&c->minkeep[1], s_mk[1]);
+  }
+  if (tile == ntiles - 1 && threadIdx.x == 0) {
+    c->n_vict = min(k, unpackA(s_excl + tot));
+    c->k_want = k;
+  }
+  scan_finish(T, ntiles);
+}
+
+__global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode) {
+  __shared__ uint32_t s_cnt[4];
+  __shared__ int s_last;
+  Ctl* c = T.ctl;
+  const uint32_t found = c->n_vict;
+  const int f0 = c->free_top;
+  uint32_t nG = 0, nAv = 0, nGL = 0;
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < found; j += gridDim.x * blockDim.x) {
+    const uint32_t v = T.victim[j];
+    const uint8_t ss = T.st[v];
+    const uint32_t fr = T.frame_of[v];
+    const bool isG = ss == ST_G;
+    uint32_t hf = UM_NONE;
+    if (isG) {
+      if (!evict_mode && T.needk[(uint32_t)f0 + j] == ST_H) hf = T.needhf[(uint32_t)f0 + j];
+      if (hf == UM_NONE) {
+        int idx = atomicSub(&c->hfree_top, 1) - 1;
+        if (idx >= 0) {
+          hf = T.hfree_stack[idx];
+        } else {
+          atomicAdd(&c->hfree_top, 1);
+          atomicExch(&c->err, 2u);
+        }
+      }
+    }
+    T.vframe[j] = fr;
+    T.vkind[j] = ss;
+    T.vhf[j] = hf;
+    T.st[v] = isG ? ST_H : ST_HD;
+    T.map[v] = UM_NONE;
+    T.frame_of[v] = UM_NONE;
+    T.hframe[v] = hf;
+    nG += isG;
+    nAv += !isG;
+    nGL += ss == ST_GL;
+    if (evict_mode) {
+      T.free_stack[f0 + j] = fr;
+      if (isG) {
+        uint32_t q = atomicAdd(&c->n_d2h, 1u);
+        T.d2h_frame[q] = fr;
+        T.d2h_hf[q] = hf;
+      }
+    }
+  }
+  {
+    uint32_t v[4] = {0u, nG, nAv, nGL};
+    const int slots[4] = {-1, S_D2H, S_D2H_AV, S_UNMAPS};
+    const long long mul[4] = {1, (long long)T.B, (long long)T.B, 1};
+    block_counts_to<4>(T, v, s_cnt, slots, mul);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(&c->vict_done, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (s_last && threadIdx.x == 0) {
+    __threadfence();
+    stat_add(T, S_EVICT, found);
+    if (c->k_want) {  // the scan covered both rings completely
+      c->disc_head = c->minkeep[0] != ~0ull ? c->minkeep[0] : c->disc_tail;
+      c->used_head = c->minkeep[1] != ~0ull ? c->minkeep[1] : c->used_tail;
+    }
+    c->minkeep[0] = c->minkeep[1] = ~0ull;
+    c->vict_done = 0;
+    if (evict_mode) {
+      c->free_top = f0 + (int)found;
+    } else {
+      const uint32_t nn = c->n_need;
+      c->f0 = (uint32_t)f0;
       c->free_top = f0 - (int)min((uint32_t)f0, nn);
       c->used_tail += c->n_rekey;
     }
@@ -814,7 +1048,10 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
   }
   unsigned long long tot;
   unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cA, 0), tot, s_scan);
-  if (threadIdx.x == 0) s_excl = lookback(T, tile, tot);
+  if (threadIdx.x < 32) {
+    unsigned long long e = lookback_warp(T, tile, tot);
+    if (threadIdx.x == 0) s_excl = e;
+  }
   __syncthreads();
   uint32_t pA = unpackA(s_excl + pre);
   const unsigned long long tail0 = s_tail0;
@@ -923,7 +1160,10 @@ __global__ void __launch_bounds__(kScanTPB) k_ring_compact(Tables T, int ring, u
   }
   unsigned long long tot;
   unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cnt, 0), tot, s_scan);
-  if (threadIdx.x == 0) s_excl = lookback(T, tile, tot);
+  if (threadIdx.x < 32) {
+    unsigned long long e = lookback_warp(T, tile, tot);
+    if (threadIdx.x == 0) s_excl = e;
+  }
   __syncthreads();
   uint32_t p = unpackA(s_excl + pre);
 #pragma unroll
@@ -1050,6 +1290,18 @@ cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, u
 
 cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, cudaStream_t s) {
   k_victims<<<1, kVictTPB, 0, s>>>(T, seq, evict_mode, want);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, uint64_t scan_bound,
+                                uint32_t max_victims, cudaStream_t s) {
+  unsigned nt = ceil_div(scan_bound ? scan_bound : 1, kScanTile);
+  k_victims_scan<<<nt, kScanTPB, 0, s>>>(T, seq, evict_mode, want);
+  cudaError_t e = cudaGetLastError();
+  if (e) return e;
+  unsigned grid = ceil_div(max_victims ? max_victims : 1, 256);
+  if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
+  k_victims_apply<<<grid, 256, 0, s>>>(T, evict_mode);
   return cudaGetLastError();
 }
 

@@ -207,3 +207,28 @@ def test_next3_radix_hashjoin(ov, mode):
     for t in (tg.gen_radix(block_bytes=B, budget_bytes=int(64 * MiB / ov) // B * B, data_bytes=32 * MiB),
               tg.gen_hashjoin(block_bytes=B, budget_bytes=int(72 * MiB / ov) // B * B, table_bytes=8 * MiB)):
         assert_parity(t, mode)
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_wide_victim_selection(mode):
+    """Sub-ops larger than kVictWideMin (8192 blocks) select victims with the multi-CTA
+    scan (k_victims_scan/k_victims_apply): large random ranges over 60k blocks with 20k
+    frames, interleaved discards (stale ring entries, DISC before USED), big evicts."""
+    B = 4096
+    base = tg.gen_random(7, block_bytes=B, arena_bytes=60000 * B, budget_bytes=20000 * B, n_ops=50,
+                         max_ranges=3, max_blocks=14000, zipf_s=0.3, mix=[50, 20, 5, 10, 10, 0, 5])
+    tb = tg.TraceBuilder(B, 60000 * B, 20000 * B)
+    for i, (o, fl, off, ln, accs) in enumerate(base.iter_ops()):
+        if o == tg.OP_TOUCH:
+            tb.touch(accs)
+        elif o == tg.OP_PREFETCH:
+            tb.prefetch(off, ln, fl)
+        elif o == tg.OP_DISCARD:
+            tb.discard(off, ln, lazy_ok=bool(fl & 1))
+        elif o == tg.OP_HOST_WRITE:
+            tb.host_write(off, ln)
+        if i % 17 == 16:
+            tb.evict(12000 * B)
+    t = tb.build()
+    for copy in ("kernel", "ce"):
+        assert_parity(t, mode, _gpu(t, mode, copy=copy))
