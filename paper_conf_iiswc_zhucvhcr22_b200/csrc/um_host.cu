@@ -414,6 +414,7 @@ struct CopyList {
 // both PCIe directions busy.  The paging stream waits for both copy streams.
 static um_status ce_subop(um_arena* a, uint32_t seq, uint32_t n) {
   CK(launch_plan_commit(a->T, seq, n, a->ps));
+  a->n_launch++;
   CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
   CK(cudaMemcpyAsync(a->hitems, a->T.xitems, sizeof(XItem) * n, cudaMemcpyDeviceToHost, a->ps));
   CK(cudaStreamSynchronize(a->ps));
@@ -443,7 +444,10 @@ static um_status ce_subop(um_arena* a, uint32_t seq, uint32_t n) {
     CK(d2d.issue(st));
     CK(wb.issue(st));
     CK(h2d.issue(st));
-    if (anyzf) CK(launch_zero_items(a->T, g0, g1, st));
+    if (anyzf) {
+      CK(launch_zero_items(a->T, g0, g1, st));
+      a->n_launch++;
+    }
     CK(sw.issue(st));
   }
   for (int i = 0; i < 2; ++i) {
@@ -488,29 +492,42 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     return UM_OK;
   }
   const uint32_t m = (uint32_t)a->ivs.size();
-  // stage lo[m], pre[m+1], w[m]
-  const uint64_t bytes_lo = 4ull * m, bytes_pre = 4ull * (m + 1), bytes_w = m;
-  const uint64_t o_lo = 0, o_pre = (bytes_lo + 15) & ~15ull, o_w = o_pre + ((bytes_pre + 15) & ~15ull);
-  const uint64_t bytes = o_w + bytes_w;
-  uint64_t off;
-  CK(a->stage.reserve(bytes, &off));
-  uint32_t* hlo = (uint32_t*)(a->stage.host + off + o_lo);
-  uint32_t* hpre = (uint32_t*)(a->stage.host + off + o_pre);
-  uint8_t* hw = a->stage.host + off + o_w;
-  uint32_t acc = 0;
-  for (uint32_t j = 0; j < m; ++j) {
-    hlo[j] = a->ivs[j].lo;
-    hpre[j] = acc;
-    hw[j] = a->ivs[j].w;
-    acc += a->ivs[j].cnt;
-  }
-  hpre[m] = acc;
-  CK(a->stage.push(off, (bytes + 15) & ~15ull, a->ps));
-  OpIv iv;
-  iv.lo = (const uint32_t*)(a->stage.dev + off + o_lo);
-  iv.pre = (const uint32_t*)(a->stage.dev + off + o_pre);
-  iv.wflag = a->stage.dev + off + o_w;
+  OpIv iv{};
   iv.m = m;
+  if (m <= kIvInline) {
+    // small list: pass it inline in the kernel parameters (no staging copy)
+    iv.inl = 1;
+    uint32_t acc = 0;
+    for (uint32_t j = 0; j < m; ++j) {
+      iv.ilo[j] = a->ivs[j].lo;
+      iv.ipre[j] = acc;
+      iv.iw[j] = a->ivs[j].w;
+      acc += a->ivs[j].cnt;
+    }
+    iv.ipre[m] = acc;
+  } else {
+    // stage lo[m], pre[m+1], w[m] through the pinned ring
+    const uint64_t bytes_lo = 4ull * m, bytes_pre = 4ull * (m + 1), bytes_w = m;
+    const uint64_t o_lo = 0, o_pre = (bytes_lo + 15) & ~15ull, o_w = o_pre + ((bytes_pre + 15) & ~15ull);
+    const uint64_t bytes = o_w + bytes_w;
+    uint64_t off;
+    CK(a->stage.reserve(bytes, &off));
+    uint32_t* hlo = (uint32_t*)(a->stage.host + off + o_lo);
+    uint32_t* hpre = (uint32_t*)(a->stage.host + off + o_pre);
+    uint8_t* hw = a->stage.host + off + o_w;
+    uint32_t acc = 0;
+    for (uint32_t j = 0; j < m; ++j) {
+      hlo[j] = a->ivs[j].lo;
+      hpre[j] = acc;
+      hw[j] = a->ivs[j].w;
+      acc += a->ivs[j].cnt;
+    }
+    hpre[m] = acc;
+    CK(a->stage.push(off, (bytes + 15) & ~15ull, a->ps));
+    iv.lo = (const uint32_t*)(a->stage.dev + off + o_lo);
+    iv.pre = (const uint32_t*)(a->stage.dev + off + o_pre);
+    iv.wflag = a->stage.dev + off + o_w;
+  }
   const uint32_t F = a->nframes;
   for (uint64_t g0 = 0; g0 < total; g0 += F) {
     const uint32_t n = (uint32_t)std::min<uint64_t>(F, total - g0);
@@ -519,23 +536,28 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     um_status st = ensure_ring_room(a, RING_USED, n);
     if (st) return st;
     cudaEvent_t sp = span_open(a);
-    CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
-    if (n > kVictWideMin)
-      CK(launch_victims_wide(a->T, seq, 0, 0, a->ub[RING_DISC] + a->ub[RING_USED], n, a->ps));
-    else
-      CK(launch_victims(a->T, seq, 0, 0, a->ps));
+    if (n <= kSmallPlan) {
+      CK(launch_plan_small(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
+      a->n_launch += 1;
+    } else {
+      CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
+      if (n > kVictWideMin)
+        CK(launch_victims_wide(a->T, seq, 0, 0, a->ub[RING_DISC] + a->ub[RING_USED], n, a->ps));
+      else
+        CK(launch_victims(a->T, seq, 0, 0, a->ps));
+      a->n_launch += n > kVictWideMin ? 3 : 2;
+    }
     span_close(a, sp, 0);
     if (use_ce(a, n)) {
       sp = span_open(a);
-      um_status st = ce_subop(a, seq, n);
+      um_status st = ce_subop(a, seq, n);   // counts its own launches
       if (st) return st;
       span_close(a, sp, 1);
-      a->n_launch += 4;
     } else {
       sp = span_open(a);
       CK(launch_service(a->T, SVC_SUBOP, seq, n, a->ps));
       span_close(a, sp, 1);
-      a->n_launch += 3;
+      a->n_launch += 1;
     }
     a->n_xfer++;
     if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP)) {
@@ -794,6 +816,7 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
       CK(launch_victims_wide(a->T, seq, 1, (uint32_t)want, a->ub[RING_DISC] + a->ub[RING_USED], (uint32_t)want, a->ps));
     else
       CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->ps));
+    a->n_launch += want > kVictWideMin ? 1 : 0;
     span_close(a, sp, 0);
     sp = span_open(a);
     if (use_ce(a, want)) {

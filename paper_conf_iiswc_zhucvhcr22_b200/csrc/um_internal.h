@@ -85,11 +85,18 @@ struct Tables {
 // A GPU-destination op's distinct blocks as sorted disjoint intervals.  Interval j
 // covers blocks [lo[j], lo[j] + pre[j+1] - pre[j]); pre[] is the op-global exclusive
 // prefix of block counts; wflag[j] = the interval holds UM_ACC_WRITE blocks.
+// Small ops (m <= kIvInline) carry the list inline in the kernel parameters (no staging
+// copy); larger ones point at a staged device copy.
+constexpr uint32_t kIvInline = 24;
 struct OpIv {
   const uint32_t* lo;
   const uint32_t* pre;
   const uint8_t* wflag;
   uint32_t m;
+  uint32_t inl;
+  uint32_t ilo[kIvInline];
+  uint32_t ipre[kIvInline + 1];
+  uint8_t iw[kIvInline];
 };
 
 constexpr int kScanTPB = 512;
@@ -110,6 +117,10 @@ cudaError_t launch_init(const Tables& T, int nhframes_alloc, cudaStream_t s);
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
                             cudaStream_t s);
 cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, cudaStream_t s);
+// K1+K2+K3 fused in one CTA for sub-ops of <= kSmallPlan blocks
+constexpr uint32_t kSmallPlan = 4096;
+cudaError_t launch_plan_small(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
+                              cudaStream_t s);
 // multi-CTA victim selection for large sub-ops (scan bound = max ring entries to scan)
 cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, uint32_t want,
                                 uint64_t scan_bound, uint32_t max_victims, cudaStream_t s);

@@ -27,12 +27,16 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
 }
 
+__device__ __forceinline__ uint32_t iv_lo(const OpIv& iv, uint32_t j) { return iv.inl ? iv.ilo[j] : iv.lo[j]; }
+__device__ __forceinline__ uint32_t iv_pre(const OpIv& iv, uint32_t j) { return iv.inl ? iv.ipre[j] : iv.pre[j]; }
+__device__ __forceinline__ uint8_t iv_w(const OpIv& iv, uint32_t j) { return iv.inl ? iv.iw[j] : iv.wflag[j]; }
+
 // Largest j in [0, m) with pre[j] <= g (pre strictly increasing, pre[0] = 0).
 __device__ __forceinline__ uint32_t iv_find(const OpIv& iv, uint32_t g) {
   uint32_t lo = 0, hi = iv.m;  // answer in [lo, hi)
   while (hi - lo > 1) {
     uint32_t mid = (lo + hi) >> 1;
-    if (iv.pre[mid] <= g) lo = mid; else hi = mid;
+    if (iv_pre(iv, mid) <= g) lo = mid; else hi = mid;
   }
   return lo;
 }
@@ -275,24 +279,26 @@ __global__ void k_poison(char* p, size_t bytes) {
 // frame (U/H/HD) are listed for K3/K4.  Every rekeyed block is appended to USED at
 // used_tail + rank with key = seq, in ascending block order.
 // ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
-                                                       int touch) {
-  __shared__ unsigned long long s_scan[kScanTPB / 32];
+template <int TPB, int IPT>
+__device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
+                                              int touch) {
+  constexpr int TILE = TPB * IPT;
+  __shared__ unsigned long long s_scan[TPB / 32];
   __shared__ unsigned long long s_excl;
   __shared__ unsigned long long s_tail0;
   __shared__ uint32_t s_cnt[6];
-  // the tile's slice of the interval list (<= kScanTile intervals), staged in smem so
+  // the tile's slice of the interval list (<= TILE intervals), staged in smem so
   // each thread's interval search runs in shared memory
-  __shared__ uint32_t s_lo[kScanTile], s_pre[kScanTile + 1];
+  __shared__ uint32_t s_lo[TILE], s_pre[TILE + 1];
   __shared__ uint32_t s_j0, s_m;
   if (threadIdx.x == 0) s_tail0 = T.ctl->used_tail;
   const uint32_t tile = take_ticket(T);
-  const uint32_t ntiles = n ? (n + kScanTile - 1) / kScanTile : 1;
-  const uint32_t tbase = tile * kScanTile;
-  const uint32_t first = tbase + threadIdx.x * kScanIPT;
+  const uint32_t ntiles = n ? (n + TILE - 1) / TILE : 1;
+  const uint32_t tbase = tile * TILE;
+  const uint32_t first = tbase + threadIdx.x * IPT;
   if (threadIdx.x == 0 && tbase < n) {
     const uint32_t ja = iv_find(iv, g0 + tbase);
-    const uint32_t jb = iv_find(iv, g0 + min(n, tbase + kScanTile) - 1);
+    const uint32_t jb = iv_find(iv, g0 + min(n, tbase + TILE) - 1);
     s_j0 = ja;
     s_m = jb - ja + 1;
   }
@@ -300,15 +306,15 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
   if (tbase < n) {
     const uint32_t j0 = s_j0, m = s_m;
     for (uint32_t q = threadIdx.x; q < m; q += blockDim.x) {
-      s_lo[q] = iv.lo[j0 + q];
-      s_pre[q] = iv.pre[j0 + q];
+      s_lo[q] = iv_lo(iv, j0 + q);
+      s_pre[q] = iv_pre(iv, j0 + q);
     }
-    if (threadIdx.x == 0) s_pre[m] = iv.pre[j0 + m];
+    if (threadIdx.x == 0) s_pre[m] = iv_pre(iv, j0 + m);
   }
   __syncthreads();
 
-  uint32_t b[kScanIPT];
-  uint8_t s[kScanIPT];
+  uint32_t b[IPT];
+  uint8_t s[IPT];
   uint32_t cN = 0, cR = 0;
   uint32_t cls[6] = {0, 0, 0, 0, 0, 0};
   unsigned needm = 0, rekm = 0;
@@ -323,7 +329,7 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
     }
     uint32_t j = lo;
 #pragma unroll
-    for (int k = 0; k < kScanIPT; ++k) {
+    for (int k = 0; k < IPT; ++k) {
       uint32_t idx = first + k;
       if (idx < n) {
         uint32_t g = g0 + idx;
@@ -344,7 +350,7 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
     }
   }
   unsigned long long tot;
-  unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cN, cR), tot, s_scan);
+  unsigned long long pre = block_excl_scan<TPB>(pack2(cN, cR), tot, s_scan);
   if (threadIdx.x < 32) {
     unsigned long long e = lookback_warp(T, tile, tot);
     if (threadIdx.x == 0) s_excl = e;
@@ -355,7 +361,7 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
   const unsigned long long tail0 = s_tail0;
   if (first < n) {
 #pragma unroll
-    for (int k = 0; k < kScanIPT; ++k) {
+    for (int k = 0; k < IPT; ++k) {
       if (first + k >= n) break;
       const uint32_t bb = b[k];
       const uint8_t ss = s[k];
@@ -407,6 +413,11 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
   }
 }
 
+__global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
+                                                       int touch) {
+  classify_body<kScanTPB, kScanIPT>(T, iv, g0, n, seq, touch);
+}
+
 // ------------------------------------------------------------------------------------
 // K3: victim selection + reclaim (PAPER §5.5: free -> (unused, empty) ->
 // discarded FIFO -> used LRU; §5.3: discarded victims need no transfer; A10:
@@ -414,7 +425,7 @@ __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32
 // ranks live & unpinned entries with a block scan and takes the first k; the head
 // advances over the maximal prefix of dead or consumed entries.
 // ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, int evict_mode, uint32_t want) {
+__device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int evict_mode, uint32_t want) {
   __shared__ unsigned long long s_scan[kVictTPB / 32];
   __shared__ unsigned long long s_minkeep;
   __shared__ uint32_t s_cnt[4];
@@ -561,6 +572,20 @@ __global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, in
       c->used_tail += c->n_rekey;
     }
   }
+}
+
+__global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, int evict_mode, uint32_t want) {
+  victims_body(T, seq, evict_mode, want);
+}
+
+// K1+K2+K3 for a sub-op that fits one tile: one CTA classifies, compacts and selects
+// victims (saves a launch per small op; same code as the multi-CTA kernels).
+__global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
+                                                         int touch) {
+  classify_body<kVictTPB, kSmallPlan / kVictTPB>(T, iv, g0, n, seq, touch);
+  __syncthreads();
+  __threadfence_block();
+  victims_body(T, seq, 0, 0);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1001,8 +1026,8 @@ __global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g
       uint32_t g = g0 + (uint32_t)(u / spb);
       uint32_t j = iv_find(iv, g);
       char* d = nullptr;
-      uint32_t bb = iv.lo[j] + (g - iv.pre[j]);
-      if (iv.wflag[j]) {
+      uint32_t bb = iv_lo(iv, j) + (g - iv_pre(iv, j));
+      if (iv_w(iv, j)) {
         uint32_t fr = T.frame_of[bb];
         if (fr != UM_NONE) d = T.frames + (size_t)fr * T.B + (size_t)(u % spb) * SEG;
       }
@@ -1290,6 +1315,12 @@ cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, u
 
 cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, cudaStream_t s) {
   k_victims<<<1, kVictTPB, 0, s>>>(T, seq, evict_mode, want);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_plan_small(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
+                              cudaStream_t s) {
+  k_plan_small<<<1, kVictTPB, 0, s>>>(T, iv, g0, n, seq, touch);
   return cudaGetLastError();
 }
 

@@ -38,31 +38,50 @@ def iteration_bounds(trace) -> list:
     return [(i * per, (i + 1) * per) for i in range(it)]
 
 
-def issue(arena: um.Arena, trace, mode: str, start: int = 0, stop: int | None = None, stream=None) -> None:
-    """Issue ops[start:stop] of the trace (no synchronization)."""
-    a = arena.handle
-    s = arena.stream_ptr if stream is None else stream
-    ops, acc = trace.ops, trace.acc
-    stop = len(ops) if stop is None else stop
+def _calls(trace, mode: str) -> list:
+    """The trace as a list of (libum function, args-after-arena) tuples, built once per
+    (trace, mode): the issue loop then only makes the ctypes calls."""
+    key = "_calls_" + mode
+    cached = trace.meta.get(key)
+    if cached is not None:
+        return cached
+    L = um.lib()
+    acc = np.ascontiguousarray(trace.acc)
+    trace.meta["_acc_keepalive"] = acc
+    base = acc.ctypes.data
     lazy = mode == "lazy"
-    for r in ops[start:stop]:
-        o = int(r["op"])
+    out = []
+    for r in trace.ops.tolist():          # (op, flags, n, off, len) as python ints
+        o, fl, n, off, ln = r
         if o == tg.OP_TOUCH:
-            i, n = int(r["off"]), int(r["n"])
-            um.um_touch_batch(a, acc[i:i + n], s)
+            out.append(("um_touch_batch", L.um_touch_batch, (base + 16 * off if n else None, n)))
         elif o == tg.OP_PREFETCH:
-            um.um_prefetch(a, int(r["off"]), int(r["len"]), int(r["flags"]), s)
+            out.append(("um_prefetch", L.um_prefetch, (off, ln, fl)))
         elif o == tg.OP_DISCARD:
-            if lazy and (int(r["flags"]) & tg.F_LAZY_OK):
-                um.um_discard_lazy(a, int(r["off"]), int(r["len"]), s)
+            if lazy and (fl & tg.F_LAZY_OK):
+                out.append(("um_discard_lazy", L.um_discard_lazy, (off, ln)))
             else:
-                um.um_discard(a, int(r["off"]), int(r["len"]), s)
+                out.append(("um_discard", L.um_discard, (off, ln)))
         elif o == tg.OP_EVICT:
-            um.um_evict(a, int(r["len"]), s)
+            out.append(("um_evict", L.um_evict, (ln,)))
         elif o == tg.OP_HOST_WRITE:
-            um.um_host_write(a, int(r["off"]), int(r["len"]), s)
+            out.append(("um_host_write", L.um_host_write, (off, ln)))
         else:
             raise ValueError(o)
+    trace.meta[key] = out
+    return out
+
+
+def issue(arena: um.Arena, trace, mode: str, start: int = 0, stop: int | None = None, stream=None) -> None:
+    """Issue ops[start:stop] of the trace through the C ABI (no synchronization)."""
+    a = arena.handle
+    s = arena.stream_ptr if stream is None else stream
+    calls = _calls(trace, mode)
+    stop = len(calls) if stop is None else stop
+    for name, fn, args in calls[start:stop]:
+        st = fn(a, *args, s)
+        if st:
+            raise um.UmError(name, st)
 
 
 def result(arena: um.Arena) -> dict:
