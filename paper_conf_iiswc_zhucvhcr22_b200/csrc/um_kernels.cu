@@ -279,7 +279,9 @@ __global__ void k_poison(char* p, size_t bytes) {
 // frame (U/H/HD) are listed for K3/K4.  Every rekeyed block is appended to USED at
 // used_tail + rank with key = seq, in ascending block order.
 // ------------------------------------------------------------------------------------
-template <int TPB, int IPT>
+// SINGLE: the whole sub-op is one tile (one CTA) -> no ticket, no look-back, counters
+// added directly (saves the dependent global round trips of the multi-CTA protocol).
+template <int TPB, int IPT, bool SINGLE = false>
 __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
                                               int touch) {
   constexpr int TILE = TPB * IPT;
@@ -292,7 +294,7 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
   __shared__ uint32_t s_lo[TILE], s_pre[TILE + 1];
   __shared__ uint32_t s_j0, s_m;
   if (threadIdx.x == 0) s_tail0 = T.ctl->used_tail;
-  const uint32_t tile = take_ticket(T);
+  const uint32_t tile = SINGLE ? 0u : take_ticket(T);
   const uint32_t ntiles = n ? (n + TILE - 1) / TILE : 1;
   const uint32_t tbase = tile * TILE;
   const uint32_t first = tbase + threadIdx.x * IPT;
@@ -351,7 +353,9 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
   }
   unsigned long long tot;
   unsigned long long pre = block_excl_scan<TPB>(pack2(cN, cR), tot, s_scan);
-  if (threadIdx.x < 32) {
+  if (SINGLE) {
+    if (threadIdx.x == 0) s_excl = 0;
+  } else if (threadIdx.x < 32) {
     unsigned long long e = lookback_warp(T, tile, tot);
     if (threadIdx.x == 0) s_excl = e;
   }
@@ -389,28 +393,32 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
   }
   // counters (classes: U H HD G GE GL)
   const long long B = T.B;
+  uint32_t v[6];
   if (touch) {
     // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE ; h2d: H ; zf: U+HD ; h2d_av: HD
-    uint32_t v[6] = {cls[0] + cls[1] + cls[2] + cls[4], cls[3] + cls[5], cls[4], cls[1], cls[0] + cls[2], cls[2]};
-    tile_counts<6>(T, tile, v, s_cnt);
+    v[0] = cls[0] + cls[1] + cls[2] + cls[4]; v[1] = cls[3] + cls[5]; v[2] = cls[4];
   } else {
-    uint32_t v[6] = {cls[3], cls[4], cls[5], cls[1], cls[0] + cls[2], cls[2]};
-    tile_counts<6>(T, tile, v, s_cnt);
+    v[0] = cls[3]; v[1] = cls[4]; v[2] = cls[5];
   }
+  v[3] = cls[1]; v[4] = cls[0] + cls[2]; v[5] = cls[2];
+  const int slots_t[6] = {S_FAULTS, S_HITS, S_REMAPS, S_H2D, S_ZF, S_H2D_AV};
+  const int slots_p[6] = {S_REFRESH, S_REMAPS, S_REVAL, S_H2D, S_ZF, S_H2D_AV};
+  const long long mul[6] = {1, 1, 1, B, B, B};
+  if (SINGLE) {
+    if (threadIdx.x == 0) {
+      T.ctl->n_need = unpackA(tot);
+      T.ctl->n_rekey = unpackB(tot);
+    }
+    block_counts_to<6>(T, v, s_cnt, touch ? slots_t : slots_p, mul);
+    return;
+  }
+  tile_counts<6>(T, tile, v, s_cnt);
   if (tile == ntiles - 1 && threadIdx.x == 0) {
     unsigned long long all = s_excl + tot;
     T.ctl->n_need = unpackA(all);
     T.ctl->n_rekey = unpackB(all);
   }
-  if (touch) {
-    const int slots[6] = {S_FAULTS, S_HITS, S_REMAPS, S_H2D, S_ZF, S_H2D_AV};
-    const long long mul[6] = {1, 1, 1, B, B, B};
-    scan_finish<6>(T, ntiles, slots, mul);
-  } else {
-    const int slots[6] = {S_REFRESH, S_REMAPS, S_REVAL, S_H2D, S_ZF, S_H2D_AV};
-    const long long mul[6] = {1, 1, 1, B, B, B};
-    scan_finish<6>(T, ntiles, slots, mul);
-  }
+  scan_finish<6>(T, ntiles, touch ? slots_t : slots_p, mul);
 }
 
 __global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
@@ -582,7 +590,7 @@ __global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, in
 // victims (saves a launch per small op; same code as the multi-CTA kernels).
 __global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
                                                          int touch) {
-  classify_body<kVictTPB, kSmallPlan / kVictTPB>(T, iv, g0, n, seq, touch);
+  classify_body<kVictTPB, kSmallPlan / kVictTPB, true>(T, iv, g0, n, seq, touch);
   __syncthreads();
   __threadfence_block();
   victims_body(T, seq, 0, 0);
@@ -1051,6 +1059,7 @@ __global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g
 //   prefetch HOST G -> H (D2H), GE/GL -> H (no transfer), HD/U -> H
 // DISC appends are ranked in ascending block order (block scan + look-back).
 // ------------------------------------------------------------------------------------
+template <bool SINGLE>
 __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
                                                         int discard_off) {
   __shared__ unsigned long long s_scan[kScanTPB / 32];
@@ -1058,7 +1067,7 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
   __shared__ unsigned long long s_tail0;
   __shared__ uint32_t s_cnt[6];
   if (threadIdx.x == 0) s_tail0 = T.ctl->disc_tail;
-  const uint32_t tile = take_ticket(T);
+  const uint32_t tile = SINGLE ? 0u : take_ticket(T);
   const uint32_t ntiles = n ? (n + kScanTile - 1) / kScanTile : 1;
   const uint32_t first = tile * kScanTile + threadIdx.x * kScanIPT;
   uint32_t cA = 0;
@@ -1073,7 +1082,9 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
   }
   unsigned long long tot;
   unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cA, 0), tot, s_scan);
-  if (threadIdx.x < 32) {
+  if (SINGLE) {
+    if (threadIdx.x == 0) s_excl = 0;
+  } else if (threadIdx.x < 32) {
     unsigned long long e = lookback_warp(T, tile, tot);
     if (threadIdx.x == 0) s_excl = e;
   }
@@ -1141,13 +1152,16 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
       }
     }
   }
-  {
-    uint32_t v[3] = {nUnmap, nD2H, nAv};
-    tile_counts<3>(T, tile, v, s_cnt);
-  }
-  if (tile == ntiles - 1 && threadIdx.x == 0) T.ctl->disc_tail = tail0 + unpackA(s_excl + tot);
+  uint32_t v[3] = {nUnmap, nD2H, nAv};
   const int slots[3] = {S_UNMAPS, S_D2H, S_D2H_AV};
   const long long mul[3] = {1, (long long)T.B, (long long)T.B};
+  if (SINGLE) {
+    if (threadIdx.x == 0) T.ctl->disc_tail = tail0 + unpackA(tot);
+    block_counts_to<3>(T, v, s_cnt, slots, mul);
+    return;
+  }
+  tile_counts<3>(T, tile, v, s_cnt);
+  if (tile == ntiles - 1 && threadIdx.x == 0) T.ctl->disc_tail = tail0 + unpackA(s_excl + tot);
   scan_finish<3>(T, ntiles, slots, mul);
 }
 
@@ -1358,7 +1372,8 @@ cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, 
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq, int discard_off,
                              cudaStream_t s) {
   unsigned nt = n ? ceil_div(n, kScanTile) : 1;
-  k_directive<<<nt, kScanTPB, 0, s>>>(T, kind, lo, n, seq, discard_off);
+  if (nt == 1) k_directive<true><<<1, kScanTPB, 0, s>>>(T, kind, lo, n, seq, discard_off);
+  else k_directive<false><<<nt, kScanTPB, 0, s>>>(T, kind, lo, n, seq, discard_off);
   return cudaGetLastError();
 }
 
