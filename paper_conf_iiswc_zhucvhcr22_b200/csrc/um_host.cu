@@ -681,8 +681,10 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   for (uint32_t i = 0; i < cfg->n_host_chunks; ++i) a->hhost.push_back((char*)cfg->host_chunks[i]);
   if (const char* v = getenv("UM_CE_MIN_BYTES")) a->ce_min_bytes = strtoull(v, nullptr, 10);
   if ((e = a->stage.init((uint8_t*)(ws + L.stage), L.stage_bytes))) return fail(e);
+  // zero the whole workspace once: every table, ring slot and list starts defined (the
+  // parity exports copy whole rings / lists; compute-sanitizer initcheck stays clean)
+  if ((e = cudaMemsetAsync(ws, 0, L.total, a->ps))) return fail(e);
   if ((e = cudaMemcpyAsync(dhc, hc.data(), 8ull * cfg->n_host_chunks, cudaMemcpyHostToDevice, a->ps))) return fail(e);
-  if ((e = cudaMemsetAsync(T.tile_status, 0, 8 * L.max_tiles, a->ps))) return fail(e);
   if ((e = launch_init(T, (int)(a->nhframes - 1), a->ps))) return fail(e);
   if (cfg->flags & UM_F_CHECK)
     if ((e = launch_poison(T, a->ps))) return fail(e);

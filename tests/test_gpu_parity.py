@@ -232,3 +232,24 @@ def test_wide_victim_selection(mode):
     t = tb.build()
     for copy in ("kernel", "ce"):
         assert_parity(t, mode, _gpu(t, mode, copy=copy))
+
+
+def _full_size_trace(iterations=2):
+    import torch
+    free, _ = torch.cuda.mem_get_info()
+    GiB = 1 << 30
+    B = 2 << 20
+    budget = min(170 * GiB, free - 6 * GiB) // B * B
+    return tg.gen_c3(block_bytes=B, budget_bytes=budget, oversub=1.5, iterations=iterations)
+
+
+@pytest.mark.parametrize("mode,copy", [("eager", "auto"), ("lazy", "kernel")])
+def test_c3_full_size(mode, copy):
+    """Parity at the bench's full size and launch configuration: C3 at 1.5x of a
+    170 GiB frame budget (255 GiB arena, 2 MiB blocks), host pool = arena - budget +
+    2 GiB, two iterations; every block's state, the queue orders, all counters and every
+    block's content tag (frames and host frames read back) against the oracle."""
+    t = _full_size_trace()
+    pool = t.arena_bytes - t.budget_bytes + (2 << 30)
+    g = _gpu(t, mode, copy=copy, host_pool_bytes=pool)
+    assert_parity(t, mode, g)
