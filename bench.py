@@ -252,6 +252,50 @@ def discard_bench(torch, um, reps=20):
     return out
 
 
+def c4_sweep(torch, um, harness):
+    """C4 (BASELINE.json configs[3]): UvmDiscard vs UvmDiscardLazy over directive size and
+    re-touch ratio, with and without memory pressure (64 KiB blocks).  Per case: kernel
+    time of the discard and of the re-touch prefetch (planning + transfer/zero-fill, from
+    um_timing), and the revive/zero-fill counts."""
+    import tracegen as tg
+    B = 64 * 1024
+    mem = um.Memory(B, 16 * GiB, 8 * GiB, host_pool_bytes=1 * GiB + 64 * MiB)
+    out = []
+    cases = [(S, p, pr) for pr in (False, True) for S in (2 * MiB, 128 * MiB, 1 * GiB, 8 * GiB)
+             for p in (0.0, 0.5, 1.0) if not (pr and S > 1 * GiB)]
+    try:
+        for S, p, pr in cases:
+            t = tg.gen_c4(S, p, block_bytes=B, pressure=pr)
+            row = {"bytes": S, "retouch": p, "pressure": pr}
+            for mode in ("eager", "lazy"):
+                a = harness.make_arena(t, mode, mem=mem, flags=um.UM_F_TIMING)
+                try:
+                    harness.alloc_buffers(a, t)
+                    harness.issue(a, t, mode, 0, 2)                  # resident + written
+                    um.um_timing(a.handle, reset=True)
+                    harness.issue(a, t, mode, 2, 3)                  # the discard
+                    td = um.um_timing(a.handle, reset=True)
+                    nxt = 3
+                    if pr:
+                        harness.issue(a, t, mode, 3, 4)              # filler (pressure)
+                        um.um_timing(a.handle, reset=True)
+                        nxt = 4
+                    harness.issue(a, t, mode, nxt, len(t))           # re-touch
+                    tr = um.um_timing(a.handle, reset=True)
+                    st = um.um_get_stats(a.handle)
+                    row[mode] = {"discard_us": td["ms_plan"] * 1e3,
+                                 "retouch_us": (tr["ms_plan"] + tr["ms_xfer"]) * 1e3,
+                                 "remaps": st["remaps"], "revalidations": st["revalidations"],
+                                 "zf_blocks": st["zf_bytes"] // B, "d2h_blocks": st["d2h_bytes"] // B}
+                finally:
+                    a.close()
+            out.append(row)
+    finally:
+        del mem
+        torch.cuda.empty_cache()
+    return out
+
+
 def c1_rate(torch, um, harness):
     """C1 tiny trace (BASELINE.json configs[0]; 10k ops, 64 KiB blocks): ops/s through
     the public API (host wall clock, synchronised at the end) — the small-op,
@@ -394,6 +438,7 @@ def main_ours(args):
     link = measure_link_peak(torch, dev)
     disc = None if args.no_discard_bench else discard_bench(torch, um)
     c1 = None if args.no_discard_bench else c1_rate(torch, um, harness)
+    c4 = None if args.no_discard_bench else c4_sweep(torch, um, harness)
 
     torch.cuda.empty_cache()
     free, total = torch.cuda.mem_get_info(dev)
@@ -483,6 +528,7 @@ def main_ours(args):
         "transfer_paths": _paths(res.get("eager"), k4, link),
         "roofline_state": state,
         "c1_directives": c1,
+        "c4_sweep": c4,
         "clocks": head["clocks"],
         "gpu_launches": tm["launches"],
         "stats_per_iter_all_ranks": stats_all,

@@ -253,3 +253,12 @@ def test_c3_full_size(mode, copy):
     pool = t.arena_bytes - t.budget_bytes + (2 << 30)
     g = _gpu(t, mode, copy=copy, host_pool_bytes=pool)
     assert_parity(t, mode, g)
+
+
+@pytest.mark.parametrize("pressure", [False, True])
+@pytest.mark.parametrize("mode", ["eager", "lazy"])
+def test_c4_sweep_cases(pressure, mode):
+    """C4 eager-vs-lazy cases (prefix and scattered re-touch) at 64 KiB blocks."""
+    for S, p, sc in [(64 << 10, 1.0, False), (32 << 20, 0.5, False), (32 << 20, 0.25, True), (256 << 20, 1.0, False)]:
+        t = tg.gen_c4(S, p, block_bytes=64 << 10, pressure=pressure, scattered=sc)
+        assert_parity(t, mode)

@@ -159,3 +159,33 @@ def test_stat_names_match_abi_order():
     body = re.search(r"typedef struct\s*\{([^}]*)\}\s*um_stats;", h).group(1)
     names = re.findall(r"\b([a-z0-9_]+)\s*[,;]", body.replace("int64_t", ""))
     assert tuple(n for n in names if not n.startswith("pad")) == STAT_NAMES
+
+
+@pytest.mark.parametrize("nb,p", [(8, 0.0), (8, 0.5), (16, 1.0), (10, 0.3)])
+@pytest.mark.parametrize("pressure", [False, True])
+@pytest.mark.parametrize("mode", ["eager", "lazy"])
+def test_c4_closed_form(nb, p, pressure, mode):
+    """C4 by hand.  nb resident written blocks are discarded, then
+    k = round(p*nb) are re-touched (prefetch + write).
+    No pressure: the pages are still resident -> k remaps (UvmDiscard re-maps, §5.7
+    L229) or k revalidations (UvmDiscardLazy's prefetch sets the dirty bits, L190); no
+    transfer, no extra zeroing.
+    Pressure (a filler of nb blocks prefetched in between, budget = nb): all nb discarded
+    pages are reclaimed first (discarded FIFO, L221) with no write-back (d2h_avoided =
+    nb); the re-touch zero-fills k blocks instead of migrating them (h2d_avoided = k,
+    L200) and evicts the k LRU filler blocks, which are valid and written back (A10)."""
+    B = 4096
+    t = tg.gen_c4(nb * B, p, block_bytes=B, pressure=pressure)
+    k = int(round(p * nb))
+    s = replay(t, mode).stats
+    if not pressure:
+        assert s["zf_bytes"] == nb * B and s["h2d_bytes"] == s["d2h_bytes"] == 0
+        assert (s["remaps"], s["revalidations"]) == ((k, 0) if mode == "eager" else (0, k))
+        assert s["unmaps"] == (nb if mode == "eager" else 0)
+    else:
+        assert s["zf_bytes"] == (2 * nb + k) * B
+        assert s["d2h_avoided_bytes"] == nb * B and s["h2d_avoided_bytes"] == k * B
+        assert s["d2h_bytes"] == k * B and s["h2d_bytes"] == 0
+        assert s["remaps"] == s["revalidations"] == 0
+        assert s["unmaps"] == nb          # eager: at discard; lazy: at reclaim (§5.6 L225)
+        assert s["evictions"] == nb + k

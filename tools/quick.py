@@ -15,3 +15,6 @@ out = {"c1": bench.c1_rate(torch, um, harness)}
 out["discard"] = [(r["bytes"], r["eager"]["kernel_us"], r["eager"]["api_us"], r["lazy"]["kernel_us"])
                   for r in bench.discard_bench(torch, um, reps=10)]
 print(json.dumps(out))
+
+out2 = bench.c4_sweep(torch, um, harness)
+print(json.dumps(out2))
