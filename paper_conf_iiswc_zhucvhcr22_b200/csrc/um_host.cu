@@ -62,7 +62,9 @@ static Layout make_layout(const um_config* c) {
   const uint64_t nf = c->budget_bytes / c->block_bytes;
   const uint64_t nh = (uint64_t)c->n_host_chunks * (c->host_chunk_bytes / c->block_bytes);
   L.cap = pow2_ceil(std::max<uint64_t>(1024, 4 * nf));
-  L.max_tiles = (std::max(nb, L.cap) + kScanTile - 1) / kScanTile + 1;
+  // tiles: classify/directive scan <= nblocks items, compaction <= cap, the wide victim
+  // scan <= |DISC| + |USED| <= 2 * cap (its bound is also clamped to 2 * cap)
+  L.max_tiles = (std::max(nb, 2 * L.cap) + kScanTile - 1) / kScanTile + 1;
   L.stage_bytes = std::min<uint64_t>(64ull << 20, 12 * nb + (1 << 20));
   uint64_t o = 0;
   auto take = [&](uint64_t bytes) {
@@ -542,7 +544,7 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     } else {
       CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
       if (n > kVictWideMin)
-        CK(launch_victims_wide(a->T, seq, 0, 0, a->ub[RING_DISC] + a->ub[RING_USED], n, a->ps));
+        CK(launch_victims_wide(a->T, seq, 0, 0, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), n, a->ps));
       else
         CK(launch_victims(a->T, seq, 0, 0, a->ps));
       a->n_launch += n > kVictWideMin ? 3 : 2;
@@ -815,7 +817,7 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
   if (want) {
     cudaEvent_t sp = span_open(a);
     if (want > kVictWideMin)
-      CK(launch_victims_wide(a->T, seq, 1, (uint32_t)want, a->ub[RING_DISC] + a->ub[RING_USED], (uint32_t)want, a->ps));
+      CK(launch_victims_wide(a->T, seq, 1, (uint32_t)want, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), (uint32_t)want, a->ps));
     else
       CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->ps));
     a->n_launch += want > kVictWideMin ? 1 : 0;

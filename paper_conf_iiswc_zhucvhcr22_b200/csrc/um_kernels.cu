@@ -114,22 +114,39 @@ __device__ unsigned long long lookback_warp(const Tables& T, uint32_t tile, unsi
   }
   if (lane == 0) st[tile] = FA | agg;
   __threadfence();
+  // each round inspects 128 predecessors (4 independent loads per lane); the closest
+  // one holding an inclusive prefix (or the start of the array) ends the walk
   unsigned long long excl = 0;
   long long p = (long long)tile - 1;
   while (true) {
-    const long long idx = p - lane;
-    unsigned long long v = FP;  // before tile 0: an inclusive prefix of 0
-    if (idx >= 0) {
-      do { v = st[idx]; } while ((v >> 62) == 0);
+    unsigned long long v[4];
+    long long pbest = -1;  // largest index in this round holding an inclusive prefix
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const long long idx = p - lane - 32 * q;
+      v[q] = 0;
+      if (idx >= 0) {
+        do { v[q] = st[idx]; } while ((v[q] >> 62) == 0);
+        if ((v[q] >> 62) == 2 && idx > pbest) pbest = idx;
+      }
     }
-    const unsigned pm = __ballot_sync(FULL, (v >> 62) == 2);
-    const int stop = pm ? __ffs(pm) - 1 : 31;
-    unsigned long long x = lane <= stop ? (v & M) : 0ull;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      long long y = __shfl_xor_sync(FULL, pbest, o);
+      pbest = y > pbest ? y : pbest;
+    }
+    const bool done = pbest >= 0 || p - 127 <= 0;   // a prefix found, or tile 0 reached
+    unsigned long long x = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const long long idx = p - lane - 32 * q;
+      if (idx >= 0 && idx >= pbest) x += v[q] & M;
+    }
 #pragma unroll
     for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(FULL, x, o);
     excl += x;
-    if (pm) break;
-    p -= 32;
+    if (done) break;
+    p -= 128;
   }
   if (lane == 0) st[tile] = FP | (excl + agg);
   __threadfence();
