@@ -74,8 +74,9 @@ __device__ __forceinline__ unsigned long long block_excl_scan(unsigned long long
   return pre;
 }
 
-// Decoupled look-back (single pass, tiles ordered by a ticket so predecessors always
-// run): returns the exclusive prefix of this tile.  Status word = flag(2b) | value(62b).
+// Decoupled look-back (single pass).  Tiles are ordered by blockIdx: CTAs are
+// dispatched in index order, so every predecessor of a waiting tile is resident or done.
+// Returns the exclusive prefix of this tile.  Status word = flag(2b) | value(62b).
 __device__ unsigned long long lookback(const Tables& T, uint32_t tile, unsigned long long agg) {
   volatile unsigned long long* st = T.tile_status;
   const unsigned long long FA = 1ull << 62, FP = 2ull << 62, M = FA - 1;
@@ -175,12 +176,6 @@ __device__ void scan_finish(const Tables& T, uint32_t ntiles) {
   }
 }
 
-__device__ __forceinline__ uint32_t take_ticket(const Tables& T) {
-  __shared__ uint32_t s_tile;
-  if (threadIdx.x == 0) s_tile = atomicAdd(&T.ctl->scan_ticket, 1u);
-  __syncthreads();
-  return s_tile;
-}
 
 __device__ __forceinline__ unsigned long long pack2(uint32_t a, uint32_t b) {
   return (unsigned long long)a | ((unsigned long long)b << 31);
@@ -296,30 +291,80 @@ __global__ void k_poison(char* p, size_t bytes) {
 // frame (U/H/HD) are listed for K3/K4.  Every rekeyed block is appended to USED at
 // used_tail + rank with key = seq, in ascending block order.
 // ------------------------------------------------------------------------------------
+// Ordered ranks with a coalesced item mapping: item (k, t) of a tile is element
+// tbase + k*TPB + t, so ascending order = (k, warp, lane).  Each warp ballots its 32
+// flags per k (two flag kinds A and B); lane 0 stores the packed popc counts
+// (A | B << 16) of every k; one warp exclusive-scans the IPT x NW counts in smem.  The
+// rank of a flagged item is then  warp offset + popc(ballot & lanes below).  Returns the
+// packed tile totals (<= TILE < 2^16 each).
+template <int TPB, int IPT>
+__device__ __forceinline__ uint32_t ordered_offsets(const unsigned (&ba)[IPT], const unsigned (&bb)[IPT], uint32_t* sm) {
+  constexpr int NW = TPB / 32, NE = IPT * NW, PER = (NE + 31) / 32;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  if (lane == 0) {
+#pragma unroll
+    for (int k = 0; k < IPT; ++k) sm[k * NW + w] = (uint32_t)__popc(ba[k]) | ((uint32_t)__popc(bb[k]) << 16);
+  }
+  __syncthreads();
+  if (w == 0) {
+    uint32_t v[PER], sum = 0;
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const int i = lane * PER + q;
+      v[q] = i < NE ? sm[i] : 0u;
+      sum += v[q];
+    }
+    uint32_t x = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    uint32_t ex = x - sum;
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const int i = lane * PER + q;
+      if (i < NE) sm[i] = ex;
+      ex += v[q];
+    }
+    if (lane == 31) sm[NE] = x;
+  }
+  __syncthreads();
+  return sm[NE];
+}
+
+__device__ __forceinline__ unsigned lanemask_lt() {
+  unsigned m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
 // SINGLE: the whole sub-op is one tile (one CTA) -> no ticket, no look-back, counters
 // added directly (saves the dependent global round trips of the multi-CTA protocol).
 template <int TPB, int IPT, bool SINGLE = false>
 __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
                                               int touch) {
-  constexpr int TILE = TPB * IPT;
-  __shared__ unsigned long long s_scan[TPB / 32];
+  constexpr int TILE = TPB * IPT, NW = TPB / 32;
+  __shared__ uint32_t s_off[IPT * NW + 1];
   __shared__ unsigned long long s_excl;
   __shared__ unsigned long long s_tail0;
   __shared__ uint32_t s_cnt[6];
-  // the tile's slice of the interval list (<= TILE intervals), staged in smem so
-  // each thread's interval search runs in shared memory
+  // the tile's slice of the interval list (<= TILE intervals), staged in smem so the
+  // per-item interval search runs in shared memory
   __shared__ uint32_t s_lo[TILE], s_pre[TILE + 1];
   __shared__ uint32_t s_j0, s_m;
-  if (threadIdx.x == 0) s_tail0 = T.ctl->used_tail;
-  const uint32_t tile = SINGLE ? 0u : take_ticket(T);
-  const uint32_t ntiles = n ? (n + TILE - 1) / TILE : 1;
+  const uint32_t tile = SINGLE ? 0u : blockIdx.x;
+  const uint32_t ntiles = SINGLE ? 1u : gridDim.x;
   const uint32_t tbase = tile * TILE;
-  const uint32_t first = tbase + threadIdx.x * IPT;
-  if (threadIdx.x == 0 && tbase < n) {
-    const uint32_t ja = iv_find(iv, g0 + tbase);
-    const uint32_t jb = iv_find(iv, g0 + min(n, tbase + TILE) - 1);
-    s_j0 = ja;
-    s_m = jb - ja + 1;
+  const int w = threadIdx.x >> 5;
+  if (threadIdx.x == 0) {
+    s_tail0 = T.ctl->used_tail;
+    if (tbase < n) {
+      const uint32_t ja = iv_find(iv, g0 + tbase);
+      const uint32_t jb = iv_find(iv, g0 + min(n, tbase + TILE) - 1);
+      s_j0 = ja;
+      s_m = jb - ja + 1;
+    }
   }
   __syncthreads();
   if (tbase < n) {
@@ -334,42 +379,38 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
 
   uint32_t b[IPT];
   uint8_t s[IPT];
-  uint32_t cN = 0, cR = 0;
+  unsigned bN[IPT], bR[IPT];
   uint32_t cls[6] = {0, 0, 0, 0, 0, 0};
-  unsigned needm = 0, rekm = 0;
-  if (first < n) {
-    uint32_t lo = 0, hi = s_m;  // largest j with s_pre[j] <= g
-    {
-      const uint32_t g = g0 + first;
+  uint32_t jlo = 0;
+  const uint32_t m = tbase < n ? s_m : 0u;
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) {
+    const uint32_t idx = tbase + k * TPB + threadIdx.x;
+    bool nd = false, rk = false;
+    b[k] = 0;
+    s[k] = 0xff;
+    if (idx < n) {
+      const uint32_t g = g0 + idx;
+      uint32_t lo = jlo, hi = m;  // largest j with s_pre[j] <= g (items ascend per thread)
       while (hi - lo > 1) {
-        uint32_t mid = (lo + hi) >> 1;
+        const uint32_t mid = (lo + hi) >> 1;
         if (s_pre[mid] <= g) lo = mid; else hi = mid;
       }
+      jlo = lo;
+      const uint32_t bb = s_lo[lo] + (g - s_pre[lo]);
+      const uint8_t ss = T.st[bb];
+      T.pin[bb] = seq;
+      b[k] = bb;
+      s[k] = ss;
+      nd = ss <= ST_HD;
+      rk = touch ? (nd || ss == ST_GE) : true;
+      cls[ss]++;
     }
-    uint32_t j = lo;
-#pragma unroll
-    for (int k = 0; k < IPT; ++k) {
-      uint32_t idx = first + k;
-      if (idx < n) {
-        uint32_t g = g0 + idx;
-        while (g >= s_pre[j + 1]) ++j;
-        uint32_t bb = s_lo[j] + (g - s_pre[j]);
-        uint8_t ss = T.st[bb];
-        T.pin[bb] = seq;
-        b[k] = bb;
-        s[k] = ss;
-        bool nd = ss <= ST_HD;
-        bool rk = touch ? (nd || ss == ST_GE) : true;
-        needm |= (unsigned)nd << k;
-        rekm |= (unsigned)rk << k;
-        cN += nd;
-        cR += rk;
-        cls[ss]++;
-      }
-    }
+    bN[k] = __ballot_sync(FULL, nd);
+    bR[k] = __ballot_sync(FULL, rk);
   }
-  unsigned long long tot;
-  unsigned long long pre = block_excl_scan<TPB>(pack2(cN, cR), tot, s_scan);
+  const uint32_t tt = ordered_offsets<TPB, IPT>(bN, bR, s_off);
+  const unsigned long long tot = pack2(tt & 0xffffu, tt >> 16);
   if (SINGLE) {
     if (threadIdx.x == 0) s_excl = 0;
   } else if (threadIdx.x < 32) {
@@ -377,33 +418,33 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
     if (threadIdx.x == 0) s_excl = e;
   }
   __syncthreads();
-  const unsigned long long base = s_excl + pre;
-  uint32_t pN = unpackA(base), pR = unpackB(base);
+  const uint32_t eN = unpackA(s_excl), eR = unpackB(s_excl);
   const unsigned long long tail0 = s_tail0;
-  if (first < n) {
+  const unsigned lt = lanemask_lt();
 #pragma unroll
-    for (int k = 0; k < IPT; ++k) {
-      if (first + k >= n) break;
-      const uint32_t bb = b[k];
-      const uint8_t ss = s[k];
-      const bool nd = (needm >> k) & 1, rk = (rekm >> k) & 1;
-      if (nd) {
-        T.need[pN] = bb;
-        T.needk[pN] = ss;
-        T.needhf[pN] = (ss == ST_H) ? T.hframe[bb] : UM_NONE;
-        ++pN;
-      }
-      if (rk) {
-        T.used_ring[(tail0 + pR) & T.cap_mask] = ((unsigned long long)seq << 32) | bb;
-        ++pR;
-        if (!nd) {
-          T.key[bb] = seq;
-          if (ss == ST_GE) {        // revive: re-map the frame kept since the discard
-            T.st[bb] = ST_G;
-            T.map[bb] = T.frame_of[bb];
-          } else if (ss == ST_GL) { // revalidate: mapping was kept (lazy)
-            T.st[bb] = ST_G;
-          }
+  for (int k = 0; k < IPT; ++k) {
+    const uint32_t idx = tbase + k * TPB + threadIdx.x;
+    if (idx >= n) continue;
+    const uint32_t bb = b[k];
+    const uint8_t ss = s[k];
+    const bool nd = (bN[k] >> (threadIdx.x & 31)) & 1, rk = (bR[k] >> (threadIdx.x & 31)) & 1;
+    const uint32_t off = s_off[k * NW + w];
+    if (nd) {
+      const uint32_t pN = eN + (off & 0xffffu) + __popc(bN[k] & lt);
+      T.need[pN] = bb;
+      T.needk[pN] = ss;
+      T.needhf[pN] = (ss == ST_H) ? T.hframe[bb] : UM_NONE;
+    }
+    if (rk) {
+      const uint32_t pR = eR + (off >> 16) + __popc(bR[k] & lt);
+      T.used_ring[(tail0 + pR) & T.cap_mask] = ((unsigned long long)seq << 32) | bb;
+      if (!nd) {
+        T.key[bb] = seq;
+        if (ss == ST_GE) {        // revive: re-map the frame kept since the discard
+          T.st[bb] = ST_G;
+          T.map[bb] = T.frame_of[bb];
+        } else if (ss == ST_GL) { // revalidate: mapping was kept (lazy)
+          T.st[bb] = ST_G;
         }
       }
     }
@@ -622,7 +663,8 @@ __global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, OpIv iv, uint
 // write-backs come from the free stack by atomic pop; ids are not observable).
 // ------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want) {
-  __shared__ unsigned long long s_scan[kScanTPB / 32];
+  constexpr int NW = kScanTPB / 32;
+  __shared__ uint32_t s_off[kScanIPT * NW + 1];
   __shared__ unsigned long long s_excl, s_dh, s_ld, s_uh, s_lu, s_mk[2];
   __shared__ uint32_t s_k;
   Ctl* c = T.ctl;
@@ -636,53 +678,56 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
     s_k = nn > f0 ? nn - f0 : 0u;
     s_mk[0] = s_mk[1] = ~0ull;
   }
-  const uint32_t tile = take_ticket(T);
+  __syncthreads();
+  const uint32_t tile = blockIdx.x;
   const uint32_t ntiles = gridDim.x;
   const unsigned long long L = s_ld + s_lu;
   const uint32_t k = s_k;
-  const unsigned long long first = (unsigned long long)tile * kScanTile + threadIdx.x * kScanIPT;
+  const unsigned long long tbase = (unsigned long long)tile * kScanTile;
+  const int w = threadIdx.x >> 5;
   uint32_t bb[kScanIPT];
-  unsigned candm = 0, livem = 0;
-  uint32_t cc = 0;
+  unsigned bC[kScanIPT], bL[kScanIPT];
 #pragma unroll
   for (int q = 0; q < kScanIPT; ++q) {
     bb[q] = 0;
-    const unsigned long long idx = first + q;
+    bool live = false, cand = false;
+    const unsigned long long idx = tbase + q * kScanTPB + threadIdx.x;
     if (k && idx < L) {
       const bool disc = idx < s_ld;
       const unsigned long long pos = disc ? s_dh + idx : s_uh + (idx - s_ld);
       const unsigned long long e = (disc ? T.disc_ring : T.used_ring)[pos & T.cap_mask];
       const uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
       const uint8_t ss = T.st[blk];
-      const bool live = (disc ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) && T.key[blk] == kk;
-      const bool cand = live && T.pin[blk] != seq;
+      live = (disc ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) && T.key[blk] == kk;
+      cand = live && T.pin[blk] != seq;
       bb[q] = blk;
-      livem |= (unsigned)live << q;
-      candm |= (unsigned)cand << q;
-      cc += cand;
     }
+    bC[q] = __ballot_sync(FULL, cand);
+    bL[q] = __ballot_sync(FULL, live);
   }
-  unsigned long long tot;
-  unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cc, 0), tot, s_scan);
+  const uint32_t tt = ordered_offsets<kScanTPB, kScanIPT>(bC, bC, s_off);
+  const unsigned long long tot = pack2(tt & 0xffffu, 0);
   if (threadIdx.x < 32) {
-    unsigned long long e = lookback_warp(T, tile, tot);
-    if (threadIdx.x == 0) s_excl = e;
+    unsigned long long ex = lookback_warp(T, tile, tot);
+    if (threadIdx.x == 0) s_excl = ex;
   }
   __syncthreads();
-  uint32_t r = unpackA(s_excl + pre);
+  const uint32_t eC = unpackA(s_excl);
+  const unsigned lt = lanemask_lt();
+  const unsigned me = 1u << (threadIdx.x & 31);
   unsigned long long mk0 = ~0ull, mk1 = ~0ull;
 #pragma unroll
   for (int q = 0; q < kScanIPT; ++q) {
     bool sel = false;
-    if ((candm >> q) & 1) {
+    if (bC[q] & me) {
+      const uint32_t r = eC + (s_off[q * NW + w] & 0xffffu) + __popc(bC[q] & lt);
       if (r < k) {
         T.victim[r] = bb[q];
         sel = true;
       }
-      ++r;
     }
-    if (((livem >> q) & 1) && !sel) {
-      const unsigned long long idx = first + q;
+    if ((bL[q] & me) && !sel) {
+      const unsigned long long idx = tbase + q * kScanTPB + threadIdx.x;
       if (idx < s_ld) mk0 = min(mk0, s_dh + idx);
       else mk1 = min(mk1, s_uh + (idx - s_ld));
     }
@@ -1079,26 +1124,28 @@ __global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g
 template <bool SINGLE>
 __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
                                                         int discard_off) {
-  __shared__ unsigned long long s_scan[kScanTPB / 32];
+  constexpr int NW = kScanTPB / 32;
+  __shared__ uint32_t s_off[kScanIPT * NW + 1];
   __shared__ unsigned long long s_excl;
   __shared__ unsigned long long s_tail0;
   __shared__ uint32_t s_cnt[6];
   if (threadIdx.x == 0) s_tail0 = T.ctl->disc_tail;
-  const uint32_t tile = SINGLE ? 0u : take_ticket(T);
-  const uint32_t ntiles = n ? (n + kScanTile - 1) / kScanTile : 1;
-  const uint32_t first = tile * kScanTile + threadIdx.x * kScanIPT;
-  uint32_t cA = 0;
+  const uint32_t tile = SINGLE ? 0u : blockIdx.x;
+  const uint32_t ntiles = SINGLE ? 1u : gridDim.x;
+  const uint32_t tbase = tile * kScanTile;
+  const int w = threadIdx.x >> 5;
+  const bool appends = !discard_off && kind != DIR_PREFETCH_HOST;
   uint8_t s[kScanIPT];
+  unsigned bA[kScanIPT], bZ[kScanIPT];
 #pragma unroll
   for (int k = 0; k < kScanIPT; ++k) {
-    s[k] = 0xff;
-    if (first + k < n) {
-      s[k] = T.st[lo + first + k];
-      cA += (!discard_off && kind != DIR_PREFETCH_HOST && s[k] == ST_G);
-    }
+    const uint32_t idx = tbase + k * kScanTPB + threadIdx.x;   // coalesced
+    s[k] = idx < n ? T.st[lo + idx] : (uint8_t)0xff;
+    bA[k] = __ballot_sync(FULL, appends && s[k] == ST_G);
+    bZ[k] = 0;
   }
-  unsigned long long tot;
-  unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cA, 0), tot, s_scan);
+  const uint32_t tt = ordered_offsets<kScanTPB, kScanIPT>(bA, bZ, s_off);
+  const unsigned long long tot = pack2(tt & 0xffffu, 0);
   if (SINGLE) {
     if (threadIdx.x == 0) s_excl = 0;
   } else if (threadIdx.x < 32) {
@@ -1106,22 +1153,24 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
     if (threadIdx.x == 0) s_excl = e;
   }
   __syncthreads();
-  uint32_t pA = unpackA(s_excl + pre);
+  const uint32_t eA = unpackA(s_excl);
+  const unsigned lt = lanemask_lt();
   const unsigned long long tail0 = s_tail0;
   // counters: unmaps, d2h, d2h_av
   uint32_t nUnmap = 0, nD2H = 0, nAv = 0;
   if (!discard_off || kind == DIR_PREFETCH_HOST) {
 #pragma unroll
     for (int k = 0; k < kScanIPT; ++k) {
-      if (first + k >= n) break;
-      const uint32_t bb = lo + first + k;
+      const uint32_t idx = tbase + k * kScanTPB + threadIdx.x;
+      if (idx >= n) continue;
+      const uint32_t bb = lo + idx;
       const uint8_t ss = s[k];
       if (kind == DIR_DISCARD || kind == DIR_DISCARD_LAZY) {
         if (ss == ST_G) {
           T.st[bb] = kind == DIR_DISCARD ? ST_GE : ST_GL;
           T.key[bb] = seq;
+          const uint32_t pA = eA + (s_off[k * NW + w] & 0xffffu) + __popc(bA[k] & lt);
           T.disc_ring[(tail0 + pA) & T.cap_mask] = ((unsigned long long)seq << 32) | bb;
-          ++pA;
           if (kind == DIR_DISCARD) {
             T.map[bb] = UM_NONE;
             ++nUnmap;
@@ -1186,7 +1235,8 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
 // K7: stable compaction of a ring's live entries [head, tail) into `dst` at [0, cnt).
 // ------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(kScanTPB) k_ring_compact(Tables T, int ring, uint64_t* dst) {
-  __shared__ unsigned long long s_scan[kScanTPB / 32];
+  constexpr int NW = kScanTPB / 32;
+  __shared__ uint32_t s_off[kScanIPT * NW + 1];
   __shared__ unsigned long long s_excl, s_head, s_n;
   Ctl* c = T.ctl;
   if (threadIdx.x == 0) {
@@ -1194,37 +1244,41 @@ __global__ void __launch_bounds__(kScanTPB) k_ring_compact(Tables T, int ring, u
     unsigned long long tl = ring == RING_USED ? c->used_tail : c->disc_tail;
     s_n = tl - s_head;
   }
-  const uint32_t tile = take_ticket(T);
+  __syncthreads();
+  const uint32_t tile = blockIdx.x;
   const uint32_t ntiles = gridDim.x;
   const uint64_t* R = ring == RING_USED ? T.used_ring : T.disc_ring;
   const unsigned long long n = s_n, head = s_head;
-  const unsigned long long first = (unsigned long long)tile * kScanTile + threadIdx.x * kScanIPT;
+  const unsigned long long tbase = (unsigned long long)tile * kScanTile;
+  const int w = threadIdx.x >> 5;
   unsigned long long e[kScanIPT];
-  unsigned livem = 0;
-  uint32_t cnt = 0;
+  unsigned bL[kScanIPT], bZ[kScanIPT];
 #pragma unroll
   for (int k = 0; k < kScanIPT; ++k) {
+    const unsigned long long idx = tbase + k * kScanTPB + threadIdx.x;
     e[k] = 0;
-    if (first + k < n) {
-      e[k] = R[(head + first + k) & T.cap_mask];
-      uint32_t blk = (uint32_t)e[k], kk = (uint32_t)(e[k] >> 32);
-      uint8_t ss = T.st[blk];
-      bool live = (ring == RING_USED ? ss == ST_G : (ss == ST_GE || ss == ST_GL)) && T.key[blk] == kk;
-      livem |= (unsigned)live << k;
-      cnt += live;
+    bool live = false;
+    if (idx < n) {
+      e[k] = R[(head + idx) & T.cap_mask];
+      const uint32_t blk = (uint32_t)e[k], kk = (uint32_t)(e[k] >> 32);
+      const uint8_t ss = T.st[blk];
+      live = (ring == RING_USED ? ss == ST_G : (ss == ST_GE || ss == ST_GL)) && T.key[blk] == kk;
     }
+    bL[k] = __ballot_sync(FULL, live);
+    bZ[k] = 0;
   }
-  unsigned long long tot;
-  unsigned long long pre = block_excl_scan<kScanTPB>(pack2(cnt, 0), tot, s_scan);
+  const uint32_t tt = ordered_offsets<kScanTPB, kScanIPT>(bL, bZ, s_off);
+  const unsigned long long tot = pack2(tt & 0xffffu, 0);
   if (threadIdx.x < 32) {
-    unsigned long long e = lookback_warp(T, tile, tot);
-    if (threadIdx.x == 0) s_excl = e;
+    unsigned long long ex = lookback_warp(T, tile, tot);
+    if (threadIdx.x == 0) s_excl = ex;
   }
   __syncthreads();
-  uint32_t p = unpackA(s_excl + pre);
+  const uint32_t eA = unpackA(s_excl);
+  const unsigned lt = lanemask_lt();
 #pragma unroll
   for (int k = 0; k < kScanIPT; ++k)
-    if ((livem >> k) & 1) dst[p++] = e[k];
+    if ((bL[k] >> (threadIdx.x & 31)) & 1) dst[eA + (s_off[k * NW + w] & 0xffffu) + __popc(bL[k] & lt)] = e[k];
   if (tile == ntiles - 1 && threadIdx.x == 0) {
     unsigned long long total = unpackA(s_excl + tot);
     if (ring == RING_USED) { c->used_head = 0; c->used_tail = total; }
