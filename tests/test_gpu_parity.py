@@ -235,11 +235,15 @@ def test_wide_victim_selection(mode):
 
 
 def _full_size_trace(iterations=2):
+    import gc
     import torch
+    gc.collect()
+    torch.cuda.empty_cache()   # the previous full-size test's frames sit in torch's cache
     free, _ = torch.cuda.mem_get_info()
     GiB = 1 << 30
     B = 2 << 20
     budget = min(170 * GiB, free - 6 * GiB) // B * B
+    assert budget >= 160 * GiB, f"only {free / GiB:.1f} GiB free for the full-size case"
     return tg.gen_c3(block_bytes=B, budget_bytes=budget, oversub=1.5, iterations=iterations)
 
 
