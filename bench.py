@@ -344,9 +344,18 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0):
         acc["off"] = blocks.astype(np.uint64) * B
         acc["len"] = B
         acc["kind"] = tg.ACC_READ
+        # a device sleep ahead of each op keeps the GPU behind the host, so every launch
+        # of the op is queued before it runs and the spans hold device time only
+        ps = torch.cuda.ExternalStream(um.um_stream(h))
+
+        def gate():
+            with torch.cuda.stream(ps):
+                torch.cuda._sleep(100_000_000)
         um.um_timing(h, reset=True)
+        gate()
         um.um_touch_batch(h, acc)
         t_touch = um.um_timing(h, reset=True)
+        gate()
         um.um_discard(h, 0, n * B)
         t_disc = um.um_timing(h, reset=True)
         st = um.um_get_stats(h)

@@ -184,6 +184,11 @@ struct um_arena {
   uint64_t* ring_buf[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};  // [ring][buffer]
   int ring_cur[2] = {0, 0};
   uint64_t ub[2] = {0, 0};  // upper bound of (tail - head) per ring
+  // exact ring tails: rings only grow by appends (every block of a GPU sub-op or of a
+  // discard range takes a slot) and compaction keeps the tail, so the host passes the
+  // tail to the appending kernels instead of having them read and publish it
+  uint64_t tail[2] = {0, 0};
+  int npar = 0;             // parity slot of the multi-CTA classify's need counter
   uint32_t B = 0, nblocks = 0, nframes = 0, nhframes = 0;
   cudaStream_t ps = nullptr;
   cudaEvent_t ev_in = nullptr, ev_out = nullptr;
@@ -315,10 +320,33 @@ static bool range_ok(um_arena* a, uint64_t off, uint64_t len) {
 
 // Sorted disjoint intervals with constant write flag from access records.
 static void build_intervals(um_arena* a, const um_access* acc, uint32_t n) {
+  const uint64_t B = a->B;
+  // Fast path (linear): records already in ascending, non-overlapping block order —
+  // e.g. a fault batch sorted by address — are the intervals (adjacent equal-W records
+  // merge).  Anything else goes through the event sort below.
+  {
+    a->ivs.clear();
+    uint64_t prev_hi = 0;
+    bool ok = true;
+    for (uint32_t i = 0; i < n && ok; ++i) {
+      if (!acc[i].len) continue;
+      const uint64_t lo = acc[i].off / B, hi = (acc[i].off + acc[i].len - 1) / B + 1;
+      const uint8_t w = (acc[i].kind & UM_ACC_WRITE) ? 1 : 0;
+      if (!a->ivs.empty() && lo < prev_hi) {
+        ok = false;
+        break;
+      }
+      if (!a->ivs.empty() && prev_hi == lo && a->ivs.back().w == w)
+        a->ivs.back().cnt += (uint32_t)(hi - lo);
+      else
+        a->ivs.push_back({(uint32_t)lo, (uint32_t)(hi - lo), w});
+      prev_hi = hi;
+    }
+    if (ok) return;
+  }
   struct Ev { uint64_t x; int dc, dw; };
   std::vector<Ev> ev;
   ev.reserve(2 * (size_t)n);
-  const uint64_t B = a->B;
   for (uint32_t i = 0; i < n; ++i) {
     if (!acc[i].len) continue;
     uint64_t lo = acc[i].off / B, hi = (acc[i].off + acc[i].len - 1) / B + 1;
@@ -531,22 +559,50 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     iv.wflag = a->stage.dev + off + o_w;
   }
   const uint32_t F = a->nframes;
+  uint32_t jcur = 0;   // interval holding the current item (items ascend across sub-ops)
+  uint64_t pcur = 0;   // its first item
   for (uint64_t g0 = 0; g0 < total; g0 += F) {
     const uint32_t n = (uint32_t)std::min<uint64_t>(F, total - g0);
     const uint32_t seq = ++a->clock;
     a->subops++;
     um_status st = ensure_ring_room(a, RING_USED, n);
     if (st) return st;
+    if (!iv.inl) {
+      // per tile of this sub-op, the interval slice its items fall in: an index the
+      // kernels would otherwise find by a dependent binary search over the staged list
+      const uint32_t tile = n <= kSmallPlan ? kSmallPlan : (uint32_t)kStTile;
+      const uint32_t nt = (n + tile - 1) / tile;
+      uint64_t off;
+      CK(a->stage.reserve(8ull * nt, &off));
+      uint32_t* tj = (uint32_t*)(a->stage.host + off);
+      auto seek = [&](uint64_t g) {
+        while (pcur + a->ivs[jcur].cnt <= g) {
+          pcur += a->ivs[jcur].cnt;
+          ++jcur;
+        }
+        return jcur;
+      };
+      for (uint32_t t = 0; t < nt; ++t) {
+        tj[2 * t] = seek(g0 + (uint64_t)t * tile);
+        tj[2 * t + 1] = seek(g0 + std::min<uint64_t>(n, (uint64_t)(t + 1) * tile) - 1);
+      }
+      CK(a->stage.push(off, 8ull * nt, a->ps));
+      iv.tj = (const uint32_t*)(a->stage.dev + off);
+    }
     cudaEvent_t sp = span_open(a);
+    const uint64_t tail0 = a->tail[RING_USED];
+    a->tail[RING_USED] += n;
     if (n <= kSmallPlan) {
-      CK(launch_plan_small(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
+      CK(launch_plan_small(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->ps));
       a->n_launch += 1;
     } else {
-      CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, a->ps));
+      CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->npar, a->ps));
       if (n > kVictWideMin)
-        CK(launch_victims_wide(a->T, seq, 0, 0, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), n, a->ps));
+        CK(launch_victims_wide(a->T, seq, 0, 0, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), n,
+                               a->npar, a->ps));
       else
-        CK(launch_victims(a->T, seq, 0, 0, a->ps));
+        CK(launch_victims(a->T, seq, 0, 0, a->npar, a->ps));
+      a->npar ^= 1;
       a->n_launch += n > kVictWideMin ? 3 : 2;
     }
     span_close(a, sp, 0);
@@ -758,7 +814,7 @@ UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, v
     if (len) {
       uint32_t lo = (uint32_t)(off / a->B), hi = (uint32_t)((off + len - 1) / a->B + 1);
       cudaEvent_t sp = span_open(a);
-      CK(launch_directive(a->T, DIR_PREFETCH_HOST, lo, hi - lo, seq, 0, a->ps));
+      CK(launch_directive(a->T, DIR_PREFETCH_HOST, lo, hi - lo, seq, 0, a->tail[RING_DISC], a->ps));
       span_close(a, sp, 0);
       const uint32_t nmax = std::min<uint32_t>(hi - lo, a->nframes);
       sp = span_open(a);
@@ -786,13 +842,21 @@ static um_status discard_common(um_arena* a, uint64_t off, uint64_t len, void* s
   const uint32_t seq = ++a->clock;
   const uint64_t lo = (off + a->B - 1) / a->B, hi = (off + len) / a->B;  // fully covered blocks
   if (hi > lo && !(a->cfg.flags & UM_F_DISCARD_OFF)) {
-    const uint32_t n = (uint32_t)(hi - lo);
-    s = ensure_ring_room(a, RING_DISC, std::min<uint32_t>(n, a->nframes));
-    if (s) return s;
-    cudaEvent_t sp = span_open(a);
-    CK(launch_directive(a->T, kind, (uint32_t)lo, n, seq, 0, a->ps));
-    span_close(a, sp, 0);
-    a->n_launch++;
+    // every block of the range takes a DISC slot (k_directive), so a range larger than
+    // the ring's free space after compaction (cap - nframes live entries) is applied in
+    // ascending chunks with the same seq: the ring stays sorted by (dkey, block)
+    const uint64_t chunk = a->L.cap - std::min<uint64_t>(a->nframes, a->L.cap / 2);
+    for (uint64_t c0 = lo; c0 < hi; c0 += chunk) {
+      const uint32_t n = (uint32_t)std::min<uint64_t>(chunk, hi - c0);
+      s = ensure_ring_room(a, RING_DISC, n);
+      if (s) return s;
+      const uint64_t tail0 = a->tail[RING_DISC];
+      a->tail[RING_DISC] += n;
+      cudaEvent_t sp = span_open(a);
+      CK(launch_directive(a->T, kind, (uint32_t)c0, n, seq, 0, tail0, a->ps));
+      span_close(a, sp, 0);
+      a->n_launch++;
+    }
   }
   return hand_out(a, stream);
 }
@@ -817,9 +881,9 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
   if (want) {
     cudaEvent_t sp = span_open(a);
     if (want > kVictWideMin)
-      CK(launch_victims_wide(a->T, seq, 1, (uint32_t)want, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), (uint32_t)want, a->ps));
+      CK(launch_victims_wide(a->T, seq, 1, (uint32_t)want, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), (uint32_t)want, a->npar, a->ps));
     else
-      CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->ps));
+      CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->npar, a->ps));
     a->n_launch += want > kVictWideMin ? 1 : 0;
     span_close(a, sp, 0);
     sp = span_open(a);
@@ -877,7 +941,10 @@ UM_API um_status um_get_stats(um_arena* a, um_stats* out) {
   if (!out) return UM_EINVAL;
   um_status s = sync_ctl(a);
   int64_t v[16];
-  for (int i = 0; i < 16; ++i) v[i] = a->hctl->stats[i];
+  for (int i = 0; i < 16; ++i) {
+    v[i] = 0;
+    for (int j = 0; j < 8; ++j) v[i] += a->hctl->stats[j][i];
+  }
   v[S_OPS] = a->ops;
   v[S_SUBOPS] = a->subops;
   memcpy(out, v, sizeof(um_stats));

@@ -32,10 +32,14 @@ struct Ctl {
   unsigned int scan_ticket, scan_done;  // decoupled look-back tile ticket / completion
   unsigned int app_units;               // D2H-only service completion counter
   unsigned int vict_done;               // wide victim apply completion counter
-  unsigned int pad[2];
+  unsigned int need_acc;                // streaming classify: need-list slots taken so far
+  unsigned int reach_tile;              // wide victim scan: first tile whose inclusive count >= k
   unsigned long long minkeep[2];        // wide victim scan: first kept ring position
   unsigned int k_want;                  // wide victim scan: victims wanted
-  long long stats[S_N];
+  unsigned int need_cnt[2];             // streaming classify: need-list slots, by sub-op parity
+  // counters, striped over 8 cache lines by CTA index (fire-and-forget atomics from
+  // thousands of CTAs do not serialise on one address); the host sums the stripes
+  long long stats[8][S_N];
 };
 
 // One need item's transfer plan (K4-CE path exports these to the host).
@@ -92,6 +96,8 @@ struct OpIv {
   const uint32_t* lo;
   const uint32_t* pre;
   const uint8_t* wflag;
+  const uint32_t* tj;   // staged lists: per tile of the current sub-op, the interval slice
+                        // [tj[2t], tj[2t+1]] its items fall in (host-computed, no search)
   uint32_t m;
   uint32_t inl;
   uint32_t ilo[kIvInline];
@@ -102,6 +108,10 @@ struct OpIv {
 constexpr int kScanTPB = 512;
 constexpr int kScanIPT = 8;
 constexpr int kScanTile = kScanTPB * kScanIPT;
+// streaming state kernels (classify, directives): no inter-CTA ordering, one wave
+constexpr int kStTPB = 256;
+constexpr int kStIPT = 8;
+constexpr int kStTile = kStTPB * kStIPT;
 constexpr int kVictTPB = 1024;
 constexpr int kVictIPT = 4;
 constexpr int kXferStages = 4;
@@ -114,21 +124,23 @@ enum RingId { RING_USED = 0, RING_DISC = 1 };
 // Launch wrappers (um_kernels.cu).  All enqueue on `s`; none synchronizes.
 cudaError_t setup_kernels();
 cudaError_t launch_init(const Tables& T, int nhframes_alloc, cudaStream_t s);
+// tail0: the ring tail before this sub-op's appends (host-tracked, exact); npar: parity
+// slot of the need counter for multi-CTA sub-ops (alternates per multi-CTA sub-op)
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
-                            cudaStream_t s);
-cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, cudaStream_t s);
+                            unsigned long long tail0, int npar, cudaStream_t s);
+cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, int npar, cudaStream_t s);
 // K1+K2+K3 fused in one CTA for sub-ops of <= kSmallPlan blocks
 constexpr uint32_t kSmallPlan = 4096;
 cudaError_t launch_plan_small(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
-                              cudaStream_t s);
+                              unsigned long long tail0, cudaStream_t s);
 // multi-CTA victim selection for large sub-ops (scan bound = max ring entries to scan)
 cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, uint32_t want,
-                                uint64_t scan_bound, uint32_t max_victims, cudaStream_t s);
+                                uint64_t scan_bound, uint32_t max_victims, int npar, cudaStream_t s);
 constexpr uint32_t kVictWideMin = 8192;
 cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max_items, cudaStream_t s);
 cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, cudaStream_t s);
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
-                             int discard_off, cudaStream_t s);
+                             int discard_off, unsigned long long tail0, cudaStream_t s);
 cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64_t cap_bound, cudaStream_t s);
 cudaError_t launch_host_write(const Tables& T, uint32_t lo, uint32_t n, uint32_t seq, cudaStream_t s);
 cudaError_t launch_tags(const Tables& T, cudaStream_t s);

@@ -9,6 +9,7 @@
 #include "um_internal.h"
 
 #include <cstdio>
+#include <cstdlib>
 
 namespace um {
 
@@ -21,6 +22,16 @@ __constant__ int c_dummy;
 // ------------------------------------------------------------------------------------
 __device__ __forceinline__ char* hptr(const Tables& T, uint32_t hf) {
   return T.hchunks[hf / T.hpc] + (size_t)(hf % T.hpc) * T.B;
+}
+
+// Programmatic dependent launch (PDL): every paging-stream kernel lets its successor be
+// scheduled as soon as all of its own CTAs are running (launch_dependents), and waits for
+// its predecessor's completion and memory (griddepcontrol.wait) before touching state.
+// The successor's launch latency then overlaps this kernel's execution.  Both are no-ops
+// for a kernel launched without the PDL attribute.
+__device__ __forceinline__ void pdl_enter() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -42,7 +53,7 @@ __device__ __forceinline__ uint32_t iv_find(const OpIv& iv, uint32_t g) {
 }
 
 __device__ __forceinline__ void stat_add(const Tables& T, int slot, long long v) {
-  if (v) atomicAdd((unsigned long long*)&T.ctl->stats[slot], (unsigned long long)v);
+  if (v) atomicAdd((unsigned long long*)&T.ctl->stats[blockIdx.x & 7][slot], (unsigned long long)v);
 }
 
 // Exclusive block scan of a 64-bit value (two packed 31-bit counts add without carry).
@@ -272,7 +283,11 @@ __global__ void k_init(Tables T, int nh) {
     c->scan_ticket = c->scan_done = c->app_units = c->vict_done = 0;
     c->minkeep[0] = c->minkeep[1] = ~0ull;
     c->k_want = 0;
-    for (int i = 0; i < S_N; ++i) c->stats[i] = 0;
+    c->need_acc = 0;
+    c->reach_tile = ~0u;
+    for (int j = 0; j < 8; ++j)
+      for (int i = 0; i < S_N; ++i) c->stats[j][i] = 0;
+    c->need_cnt[0] = c->need_cnt[1] = 0;
   }
 }
 
@@ -339,54 +354,44 @@ __device__ __forceinline__ unsigned lanemask_lt() {
   return m;
 }
 
-// SINGLE: the whole sub-op is one tile (one CTA) -> no ticket, no look-back, counters
-// added directly (saves the dependent global round trips of the multi-CTA protocol).
-template <int TPB, int IPT, bool SINGLE = false>
-__device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
-                                              int touch) {
+// K1/K2 for a sub-op that fits one CTA (k_plan_small): classify, pin, list the blocks
+// needing a frame in ascending order, and give every block of the sub-op its USED slot
+// tail0 + (its rank in the sub-op) -- the same dead-slot rule as the streaming kernel
+// below, so the host knows every ring tail exactly.
+template <int TPB, int IPT>
+__device__ __forceinline__ void classify_single(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
+                                                int touch, unsigned long long tail0) {
   constexpr int TILE = TPB * IPT, NW = TPB / 32;
   __shared__ uint32_t s_off[IPT * NW + 1];
-  __shared__ unsigned long long s_excl;
-  __shared__ unsigned long long s_tail0;
   __shared__ uint32_t s_cnt[6];
-  // the tile's slice of the interval list (<= TILE intervals), staged in smem so the
+  // the sub-op's slice of the interval list (<= TILE intervals), staged in smem so the
   // per-item interval search runs in shared memory
   __shared__ uint32_t s_lo[TILE], s_pre[TILE + 1];
   __shared__ uint32_t s_j0, s_m;
-  const uint32_t tile = SINGLE ? 0u : blockIdx.x;
-  const uint32_t ntiles = SINGLE ? 1u : gridDim.x;
-  const uint32_t tbase = tile * TILE;
   const int w = threadIdx.x >> 5;
   if (threadIdx.x == 0) {
-    s_tail0 = T.ctl->used_tail;
-    if (tbase < n) {
-      const uint32_t ja = iv_find(iv, g0 + tbase);
-      const uint32_t jb = iv_find(iv, g0 + min(n, tbase + TILE) - 1);
-      s_j0 = ja;
-      s_m = jb - ja + 1;
-    }
+    const uint32_t ja = iv.inl ? iv_find(iv, g0) : iv.tj[0];
+    const uint32_t jb = iv.inl ? iv_find(iv, g0 + n - 1) : iv.tj[1];
+    s_j0 = ja;
+    s_m = jb - ja + 1;
   }
   __syncthreads();
-  if (tbase < n) {
-    const uint32_t j0 = s_j0, m = s_m;
-    for (uint32_t q = threadIdx.x; q < m; q += blockDim.x) {
-      s_lo[q] = iv_lo(iv, j0 + q);
-      s_pre[q] = iv_pre(iv, j0 + q);
-    }
-    if (threadIdx.x == 0) s_pre[m] = iv_pre(iv, j0 + m);
+  const uint32_t j0 = s_j0, m = s_m;
+  for (uint32_t q = threadIdx.x; q <= m; q += blockDim.x) {
+    if (q < m) s_lo[q] = iv_lo(iv, j0 + q);
+    s_pre[q] = iv_pre(iv, j0 + q);
   }
   __syncthreads();
-
+  const unsigned long long kseq = (unsigned long long)seq << 32;
   uint32_t b[IPT];
   uint8_t s[IPT];
-  unsigned bN[IPT], bR[IPT];
-  uint32_t cls[6] = {0, 0, 0, 0, 0, 0};
+  unsigned bN[IPT];
+  uint32_t cls = 0;   // 4 bits per class U H HD G GE GL
   uint32_t jlo = 0;
-  const uint32_t m = tbase < n ? s_m : 0u;
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
-    const uint32_t idx = tbase + k * TPB + threadIdx.x;
-    bool nd = false, rk = false;
+    const uint32_t idx = k * TPB + threadIdx.x;
+    bool nd = false;
     b[k] = 0;
     s[k] = 0xff;
     if (idx < n) {
@@ -400,88 +405,225 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
       const uint32_t bb = s_lo[lo] + (g - s_pre[lo]);
       const uint8_t ss = T.st[bb];
       T.pin[bb] = seq;
+      T.used_ring[(tail0 + idx) & T.cap_mask] = kseq | bb;
       b[k] = bb;
       s[k] = ss;
       nd = ss <= ST_HD;
-      rk = touch ? (nd || ss == ST_GE) : true;
-      cls[ss]++;
+      cls += 1u << (4 * ss);
     }
     bN[k] = __ballot_sync(FULL, nd);
-    bR[k] = __ballot_sync(FULL, rk);
   }
-  const uint32_t tt = ordered_offsets<TPB, IPT>(bN, bR, s_off);
-  const unsigned long long tot = pack2(tt & 0xffffu, tt >> 16);
-  if (SINGLE) {
-    if (threadIdx.x == 0) s_excl = 0;
-  } else if (threadIdx.x < 32) {
-    unsigned long long e = lookback_warp(T, tile, tot);
-    if (threadIdx.x == 0) s_excl = e;
-  }
-  __syncthreads();
-  const uint32_t eN = unpackA(s_excl), eR = unpackB(s_excl);
-  const unsigned long long tail0 = s_tail0;
+  const uint32_t tt = ordered_offsets<TPB, IPT>(bN, bN, s_off);
   const unsigned lt = lanemask_lt();
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
-    const uint32_t idx = tbase + k * TPB + threadIdx.x;
+    const uint32_t idx = k * TPB + threadIdx.x;
     if (idx >= n) continue;
     const uint32_t bb = b[k];
     const uint8_t ss = s[k];
-    const bool nd = (bN[k] >> (threadIdx.x & 31)) & 1, rk = (bR[k] >> (threadIdx.x & 31)) & 1;
-    const uint32_t off = s_off[k * NW + w];
-    if (nd) {
-      const uint32_t pN = eN + (off & 0xffffu) + __popc(bN[k] & lt);
+    if ((bN[k] >> (threadIdx.x & 31)) & 1) {
+      const uint32_t pN = (s_off[k * NW + w] & 0xffffu) + __popc(bN[k] & lt);
       T.need[pN] = bb;
       T.needk[pN] = ss;
       T.needhf[pN] = (ss == ST_H) ? T.hframe[bb] : UM_NONE;
-    }
-    if (rk) {
-      const uint32_t pR = eR + (off >> 16) + __popc(bR[k] & lt);
-      T.used_ring[(tail0 + pR) & T.cap_mask] = ((unsigned long long)seq << 32) | bb;
-      if (!nd) {
-        T.key[bb] = seq;
-        if (ss == ST_GE) {        // revive: re-map the frame kept since the discard
-          T.st[bb] = ST_G;
-          T.map[bb] = T.frame_of[bb];
-        } else if (ss == ST_GL) { // revalidate: mapping was kept (lazy)
-          T.st[bb] = ST_G;
-        }
-      }
+    } else if (ss == ST_GE) {   // revive: re-map the frame kept since the discard (L229)
+      T.st[bb] = ST_G;
+      T.key[bb] = seq;
+      T.map[bb] = T.frame_of[bb];
+    } else if (!touch) {
+      T.key[bb] = seq;          // refresh (G) / revalidate (GL -> G, L190)
+      if (ss == ST_GL) T.st[bb] = ST_G;
     }
   }
   // counters (classes: U H HD G GE GL)
   const long long B = T.B;
+  const uint32_t c0 = cls & 15u, c1 = (cls >> 4) & 15u, c2 = (cls >> 8) & 15u, c3 = (cls >> 12) & 15u,
+                 c4 = (cls >> 16) & 15u, c5 = (cls >> 20) & 15u;
   uint32_t v[6];
   if (touch) {
     // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE ; h2d: H ; zf: U+HD ; h2d_av: HD
-    v[0] = cls[0] + cls[1] + cls[2] + cls[4]; v[1] = cls[3] + cls[5]; v[2] = cls[4];
+    v[0] = c0 + c1 + c2 + c4; v[1] = c3 + c5; v[2] = c4;
   } else {
-    v[0] = cls[3]; v[1] = cls[4]; v[2] = cls[5];
+    v[0] = c3; v[1] = c4; v[2] = c5;
   }
-  v[3] = cls[1]; v[4] = cls[0] + cls[2]; v[5] = cls[2];
+  v[3] = c1; v[4] = c0 + c2; v[5] = c2;
   const int slots_t[6] = {S_FAULTS, S_HITS, S_REMAPS, S_H2D, S_ZF, S_H2D_AV};
   const int slots_p[6] = {S_REFRESH, S_REMAPS, S_REVAL, S_H2D, S_ZF, S_H2D_AV};
   const long long mul[6] = {1, 1, 1, B, B, B};
-  if (SINGLE) {
-    if (threadIdx.x == 0) {
-      T.ctl->n_need = unpackA(tot);
-      T.ctl->n_rekey = unpackB(tot);
-    }
-    block_counts_to<6>(T, v, s_cnt, touch ? slots_t : slots_p, mul);
-    return;
+  if (threadIdx.x == 0) {
+    T.ctl->n_need = tt & 0xffffu;
+    T.ctl->n_rekey = n;
   }
-  tile_counts<6>(T, tile, v, s_cnt);
-  if (tile == ntiles - 1 && threadIdx.x == 0) {
-    unsigned long long all = s_excl + tot;
-    T.ctl->n_need = unpackA(all);
-    T.ctl->n_rekey = unpackB(all);
-  }
-  scan_finish<6>(T, ntiles, touch ? slots_t : slots_p, mul);
+  block_counts_to<6>(T, v, s_cnt, touch ? slots_t : slots_p, mul);
 }
 
-__global__ void __launch_bounds__(kScanTPB) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
-                                                       int touch) {
-  classify_body<kScanTPB, kScanIPT>(T, iv, g0, n, seq, touch);
+// ------------------------------------------------------------------------------------
+// Streaming K1/K2 for multi-CTA sub-ops: no inter-CTA ordering at all.
+//  * USED: every block of the sub-op gets the slot used_tail + (its rank in the sub-op)
+//    with entry (seq, b), rekeyed or not.  The rank is the block's position in the
+//    sorted distinct list, so the slots are in ascending block order; an entry whose
+//    block does not take key = seq in state G here is dead by the liveness rule
+//    (st == G && key == entry key) and stays dead, since seq is never reissued.
+//  * need list: its order is not observable (frame ids and the victim<->newcomer
+//    pairing are internal), so slots come from one atomic per CTA.
+//  * counters: per-tile partials summed by the last CTA (no same-address atomics).
+// ------------------------------------------------------------------------------------
+
+// Exclusive CTA scan of one 32-bit count per thread; returns the prefix, total in `tot`.
+template <int TPB>
+__device__ __forceinline__ uint32_t cta_excl_scan(uint32_t v, uint32_t& tot, uint32_t* sm /*[TPB/32]*/) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) sm[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t t = lane < TPB / 32 ? sm[lane] : 0u;
+    uint32_t ti = t;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(FULL, ti, o);
+      if (lane >= o) ti += y;
+    }
+    if (lane < TPB / 32) sm[lane] = ti - t;   // exclusive warp offsets
+    if (lane == TPB / 32 - 1) sm[TPB / 32] = ti;
+  }
+  __syncthreads();
+  const uint32_t pre = sm[w] + x - v;
+  tot = sm[TPB / 32];
+  __syncthreads();
+  return pre;
+}
+
+// Last-CTA epilogue of a streaming launch: the CTA that finishes last (completion
+// ticket) sums the per-tile counter partials and adds them once.  Returns true in
+// that CTA (uniformly), so the caller can publish launch-wide results.
+template <int NC>
+__device__ bool grid_finish(const Tables& T, const int (&slots)[NC], const long long (&mul)[NC]) {
+  __shared__ int s_last;
+  __shared__ unsigned long long s_sum[NC];
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(&T.ctl->scan_done, 1u) == gridDim.x - 1;
+  }
+  if (threadIdx.x < NC) s_sum[threadIdx.x] = 0;
+  __syncthreads();
+  if (!s_last) return false;
+  __threadfence();
+  const uint32_t nt = gridDim.x;
+  for (int k = 0; k < NC; ++k) {
+    unsigned long long acc = 0;
+    for (uint32_t t = threadIdx.x; t < nt; t += blockDim.x) acc += ((volatile uint32_t*)T.tile_cnt)[t * 8 + k];
+    for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
+    if ((threadIdx.x & 31) == 0 && acc) atomicAdd(&s_sum[k], acc);
+  }
+  __syncthreads();
+  if (threadIdx.x < NC && slots[threadIdx.x] >= 0) stat_add(T, slots[threadIdx.x], (long long)s_sum[threadIdx.x] * mul[threadIdx.x]);
+  if (threadIdx.x == 0) T.ctl->scan_done = 0;
+  return true;
+}
+
+__global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
+                                                        int touch, unsigned long long tail0, int npar) {
+  pdl_enter();
+  constexpr int TPB = kStTPB, IPT = kStIPT, TILE = kStTile;
+  __shared__ uint32_t s_lo[TILE], s_pre[TILE + 1];
+  __shared__ uint32_t s_j0, s_m, s_base;
+  __shared__ uint32_t s_sc[TPB / 32 + 1];
+  __shared__ uint32_t s_cnt[8];
+  const uint32_t tile = blockIdx.x, tbase = tile * TILE;
+  if (threadIdx.x == 0) {
+    const uint32_t ja = iv.inl ? iv_find(iv, g0 + tbase) : iv.tj[2 * tile];
+    const uint32_t jb = iv.inl ? iv_find(iv, g0 + min(n, tbase + TILE) - 1) : iv.tj[2 * tile + 1];
+    s_j0 = ja;
+    s_m = jb - ja + 1;
+  }
+  __syncthreads();
+  const uint32_t j0 = s_j0, m = s_m;
+  for (uint32_t q = threadIdx.x; q <= m; q += TPB) {
+    if (q < m) s_lo[q] = iv_lo(iv, j0 + q);
+    s_pre[q] = iv_pre(iv, j0 + q);
+  }
+  __syncthreads();
+  const unsigned long long kseq = (unsigned long long)seq << 32;
+  uint32_t b[IPT];
+  uint8_t s[IPT];
+  uint32_t cls = 0;   // per-class counts (<= IPT < 16 each), 4 bits per class U H HD G GE GL
+  uint32_t nneed = 0, jlo = 0;
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) {
+    const uint32_t idx = tbase + k * TPB + threadIdx.x;
+    s[k] = 0xff;
+    b[k] = 0;
+    if (idx < n) {
+      const uint32_t g = g0 + idx;
+      uint32_t lo = jlo, hi = m;   // largest j with s_pre[j] <= g (a thread's items ascend)
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (s_pre[mid] <= g) lo = mid; else hi = mid;
+      }
+      jlo = lo;
+      const uint32_t bb = s_lo[lo] + (g - s_pre[lo]);
+      b[k] = bb;
+      s[k] = T.st[bb];
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) {
+    const uint32_t idx = tbase + k * TPB + threadIdx.x;
+    if (idx < n) {
+      T.pin[b[k]] = seq;
+      T.used_ring[(tail0 + idx) & T.cap_mask] = kseq | b[k];
+      nneed += s[k] <= ST_HD;
+      cls += 1u << (4 * s[k]);
+    }
+  }
+  uint32_t tot;
+  const uint32_t pre = cta_excl_scan<TPB>(nneed, tot, s_sc);
+  if (threadIdx.x == 0) s_base = tot ? atomicAdd(&T.ctl->need_cnt[npar], tot) : 0u;
+  __syncthreads();
+  uint32_t pos = s_base + pre;
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) {
+    const uint8_t ss = s[k];
+    if (ss == 0xff) continue;
+    const uint32_t bb = b[k];
+    if (ss <= ST_HD) {
+      T.need[pos] = bb;
+      T.needk[pos] = ss;
+      T.needhf[pos] = ss == ST_H ? T.hframe[bb] : UM_NONE;
+      ++pos;
+    } else if (ss == ST_GE) {      // revive: re-map the frame kept since the discard (L229)
+      T.st[bb] = ST_G;
+      T.key[bb] = seq;
+      T.map[bb] = T.frame_of[bb];
+    } else if (!touch) {
+      T.key[bb] = seq;             // refresh (G) / revalidate (GL -> G, L190)
+      if (ss == ST_GL) T.st[bb] = ST_G;
+    }
+  }
+  // counters (classes: U H HD G GE GL)
+  const long long B = T.B;
+  const uint32_t c0 = cls & 15u, c1 = (cls >> 4) & 15u, c2 = (cls >> 8) & 15u, c3 = (cls >> 12) & 15u,
+                 c4 = (cls >> 16) & 15u, c5 = (cls >> 20) & 15u;
+  uint32_t v[6];
+  if (touch) {
+    // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE
+    v[0] = c0 + c1 + c2 + c4; v[1] = c3 + c5; v[2] = c4;
+  } else {
+    v[0] = c3; v[1] = c4; v[2] = c5;   // refreshes, remaps, revalidations
+  }
+  v[3] = c1; v[4] = c0 + c2; v[5] = c2;   // h2d, zf, h2d_avoided
+  const int slots_t[6] = {S_FAULTS, S_HITS, S_REMAPS, S_H2D, S_ZF, S_H2D_AV};
+  const int slots_p[6] = {S_REFRESH, S_REMAPS, S_REVAL, S_H2D, S_ZF, S_H2D_AV};
+  const long long mul[6] = {1, 1, 1, B, B, B};
+  block_counts_to<6>(T, v, s_cnt, touch ? slots_t : slots_p, mul);
+  if (blockIdx.x == 0 && threadIdx.x == 0) T.ctl->n_rekey = n;   // USED slots appended
 }
 
 // ------------------------------------------------------------------------------------
@@ -640,15 +782,25 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
   }
 }
 
-__global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, int evict_mode, uint32_t want) {
+__global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, int evict_mode, uint32_t want,
+                                                      int npar) {
+  pdl_enter();
+  if (!evict_mode && threadIdx.x == 0) {
+    // publish the streaming classify's need count; clear the other parity slot for the
+    // next multi-CTA sub-op (nothing reads it until then)
+    T.ctl->n_need = T.ctl->need_cnt[npar];
+    T.ctl->need_cnt[npar ^ 1] = 0;
+  }
+  __syncthreads();
   victims_body(T, seq, evict_mode, want);
 }
 
 // K1+K2+K3 for a sub-op that fits one tile: one CTA classifies, compacts and selects
 // victims (saves a launch per small op; same code as the multi-CTA kernels).
 __global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
-                                                         int touch) {
-  classify_body<kVictTPB, kSmallPlan / kVictTPB, true>(T, iv, g0, n, seq, touch);
+                                                         int touch, unsigned long long tail0) {
+  pdl_enter();
+  classify_single<kVictTPB, kSmallPlan / kVictTPB>(T, iv, g0, n, seq, touch, tail0);
   __syncthreads();
   __threadfence_block();
   victims_body(T, seq, 0, 0);
@@ -656,17 +808,26 @@ __global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, OpIv iv, uint
 
 // ------------------------------------------------------------------------------------
 // K3 (wide): the same victim rule for large sub-ops, over all SMs.  Pass 1 scans the
-// concatenation DISC[head,tail) ++ USED[head,tail) in tiles: candidates (live, not
-// pinned) are ranked with a block scan + decoupled look-back, rank < k are the victims
-// (exactly the first k in queue order), and the first kept position of each ring is
-// found with atomicMin.  Pass 2 reclaims the victims in parallel (host frames for
-// write-backs come from the free stack by atomic pop; ids are not observable).
+// concatenation DISC[head,tail) ++ USED[head,tail) in tiles taken in ascending order
+// from a ticket by a persistent grid (all CTAs resident): candidates (live, not pinned)
+// are ranked with a block scan + decoupled look-back, rank < k are the victims (exactly
+// the first k in queue order).  The first tile whose inclusive count reaches k is
+// recorded; tiles fetched after that is known are not read at all (their status is
+// published as "k reached"), so a scan stops soon after its k-th candidate instead of
+// reading the whole ring.  Ring heads may advance over examined dead/consumed entries
+// only: the first kept live entry, or the first entry of an unexamined tile, bounds
+// them.  Pass 2 reclaims the victims in parallel (host frames for write-backs come
+// from the free stack, one atomic per CTA chunk; ids are not observable).
 // ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want) {
+__global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want,
+                                                            int npar) {
+  pdl_enter();
   constexpr int NW = kScanTPB / 32;
+  const unsigned long long FP = 2ull << 62;
   __shared__ uint32_t s_off[kScanIPT * NW + 1];
   __shared__ unsigned long long s_excl, s_dh, s_ld, s_uh, s_lu, s_mk[2];
-  __shared__ uint32_t s_k;
+  __shared__ uint32_t s_k, s_nn, s_f0, s_tile, s_skip;
+  __shared__ int s_last;
   Ctl* c = T.ctl;
   if (threadIdx.x == 0) {
     s_dh = c->disc_head;
@@ -674,63 +835,97 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
     s_uh = c->used_head;
     s_lu = c->used_tail - c->used_head;
     const uint32_t f0 = (uint32_t)c->free_top;
-    const uint32_t nn = evict_mode ? want : c->n_need;
+    const uint32_t nn = evict_mode ? want : c->need_cnt[npar];
     s_k = nn > f0 ? nn - f0 : 0u;
+    s_nn = nn;
+    s_f0 = f0;
     s_mk[0] = s_mk[1] = ~0ull;
+    if (blockIdx.x == 0 && !evict_mode) {
+      c->n_need = nn;              // publish the streaming classify's need count
+      c->need_cnt[npar ^ 1] = 0;   // and clear the other parity slot (read by no one now)
+    }
   }
   __syncthreads();
-  const uint32_t tile = blockIdx.x;
-  const uint32_t ntiles = gridDim.x;
   const unsigned long long L = s_ld + s_lu;
   const uint32_t k = s_k;
-  const unsigned long long tbase = (unsigned long long)tile * kScanTile;
+  const uint32_t ntiles = k ? (uint32_t)((L + kScanTile - 1) / kScanTile) : 0u;
   const int w = threadIdx.x >> 5;
-  uint32_t bb[kScanIPT];
-  unsigned bC[kScanIPT], bL[kScanIPT];
-#pragma unroll
-  for (int q = 0; q < kScanIPT; ++q) {
-    bb[q] = 0;
-    bool live = false, cand = false;
-    const unsigned long long idx = tbase + q * kScanTPB + threadIdx.x;
-    if (k && idx < L) {
-      const bool disc = idx < s_ld;
-      const unsigned long long pos = disc ? s_dh + idx : s_uh + (idx - s_ld);
-      const unsigned long long e = (disc ? T.disc_ring : T.used_ring)[pos & T.cap_mask];
-      const uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
-      const uint8_t ss = T.st[blk];
-      live = (disc ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) && T.key[blk] == kk;
-      cand = live && T.pin[blk] != seq;
-      bb[q] = blk;
-    }
-    bC[q] = __ballot_sync(FULL, cand);
-    bL[q] = __ballot_sync(FULL, live);
-  }
-  const uint32_t tt = ordered_offsets<kScanTPB, kScanIPT>(bC, bC, s_off);
-  const unsigned long long tot = pack2(tt & 0xffffu, 0);
-  if (threadIdx.x < 32) {
-    unsigned long long ex = lookback_warp(T, tile, tot);
-    if (threadIdx.x == 0) s_excl = ex;
-  }
-  __syncthreads();
-  const uint32_t eC = unpackA(s_excl);
   const unsigned lt = lanemask_lt();
   const unsigned me = 1u << (threadIdx.x & 31);
   unsigned long long mk0 = ~0ull, mk1 = ~0ull;
+  while (true) {
+    if (threadIdx.x == 0) {
+      const uint32_t t = atomicAdd(&c->scan_ticket, 1u);
+      s_tile = t;
+      s_skip = t >= ntiles ? 2u : (*(volatile uint32_t*)&c->reach_tile < t ? 1u : 0u);
+    }
+    __syncthreads();
+    const uint32_t tile = s_tile, skip = s_skip;
+    __syncthreads();
+    if (skip == 2u) break;
+    const unsigned long long tbase = (unsigned long long)tile * kScanTile;
+    if (skip == 1u) {
+      // every later ticket skips as well, so this CTA is done
+      if (threadIdx.x == 0) {
+        ((volatile unsigned long long*)T.tile_status)[tile] = FP | pack2(k, 0);
+        __threadfence();
+        if (tbase < s_ld) {
+          mk0 = min(mk0, s_dh + tbase);
+          mk1 = min(mk1, s_uh);
+        } else {
+          mk1 = min(mk1, s_uh + (tbase - s_ld));
+        }
+      }
+      break;
+    }
+    uint32_t bb[kScanIPT];
+    unsigned bC[kScanIPT], bL[kScanIPT];
 #pragma unroll
-  for (int q = 0; q < kScanIPT; ++q) {
-    bool sel = false;
-    if (bC[q] & me) {
-      const uint32_t r = eC + (s_off[q * NW + w] & 0xffffu) + __popc(bC[q] & lt);
-      if (r < k) {
-        T.victim[r] = bb[q];
-        sel = true;
+    for (int q = 0; q < kScanIPT; ++q) {
+      bb[q] = 0;
+      bool live = false, cand = false;
+      const unsigned long long idx = tbase + q * kScanTPB + threadIdx.x;
+      if (idx < L) {
+        const bool disc = idx < s_ld;
+        const unsigned long long pos = disc ? s_dh + idx : s_uh + (idx - s_ld);
+        const unsigned long long e = (disc ? T.disc_ring : T.used_ring)[pos & T.cap_mask];
+        const uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
+        const uint8_t ss = T.st[blk];
+        live = (disc ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) && T.key[blk] == kk;
+        cand = live && T.pin[blk] != seq;
+        bb[q] = blk;
+      }
+      bC[q] = __ballot_sync(FULL, cand);
+      bL[q] = __ballot_sync(FULL, live);
+    }
+    const uint32_t tt = ordered_offsets<kScanTPB, kScanIPT>(bC, bC, s_off);
+    const unsigned long long tot = pack2(tt & 0xffffu, 0);
+    if (threadIdx.x < 32) {
+      unsigned long long ex = lookback_warp(T, tile, tot);
+      if (threadIdx.x == 0) {
+        s_excl = ex;
+        if (unpackA(ex) + unpackA(tot) >= k) atomicMin(&c->reach_tile, tile);
       }
     }
-    if ((bL[q] & me) && !sel) {
-      const unsigned long long idx = tbase + q * kScanTPB + threadIdx.x;
-      if (idx < s_ld) mk0 = min(mk0, s_dh + idx);
-      else mk1 = min(mk1, s_uh + (idx - s_ld));
+    __syncthreads();
+    const uint32_t eC = unpackA(s_excl);
+#pragma unroll
+    for (int q = 0; q < kScanIPT; ++q) {
+      bool sel = false;
+      if (bC[q] & me) {
+        const uint32_t r = eC + (s_off[q * NW + w] & 0xffffu) + __popc(bC[q] & lt);
+        if (r < k) {
+          T.victim[r] = bb[q];
+          sel = true;
+        }
+      }
+      if ((bL[q] & me) && !sel) {
+        const unsigned long long idx = tbase + q * kScanTPB + threadIdx.x;
+        if (idx < s_ld) mk0 = min(mk0, s_dh + idx);
+        else mk1 = min(mk1, s_uh + (idx - s_ld));
+      }
     }
+    __syncthreads();
   }
   if (mk0 != ~0ull) atomicMin(&s_mk[0], mk0);
   if (mk1 != ~0ull) atomicMin(&s_mk[1], mk1);
@@ -738,88 +933,122 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
   if (threadIdx.x == 0) {
     if (s_mk[0] != ~0ull) atomicMin(&c->minkeep[0], s_mk[0]);
     if (s_mk[1] != ~0ull) atomicMin(&c->minkeep[1], s_mk[1]);
+    __threadfence();
+    s_last = atomicAdd(&c->scan_done, 1u) == gridDim.x - 1;
   }
-  if (tile == ntiles - 1 && threadIdx.x == 0) {
-    c->n_vict = min(k, unpackA(s_excl + tot));
-    c->k_want = k;
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    const uint32_t fetched = min(ntiles, *(volatile uint32_t*)&c->scan_ticket);
+    for (uint32_t i = threadIdx.x; i < fetched; i += blockDim.x) T.tile_status[i] = 0ull;
+    if (threadIdx.x == 0) {
+      const uint32_t reach = *(volatile uint32_t*)&c->reach_tile;
+      uint32_t found = 0;
+      if (k) found = reach != ~0u ? k : unpackA(((volatile unsigned long long*)T.tile_status)[ntiles - 1] & ((1ull << 62) - 1));
+      found = min(k, found);
+      // victim bookkeeping for the apply pass (which reads f0 / n_vict only)
+      c->n_vict = found;
+      stat_add(T, S_EVICT, found);
+      if (k) {
+        const unsigned long long m0 = *(volatile unsigned long long*)&c->minkeep[0];
+        const unsigned long long m1 = *(volatile unsigned long long*)&c->minkeep[1];
+        c->disc_head = m0 != ~0ull ? m0 : c->disc_tail;
+        c->used_head = m1 != ~0ull ? m1 : c->used_tail;
+      }
+      c->minkeep[0] = c->minkeep[1] = ~0ull;
+      const int f0 = (int)s_f0;
+      c->f0 = (uint32_t)f0;
+      if (evict_mode) {
+        c->free_top = f0 + (int)found;
+      } else {
+        c->free_top = f0 - (int)min((uint32_t)f0, s_nn);
+        c->used_tail += c->n_rekey;
+      }
+      c->scan_ticket = 0;
+      c->scan_done = 0;
+      c->reach_tile = ~0u;
+    }
+    __threadfence();
   }
-  scan_finish(T, ntiles);
 }
 
 __global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode) {
-  __shared__ uint32_t s_cnt[4];
-  __shared__ int s_last;
+  pdl_enter();
+  constexpr int TPB = 256;
+  __shared__ uint32_t s_cnt[8];
+  __shared__ unsigned long long s_sc[TPB / 32];
+  __shared__ int s_hb;
+  __shared__ uint32_t s_hav, s_db;
   Ctl* c = T.ctl;
   const uint32_t found = c->n_vict;
-  const int f0 = c->free_top;
+  const int f0 = (int)c->f0;   // free_top when the victims were chosen (set by the scan)
+  // contiguous chunk of victims per CTA; one host-frame pop (and D2H-list append) per
+  // 256 victims instead of one same-address atomic per victim
+  const uint32_t j0 = (uint32_t)((unsigned long long)found * blockIdx.x / gridDim.x);
+  const uint32_t j1 = (uint32_t)((unsigned long long)found * (blockIdx.x + 1) / gridDim.x);
   uint32_t nG = 0, nAv = 0, nGL = 0;
-  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < found; j += gridDim.x * blockDim.x) {
-    const uint32_t v = T.victim[j];
-    const uint8_t ss = T.st[v];
-    const uint32_t fr = T.frame_of[v];
-    const bool isG = ss == ST_G;
-    uint32_t hf = UM_NONE;
-    if (isG) {
-      if (!evict_mode && T.needk[(uint32_t)f0 + j] == ST_H) hf = T.needhf[(uint32_t)f0 + j];
-      if (hf == UM_NONE) {
-        int idx = atomicSub(&c->hfree_top, 1) - 1;
-        if (idx >= 0) {
-          hf = T.hfree_stack[idx];
-        } else {
-          atomicAdd(&c->hfree_top, 1);
-          atomicExch(&c->err, 2u);
+  for (uint32_t base = j0; base < j1; base += TPB) {
+    const uint32_t j = base + threadIdx.x;
+    uint32_t v = 0, fr = UM_NONE, hf = UM_NONE;
+    uint8_t ss = 0;
+    bool isG = false, needA = false;
+    if (j < j1) {
+      v = T.victim[j];
+      ss = T.st[v];
+      fr = T.frame_of[v];
+      isG = ss == ST_G;
+      if (isG && !evict_mode && T.needk[(uint32_t)f0 + j] == ST_H) hf = T.needhf[(uint32_t)f0 + j];
+      needA = isG && hf == UM_NONE;
+    }
+    unsigned long long tot;
+    const unsigned long long pre = block_excl_scan<TPB>(pack2(needA, evict_mode && isG), tot, s_sc);
+    if (threadIdx.x == 0) {
+      const uint32_t tA = unpackA(tot), tD = unpackB(tot);
+      s_hb = 0;
+      s_hav = 0;
+      if (tA) {
+        const int old = atomicSub(&c->hfree_top, (int)tA);
+        const int avail = old < 0 ? 0 : (old < (int)tA ? old : (int)tA);
+        if (avail < (int)tA) {
+          atomicAdd(&c->hfree_top, (int)tA - avail);
+          atomicExch(&c->err, 2u);   // host-frame pool exhausted -> UM_ENOMEM
+        }
+        s_hb = old;
+        s_hav = (uint32_t)avail;
+      }
+      s_db = tD ? atomicAdd(&c->n_d2h, tD) : 0u;
+    }
+    __syncthreads();
+    if (j < j1) {
+      if (needA) {
+        const uint32_t r = unpackA(pre);
+        hf = r < s_hav ? T.hfree_stack[s_hb - 1 - (int)r] : UM_NONE;
+      }
+      T.vframe[j] = fr;
+      T.vkind[j] = ss;
+      T.vhf[j] = hf;
+      T.st[v] = isG ? ST_H : ST_HD;
+      T.map[v] = UM_NONE;
+      T.frame_of[v] = UM_NONE;
+      T.hframe[v] = hf;
+      nG += isG;
+      nAv += !isG;
+      nGL += ss == ST_GL;
+      if (evict_mode) {
+        T.free_stack[f0 + j] = fr;
+        if (isG) {
+          const uint32_t q = s_db + unpackB(pre);
+          T.d2h_frame[q] = fr;
+          T.d2h_hf[q] = hf;
         }
       }
     }
-    T.vframe[j] = fr;
-    T.vkind[j] = ss;
-    T.vhf[j] = hf;
-    T.st[v] = isG ? ST_H : ST_HD;
-    T.map[v] = UM_NONE;
-    T.frame_of[v] = UM_NONE;
-    T.hframe[v] = hf;
-    nG += isG;
-    nAv += !isG;
-    nGL += ss == ST_GL;
-    if (evict_mode) {
-      T.free_stack[f0 + j] = fr;
-      if (isG) {
-        uint32_t q = atomicAdd(&c->n_d2h, 1u);
-        T.d2h_frame[q] = fr;
-        T.d2h_hf[q] = hf;
-      }
-    }
+    __syncthreads();
   }
-  {
-    uint32_t v[4] = {0u, nG, nAv, nGL};
-    const int slots[4] = {-1, S_D2H, S_D2H_AV, S_UNMAPS};
-    const long long mul[4] = {1, (long long)T.B, (long long)T.B, 1};
-    block_counts_to<4>(T, v, s_cnt, slots, mul);
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    s_last = atomicAdd(&c->vict_done, 1u) == gridDim.x - 1;
-  }
-  __syncthreads();
-  if (s_last && threadIdx.x == 0) {
-    __threadfence();
-    stat_add(T, S_EVICT, found);
-    if (c->k_want) {  // the scan covered both rings completely
-      c->disc_head = c->minkeep[0] != ~0ull ? c->minkeep[0] : c->disc_tail;
-      c->used_head = c->minkeep[1] != ~0ull ? c->minkeep[1] : c->used_tail;
-    }
-    c->minkeep[0] = c->minkeep[1] = ~0ull;
-    c->vict_done = 0;
-    if (evict_mode) {
-      c->free_top = f0 + (int)found;
-    } else {
-      const uint32_t nn = c->n_need;
-      c->f0 = (uint32_t)f0;
-      c->free_top = f0 - (int)min((uint32_t)f0, nn);
-      c->used_tail += c->n_rekey;
-    }
-  }
+  uint32_t v[3] = {nG, nAv, nGL};
+  const int slots[3] = {S_D2H, S_D2H_AV, S_UNMAPS};
+  const long long mul[3] = {(long long)T.B, (long long)T.B, 1};
+  block_counts_to<3>(T, v, s_cnt, slots, mul);
 }
 
 // ------------------------------------------------------------------------------------
@@ -920,6 +1149,7 @@ struct Unit {
 };
 
 __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t seq) {
+  pdl_enter();
   extern __shared__ __align__(128) char smem[];
   __shared__ __align__(8) uint64_t bar[kXferStages];
   const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
@@ -1041,6 +1271,7 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
 // items that need it runs as a kernel on the copy streams.
 // ------------------------------------------------------------------------------------
 __global__ void k_plan_commit(Tables T, uint32_t seq) {
+  pdl_enter();
   const uint32_t n = T.ctl->n_need, f0 = T.ctl->f0, nfu = min(f0, n);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     XItem x = item_plan(T, i, f0, nfu);
@@ -1086,6 +1317,7 @@ __global__ void __launch_bounds__(256) k_zero_items(Tables T, uint32_t i0, uint3
 // 16-byte pattern {s, ~s}, written through its frame (G or GL blocks are mapped).
 // ------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq) {
+  pdl_enter();
   __shared__ char* s_dst;
   __shared__ uint32_t s_blk;
   const uint32_t SEG = T.B < kFillSeg ? T.B : kFillSeg;
@@ -1119,58 +1351,82 @@ __global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g
 //   discard      G -> GE (unmap, DISC append), GL -> GE, H -> HD
 //   discard_lazy G -> GL (DISC append, mapping kept), H -> HD
 //   prefetch HOST G -> H (D2H), GE/GL -> H (no transfer), HD/U -> H
-// DISC appends are ranked in ascending block order (block scan + look-back).
+// Streaming: block lo + idx owns DISC slot disc_tail + idx (entry (seq, b)); the slot
+// is live only if the block turns GE/GL with dkey = seq here, so the ring stays sorted
+// by (dkey, block) without ranking.  Frame / host-frame stack traffic and the D2H list
+// take one atomic per CTA (their order is not observable).  The last CTA publishes
+// disc_tail and the counters.
 // ------------------------------------------------------------------------------------
-template <bool SINGLE>
-__global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
-                                                        int discard_off) {
-  constexpr int NW = kScanTPB / 32;
-  __shared__ uint32_t s_off[kScanIPT * NW + 1];
-  __shared__ unsigned long long s_excl;
-  __shared__ unsigned long long s_tail0;
-  __shared__ uint32_t s_cnt[6];
-  if (threadIdx.x == 0) s_tail0 = T.ctl->disc_tail;
-  const uint32_t tile = SINGLE ? 0u : blockIdx.x;
-  const uint32_t ntiles = SINGLE ? 1u : gridDim.x;
-  const uint32_t tbase = tile * kScanTile;
-  const int w = threadIdx.x >> 5;
-  const bool appends = !discard_off && kind != DIR_PREFETCH_HOST;
-  uint8_t s[kScanIPT];
-  unsigned bA[kScanIPT], bZ[kScanIPT];
+__global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
+                                                         int discard_off, unsigned long long tail0) {
+  pdl_enter();
+  constexpr int TPB = kStTPB, IPT = kStIPT, TILE = kStTile;
+  __shared__ unsigned long long s_sc[TPB / 32];
+  __shared__ int s_hb, s_fb;
+  __shared__ uint32_t s_db, s_hav;
+  __shared__ uint32_t s_cnt[8];
+  Ctl* c = T.ctl;
+  const uint32_t tbase = blockIdx.x * TILE;
+  const bool disc = kind == DIR_DISCARD || kind == DIR_DISCARD_LAZY;
+  const bool active = !discard_off || kind == DIR_PREFETCH_HOST;
+  uint8_t s[IPT];
+  uint32_t hasf = 0;   // bit k: item k is an H block holding a host frame (discard)
+  // per-thread counts of stack / list traffic: A = host frames (released by a discard
+  // of an H block holding one, taken by a prefetch HOST of G), F = GPU frames freed
+  // (prefetch HOST)
+  uint32_t nA = 0, nF = 0;
 #pragma unroll
-  for (int k = 0; k < kScanIPT; ++k) {
-    const uint32_t idx = tbase + k * kScanTPB + threadIdx.x;   // coalesced
+  for (int k = 0; k < IPT; ++k) {
+    const uint32_t idx = tbase + k * TPB + threadIdx.x;   // coalesced
     s[k] = idx < n ? T.st[lo + idx] : (uint8_t)0xff;
-    bA[k] = __ballot_sync(FULL, appends && s[k] == ST_G);
-    bZ[k] = 0;
+    if (disc) {
+      if (s[k] == ST_H && T.hframe[lo + idx] != UM_NONE) {
+        hasf |= 1u << k;
+        ++nA;
+      }
+    } else {
+      nA += s[k] == ST_G;
+      nF += s[k] == ST_G || s[k] == ST_GE || s[k] == ST_GL;
+    }
   }
-  const uint32_t tt = ordered_offsets<kScanTPB, kScanIPT>(bA, bZ, s_off);
-  const unsigned long long tot = pack2(tt & 0xffffu, 0);
-  if (SINGLE) {
-    if (threadIdx.x == 0) s_excl = 0;
-  } else if (threadIdx.x < 32) {
-    unsigned long long e = lookback_warp(T, tile, tot);
-    if (threadIdx.x == 0) s_excl = e;
+  const unsigned long long kseq = (unsigned long long)seq << 32;
+  unsigned long long tot;
+  const unsigned long long pre = block_excl_scan<TPB>(active ? pack2(nA, nF) : 0ull, tot, s_sc);
+  if (threadIdx.x == 0) {
+    const uint32_t tA = unpackA(tot), tF = unpackB(tot);
+    s_hb = 0; s_fb = 0; s_db = 0; s_hav = tA;
+    if (disc) {
+      if (tA) s_hb = atomicAdd(&c->hfree_top, (int)tA);            // release: push
+    } else {
+      if (tA) {                                                     // take: pop
+        const int old = atomicSub(&c->hfree_top, (int)tA);
+        const int avail = old < 0 ? 0 : (old < (int)tA ? old : (int)tA);
+        if (avail < (int)tA) {
+          atomicAdd(&c->hfree_top, (int)tA - avail);
+          atomicExch(&c->err, 2u);                                  // -> UM_ENOMEM
+        }
+        s_hb = old;          // this CTA owns hfree_stack[old - avail, old)
+        s_hav = (uint32_t)avail;
+        s_db = atomicAdd(&c->n_d2h, tA);
+      }
+      if (tF) s_fb = atomicAdd(&c->free_top, (int)tF);
+    }
   }
   __syncthreads();
-  const uint32_t eA = unpackA(s_excl);
-  const unsigned lt = lanemask_lt();
-  const unsigned long long tail0 = s_tail0;
-  // counters: unmaps, d2h, d2h_av
+  uint32_t rA = unpackA(pre), rF = unpackB(pre);
   uint32_t nUnmap = 0, nD2H = 0, nAv = 0;
-  if (!discard_off || kind == DIR_PREFETCH_HOST) {
+  if (active) {
 #pragma unroll
-    for (int k = 0; k < kScanIPT; ++k) {
-      const uint32_t idx = tbase + k * kScanTPB + threadIdx.x;
+    for (int k = 0; k < IPT; ++k) {
+      const uint32_t idx = tbase + k * TPB + threadIdx.x;
       if (idx >= n) continue;
       const uint32_t bb = lo + idx;
       const uint8_t ss = s[k];
-      if (kind == DIR_DISCARD || kind == DIR_DISCARD_LAZY) {
+      if (disc) {
+        T.disc_ring[(tail0 + idx) & T.cap_mask] = kseq | bb;
         if (ss == ST_G) {
           T.st[bb] = kind == DIR_DISCARD ? ST_GE : ST_GL;
           T.key[bb] = seq;
-          const uint32_t pA = eA + (s_off[k * NW + w] & 0xffffu) + __popc(bA[k] & lt);
-          T.disc_ring[(tail0 + pA) & T.cap_mask] = ((unsigned long long)seq << 32) | bb;
           if (kind == DIR_DISCARD) {
             T.map[bb] = UM_NONE;
             ++nUnmap;
@@ -1181,36 +1437,28 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
           ++nUnmap;
         } else if (ss == ST_H) {
           T.st[bb] = ST_HD;
-          uint32_t hf = T.hframe[bb];
-          if (hf != UM_NONE) {  // the host copy is released (reading R1)
+          if ((hasf >> k) & 1u) {   // the host copy is released (reading R1)
+            T.hfree_stack[s_hb + rA] = T.hframe[bb];
             T.hframe[bb] = UM_NONE;
-            int idx = atomicAdd(&T.ctl->hfree_top, 1);
-            T.hfree_stack[idx] = hf;
+            ++rA;
           }
         }
       } else {  // prefetch to HOST
         if (ss == ST_G || ss == ST_GE || ss == ST_GL) {
-          uint32_t fr = T.frame_of[bb];
+          const uint32_t fr = T.frame_of[bb];
           if (ss == ST_G) {
-            int idx = atomicSub(&T.ctl->hfree_top, 1) - 1;
-            uint32_t hf = UM_NONE;
-            if (idx >= 0) {
-              hf = T.hfree_stack[idx];
-            } else {
-              atomicAdd(&T.ctl->hfree_top, 1);
-              atomicExch(&T.ctl->err, 2u);
-            }
-            uint32_t q = atomicAdd(&T.ctl->n_d2h, 1u);
-            T.d2h_frame[q] = fr;
-            T.d2h_hf[q] = hf;
+            const uint32_t hf = rA < s_hav ? T.hfree_stack[s_hb - 1 - (int)rA] : UM_NONE;
+            T.d2h_frame[s_db + rA] = fr;
+            T.d2h_hf[s_db + rA] = hf;
             T.hframe[bb] = hf;
+            ++rA;
             ++nD2H;
           } else {
             ++nAv;
             if (ss == ST_GL) ++nUnmap;
           }
-          int fi = atomicAdd(&T.ctl->free_top, 1);
-          T.free_stack[fi] = fr;
+          T.free_stack[s_fb + rF] = fr;
+          ++rF;
           T.frame_of[bb] = UM_NONE;
           T.map[bb] = UM_NONE;
         }
@@ -1221,45 +1469,44 @@ __global__ void __launch_bounds__(kScanTPB) k_directive(Tables T, int kind, uint
   uint32_t v[3] = {nUnmap, nD2H, nAv};
   const int slots[3] = {S_UNMAPS, S_D2H, S_D2H_AV};
   const long long mul[3] = {1, (long long)T.B, (long long)T.B};
-  if (SINGLE) {
-    if (threadIdx.x == 0) T.ctl->disc_tail = tail0 + unpackA(tot);
-    block_counts_to<3>(T, v, s_cnt, slots, mul);
-    return;
-  }
-  tile_counts<3>(T, tile, v, s_cnt);
-  if (tile == ntiles - 1 && threadIdx.x == 0) T.ctl->disc_tail = tail0 + unpackA(s_excl + tot);
-  scan_finish<3>(T, ntiles, slots, mul);
+  block_counts_to<3>(T, v, s_cnt, slots, mul);
+  // the host passes the exact tail; nothing in this launch reads c->disc_tail
+  if (blockIdx.x == 0 && threadIdx.x == 0 && disc && active) c->disc_tail = tail0 + n;
 }
 
 // ------------------------------------------------------------------------------------
-// K7: stable compaction of a ring's live entries [head, tail) into `dst` at [0, cnt).
+// K7: stable compaction of a ring's live entries [head, tail) into `dst`, right-aligned:
+// the live entries keep their order and end at the same tail, so ring tails only ever
+// grow by appends and the host knows them exactly (it passes them to the appending
+// kernels).  Entries are ranked from the tail backwards (tile 0 holds the newest).
 // ------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(kScanTPB) k_ring_compact(Tables T, int ring, uint64_t* dst) {
+  pdl_enter();
   constexpr int NW = kScanTPB / 32;
   __shared__ uint32_t s_off[kScanIPT * NW + 1];
-  __shared__ unsigned long long s_excl, s_head, s_n;
+  __shared__ unsigned long long s_excl, s_tail, s_n;
   Ctl* c = T.ctl;
   if (threadIdx.x == 0) {
-    s_head = ring == RING_USED ? c->used_head : c->disc_head;
-    unsigned long long tl = ring == RING_USED ? c->used_tail : c->disc_tail;
-    s_n = tl - s_head;
+    const unsigned long long hd = ring == RING_USED ? c->used_head : c->disc_head;
+    s_tail = ring == RING_USED ? c->used_tail : c->disc_tail;
+    s_n = s_tail - hd;
   }
   __syncthreads();
   const uint32_t tile = blockIdx.x;
   const uint32_t ntiles = gridDim.x;
   const uint64_t* R = ring == RING_USED ? T.used_ring : T.disc_ring;
-  const unsigned long long n = s_n, head = s_head;
+  const unsigned long long n = s_n, tail = s_tail;
   const unsigned long long tbase = (unsigned long long)tile * kScanTile;
   const int w = threadIdx.x >> 5;
   unsigned long long e[kScanIPT];
   unsigned bL[kScanIPT], bZ[kScanIPT];
 #pragma unroll
   for (int k = 0; k < kScanIPT; ++k) {
-    const unsigned long long idx = tbase + k * kScanTPB + threadIdx.x;
+    const unsigned long long ri = tbase + k * kScanTPB + threadIdx.x;   // rank from the tail
     e[k] = 0;
     bool live = false;
-    if (idx < n) {
-      e[k] = R[(head + idx) & T.cap_mask];
+    if (ri < n) {
+      e[k] = R[(tail - 1 - ri) & T.cap_mask];
       const uint32_t blk = (uint32_t)e[k], kk = (uint32_t)(e[k] >> 32);
       const uint8_t ss = T.st[blk];
       live = (ring == RING_USED ? ss == ST_G : (ss == ST_GE || ss == ST_GL)) && T.key[blk] == kk;
@@ -1278,11 +1525,12 @@ __global__ void __launch_bounds__(kScanTPB) k_ring_compact(Tables T, int ring, u
   const unsigned lt = lanemask_lt();
 #pragma unroll
   for (int k = 0; k < kScanIPT; ++k)
-    if ((bL[k] >> (threadIdx.x & 31)) & 1) dst[eA + (s_off[k * NW + w] & 0xffffu) + __popc(bL[k] & lt)] = e[k];
+    if ((bL[k] >> (threadIdx.x & 31)) & 1)
+      dst[(tail - 1 - (eA + (s_off[k * NW + w] & 0xffffu) + __popc(bL[k] & lt))) & T.cap_mask] = e[k];
   if (tile == ntiles - 1 && threadIdx.x == 0) {
-    unsigned long long total = unpackA(s_excl + tot);
-    if (ring == RING_USED) { c->used_head = 0; c->used_tail = total; }
-    else { c->disc_head = 0; c->disc_tail = total; }
+    const unsigned long long total = unpackA(s_excl + tot);
+    if (ring == RING_USED) c->used_head = tail - total;
+    else c->disc_head = tail - total;
   }
   scan_finish(T, ntiles);
 }
@@ -1368,6 +1616,8 @@ __global__ void __launch_bounds__(256) k_tags(Tables T) {
 // launch wrappers
 // ------------------------------------------------------------------------------------
 static int g_nsm = 0;
+static int g_vscan_occ = 1;   // resident k_victims_scan CTAs per SM
+static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch (A/B)
 
 cudaError_t setup_kernels() {
   int dev;
@@ -1375,8 +1625,30 @@ cudaError_t setup_kernels() {
   if (e) return e;
   e = cudaDeviceGetAttribute(&g_nsm, cudaDevAttrMultiProcessorCount, dev);
   if (e) return e;
+  if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_vscan_occ, k_victims_scan, kScanTPB, 0);
+  if (e) return e;
+  if (g_vscan_occ < 1) g_vscan_occ = 1;
   int smem = (int)(kXferChunk * (1 + 2 * kXferStages));
   return cudaFuncSetAttribute(k_service, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+}
+
+
+// Launch on `s` with programmatic stream serialization (see pdl_enter).
+template <typename... KArgs, typename... Args>
+static cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
+                              Args... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = g_pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
 }
 
 static inline unsigned ceil_div(unsigned long long a, unsigned long long b) { return (unsigned)((a + b - 1) / b); }
@@ -1392,32 +1664,40 @@ cudaError_t launch_poison(const Tables& T, cudaStream_t s) {
 }
 
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
-                            cudaStream_t s) {
-  unsigned nt = n ? ceil_div(n, kScanTile) : 1;
-  k_classify<<<nt, kScanTPB, 0, s>>>(T, iv, g0, n, seq, touch);
+                            unsigned long long tail0, int npar, cudaStream_t s) {
+  unsigned nt = n ? ceil_div(n, kStTile) : 1;
+  cudaError_t le__ = launch_pdl(k_classify, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 
-cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, cudaStream_t s) {
-  k_victims<<<1, kVictTPB, 0, s>>>(T, seq, evict_mode, want);
+cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, int npar, cudaStream_t s) {
+  cudaError_t le__ = launch_pdl(k_victims, dim3(1), dim3(kVictTPB), 0, s, T, seq, evict_mode, want, npar);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 
 cudaError_t launch_plan_small(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
-                              cudaStream_t s) {
-  k_plan_small<<<1, kVictTPB, 0, s>>>(T, iv, g0, n, seq, touch);
+                              unsigned long long tail0, cudaStream_t s) {
+  cudaError_t le__ = launch_pdl(k_plan_small, dim3(1), dim3(kVictTPB), 0, s, T, iv, g0, n, seq, touch, tail0);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 
 cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, uint64_t scan_bound,
-                                uint32_t max_victims, cudaStream_t s) {
+                                uint32_t max_victims, int npar, cudaStream_t s) {
+  // persistent scan grid: never more CTAs than can be resident (tiles are taken from a
+  // ticket in order and a tile may wait on its predecessors' status)
   unsigned nt = ceil_div(scan_bound ? scan_bound : 1, kScanTile);
-  k_victims_scan<<<nt, kScanTPB, 0, s>>>(T, seq, evict_mode, want);
+  const unsigned cap = (unsigned)(g_nsm * g_vscan_occ);
+  cudaError_t le__ = launch_pdl(k_victims_scan, dim3(nt < cap ? nt : cap), dim3(kScanTPB), 0, s, T, seq, evict_mode, want, npar);
+  if (le__) return le__;
   cudaError_t e = cudaGetLastError();
   if (e) return e;
-  unsigned grid = ceil_div(max_victims ? max_victims : 1, 256);
-  if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
-  k_victims_apply<<<grid, 256, 0, s>>>(T, evict_mode);
+  unsigned grid = ceil_div(max_victims ? max_victims : 1, 1024);
+  if (grid > (unsigned)g_nsm * 4) grid = g_nsm * 4;
+  le__ = launch_pdl(k_victims_apply, dim3(grid), dim3(256), 0, s, T, evict_mode);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 
@@ -1427,7 +1707,8 @@ cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max
   unsigned grid = (unsigned)(units < (unsigned long long)g_nsm ? units : (unsigned long long)g_nsm);
   if (grid == 0) grid = 1;
   size_t smem = (size_t)CH * (1 + 2 * kXferStages);
-  k_service<<<grid, 32, smem, s>>>(T, mode, seq);
+  cudaError_t le__ = launch_pdl(k_service, dim3(grid), dim3(32), smem, s, T, mode, seq);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 
@@ -1436,21 +1717,23 @@ cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, 
   unsigned long long units = (unsigned long long)n * (T.B / SEG);
   unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
   if (!grid) return cudaSuccess;
-  k_app_stamp<<<grid, 256, 0, s>>>(T, iv, g0, n, seq);
+  cudaError_t le__ = launch_pdl(k_app_stamp, dim3(grid), dim3(256), 0, s, T, iv, g0, n, seq);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq, int discard_off,
-                             cudaStream_t s) {
-  unsigned nt = n ? ceil_div(n, kScanTile) : 1;
-  if (nt == 1) k_directive<true><<<1, kScanTPB, 0, s>>>(T, kind, lo, n, seq, discard_off);
-  else k_directive<false><<<nt, kScanTPB, 0, s>>>(T, kind, lo, n, seq, discard_off);
+                             unsigned long long tail0, cudaStream_t s) {
+  unsigned nt = n ? ceil_div(n, kStTile) : 1;
+  cudaError_t le__ = launch_pdl(k_directive, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq, discard_off, tail0);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 
 cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64_t cap_bound, cudaStream_t s) {
   unsigned nt = ceil_div(cap_bound ? cap_bound : 1, kScanTile);
-  k_ring_compact<<<nt, kScanTPB, 0, s>>>(T, ring, dst);
+  cudaError_t le__ = launch_pdl(k_ring_compact, dim3(nt), dim3(kScanTPB), 0, s, T, ring, dst);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 
@@ -1466,7 +1749,8 @@ cudaError_t launch_host_write(const Tables& T, uint32_t lo, uint32_t n, uint32_t
 
 cudaError_t launch_plan_commit(const Tables& T, uint32_t seq, uint32_t max_items, cudaStream_t s) {
   unsigned grid = ceil_div(max_items ? max_items : 1, 256);
-  k_plan_commit<<<grid, 256, 0, s>>>(T, seq);
+  cudaError_t le__ = launch_pdl(k_plan_commit, dim3(grid), dim3(256), 0, s, T, seq);
+  if (le__) return le__;
   return cudaGetLastError();
 }
 

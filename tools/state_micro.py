@@ -24,6 +24,15 @@ nf = (1 << 21) + (1 << 20)
 n = 1 << 21
 a = um.Arena(B, nb * B, nf * B, flags=um.UM_F_TIMING | um.UM_F_COPY_KERNEL, host_pool_bytes=1 << 30)
 h = a.handle
+# Gate: a ~50 ms device sleep on the paging stream before each op, so every launch of the
+# op is queued before the GPU reaches it and the timed spans hold device time only (no
+# host enqueue gaps between the kernels).
+_ps = torch.cuda.ExternalStream(a.stream_ptr)
+
+
+def gate():
+    with torch.cuda.stream(_ps):
+        torch.cuda._sleep(100_000_000)
 rng = np.random.default_rng(0)
 out = {}
 
@@ -35,14 +44,17 @@ def touch_random(tag):
     acc["len"] = B
     acc["kind"] = tg.ACC_READ
     um.um_timing(h, reset=True)
+    gate()
     um.um_touch_batch(h, acc)
     out[tag] = um.um_timing(h, reset=True)
 
 
 for rep in range(2):
     touch_random(f"touch_random_{rep}")
+    gate()
     um.um_discard(h, 0, n * B)
     out[f"discard_{rep}"] = um.um_timing(h, reset=True)
+    gate()
     um.um_prefetch(h, 0, n * B, um.UM_DST_GPU)
     out[f"prefetch_revive_{rep}"] = um.um_timing(h, reset=True)
 out["stats"] = um.um_get_stats(h)
