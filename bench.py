@@ -321,11 +321,31 @@ def c1_rate(torch, um, harness):
         arena.close()
 
 
+def _hbm_peak():
+    """Measured HBM copy bandwidth (MEASURED_PEAKS.json, driver-written), else the
+    profiling guide's fallback."""
+    try:
+        with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "MEASURED_PEAKS.json")) as f:
+            return float(json.load(f)["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs (copy, read+write), burst"
+    except Exception:
+        return 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
+
+
 def state_bench(torch, um, mem, budget, arena_bytes, seed=0):
     """State-kernel microbench (SURVEY §8(d) last row): C3-64K-sized tables (64 KiB blocks
-    over the same 170 GiB of frames / 255 GiB arena), one touch_batch of 2^21 distinct
-    uniformly random blocks, then one 2^21-block discard.  Planning kernels timed apart
-    from the zero-fill (um_timing); algorithmic bytes per block as in DESIGN.md §5."""
+    over the same frame budget / 1.5x arena), each op on a cold L2 (the previous op's
+    zero-fill streams GBs through it):
+      touch_random   one touch_batch of 2^21 distinct uniformly random blocks (all U)
+      discard        one eager discard of blocks [0, 2^21)
+      touch_pressure a second 2^21-block random touch: revives, zero-fills and reclaims
+                     discarded frames (victim scan + apply)
+    Planning kernels are timed apart from the zero-fill (um_timing spans, CUDA events on
+    the paging stream).  Algorithmic bytes per unit:
+      classify  per block 9 (interval record) + 4 sk rd + 4 pin wr + 8 USED slot;
+                per need item + 9 (need, needk, needhf); per revive + 12 (frame_of rd,
+                sk wr, map wr); per H block + 4 (hframe rd)
+      victims   per victim 12 (ring entry + sk) + 42 (apply: lists, sk/frame_of/map/hframe)
+      directive per block 4 sk rd + 8 DISC slot; per G block + 8 (sk wr, map wr)"""
     import numpy as np
     import tracegen as tg
     B = 64 * 1024
@@ -339,11 +359,16 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0):
     h = um.um_arena_create(cfg)
     try:
         rng = np.random.default_rng(seed)
-        blocks = np.sort(rng.choice(nb, size=n, replace=False))
-        acc = np.zeros(n, dtype=tg.ACC_DTYPE)
-        acc["off"] = blocks.astype(np.uint64) * B
-        acc["len"] = B
-        acc["kind"] = tg.ACC_READ
+
+        def records(blocks):
+            acc = np.zeros(len(blocks), dtype=tg.ACC_DTYPE)
+            acc["off"] = blocks.astype(np.uint64) * B
+            acc["len"] = B
+            acc["kind"] = tg.ACC_READ
+            return acc
+        b0 = np.sort(rng.choice(nb, size=n, replace=False))
+        b1 = np.sort(rng.choice(nb, size=n, replace=False))
+        acc0, acc1 = records(b0), records(b1)
         # a device sleep ahead of each op keeps the GPU behind the host, so every launch
         # of the op is queued before it runs and the spans hold device time only
         ps = torch.cuda.ExternalStream(um.um_stream(h))
@@ -351,29 +376,44 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0):
         def gate():
             with torch.cuda.stream(ps):
                 torch.cuda._sleep(100_000_000)
-        um.um_timing(h, reset=True)
-        gate()
-        um.um_touch_batch(h, acc)
-        t_touch = um.um_timing(h, reset=True)
-        gate()
-        um.um_discard(h, 0, n * B)
-        t_disc = um.um_timing(h, reset=True)
-        st = um.um_get_stats(h)
-        assert st["zf_bytes"] == n * B
-        g_in = int(np.count_nonzero(blocks < n))        # G blocks inside the discarded range
-        # bytes per block: classify 1 st + 4 pin + 8 ring + 9 need list + 4 hframe + 8 intervals;
-        # victims: none needed (frames free).  directive: 1 st rd; G: 1 st + 4 key + 4 map + 8 DISC
-        cls_bytes = n * (1 + 4 + 8 + 9 + 4 + 8)
-        dir_bytes = n * 1 + g_in * (1 + 4 + 4 + 8)
-        peak = 6548.5
-        def rl(name, by, ms):
+
+        def timed(fn):
+            s0 = um.um_get_stats(h)
+            um.um_timing(h, reset=True)
+            gate()
+            fn()
+            t = um.um_timing(h, reset=True)
+            s1 = um.um_get_stats(h)
+            return t, {k: s1[k] - s0[k] for k in s1}
+        t_touch, d0 = timed(lambda: um.um_touch_batch(h, acc0))
+        t_disc, d1 = timed(lambda: um.um_discard(h, 0, n * B))
+        t_pres, d2 = timed(lambda: um.um_touch_batch(h, acc1))
+        assert d0["zf_bytes"] == n * B
+        g_in = int(np.count_nonzero(b0 < n))             # G blocks inside the discarded range
+        assert d1["unmaps"] == g_in
+
+        def cls_bytes(d):
+            need = d["faults"] - d["remaps"]
+            return n * (9 + 4 + 4 + 8) + need * 9 + d["remaps"] * 12 + (d["h2d_bytes"] // B) * 4
+        touch_bytes = cls_bytes(d0)
+        pres_bytes = cls_bytes(d2) + d2["evictions"] * (12 + 42)
+        dir_bytes = n * (4 + 8) + g_in * 8
+        peak, peak_src = _hbm_peak()
+
+        def rl(name, by, ms, extra=None):
             a = by / (ms / 1e3) / 1e9 if ms else None
-            return {"kernel": name, "bound": "hbm", "achieved": a, "peak": peak, "unit": "GB/s",
-                    "frac": a / peak if a else None, "algorithmic_bytes": by, "ms": ms, "blocks": n}
-        return {"touch_2^21_random": rl("k_classify+k_victims", cls_bytes, t_touch["ms_plan"]),
+            r = {"kernel": name, "bound": "hbm", "achieved": a, "peak": peak, "unit": "GB/s",
+                 "frac": a / peak if a else None, "algorithmic_bytes": by, "ms": ms, "blocks": n}
+            r.update(extra or {})
+            return r
+        return {"touch_2^21_random": rl("k_classify + k_victims_scan/apply (k = 0)", touch_bytes, t_touch["ms_plan"]),
                 "discard_2^21": rl("k_directive", dir_bytes, t_disc["ms_plan"]),
+                "touch_2^21_pressure": rl("k_classify + k_victims_scan + k_victims_apply", pres_bytes, t_pres["ms_plan"],
+                                          {"victims": d2["evictions"], "remaps": d2["remaps"]}),
                 "zero_fill_gbs": (n * B) / (t_touch["ms_xfer"] / 1e3) / 1e9 if t_touch["ms_xfer"] else None,
-                "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, read+write)", "nblocks": nb}
+                "peak_source": peak_src, "nblocks": nb, "nframes": budget // B,
+                "timing": "CUDA events around each op's planning launches on the paging stream; every launch "
+                          "queued behind a device sleep; L2 cold (the previous op's zero-fill flushes it)"}
     finally:
         um.um_arena_destroy(h)
         del ws

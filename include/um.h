@@ -50,7 +50,8 @@ typedef struct um_arena um_arena; /* opaque; library-owned host bookkeeping */
 typedef enum {
   UM_OK = 0,
   UM_EINVAL = -1, /* bad argument / range; nothing enqueued                              */
-  UM_ENOMEM = -2, /* arena (um_alloc) or host-frame pool exhausted; sticky when on device */
+  UM_ENOMEM = -2, /* arena (um_alloc) or host-frame pool exhausted (sticky when on device), or
+                     the arena's 2^29 - 1 sequence numbers (one per sub-op) used up (sticky) */
   UM_ECUDA = -3,  /* CUDA error; sticky                                                   */
   UM_EBUSY = -4   /* concurrent call on the same arena                                   */
 } um_status;

@@ -28,10 +28,11 @@ namespace {
 constexpr uint64_t kAlign = 256;
 
 struct Layout {
-  uint64_t st, key, frame_of, map, hframe, pin, free_stack, hfree_stack;
+  uint64_t sk, frame_of, map, hframe, pin, free_stack, hfree_stack;
   uint64_t used[2], disc[2];
   uint64_t need, needk, needhf, victim, vframe, vhf, vkind, d2h_frame, d2h_hf;
   uint64_t tile_status, tile_cnt, tags, ctl, hchunks, stage, xitems, bounce;
+  uint64_t obits, wbits, dlo, dpre, dw;
   uint64_t stage_bytes, max_tiles, cap, total, ce_group, bounce_bytes;
 };
 
@@ -72,8 +73,7 @@ static Layout make_layout(const um_config* c) {
     o += (bytes + kAlign - 1) / kAlign * kAlign;
     return r;
   };
-  L.st = take(nb);
-  L.key = take(4 * nb);
+  L.sk = take(4 * nb);
   L.frame_of = take(4 * nb);
   L.map = take(4 * nb);
   L.hframe = take(4 * nb);
@@ -103,6 +103,12 @@ static Layout make_layout(const um_config* c) {
   L.ce_group = std::max<uint64_t>(1, std::min<uint64_t>(1024, (64ull << 20) / c->block_bytes));
   L.bounce_bytes = 2 * L.ce_group * c->block_bytes;
   L.bounce = take(L.bounce_bytes);
+  const uint64_t nw = (nb + 31) / 32;
+  L.obits = take(4 * nw);
+  L.wbits = take(4 * nw);
+  L.dlo = take(4 * nb);
+  L.dpre = take(4 * (nb + 1));
+  L.dw = take(nb);
   L.total = o;
   return L;
 }
@@ -189,6 +195,12 @@ struct um_arena {
   // tail to the appending kernels instead of having them read and publish it
   uint64_t tail[2] = {0, 0};
   int npar = 0;             // parity slot of the multi-CTA classify's need counter
+  // device intake result for the current op (intervals in T.dlo/dpre/dw)
+  bool dev_iv = false, dev_anyw = false;
+  uint32_t dev_m = 0;
+  uint64_t dev_total = 0;
+  std::vector<uint32_t> hpre;   // interval prefix of the current op (host copy, for tile tables)
+  std::vector<MarkRec> mark;    // scratch: split records
   uint32_t B = 0, nblocks = 0, nframes = 0, nhframes = 0;
   cudaStream_t ps = nullptr;
   cudaEvent_t ev_in = nullptr, ev_out = nullptr;
@@ -311,6 +323,17 @@ static um_status ensure_ring_room(um_arena* a, int ring, uint64_t appends) {
   a->ring_cur[ring] = nxt;
   set_ring_ptrs(a);
   a->ub[ring] = std::min<uint64_t>(a->nframes, a->L.cap) + appends;
+  return UM_OK;
+}
+
+// Keys live in the upper 29 bits of the packed state word, so an arena has 2^29 - 1
+// sequence numbers; an op that would need more fails with UM_ENOMEM (sticky).
+constexpr uint64_t kSeqLimit = (1ull << 29) - 1;
+static um_status seq_room(um_arena* a, uint64_t k) {
+  if ((uint64_t)a->clock + k > kSeqLimit) {
+    a->sticky = UM_ENOMEM;
+    return UM_ENOMEM;
+  }
   return UM_OK;
 }
 
@@ -507,13 +530,97 @@ static um_status ce_d2h_only(um_arena* a, uint32_t nmax) {
   return UM_OK;
 }
 
+// True when the records are in ascending, non-overlapping block order (then they are the
+// intervals and no dedupe is needed).
+static bool sorted_disjoint(um_arena* a, const um_access* acc, uint32_t n) {
+  uint64_t prev_hi = 0;
+  bool any = false;
+  for (uint32_t i = 0; i < n; ++i) {
+    if (!acc[i].len) continue;
+    const uint64_t lo = acc[i].off / a->B, hi = (acc[i].off + acc[i].len - 1) / a->B + 1;
+    if (any && lo < prev_hi) return false;
+    prev_hi = hi;
+    any = true;
+  }
+  return true;
+}
+
+// Device intake: dedupe a batch of accesses on the GPU.  The host converts
+// each record to blocks and splits it into pieces of <= kMarkMaxBlocks (argument
+// marshalling), stages the pieces, and the kernels build the sorted disjoint interval
+// list in HBM.  One sync reads the interval count and the prefix array back: the host
+// needs them to number the sub-ops and index tiles, not to compute anything.
+static um_status device_intake(um_arena* a, const um_access* acc, uint32_t n) {
+  const uint64_t B = a->B;
+  uint64_t bmin = ~0ull, bmax = 0;
+  bool anyw = false;
+  auto& mk = a->mark;
+  mk.clear();
+  for (uint32_t i = 0; i < n; ++i) {
+    if (!acc[i].len) continue;
+    const uint64_t lo = acc[i].off / B, hi = (acc[i].off + acc[i].len - 1) / B + 1;
+    const uint32_t w = (acc[i].kind & UM_ACC_WRITE) ? 1u : 0u;
+    anyw |= w != 0;
+    bmin = std::min(bmin, lo);
+    bmax = std::max(bmax, hi);
+    for (uint64_t x = lo; x < hi; x += kMarkMaxBlocks)
+      mk.push_back({(uint32_t)x, (uint32_t)std::min<uint64_t>(kMarkMaxBlocks, hi - x), w, 0u});
+  }
+  if (mk.empty()) {
+    a->dev_iv = true;
+    a->dev_m = 0;
+    a->dev_total = 0;
+    a->dev_anyw = false;
+    a->hpre.assign(1, 0u);
+    return UM_OK;
+  }
+  const uint64_t per = std::max<uint64_t>(1, (a->L.stage_bytes / 2) / sizeof(MarkRec));
+  for (size_t c0 = 0; c0 < mk.size(); c0 += per) {
+    const size_t cn = std::min<size_t>(per, mk.size() - c0);
+    uint64_t off;
+    CK(a->stage.reserve(cn * sizeof(MarkRec), &off));
+    memcpy(a->stage.host + off, mk.data() + c0, cn * sizeof(MarkRec));
+    CK(a->stage.push(off, (cn * sizeof(MarkRec) + 15) & ~15ull, a->ps));
+    CK(launch_mark(a->T, (const MarkRec*)(a->stage.dev + off), (uint32_t)cn, a->ps));
+  }
+  const uint32_t w0 = (uint32_t)(bmin >> 5), w1 = (uint32_t)((bmax + 31) >> 5);
+  CK(launch_runs(a->T, w0, w1, a->ps));
+  CK(launch_intake_clear(a->T, w0, w1, a->ps));
+  a->n_launch += 2 + (mk.size() + per - 1) / per;
+  CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaStreamSynchronize(a->ps));
+  const uint32_t m = a->hctl->iv_m;
+  a->hpre.resize((size_t)m + 1);
+  CK(cudaMemcpyAsync(a->hpre.data(), a->T.dpre, 4ull * (m + 1), cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaStreamSynchronize(a->ps));
+  a->dev_iv = true;
+  a->dev_m = m;
+  a->dev_total = a->hctl->iv_d;
+  a->dev_anyw = anyw;
+  return UM_OK;
+}
+
 // Enqueue the K1/K2 -> K3 -> K4/K5/K6 (-> K9) chain for every sub-op of a GPU op.
 static um_status run_gpu_op(um_arena* a, int touch) {
   uint64_t total = 0;
   bool anyw = false;
-  for (auto& v : a->ivs) {
-    total += v.cnt;
-    anyw |= v.w;
+  const bool dev = a->dev_iv;
+  a->dev_iv = false;
+  if (dev) {
+    total = a->dev_total;
+    anyw = a->dev_anyw;
+  } else {
+    a->hpre.resize(a->ivs.size() + 1);
+    for (size_t j = 0; j < a->ivs.size(); ++j) {
+      a->hpre[j] = (uint32_t)total;
+      total += a->ivs[j].cnt;
+      anyw |= a->ivs[j].w;
+    }
+    a->hpre[a->ivs.size()] = (uint32_t)total;
+  }
+  {
+    um_status sr = seq_room(a, total ? (total + a->nframes - 1) / a->nframes : 1);
+    if (sr) return sr;
   }
   a->ops++;
   if (total == 0) {
@@ -521,10 +628,15 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     a->subops++;
     return UM_OK;
   }
-  const uint32_t m = (uint32_t)a->ivs.size();
+  const uint32_t m = dev ? a->dev_m : (uint32_t)a->ivs.size();
   OpIv iv{};
   iv.m = m;
-  if (m <= kIvInline) {
+  if (dev) {
+    // intervals made on the device by the intake kernels (already in HBM)
+    iv.lo = a->T.dlo;
+    iv.pre = a->T.dpre;
+    iv.wflag = a->T.dw;
+  } else if (m <= kIvInline) {
     // small list: pass it inline in the kernel parameters (no staging copy)
     iv.inl = 1;
     uint32_t acc = 0;
@@ -560,7 +672,7 @@ static um_status run_gpu_op(um_arena* a, int touch) {
   }
   const uint32_t F = a->nframes;
   uint32_t jcur = 0;   // interval holding the current item (items ascend across sub-ops)
-  uint64_t pcur = 0;   // its first item
+  const uint32_t* hp = a->hpre.data();
   for (uint64_t g0 = 0; g0 < total; g0 += F) {
     const uint32_t n = (uint32_t)std::min<uint64_t>(F, total - g0);
     const uint32_t seq = ++a->clock;
@@ -570,16 +682,13 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     if (!iv.inl) {
       // per tile of this sub-op, the interval slice its items fall in: an index the
       // kernels would otherwise find by a dependent binary search over the staged list
-      const uint32_t tile = n <= kSmallPlan ? kSmallPlan : (uint32_t)kStTile;
+      const uint32_t tile = n <= kSmallPlan ? kSmallPlan : (uint32_t)kClsTile;
       const uint32_t nt = (n + tile - 1) / tile;
       uint64_t off;
       CK(a->stage.reserve(8ull * nt, &off));
       uint32_t* tj = (uint32_t*)(a->stage.host + off);
       auto seek = [&](uint64_t g) {
-        while (pcur + a->ivs[jcur].cnt <= g) {
-          pcur += a->ivs[jcur].cnt;
-          ++jcur;
-        }
+        while (hp[jcur + 1] <= g) ++jcur;
         return jcur;
       };
       for (uint32_t t = 0; t < nt; ++t) {
@@ -673,8 +782,7 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   if ((e = setup_kernels())) return fail(e);
   char* ws = (char*)cfg->workspace;
   Tables& T = a->T;
-  T.st = (uint8_t*)(ws + L.st);
-  T.key = (uint32_t*)(ws + L.key);
+  T.sk = (uint32_t*)(ws + L.sk);
   T.frame_of = (uint32_t*)(ws + L.frame_of);
   T.map = (uint32_t*)(ws + L.map);
   T.hframe = (uint32_t*)(ws + L.hframe);
@@ -700,6 +808,11 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   T.tags = (uint64_t*)(ws + L.tags);
   T.ctl = (Ctl*)(ws + L.ctl);
   T.xitems = (XItem*)(ws + L.xitems);
+  T.obits = (uint32_t*)(ws + L.obits);
+  T.wbits = (uint32_t*)(ws + L.wbits);
+  T.dlo = (uint32_t*)(ws + L.dlo);
+  T.dpre = (uint32_t*)(ws + L.dpre);
+  T.dw = (uint8_t*)(ws + L.dw);
   a->bounce = ws + L.bounce;
   T.frames = (char*)cfg->frames;
   T.hpc = hpc;
@@ -786,9 +899,17 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
   if (n && !acc) return UM_EINVAL;
   for (uint32_t i = 0; i < n; ++i)
     if (!range_ok(a, acc[i].off, acc[i].len)) return UM_EINVAL;
-  build_intervals(a, acc, n);
   um_status s = hand_in(a, stream);
   if (s) return s;
+  // a batch of more records than fit inline that is not already sorted and disjoint is
+  // deduplicated on the device; otherwise the records (or the <= kIvInline records after a
+  // 2n-event merge while they are packed into the kernel arguments) are the intervals
+  if (n > kIvInline && a->nblocks < (1u << 31) && !sorted_disjoint(a, acc, n)) {
+    s = device_intake(a, acc, n);
+    if (s) return s;
+  } else {
+    build_intervals(a, acc, n);
+  }
   s = run_gpu_op(a, 1);
   if (s) return s;
   return hand_out(a, stream);
@@ -808,6 +929,7 @@ UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, v
     s = run_gpu_op(a, 0);
     if (s) return s;
   } else {
+    if ((s = seq_room(a, 1))) return s;
     a->ops++;
     a->subops++;
     const uint32_t seq = ++a->clock;
@@ -837,6 +959,7 @@ static um_status discard_common(um_arena* a, uint64_t off, uint64_t len, void* s
   if (!range_ok(a, off, len)) return UM_EINVAL;
   um_status s = hand_in(a, stream);
   if (s) return s;
+  if ((s = seq_room(a, 1))) return s;
   a->ops++;
   a->subops++;
   const uint32_t seq = ++a->clock;
@@ -873,6 +996,7 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
   ENTER(a);
   um_status s = hand_in(a, stream);
   if (s) return s;
+  if ((s = seq_room(a, 1))) return s;
   a->ops++;
   a->subops++;
   const uint32_t seq = ++a->clock;
@@ -905,6 +1029,7 @@ UM_API um_status um_host_write(um_arena* a, uint64_t off, uint64_t len, void* st
   if (!range_ok(a, off, len)) return UM_EINVAL;
   um_status s = hand_in(a, stream);
   if (s) return s;
+  if ((s = seq_room(a, 1))) return s;
   a->ops++;
   a->subops++;
   const uint32_t seq = ++a->clock;
@@ -956,10 +1081,10 @@ UM_API um_status um_dump(um_arena* a, uint8_t* st, uint32_t* used_order, uint32_
   ENTER(a);
   um_status s = sync_ctl(a);
   if (s) return s;
+  std::vector<uint32_t> hsk(a->nblocks);
+  CK(cudaMemcpy(hsk.data(), a->T.sk, 4ull * a->nblocks, cudaMemcpyDeviceToHost));
   std::vector<uint8_t> hst(a->nblocks);
-  std::vector<uint32_t> hkey(a->nblocks);
-  CK(cudaMemcpy(hst.data(), a->T.st, a->nblocks, cudaMemcpyDeviceToHost));
-  CK(cudaMemcpy(hkey.data(), a->T.key, 4ull * a->nblocks, cudaMemcpyDeviceToHost));
+  for (uint32_t b = 0; b < a->nblocks; ++b) hst[b] = (uint8_t)(hsk[b] & 7u);
   if (st) memcpy(st, hst.data(), a->nblocks);
   std::vector<uint64_t> ring(a->L.cap);
   for (int r = 0; r < 2; ++r) {
@@ -974,7 +1099,7 @@ UM_API um_status um_dump(um_arena* a, uint8_t* st, uint32_t* used_order, uint32_
       uint64_t e = ring[p & (a->L.cap - 1)];
       uint32_t b = (uint32_t)e, k = (uint32_t)(e >> 32);
       uint8_t x = hst[b];
-      bool live = (r == RING_USED ? x == ST_G : (x == ST_GE || x == ST_GL)) && hkey[b] == k;
+      bool live = (r == RING_USED ? x == ST_G : (x == ST_GE || x == ST_GL)) && (hsk[b] >> 3) == k;
       if (live) {
         if (outp && cnt < a->nframes) outp[cnt] = b;
         ++cnt;

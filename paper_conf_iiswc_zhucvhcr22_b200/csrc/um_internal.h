@@ -34,6 +34,7 @@ struct Ctl {
   unsigned int vict_done;               // wide victim apply completion counter
   unsigned int need_acc;                // streaming classify: need-list slots taken so far
   unsigned int reach_tile;              // wide victim scan: first tile whose inclusive count >= k
+  unsigned int iv_m, iv_d;              // device intake: intervals produced, distinct blocks
   unsigned long long minkeep[2];        // wide victim scan: first kept ring position
   unsigned int k_want;                  // wide victim scan: victims wanted
   unsigned int need_cnt[2];             // streaming classify: need-list slots, by sub-op parity
@@ -53,8 +54,8 @@ enum { XI_H2D = 1u, XI_ZF = 2u, XI_D2H = 4u, XI_SWAP = 8u };
 
 // Everything a kernel needs, passed by value.
 struct Tables {
-  uint8_t* st;          // [nblocks] state
-  uint32_t* key;        // [nblocks] ukey / dkey (seq)
+  uint32_t* sk;         // [nblocks] packed state word (key << 3) | state, key = ukey or
+                        // dkey (a seq < 2^29): one load decides whether a ring entry is live
   uint32_t* frame_of;   // [nblocks] GPU frame (G/GE/GL) or NONE
   uint32_t* map;        // [nblocks] app-visible table: frame if mapped (G/GL) else NONE
   uint32_t* hframe;     // [nblocks] host frame holding the block's data (H only) or NONE
@@ -77,6 +78,12 @@ struct Tables {
   uint32_t* tile_cnt;   // [max tiles * 8] per-tile counter partials
   uint64_t* tags;       // [nblocks] content tags (harness)
   XItem* xitems;        // [nframes] exported plan of the current sub-op (K4-CE path)
+  // device intake (dedupe of unsorted / overlapping access batches, SURVEY A1 "op bitmap")
+  uint32_t* obits;      // [nwords] blocks touched by the batch (cleared after each batch)
+  uint32_t* wbits;      // [nwords] ... with a WRITE access
+  uint32_t* dlo;        // [nblocks] produced intervals: first block
+  uint32_t* dpre;       // [nblocks + 1] exclusive prefix of interval lengths (pre[m] = D)
+  uint8_t* dw;          // [nblocks] write flag per interval
   Ctl* ctl;
   char* frames;             // device, nframes * B
   char* const* hchunks;     // device array of host-chunk device pointers
@@ -112,6 +119,9 @@ constexpr int kScanTile = kScanTPB * kScanIPT;
 constexpr int kStTPB = 256;
 constexpr int kStIPT = 8;
 constexpr int kStTile = kStTPB * kStIPT;
+// multi-CTA classify: items per thread (two dependent gathers each)
+constexpr int kClsIPT = 8;
+constexpr int kClsTile = kStTPB * kClsIPT;
 constexpr int kVictTPB = 1024;
 constexpr int kVictIPT = 4;
 constexpr int kXferStages = 4;
@@ -147,5 +157,13 @@ cudaError_t launch_tags(const Tables& T, cudaStream_t s);
 cudaError_t launch_plan_commit(const Tables& T, uint32_t seq, uint32_t max_items, cudaStream_t s);
 cudaError_t launch_zero_items(const Tables& T, uint32_t i0, uint32_t i1, cudaStream_t s);
 cudaError_t launch_poison(const Tables& T, cudaStream_t s);
+// Device intake: mark a staged record chunk into the op bitmaps; turn the bitmap words
+// [w0, w1) into sorted disjoint intervals (dlo/dpre/dw, ctl->iv_m / iv_d); clear them.
+// Records must not cover more than kMarkMaxBlocks blocks each (the host splits them).
+constexpr uint32_t kMarkMaxBlocks = 1024;
+struct MarkRec { uint32_t lo, cnt, w, pad; };   // one staged (split) record, in blocks
+cudaError_t launch_mark(const Tables& T, const MarkRec* rec, uint32_t n, cudaStream_t s);
+cudaError_t launch_runs(const Tables& T, uint32_t w0, uint32_t w1, cudaStream_t s);
+cudaError_t launch_intake_clear(const Tables& T, uint32_t w0, uint32_t w1, cudaStream_t s);
 
 }  // namespace um

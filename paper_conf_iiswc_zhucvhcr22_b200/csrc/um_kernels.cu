@@ -10,6 +10,7 @@
 
 #include <cstdio>
 #include <cstdlib>
+#include <algorithm>
 
 namespace um {
 
@@ -32,6 +33,18 @@ __device__ __forceinline__ char* hptr(const Tables& T, uint32_t hf) {
 __device__ __forceinline__ void pdl_enter() {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   asm volatile("griddepcontrol.wait;" ::: "memory");
+}
+
+// Packed per-block state word (Tables::sk): bits 0-2 = state, bits 3-31 = key (seq).
+__device__ __forceinline__ uint8_t st_of(uint32_t w) { return (uint8_t)(w & 7u); }
+__device__ __forceinline__ uint32_t key_of(uint32_t w) { return w >> 3; }
+__device__ __forceinline__ uint32_t mk_sk(uint8_t st, uint32_t key) { return (key << 3) | st; }
+__device__ __forceinline__ uint8_t ld_st(const Tables& T, uint32_t b) { return st_of(T.sk[b]); }
+// liveness of ring entry (key kk, block b) whose ring holds state set {G} (USED) or {GE, GL} (DISC)
+__device__ __forceinline__ bool entry_live(const Tables& T, bool disc, uint32_t blk, uint32_t kk) {
+  const uint32_t w = T.sk[blk];
+  const uint8_t ss = st_of(w);
+  return (disc ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) && key_of(w) == kk;
 }
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -265,8 +278,7 @@ __device__ void scan_finish(const Tables& T, uint32_t ntiles, const int (&slots)
 __global__ void k_init(Tables T, int nh) {
   size_t tid = blockIdx.x * (size_t)blockDim.x + threadIdx.x, str = (size_t)gridDim.x * blockDim.x;
   for (size_t i = tid; i < T.nblocks; i += str) {
-    T.st[i] = ST_U;
-    T.key[i] = 0;
+    T.sk[i] = mk_sk(ST_U, 0);
     T.frame_of[i] = UM_NONE;
     T.map[i] = UM_NONE;
     T.hframe[i] = UM_NONE;
@@ -403,7 +415,7 @@ __device__ __forceinline__ void classify_single(const Tables& T, const OpIv& iv,
       }
       jlo = lo;
       const uint32_t bb = s_lo[lo] + (g - s_pre[lo]);
-      const uint8_t ss = T.st[bb];
+      const uint8_t ss = ld_st(T, bb);
       T.pin[bb] = seq;
       T.used_ring[(tail0 + idx) & T.cap_mask] = kseq | bb;
       b[k] = bb;
@@ -427,12 +439,10 @@ __device__ __forceinline__ void classify_single(const Tables& T, const OpIv& iv,
       T.needk[pN] = ss;
       T.needhf[pN] = (ss == ST_H) ? T.hframe[bb] : UM_NONE;
     } else if (ss == ST_GE) {   // revive: re-map the frame kept since the discard (L229)
-      T.st[bb] = ST_G;
-      T.key[bb] = seq;
+      T.sk[bb] = mk_sk(ST_G, seq);
       T.map[bb] = T.frame_of[bb];
     } else if (!touch) {
-      T.key[bb] = seq;          // refresh (G) / revalidate (GL -> G, L190)
-      if (ss == ST_GL) T.st[bb] = ST_G;
+      T.sk[bb] = mk_sk(ST_G, seq);   // refresh (G) / revalidate (GL -> G, L190)
     }
   }
   // counters (classes: U H HD G GE GL)
@@ -528,13 +538,13 @@ __device__ bool grid_finish(const Tables& T, const int (&slots)[NC], const long 
   return true;
 }
 
-__global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
+__global__ void __launch_bounds__(kStTPB, 5) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
                                                         int touch, unsigned long long tail0, int npar) {
   pdl_enter();
-  constexpr int TPB = kStTPB, IPT = kStIPT, TILE = kStTile;
+  constexpr int TPB = kStTPB, IPT = kClsIPT, TILE = kClsTile;
   __shared__ uint32_t s_lo[TILE], s_pre[TILE + 1];
   __shared__ uint32_t s_j0, s_m, s_base;
-  __shared__ uint32_t s_sc[TPB / 32 + 1];
+  __shared__ uint32_t s_off[IPT * (TPB / 32) + 1];
   __shared__ uint32_t s_cnt[8];
   const uint32_t tile = blockIdx.x, tbase = tile * TILE;
   if (threadIdx.x == 0) {
@@ -553,8 +563,8 @@ __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, OpIv iv, uint3
   const unsigned long long kseq = (unsigned long long)seq << 32;
   uint32_t b[IPT];
   uint8_t s[IPT];
-  uint32_t cls = 0;   // per-class counts (<= IPT < 16 each), 4 bits per class U H HD G GE GL
-  uint32_t nneed = 0, jlo = 0;
+  uint32_t cls = 0;   // per-class counts (<= IPT < 32 each), 5 bits per class U H HD G GE GL
+  uint32_t jlo = 0;
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint32_t idx = tbase + k * TPB + threadIdx.x;
@@ -570,47 +580,58 @@ __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, OpIv iv, uint3
       jlo = lo;
       const uint32_t bb = s_lo[lo] + (g - s_pre[lo]);
       b[k] = bb;
-      s[k] = T.st[bb];
+      s[k] = ld_st(T, bb);
     }
   }
+  // second dependent loads, all issued before any store (stores could alias them): the
+  // host frame of an H block, the kept frame of a GE block
+  uint32_t aux[IPT];
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) {
+    aux[k] = UM_NONE;
+    if (s[k] == ST_H) aux[k] = T.hframe[b[k]];
+    else if (s[k] == ST_GE) aux[k] = T.frame_of[b[k]];
+  }
+  unsigned bN[IPT];
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint32_t idx = tbase + k * TPB + threadIdx.x;
     if (idx < n) {
       T.pin[b[k]] = seq;
       T.used_ring[(tail0 + idx) & T.cap_mask] = kseq | b[k];
-      nneed += s[k] <= ST_HD;
-      cls += 1u << (4 * s[k]);
+      cls += 1u << (5 * s[k]);
     }
+    bN[k] = __ballot_sync(FULL, s[k] <= ST_HD);   // 0xff (no item) is > ST_HD
   }
-  uint32_t tot;
-  const uint32_t pre = cta_excl_scan<TPB>(nneed, tot, s_sc);
+  // need-list slots: one atomic per CTA for the base, then warp-ballot ranks so that
+  // consecutive lanes write consecutive slots (coalesced stores)
+  const uint32_t tot = ordered_offsets<TPB, IPT>(bN, bN, s_off) & 0xffffu;
   if (threadIdx.x == 0) s_base = tot ? atomicAdd(&T.ctl->need_cnt[npar], tot) : 0u;
   __syncthreads();
-  uint32_t pos = s_base + pre;
+  const uint32_t base = s_base;
+  const unsigned lt = lanemask_lt();
+  const int w = threadIdx.x >> 5;
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint8_t ss = s[k];
     if (ss == 0xff) continue;
     const uint32_t bb = b[k];
     if (ss <= ST_HD) {
+      const uint32_t pos = base + (s_off[k * (TPB / 32) + w] & 0xffffu) + __popc(bN[k] & lt);
       T.need[pos] = bb;
       T.needk[pos] = ss;
-      T.needhf[pos] = ss == ST_H ? T.hframe[bb] : UM_NONE;
-      ++pos;
+      T.needhf[pos] = aux[k];
     } else if (ss == ST_GE) {      // revive: re-map the frame kept since the discard (L229)
-      T.st[bb] = ST_G;
-      T.key[bb] = seq;
-      T.map[bb] = T.frame_of[bb];
+      T.sk[bb] = mk_sk(ST_G, seq);
+      T.map[bb] = aux[k];
     } else if (!touch) {
-      T.key[bb] = seq;             // refresh (G) / revalidate (GL -> G, L190)
-      if (ss == ST_GL) T.st[bb] = ST_G;
+      T.sk[bb] = mk_sk(ST_G, seq);   // refresh (G) / revalidate (GL -> G, L190)
     }
   }
   // counters (classes: U H HD G GE GL)
   const long long B = T.B;
-  const uint32_t c0 = cls & 15u, c1 = (cls >> 4) & 15u, c2 = (cls >> 8) & 15u, c3 = (cls >> 12) & 15u,
-                 c4 = (cls >> 16) & 15u, c5 = (cls >> 20) & 15u;
+  const uint32_t c0 = cls & 31u, c1 = (cls >> 5) & 31u, c2 = (cls >> 10) & 31u, c3 = (cls >> 15) & 31u,
+                 c4 = (cls >> 20) & 31u, c5 = (cls >> 25) & 31u;
   uint32_t v[6];
   if (touch) {
     // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE
@@ -665,8 +686,7 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
         if (first + q < w) {
           unsigned long long e = R[(pos + first + q) & T.cap_mask];
           uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
-          uint8_t ss = T.st[blk];
-          bool live = (ring == RING_USED ? ss == ST_G : (ss == ST_GE || ss == ST_GL)) && T.key[blk] == kk;
+          bool live = entry_live(T, ring == RING_DISC, blk, kk);
           bool cand = live && T.pin[blk] != seq;
           bb[q] = blk;
           livem |= (unsigned)live << q;
@@ -723,7 +743,7 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
     uint32_t isG = 0, needA = 0;
     if (j < found) {
       v = T.victim[j];
-      ss = T.st[v];
+      ss = ld_st(T, v);
       fr = T.frame_of[v];
       isG = ss == ST_G;
       if (isG && !evict_mode) {
@@ -745,7 +765,7 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
       T.vframe[j] = fr;
       T.vkind[j] = ss;
       T.vhf[j] = hf;
-      T.st[v] = isG ? ST_H : ST_HD;
+      T.sk[v] = mk_sk(isG ? ST_H : ST_HD, 0);
       T.map[v] = UM_NONE;
       T.frame_of[v] = UM_NONE;
       T.hframe[v] = hf;
@@ -890,8 +910,7 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
         const unsigned long long pos = disc ? s_dh + idx : s_uh + (idx - s_ld);
         const unsigned long long e = (disc ? T.disc_ring : T.used_ring)[pos & T.cap_mask];
         const uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
-        const uint8_t ss = T.st[blk];
-        live = (disc ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) && T.key[blk] == kk;
+        live = entry_live(T, disc, blk, kk);
         cand = live && T.pin[blk] != seq;
         bb[q] = blk;
       }
@@ -994,7 +1013,7 @@ __global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode)
     bool isG = false, needA = false;
     if (j < j1) {
       v = T.victim[j];
-      ss = T.st[v];
+      ss = ld_st(T, v);
       fr = T.frame_of[v];
       isG = ss == ST_G;
       if (isG && !evict_mode && T.needk[(uint32_t)f0 + j] == ST_H) hf = T.needhf[(uint32_t)f0 + j];
@@ -1027,7 +1046,7 @@ __global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode)
       T.vframe[j] = fr;
       T.vkind[j] = ss;
       T.vhf[j] = hf;
-      T.st[v] = isG ? ST_H : ST_HD;
+      T.sk[v] = mk_sk(isG ? ST_H : ST_HD, 0);
       T.map[v] = UM_NONE;
       T.frame_of[v] = UM_NONE;
       T.hframe[v] = hf;
@@ -1126,8 +1145,7 @@ __device__ __forceinline__ XItem item_plan(const Tables& T, uint32_t i, uint32_t
 // is recycled unless it was handed to the victim.
 __device__ __forceinline__ void item_commit(const Tables& T, uint32_t i, const XItem& x, uint32_t seq) {
   const uint32_t bb = T.need[i];
-  T.st[bb] = ST_G;
-  T.key[bb] = seq;
+  T.sk[bb] = mk_sk(ST_G, seq);
   T.frame_of[bb] = x.fr;
   T.map[bb] = x.fr;
   const uint32_t hf = T.needhf[i];
@@ -1366,9 +1384,14 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
   __shared__ uint32_t s_db, s_hav;
   __shared__ uint32_t s_cnt[8];
   Ctl* c = T.ctl;
-  const uint32_t tbase = blockIdx.x * TILE;
   const bool disc = kind == DIR_DISCARD || kind == DIR_DISCARD_LAZY;
   const bool active = !discard_off || kind == DIR_PREFETCH_HOST;
+  const unsigned long long kseq = (unsigned long long)seq << 32;
+  uint32_t nUnmap = 0, nD2H = 0, nAv = 0;
+  // persistent grid (resident CTAs) striding over tiles of TILE blocks
+  const uint32_t ntiles = (n + TILE - 1) / TILE;
+  for (uint32_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+  const uint32_t tbase = tile * TILE;
   uint8_t s[IPT];
   uint32_t hasf = 0;   // bit k: item k is an H block holding a host frame (discard)
   // per-thread counts of stack / list traffic: A = host frames (released by a discard
@@ -1378,7 +1401,7 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint32_t idx = tbase + k * TPB + threadIdx.x;   // coalesced
-    s[k] = idx < n ? T.st[lo + idx] : (uint8_t)0xff;
+    s[k] = idx < n ? ld_st(T, lo + idx) : (uint8_t)0xff;
     if (disc) {
       if (s[k] == ST_H && T.hframe[lo + idx] != UM_NONE) {
         hasf |= 1u << k;
@@ -1389,7 +1412,6 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
       nF += s[k] == ST_G || s[k] == ST_GE || s[k] == ST_GL;
     }
   }
-  const unsigned long long kseq = (unsigned long long)seq << 32;
   unsigned long long tot;
   const unsigned long long pre = block_excl_scan<TPB>(active ? pack2(nA, nF) : 0ull, tot, s_sc);
   if (threadIdx.x == 0) {
@@ -1414,7 +1436,6 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
   }
   __syncthreads();
   uint32_t rA = unpackA(pre), rF = unpackB(pre);
-  uint32_t nUnmap = 0, nD2H = 0, nAv = 0;
   if (active) {
 #pragma unroll
     for (int k = 0; k < IPT; ++k) {
@@ -1425,18 +1446,17 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
       if (disc) {
         T.disc_ring[(tail0 + idx) & T.cap_mask] = kseq | bb;
         if (ss == ST_G) {
-          T.st[bb] = kind == DIR_DISCARD ? ST_GE : ST_GL;
-          T.key[bb] = seq;
+          T.sk[bb] = mk_sk(kind == DIR_DISCARD ? ST_GE : ST_GL, seq);
           if (kind == DIR_DISCARD) {
             T.map[bb] = UM_NONE;
             ++nUnmap;
           }
         } else if (ss == ST_GL && kind == DIR_DISCARD) {
-          T.st[bb] = ST_GE;
+          T.sk[bb] = (T.sk[bb] & ~7u) | ST_GE;   // keeps its dkey (A6)
           T.map[bb] = UM_NONE;
           ++nUnmap;
         } else if (ss == ST_H) {
-          T.st[bb] = ST_HD;
+          T.sk[bb] = mk_sk(ST_HD, 0);
           if ((hasf >> k) & 1u) {   // the host copy is released (reading R1)
             T.hfree_stack[s_hb + rA] = T.hframe[bb];
             T.hframe[bb] = UM_NONE;
@@ -1462,9 +1482,11 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
           T.frame_of[bb] = UM_NONE;
           T.map[bb] = UM_NONE;
         }
-        if (ss != ST_H) T.st[bb] = ST_H;
+        if (ss != ST_H) T.sk[bb] = mk_sk(ST_H, 0);
       }
     }
+  }
+  __syncthreads();   // s_hb / s_fb / s_db are rewritten by the next tile
   }
   uint32_t v[3] = {nUnmap, nD2H, nAv};
   const int slots[3] = {S_UNMAPS, S_D2H, S_D2H_AV};
@@ -1508,8 +1530,7 @@ __global__ void __launch_bounds__(kScanTPB) k_ring_compact(Tables T, int ring, u
     if (ri < n) {
       e[k] = R[(tail - 1 - ri) & T.cap_mask];
       const uint32_t blk = (uint32_t)e[k], kk = (uint32_t)(e[k] >> 32);
-      const uint8_t ss = T.st[blk];
-      live = (ring == RING_USED ? ss == ST_G : (ss == ST_GE || ss == ST_GL)) && T.key[blk] == kk;
+      live = entry_live(T, ring == RING_DISC, blk, kk);
     }
     bL[k] = __ballot_sync(FULL, live);
     bZ[k] = 0;
@@ -1536,12 +1557,107 @@ __global__ void __launch_bounds__(kScanTPB) k_ring_compact(Tables T, int ring, u
 }
 
 // ------------------------------------------------------------------------------------
+// Device intake ("dedupe with the op bitmap"): a batch of accesses that is
+// not already sorted and disjoint is deduplicated here, not on the host.
+//   k_mark        every (split) record ORs its block range into obits (and wbits for a
+//                 WRITE access): the union, duplicates and overlaps collapse for free
+//   k_runs        one ordered scan over the bitmap words turns set-bit runs into sorted
+//                 disjoint intervals (a run also breaks where the write flag changes):
+//                 interval j = (first block, rank of that block among all set bits, W),
+//                 ranked by block scan + decoupled look-back over word tiles
+//   k_intake_clear zeroes the words again for the next batch
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_mark(Tables T, const MarkRec* rec, uint32_t n) {
+  pdl_enter();
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const MarkRec r = rec[i];
+    const uint32_t lo = r.lo, hi = r.lo + r.cnt;   // blocks [lo, hi), cnt <= kMarkMaxBlocks
+    for (uint32_t w = lo >> 5; w <= (hi - 1) >> 5; ++w) {
+      const uint32_t a = max(lo, w << 5) - (w << 5), b = min(hi, (w + 1) << 5) - (w << 5);   // bits [a, b)
+      const uint32_t mask = (b - a == 32) ? FULL : (((1u << (b - a)) - 1u) << a);
+      atomicOr(&T.obits[w], mask);
+      if (r.w) atomicOr(&T.wbits[w], mask);
+    }
+  }
+}
+
+constexpr int kRunTPB = 512, kRunIPT = 8, kRunTile = kRunTPB * kRunIPT;   // words per tile
+
+__global__ void __launch_bounds__(kRunTPB) k_runs(Tables T, uint32_t w0, uint32_t w1) {
+  pdl_enter();
+  __shared__ unsigned long long s_sc[kRunTPB / 32];
+  __shared__ unsigned long long s_excl;
+  const uint32_t tile = blockIdx.x, ntiles = gridDim.x;
+  const uint32_t first = w0 + tile * kRunTile + threadIdx.x * kRunIPT;   // this thread's words
+  uint32_t o[kRunIPT], wb[kRunIPT], st[kRunIPT];
+  uint32_t co = 0, cw = 0;   // carry: top bit of the previous word
+  if (first < w1 && first > w0) {
+    co = T.obits[first - 1] >> 31;
+    cw = T.wbits[first - 1] >> 31;
+  }
+  uint32_t nS = 0, nB = 0;
+#pragma unroll
+  for (int q = 0; q < kRunIPT; ++q) {
+    const uint32_t w = first + q;
+    o[q] = w < w1 ? T.obits[w] : 0u;
+    wb[q] = w < w1 ? T.wbits[w] : 0u;
+  }
+#pragma unroll
+  for (int q = 0; q < kRunIPT; ++q) {
+    // bit i starts an interval if it is set and (bit i-1 is clear or has the other W)
+    const uint32_t P = (o[q] << 1) | co, PW = (wb[q] << 1) | cw;
+    st[q] = o[q] & (~P | (wb[q] ^ PW));
+    co = o[q] >> 31;
+    cw = wb[q] >> 31;
+    nS += __popc(st[q]);
+    nB += __popc(o[q]);
+  }
+  unsigned long long tot;
+  const unsigned long long pre = block_excl_scan<kRunTPB>(pack2(nS, nB), tot, s_sc);
+  if (threadIdx.x < 32) {
+    const unsigned long long ex = lookback_warp(T, tile, tot);
+    if (threadIdx.x == 0) s_excl = ex;
+  }
+  __syncthreads();
+  uint32_t J = unpackA(s_excl) + unpackA(pre), R = unpackB(s_excl) + unpackB(pre);
+#pragma unroll
+  for (int q = 0; q < kRunIPT; ++q) {
+    uint32_t m = st[q];
+    while (m) {
+      const int i = __ffs(m) - 1;
+      m &= m - 1;
+      const uint32_t below = (1u << i) - 1u;
+      T.dlo[J] = (first + q) * 32u + (uint32_t)i;
+      T.dpre[J] = R + __popc(o[q] & below);
+      T.dw[J] = (uint8_t)((wb[q] >> i) & 1u);
+      ++J;
+    }
+    R += __popc(o[q]);
+  }
+  if (tile == ntiles - 1 && threadIdx.x == 0) {
+    const unsigned long long all = s_excl + tot;
+    T.ctl->iv_m = unpackA(all);
+    T.ctl->iv_d = unpackB(all);
+    T.dpre[unpackA(all)] = unpackB(all);
+  }
+  scan_finish(T, ntiles);
+}
+
+__global__ void __launch_bounds__(256) k_intake_clear(Tables T, uint32_t w0, uint32_t w1) {
+  pdl_enter();
+  for (uint32_t w = w0 + blockIdx.x * blockDim.x + threadIdx.x; w < w1; w += gridDim.x * blockDim.x) {
+    T.obits[w] = 0u;
+    T.wbits[w] = 0u;
+  }
+}
+
+// ------------------------------------------------------------------------------------
 // Harness: host writes (Listing 6 "Generate data, labels").
 // ------------------------------------------------------------------------------------
 __global__ void k_hw_alloc(Tables T, uint32_t lo, uint32_t n) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     uint32_t bb = lo + i;
-    if (T.st[bb] != ST_H) {
+    if (ld_st(T, bb) != ST_H) {
       atomicExch(&T.ctl->err, 1u);
       continue;
     }
@@ -1564,7 +1680,7 @@ __global__ void __launch_bounds__(256) k_hw_fill(Tables T, uint32_t lo, uint32_t
   for (unsigned long long u = blockIdx.x; u < units; u += gridDim.x) {
     uint32_t bb = lo + (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
     uint32_t hf = T.hframe[bb];
-    if (hf == UM_NONE || T.st[bb] != ST_H) continue;
+    if (hf == UM_NONE || ld_st(T, bb) != ST_H) continue;
     unsigned long long sv = ((unsigned long long)seq << 32) | bb;
     uint4 pat = make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32));
     uint4* dst = reinterpret_cast<uint4*>(hptr(T, hf) + (size_t)ch * CH);
@@ -1578,7 +1694,7 @@ __global__ void __launch_bounds__(256) k_hw_fill(Tables T, uint32_t lo, uint32_t
 __global__ void __launch_bounds__(256) k_tags(Tables T) {
   __shared__ int s_ok, s_zero;
   for (uint32_t bb = blockIdx.x; bb < T.nblocks; bb += gridDim.x) {
-    uint8_t ss = T.st[bb];
+    uint8_t ss = ld_st(T, bb);
     const uint4* src = nullptr;
     if (ss == ST_G || ss == ST_GE || ss == ST_GL) {
       uint32_t fr = T.frame_of[bb];
@@ -1618,6 +1734,7 @@ __global__ void __launch_bounds__(256) k_tags(Tables T) {
 static int g_nsm = 0;
 static int g_vscan_occ = 1;   // resident k_victims_scan CTAs per SM
 static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch (A/B)
+static int g_dir_occ = 8;     // resident k_directive CTAs per SM (persistent grid)
 
 cudaError_t setup_kernels() {
   int dev;
@@ -1626,9 +1743,29 @@ cudaError_t setup_kernels() {
   e = cudaDeviceGetAttribute(&g_nsm, cudaDevAttrMultiProcessorCount, dev);
   if (e) return e;
   if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
+  // One L1/shared carveout for every paging kernel: k_service needs 144 KB of shared
+  // memory, and a carveout change between consecutive kernels forces the SM to drain.
+  // UM_CARVEOUT=0 keeps the driver's per-kernel choice (A/B).
+  bool carve = true;
+  if (const char* v = getenv("UM_CARVEOUT")) carve = atoi(v) != 0;
+  if (carve) {
+    const void* ks[] = {(const void*)k_classify, (const void*)k_victims, (const void*)k_plan_small,
+                        (const void*)k_victims_scan, (const void*)k_victims_apply, (const void*)k_service,
+                        (const void*)k_app_stamp, (const void*)k_directive, (const void*)k_ring_compact,
+                        (const void*)k_plan_commit, (const void*)k_zero_items, (const void*)k_mark,
+                        (const void*)k_runs, (const void*)k_intake_clear};
+    for (const void* k : ks) {
+      e = cudaFuncSetAttribute(k, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
+      if (e) return e;
+    }
+  }
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_vscan_occ, k_victims_scan, kScanTPB, 0);
   if (e) return e;
   if (g_vscan_occ < 1) g_vscan_occ = 1;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_dir_occ, k_directive, kStTPB, 0);
+  if (e) return e;
+  if (g_dir_occ < 1) g_dir_occ = 1;
+  if (const char* v = getenv("UM_DIR_OCC")) g_dir_occ = std::max(1, atoi(v));
   int smem = (int)(kXferChunk * (1 + 2 * kXferStages));
   return cudaFuncSetAttribute(k_service, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
 }
@@ -1665,7 +1802,7 @@ cudaError_t launch_poison(const Tables& T, cudaStream_t s) {
 
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
                             unsigned long long tail0, int npar, cudaStream_t s) {
-  unsigned nt = n ? ceil_div(n, kStTile) : 1;
+  unsigned nt = n ? ceil_div(n, kClsTile) : 1;
   cudaError_t le__ = launch_pdl(k_classify, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar);
   if (le__) return le__;
   return cudaGetLastError();
@@ -1725,6 +1862,7 @@ cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, 
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq, int discard_off,
                              unsigned long long tail0, cudaStream_t s) {
   unsigned nt = n ? ceil_div(n, kStTile) : 1;
+  if (nt > (unsigned)(g_nsm * g_dir_occ)) nt = (unsigned)(g_nsm * g_dir_occ);   // persistent
   cudaError_t le__ = launch_pdl(k_directive, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq, discard_off, tail0);
   if (le__) return le__;
   return cudaGetLastError();
@@ -1767,6 +1905,31 @@ cudaError_t launch_tags(const Tables& T, cudaStream_t s) {
   unsigned grid = T.nblocks < (uint32_t)g_nsm * 16 ? T.nblocks : (unsigned)g_nsm * 16;
   if (!grid) grid = 1;
   k_tags<<<grid, 256, 0, s>>>(T);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_mark(const Tables& T, const MarkRec* rec, uint32_t n, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  unsigned grid = ceil_div(n, 256);
+  if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
+  cudaError_t e = launch_pdl(k_mark, dim3(grid), dim3(256), 0, s, T, rec, n);
+  if (e) return e;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_runs(const Tables& T, uint32_t w0, uint32_t w1, cudaStream_t s) {
+  unsigned nt = w1 > w0 ? ceil_div(w1 - w0, kRunTile) : 1;
+  cudaError_t e = launch_pdl(k_runs, dim3(nt), dim3(kRunTPB), 0, s, T, w0, w1);
+  if (e) return e;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_intake_clear(const Tables& T, uint32_t w0, uint32_t w1, cudaStream_t s) {
+  if (w1 <= w0) return cudaSuccess;
+  unsigned grid = ceil_div(w1 - w0, 256);
+  if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
+  cudaError_t e = launch_pdl(k_intake_clear, dim3(grid), dim3(256), 0, s, T, w0, w1);
+  if (e) return e;
   return cudaGetLastError();
 }
 

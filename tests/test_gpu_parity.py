@@ -266,3 +266,23 @@ def test_c4_sweep_cases(pressure, mode):
     for S, p, sc in [(64 << 10, 1.0, False), (32 << 20, 0.5, False), (32 << 20, 0.25, True), (256 << 20, 1.0, False)]:
         t = tg.gen_c4(S, p, block_bytes=64 << 10, pressure=pressure, scattered=sc)
         assert_parity(t, mode)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_device_intake(seed, mode):
+    """Touch batches of 1-200 unsorted, overlapping ranges with mixed W flags: batches of
+    more than 24 records are deduplicated on the device (op bitmap: k_mark, k_runs,
+    SURVEY §8(a) A1); distinct blocks often exceed nframes (sub-op splitting)."""
+    t = tg.gen_random(seed, block_bytes=64 << 10, arena_bytes=32 << 20, budget_bytes=4 << 20, n_ops=400,
+                      max_ranges=200, max_blocks=8, zipf_s=0.8)
+    assert_parity(t, mode)
+
+
+@pytest.mark.parametrize("mode", ["eager", "lazy"])
+def test_device_intake_wide(mode):
+    """Device-intake batches whose sub-ops exceed 4096 blocks (multi-CTA classify on the
+    device-made interval list, wide victim scan) and span several sub-ops."""
+    t = tg.gen_random(7, block_bytes=4 << 10, arena_bytes=64 << 20, budget_bytes=24 << 20, n_ops=120,
+                      max_ranges=1500, max_blocks=32, zipf_s=0.6)
+    assert_parity(t, mode)
