@@ -65,7 +65,7 @@ static Layout make_layout(const um_config* c) {
   L.cap = pow2_ceil(std::max<uint64_t>(1024, 4 * nf));
   // tiles: classify/directive scan <= nblocks items, compaction <= cap, the wide victim
   // scan <= |DISC| + |USED| <= 2 * cap (its bound is also clamped to 2 * cap)
-  L.max_tiles = (std::max(nb, 2 * L.cap) + kScanTile - 1) / kScanTile + 1;
+  L.max_tiles = (std::max(nb, 2 * L.cap) + 2048 - 1) / 2048 + 1;   // smallest scan tile: 2048 items
   L.stage_bytes = std::min<uint64_t>(64ull << 20, 12 * nb + (1 << 20));
   uint64_t o = 0;
   auto take = [&](uint64_t bytes) {

@@ -839,12 +839,14 @@ __global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, OpIv iv, uint
 // them.  Pass 2 reclaims the victims in parallel (host frames for write-backs come
 // from the free stack, one atomic per CTA chunk; ids are not observable).
 // ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want,
+constexpr int kVsTPB = 256, kVsIPT = 8, kVsTile = kVsTPB * kVsIPT;   // victim scan tiles
+
+__global__ void __launch_bounds__(kVsTPB, 6) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want,
                                                             int npar) {
   pdl_enter();
-  constexpr int NW = kScanTPB / 32;
+  constexpr int NW = kVsTPB / 32;
   const unsigned long long FP = 2ull << 62;
-  __shared__ uint32_t s_off[kScanIPT * NW + 1];
+  __shared__ uint32_t s_off[kVsIPT * NW + 1];
   __shared__ unsigned long long s_excl, s_dh, s_ld, s_uh, s_lu, s_mk[2];
   __shared__ uint32_t s_k, s_nn, s_f0, s_tile, s_skip;
   __shared__ int s_last;
@@ -868,7 +870,7 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
   __syncthreads();
   const unsigned long long L = s_ld + s_lu;
   const uint32_t k = s_k;
-  const uint32_t ntiles = k ? (uint32_t)((L + kScanTile - 1) / kScanTile) : 0u;
+  const uint32_t ntiles = k ? (uint32_t)((L + kVsTile - 1) / kVsTile) : 0u;
   const int w = threadIdx.x >> 5;
   const unsigned lt = lanemask_lt();
   const unsigned me = 1u << (threadIdx.x & 31);
@@ -883,7 +885,7 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
     const uint32_t tile = s_tile, skip = s_skip;
     __syncthreads();
     if (skip == 2u) break;
-    const unsigned long long tbase = (unsigned long long)tile * kScanTile;
+    const unsigned long long tbase = (unsigned long long)tile * kVsTile;
     if (skip == 1u) {
       // every later ticket skips as well, so this CTA is done
       if (threadIdx.x == 0) {
@@ -898,13 +900,13 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
       }
       break;
     }
-    uint32_t bb[kScanIPT];
-    unsigned bC[kScanIPT], bL[kScanIPT];
+    uint32_t bb[kVsIPT];
+    unsigned bC[kVsIPT], bL[kVsIPT];
 #pragma unroll
-    for (int q = 0; q < kScanIPT; ++q) {
+    for (int q = 0; q < kVsIPT; ++q) {
       bb[q] = 0;
       bool live = false, cand = false;
-      const unsigned long long idx = tbase + q * kScanTPB + threadIdx.x;
+      const unsigned long long idx = tbase + q * kVsTPB + threadIdx.x;
       if (idx < L) {
         const bool disc = idx < s_ld;
         const unsigned long long pos = disc ? s_dh + idx : s_uh + (idx - s_ld);
@@ -917,7 +919,7 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
       bC[q] = __ballot_sync(FULL, cand);
       bL[q] = __ballot_sync(FULL, live);
     }
-    const uint32_t tt = ordered_offsets<kScanTPB, kScanIPT>(bC, bC, s_off);
+    const uint32_t tt = ordered_offsets<kVsTPB, kVsIPT>(bC, bC, s_off);
     const unsigned long long tot = pack2(tt & 0xffffu, 0);
     if (threadIdx.x < 32) {
       unsigned long long ex = lookback_warp(T, tile, tot);
@@ -929,7 +931,7 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
     __syncthreads();
     const uint32_t eC = unpackA(s_excl);
 #pragma unroll
-    for (int q = 0; q < kScanIPT; ++q) {
+    for (int q = 0; q < kVsIPT; ++q) {
       bool sel = false;
       if (bC[q] & me) {
         const uint32_t r = eC + (s_off[q * NW + w] & 0xffffu) + __popc(bC[q] & lt);
@@ -939,7 +941,7 @@ __global__ void __launch_bounds__(kScanTPB) k_victims_scan(Tables T, uint32_t se
         }
       }
       if ((bL[q] & me) && !sel) {
-        const unsigned long long idx = tbase + q * kScanTPB + threadIdx.x;
+        const unsigned long long idx = tbase + q * kVsTPB + threadIdx.x;
         if (idx < s_ld) mk0 = min(mk0, s_dh + idx);
         else mk1 = min(mk1, s_uh + (idx - s_ld));
       }
@@ -1743,10 +1745,10 @@ cudaError_t setup_kernels() {
   e = cudaDeviceGetAttribute(&g_nsm, cudaDevAttrMultiProcessorCount, dev);
   if (e) return e;
   if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
-  // One L1/shared carveout for every paging kernel: k_service needs 144 KB of shared
-  // memory, and a carveout change between consecutive kernels forces the SM to drain.
-  // UM_CARVEOUT=0 keeps the driver's per-kernel choice (A/B).
-  bool carve = true;
+  // Optionally one L1/shared carveout for every paging kernel (k_service needs 144 KB of
+  // shared memory; a carveout change between consecutive kernels can force an SM drain).
+  // UM_CARVEOUT=1 turns it on (A/B; off by default).
+  bool carve = false;   // measured: no effect on the C1 small-op rate (B200, r01)
   if (const char* v = getenv("UM_CARVEOUT")) carve = atoi(v) != 0;
   if (carve) {
     const void* ks[] = {(const void*)k_classify, (const void*)k_victims, (const void*)k_plan_small,
@@ -1759,7 +1761,7 @@ cudaError_t setup_kernels() {
       if (e) return e;
     }
   }
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_vscan_occ, k_victims_scan, kScanTPB, 0);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_vscan_occ, k_victims_scan, kVsTPB, 0);
   if (e) return e;
   if (g_vscan_occ < 1) g_vscan_occ = 1;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_dir_occ, k_directive, kStTPB, 0);
@@ -1825,14 +1827,14 @@ cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, u
                                 uint32_t max_victims, int npar, cudaStream_t s) {
   // persistent scan grid: never more CTAs than can be resident (tiles are taken from a
   // ticket in order and a tile may wait on its predecessors' status)
-  unsigned nt = ceil_div(scan_bound ? scan_bound : 1, kScanTile);
+  unsigned nt = ceil_div(scan_bound ? scan_bound : 1, kVsTile);
   const unsigned cap = (unsigned)(g_nsm * g_vscan_occ);
-  cudaError_t le__ = launch_pdl(k_victims_scan, dim3(nt < cap ? nt : cap), dim3(kScanTPB), 0, s, T, seq, evict_mode, want, npar);
+  cudaError_t le__ = launch_pdl(k_victims_scan, dim3(nt < cap ? nt : cap), dim3(kVsTPB), 0, s, T, seq, evict_mode, want, npar);
   if (le__) return le__;
   cudaError_t e = cudaGetLastError();
   if (e) return e;
-  unsigned grid = ceil_div(max_victims ? max_victims : 1, 1024);
-  if (grid > (unsigned)g_nsm * 4) grid = g_nsm * 4;
+  unsigned grid = ceil_div(max_victims ? max_victims : 1, 512);
+  if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
   le__ = launch_pdl(k_victims_apply, dim3(grid), dim3(256), 0, s, T, evict_mode);
   if (le__) return le__;
   return cudaGetLastError();
