@@ -120,7 +120,7 @@ constexpr int kStTPB = 256;
 constexpr int kStIPT = 8;
 constexpr int kStTile = kStTPB * kStIPT;
 // multi-CTA classify: items per thread (two dependent gathers each)
-constexpr int kClsIPT = 8;
+constexpr int kClsIPT = 4;
 constexpr int kClsTile = kStTPB * kClsIPT;
 constexpr int kVictTPB = 1024;
 constexpr int kVictIPT = 4;

@@ -538,7 +538,7 @@ __device__ bool grid_finish(const Tables& T, const int (&slots)[NC], const long 
   return true;
 }
 
-__global__ void __launch_bounds__(kStTPB, 5) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
+__global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
                                                         int touch, unsigned long long tail0, int npar) {
   pdl_enter();
   constexpr int TPB = kStTPB, IPT = kClsIPT, TILE = kClsTile;
