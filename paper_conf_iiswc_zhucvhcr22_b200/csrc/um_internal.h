@@ -38,6 +38,7 @@ struct Ctl {
   unsigned long long minkeep[2];        // wide victim scan: first kept ring position
   unsigned int k_want;                  // wide victim scan: victims wanted
   unsigned int need_cnt[2];             // streaming classify: need-list slots, by sub-op parity
+  unsigned int k0_take, k0_pend;        // wide victim scan with k = 0: frames to take, pending flag
   // counters, striped over 8 cache lines by CTA index (fire-and-forget atomics from
   // thousands of CTAs do not serialise on one address); the host sums the stripes
   long long stats[8][S_N];

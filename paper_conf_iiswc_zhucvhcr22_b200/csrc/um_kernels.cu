@@ -219,7 +219,9 @@ __device__ __forceinline__ void block_counts_to(const Tables& T, uint32_t (&c)[N
     if ((threadIdx.x & 31) == 0 && v) atomicAdd(&sm[i], v);
   }
   __syncthreads();
-  if (threadIdx.x < NC && slots[threadIdx.x] >= 0) stat_add(T, slots[threadIdx.x], (long long)sm[threadIdx.x] * mul[threadIdx.x]);
+#pragma unroll
+  for (int i = 0; i < NC; ++i)   // static indices: the slot tables stay in registers
+    if (threadIdx.x == i && slots[i] >= 0) stat_add(T, slots[i], (long long)sm[i] * mul[i]);
 }
 
 // Multi-CTA scans do not add their counters with same-address atomics (thousands of
@@ -263,7 +265,9 @@ __device__ void scan_finish(const Tables& T, uint32_t ntiles, const int (&slots)
     }
     for (uint32_t i = threadIdx.x; i < ntiles; i += blockDim.x) T.tile_status[i] = 0ull;
     __syncthreads();
-    if (threadIdx.x < NC && slots[threadIdx.x] >= 0) stat_add(T, slots[threadIdx.x], (long long)s_sum[threadIdx.x] * mul[threadIdx.x]);
+#pragma unroll
+    for (int i = 0; i < NC; ++i)
+      if (threadIdx.x == i && slots[i] >= 0) stat_add(T, slots[i], (long long)s_sum[i] * mul[i]);
     if (threadIdx.x == 0) {
       T.ctl->scan_done = 0;
       T.ctl->scan_ticket = 0;
@@ -300,6 +304,7 @@ __global__ void k_init(Tables T, int nh) {
     for (int j = 0; j < 8; ++j)
       for (int i = 0; i < S_N; ++i) c->stats[j][i] = 0;
     c->need_cnt[0] = c->need_cnt[1] = 0;
+    c->k0_take = c->k0_pend = 0;
   }
 }
 
@@ -533,55 +538,84 @@ __device__ bool grid_finish(const Tables& T, const int (&slots)[NC], const long 
     if ((threadIdx.x & 31) == 0 && acc) atomicAdd(&s_sum[k], acc);
   }
   __syncthreads();
-  if (threadIdx.x < NC && slots[threadIdx.x] >= 0) stat_add(T, slots[threadIdx.x], (long long)s_sum[threadIdx.x] * mul[threadIdx.x]);
+#pragma unroll
+  for (int i = 0; i < NC; ++i)
+    if (threadIdx.x == i && slots[i] >= 0) stat_add(T, slots[i], (long long)s_sum[i] * mul[i]);
   if (threadIdx.x == 0) T.ctl->scan_done = 0;
   return true;
 }
 
-__global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
-                                                        int touch, unsigned long long tail0, int npar) {
+__global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
+                                                        uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
+                                                        int npar) {
   pdl_enter();
-  constexpr int TPB = kStTPB, IPT = kClsIPT, TILE = kClsTile;
-  __shared__ uint32_t s_lo[TILE], s_pre[TILE + 1];
-  __shared__ uint32_t s_j0, s_m, s_base;
-  __shared__ uint32_t s_off[IPT * (TPB / 32) + 1];
+  constexpr int TPB = kStTPB, IPT = kClsIPT, TILE = kClsTile, NW = TPB / 32, NWORD = TILE / 32;
+  static_assert(NWORD <= 32, "one bitmap word per lane");
+  // Interval lookup without a search: the tile's interval slice [ja, jb] is staged as
+  // d[q] = lo - pre (block = rank + d), and the start of every slice interval but the
+  // first sets one bit of a TILE-bit map at its in-tile position.  The interval of item
+  // i is then the number of set bits in [0, i] (a warp prefix of word popcounts plus one
+  // masked popc), so every item costs O(1) instead of a log2(TILE)-step dependent search.
+  __shared__ uint32_t s_d[TILE];
+  __shared__ uint32_t s_bits[NWORD];
+  __shared__ uint32_t s_base;
+  __shared__ uint32_t s_off[IPT * NW + 1];
   __shared__ uint32_t s_cnt[8];
-  const uint32_t tile = blockIdx.x, tbase = tile * TILE;
-  if (threadIdx.x == 0) {
-    const uint32_t ja = iv.inl ? iv_find(iv, g0 + tbase) : iv.tj[2 * tile];
-    const uint32_t jb = iv.inl ? iv_find(iv, g0 + min(n, tbase + TILE) - 1) : iv.tj[2 * tile + 1];
-    s_j0 = ja;
-    s_m = jb - ja + 1;
+  const uint32_t tile = blockIdx.x, tbase = tile * TILE, gt = g0 + tbase;
+  const uint32_t ja = iv.inl ? iv_find(iv, gt) : iv.tj[2 * tile];
+  const uint32_t jb = iv.inl ? iv_find(iv, g0 + min(n, tbase + TILE) - 1) : iv.tj[2 * tile + 1];
+  const uint32_t m = jb - ja + 1;   // <= TILE (every slice interval holds an item of the tile)
+  uint32_t qlo[IPT], qpre[IPT];
+#pragma unroll
+  for (int r = 0; r < IPT; ++r) {
+    const uint32_t q = r * TPB + threadIdx.x;
+    if (q < m) {
+      qlo[r] = iv_lo(iv, ja + q);
+      qpre[r] = iv_pre(iv, ja + q);
+    }
+  }
+  if (threadIdx.x < NWORD) s_bits[threadIdx.x] = 0u;
+  __syncthreads();
+#pragma unroll
+  for (int r = 0; r < IPT; ++r) {
+    const uint32_t q = r * TPB + threadIdx.x;
+    if (q < m) {
+      s_d[q] = qlo[r] - qpre[r];
+      if (q) {
+        const uint32_t pos = qpre[r] - gt;   // in (0, TILE)
+        atomicOr(&s_bits[pos >> 5], 1u << (pos & 31));
+      }
+    }
   }
   __syncthreads();
-  const uint32_t j0 = s_j0, m = s_m;
-  for (uint32_t q = threadIdx.x; q <= m; q += TPB) {
-    if (q < m) s_lo[q] = iv_lo(iv, j0 + q);
-    s_pre[q] = iv_pre(iv, j0 + q);
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t wexcl;   // lane l: set bits in words [0, l)
+  {
+    const uint32_t c = lane < NWORD ? __popc(s_bits[lane]) : 0u;
+    uint32_t x = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    wexcl = x - c;
   }
-  __syncthreads();
+  const unsigned le = lanemask_lt() | (1u << lane);
   const unsigned long long kseq = (unsigned long long)seq << 32;
   uint32_t b[IPT];
   uint8_t s[IPT];
   uint32_t cls = 0;   // per-class counts (<= IPT < 32 each), 5 bits per class U H HD G GE GL
-  uint32_t jlo = 0;
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint32_t idx = tbase + k * TPB + threadIdx.x;
-    s[k] = 0xff;
-    b[k] = 0;
-    if (idx < n) {
-      const uint32_t g = g0 + idx;
-      uint32_t lo = jlo, hi = m;   // largest j with s_pre[j] <= g (a thread's items ascend)
-      while (hi - lo > 1) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (s_pre[mid] <= g) lo = mid; else hi = mid;
-      }
-      jlo = lo;
-      const uint32_t bb = s_lo[lo] + (g - s_pre[lo]);
-      b[k] = bb;
-      s[k] = ld_st(T, bb);
-    }
+    const int wi = k * NW + w;   // bitmap word of item (k, thread): in-tile position k*TPB + tid
+    const uint32_t j = __shfl_sync(FULL, wexcl, wi) + __popc(s_bits[wi] & le);
+    b[k] = g0 + idx + s_d[j];
+  }
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) {
+    const uint32_t idx = tbase + k * TPB + threadIdx.x;
+    s[k] = idx < n ? ld_st(T, b[k]) : (uint8_t)0xff;
   }
   // second dependent loads, all issued before any store (stores could alias them): the
   // host frame of an H block, the kept frame of a GE block
@@ -610,7 +644,6 @@ __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, OpIv iv, uint3
   __syncthreads();
   const uint32_t base = s_base;
   const unsigned lt = lanemask_lt();
-  const int w = threadIdx.x >> 5;
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint8_t ss = s[k];
@@ -817,7 +850,7 @@ __global__ void __launch_bounds__(kVictTPB) k_victims(Tables T, uint32_t seq, in
 
 // K1+K2+K3 for a sub-op that fits one tile: one CTA classifies, compacts and selects
 // victims (saves a launch per small op; same code as the multi-CTA kernels).
-__global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
+__global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, const __grid_constant__ OpIv iv, uint32_t g0, uint32_t n, uint32_t seq,
                                                          int touch, unsigned long long tail0) {
   pdl_enter();
   classify_single<kVictTPB, kSmallPlan / kVictTPB>(T, iv, g0, n, seq, touch, tail0);
@@ -841,7 +874,7 @@ __global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, OpIv iv, uint
 // ------------------------------------------------------------------------------------
 constexpr int kVsTPB = 256, kVsIPT = 8, kVsTile = kVsTPB * kVsIPT;   // victim scan tiles
 
-__global__ void __launch_bounds__(kVsTPB, 6) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want,
+__global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want,
                                                             int npar) {
   pdl_enter();
   constexpr int NW = kVsTPB / 32;
@@ -868,6 +901,20 @@ __global__ void __launch_bounds__(kVsTPB, 6) k_victims_scan(Tables T, uint32_t s
     }
   }
   __syncthreads();
+  if (s_k == 0) {
+    // nothing to evict (the sub-op's need fits the free frames): one CTA does the
+    // bookkeeping of an empty victim list, the others exit; no ticket, look-back or
+    // completion counter is touched, so they stay clean for the next scan
+    // free_top and used_tail are advanced by k_victims_apply, which runs after this
+    // grid completes: other CTAs of this grid may still be reading free_top
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      c->n_vict = 0;
+      c->f0 = s_f0;
+      c->k0_take = evict_mode ? 0u : min(s_f0, s_nn);
+      c->k0_pend = evict_mode ? 0u : 1u;
+    }
+    return;
+  }
   const unsigned long long L = s_ld + s_lu;
   const uint32_t k = s_k;
   const uint32_t ntiles = k ? (uint32_t)((L + kVsTile - 1) / kVsTile) : 0u;
@@ -900,25 +947,35 @@ __global__ void __launch_bounds__(kVsTPB, 6) k_victims_scan(Tables T, uint32_t s
       }
       break;
     }
-    uint32_t bb[kVsIPT];
+    // three load phases, each with all kVsIPT loads in flight: ring entries, the state
+    // words of their blocks (liveness), the pin words of live entries
+    uint32_t bb[kVsIPT], kk[kVsIPT], wv[kVsIPT];
     unsigned bC[kVsIPT], bL[kVsIPT];
 #pragma unroll
     for (int q = 0; q < kVsIPT; ++q) {
-      bb[q] = 0;
-      bool live = false, cand = false;
       const unsigned long long idx = tbase + q * kVsTPB + threadIdx.x;
+      unsigned long long e = ~0ull;
       if (idx < L) {
         const bool disc = idx < s_ld;
         const unsigned long long pos = disc ? s_dh + idx : s_uh + (idx - s_ld);
-        const unsigned long long e = (disc ? T.disc_ring : T.used_ring)[pos & T.cap_mask];
-        const uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
-        live = entry_live(T, disc, blk, kk);
-        cand = live && T.pin[blk] != seq;
-        bb[q] = blk;
+        e = (disc ? T.disc_ring : T.used_ring)[pos & T.cap_mask];
       }
-      bC[q] = __ballot_sync(FULL, cand);
+      bb[q] = (uint32_t)e;
+      kk[q] = (uint32_t)(e >> 32);
+    }
+#pragma unroll
+    for (int q = 0; q < kVsIPT; ++q) wv[q] = bb[q] != UM_NONE ? T.sk[bb[q]] : 0u;
+#pragma unroll
+    for (int q = 0; q < kVsIPT; ++q) {
+      const unsigned long long idx = tbase + q * kVsTPB + threadIdx.x;
+      const uint8_t ss = st_of(wv[q]);
+      const bool live = bb[q] != UM_NONE && (idx < s_ld ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) &&
+                        key_of(wv[q]) == kk[q];
+      wv[q] = live ? T.pin[bb[q]] : seq;   // not a candidate unless live and unpinned
       bL[q] = __ballot_sync(FULL, live);
     }
+#pragma unroll
+    for (int q = 0; q < kVsIPT; ++q) bC[q] = __ballot_sync(FULL, wv[q] != seq);
     const uint32_t tt = ordered_offsets<kVsTPB, kVsIPT>(bC, bC, s_off);
     const unsigned long long tot = pack2(tt & 0xffffu, 0);
     if (threadIdx.x < 32) {
@@ -995,34 +1052,64 @@ __global__ void __launch_bounds__(kVsTPB, 6) k_victims_scan(Tables T, uint32_t s
 
 __global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode) {
   pdl_enter();
-  constexpr int TPB = 256;
+  constexpr int TPB = 256, AIPT = 4, CH = TPB * AIPT;
   __shared__ uint32_t s_cnt[8];
   __shared__ unsigned long long s_sc[TPB / 32];
   __shared__ int s_hb;
   __shared__ uint32_t s_hav, s_db;
   Ctl* c = T.ctl;
   const uint32_t found = c->n_vict;
+  if (found == 0) {            // uniform: no victims, no counters
+    if (blockIdx.x == 0 && threadIdx.x == 0 && c->k0_pend) {   // bookkeeping of the k = 0 scan
+      c->free_top -= (int)c->k0_take;
+      c->used_tail += c->n_rekey;
+      c->k0_pend = 0;
+    }
+    return;
+  }
   const int f0 = (int)c->f0;   // free_top when the victims were chosen (set by the scan)
   // contiguous chunk of victims per CTA; one host-frame pop (and D2H-list append) per
-  // 256 victims instead of one same-address atomic per victim
+  // chunk of CH victims instead of one same-address atomic per victim.  Item (q, t) of a
+  // chunk is victim base + q * TPB + t (coalesced); every load phase keeps AIPT loads
+  // of a thread in flight.
   const uint32_t j0 = (uint32_t)((unsigned long long)found * blockIdx.x / gridDim.x);
   const uint32_t j1 = (uint32_t)((unsigned long long)found * (blockIdx.x + 1) / gridDim.x);
   uint32_t nG = 0, nAv = 0, nGL = 0;
-  for (uint32_t base = j0; base < j1; base += TPB) {
-    const uint32_t j = base + threadIdx.x;
-    uint32_t v = 0, fr = UM_NONE, hf = UM_NONE;
-    uint8_t ss = 0;
-    bool isG = false, needA = false;
-    if (j < j1) {
-      v = T.victim[j];
-      ss = ld_st(T, v);
-      fr = T.frame_of[v];
-      isG = ss == ST_G;
-      if (isG && !evict_mode && T.needk[(uint32_t)f0 + j] == ST_H) hf = T.needhf[(uint32_t)f0 + j];
-      needA = isG && hf == UM_NONE;
+  for (uint32_t base = j0; base < j1; base += CH) {
+    uint32_t v[AIPT], fr[AIPT], hf[AIPT];
+    uint8_t ss[AIPT], nk[AIPT];
+#pragma unroll
+    for (int q = 0; q < AIPT; ++q) {
+      const uint32_t j = base + q * TPB + threadIdx.x;
+      v[q] = j < j1 ? T.victim[j] : UM_NONE;
+      nk[q] = (j < j1 && !evict_mode) ? T.needk[(uint32_t)f0 + j] : (uint8_t)0xff;
+    }
+#pragma unroll
+    for (int q = 0; q < AIPT; ++q) {
+      ss[q] = v[q] != UM_NONE ? ld_st(T, v[q]) : (uint8_t)0xff;
+      fr[q] = v[q] != UM_NONE ? T.frame_of[v[q]] : UM_NONE;
+    }
+    uint32_t mA = 0, cA = 0, cD = 0;   // bit q: needs a host frame from the pool
+#pragma unroll
+    for (int q = 0; q < AIPT; ++q) {
+      const uint32_t j = base + q * TPB + threadIdx.x;
+      const bool isG = ss[q] == ST_G;
+      // a write-back victim's bytes land in the host frame of the block migrating into
+      // its frame (fused swap, R5) when there is one
+      hf[q] = (isG && nk[q] == ST_H) ? T.needhf[(uint32_t)f0 + j] : UM_NONE;
+      (void)j;
+    }
+#pragma unroll
+    for (int q = 0; q < AIPT; ++q) {
+      const bool isG = ss[q] == ST_G;
+      if (isG && hf[q] == UM_NONE) {
+        mA |= 1u << q;
+        ++cA;
+      }
+      cD += evict_mode && isG;
     }
     unsigned long long tot;
-    const unsigned long long pre = block_excl_scan<TPB>(pack2(needA, evict_mode && isG), tot, s_sc);
+    const unsigned long long pre = block_excl_scan<TPB>(pack2(cA, cD), tot, s_sc);
     if (threadIdx.x == 0) {
       const uint32_t tA = unpackA(tot), tD = unpackB(tot);
       s_hb = 0;
@@ -1040,36 +1127,44 @@ __global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode)
       s_db = tD ? atomicAdd(&c->n_d2h, tD) : 0u;
     }
     __syncthreads();
-    if (j < j1) {
-      if (needA) {
-        const uint32_t r = unpackA(pre);
-        hf = r < s_hav ? T.hfree_stack[s_hb - 1 - (int)r] : UM_NONE;
+    uint32_t rA = unpackA(pre), rD = unpackB(pre);
+#pragma unroll
+    for (int q = 0; q < AIPT; ++q) {
+      if ((mA >> q) & 1u) {
+        hf[q] = rA < s_hav ? T.hfree_stack[s_hb - 1 - (int)rA] : UM_NONE;
+        ++rA;
       }
-      T.vframe[j] = fr;
-      T.vkind[j] = ss;
-      T.vhf[j] = hf;
-      T.sk[v] = mk_sk(isG ? ST_H : ST_HD, 0);
-      T.map[v] = UM_NONE;
-      T.frame_of[v] = UM_NONE;
-      T.hframe[v] = hf;
+    }
+#pragma unroll
+    for (int q = 0; q < AIPT; ++q) {
+      const uint32_t j = base + q * TPB + threadIdx.x;
+      if (v[q] == UM_NONE) continue;
+      const bool isG = ss[q] == ST_G;
+      T.vframe[j] = fr[q];
+      T.vkind[j] = ss[q];
+      T.vhf[j] = hf[q];
+      T.sk[v[q]] = mk_sk(isG ? ST_H : ST_HD, 0);
+      T.map[v[q]] = UM_NONE;
+      T.frame_of[v[q]] = UM_NONE;
+      T.hframe[v[q]] = hf[q];
       nG += isG;
       nAv += !isG;
-      nGL += ss == ST_GL;
+      nGL += ss[q] == ST_GL;
       if (evict_mode) {
-        T.free_stack[f0 + j] = fr;
+        T.free_stack[f0 + j] = fr[q];
         if (isG) {
-          const uint32_t q = s_db + unpackB(pre);
-          T.d2h_frame[q] = fr;
-          T.d2h_hf[q] = hf;
+          T.d2h_frame[s_db + rD] = fr[q];
+          T.d2h_hf[s_db + rD] = hf[q];
+          ++rD;
         }
       }
     }
     __syncthreads();
   }
-  uint32_t v[3] = {nG, nAv, nGL};
+  uint32_t cnt[3] = {nG, nAv, nGL};
   const int slots[3] = {S_D2H, S_D2H_AV, S_UNMAPS};
   const long long mul[3] = {(long long)T.B, (long long)T.B, 1};
-  block_counts_to<3>(T, v, s_cnt, slots, mul);
+  block_counts_to<3>(T, cnt, s_cnt, slots, mul);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1336,7 +1431,7 @@ __global__ void __launch_bounds__(256) k_zero_items(Tables T, uint32_t i0, uint3
 // UM_ACC_WRITE access receives the content stamp s = (seq << 32) | block as the
 // 16-byte pattern {s, ~s}, written through its frame (G or GL blocks are mapped).
 // ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq) {
+__global__ void __launch_bounds__(256) k_app_stamp(Tables T, const __grid_constant__ OpIv iv, uint32_t g0, uint32_t n, uint32_t seq) {
   pdl_enter();
   __shared__ char* s_dst;
   __shared__ uint32_t s_blk;
@@ -1377,7 +1472,7 @@ __global__ void __launch_bounds__(256) k_app_stamp(Tables T, OpIv iv, uint32_t g
 // take one atomic per CTA (their order is not observable).  The last CTA publishes
 // disc_tail and the counters.
 // ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
+__global__ void __launch_bounds__(kStTPB, 6) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
                                                          int discard_off, unsigned long long tail0) {
   pdl_enter();
   constexpr int TPB = kStTPB, IPT = kStIPT, TILE = kStTile;
@@ -1400,12 +1495,20 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
   // of an H block holding one, taken by a prefetch HOST of G), F = GPU frames freed
   // (prefetch HOST)
   uint32_t nA = 0, nF = 0;
+  // all state loads first (one basic block: IPT gathers in flight), then the
+  // dependent host-frame loads of H blocks (predicated, again all in flight)
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint32_t idx = tbase + k * TPB + threadIdx.x;   // coalesced
     s[k] = idx < n ? ld_st(T, lo + idx) : (uint8_t)0xff;
+  }
+  uint32_t hfv[IPT];
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) hfv[k] = (disc && s[k] == ST_H) ? T.hframe[lo + tbase + k * TPB + threadIdx.x] : UM_NONE;
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) {
     if (disc) {
-      if (s[k] == ST_H && T.hframe[lo + idx] != UM_NONE) {
+      if (hfv[k] != UM_NONE) {
         hasf |= 1u << k;
         ++nA;
       }
@@ -1414,8 +1517,13 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
       nF += s[k] == ST_G || s[k] == ST_GE || s[k] == ST_GL;
     }
   }
+  // frame / host-frame stack traffic in this tile: ranked by a block scan, based by one
+  // atomic per CTA -- skipped (one predicated barrier) when the tile has none, e.g. a
+  // discard of GPU-resident data
+  unsigned long long pre = 0ull;
+  if (__syncthreads_or(active && (nA | nF))) {
   unsigned long long tot;
-  const unsigned long long pre = block_excl_scan<TPB>(active ? pack2(nA, nF) : 0ull, tot, s_sc);
+  pre = block_excl_scan<TPB>(active ? pack2(nA, nF) : 0ull, tot, s_sc);
   if (threadIdx.x == 0) {
     const uint32_t tA = unpackA(tot), tF = unpackB(tot);
     s_hb = 0; s_fb = 0; s_db = 0; s_hav = tA;
@@ -1437,6 +1545,7 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
     }
   }
   __syncthreads();
+  }
   uint32_t rA = unpackA(pre), rF = unpackB(pre);
   if (active) {
 #pragma unroll
@@ -1460,7 +1569,7 @@ __global__ void __launch_bounds__(kStTPB, 8) k_directive(Tables T, int kind, uin
         } else if (ss == ST_H) {
           T.sk[bb] = mk_sk(ST_HD, 0);
           if ((hasf >> k) & 1u) {   // the host copy is released (reading R1)
-            T.hfree_stack[s_hb + rA] = T.hframe[bb];
+            T.hfree_stack[s_hb + rA] = hfv[k];
             T.hframe[bb] = UM_NONE;
             ++rA;
           }
@@ -1833,7 +1942,7 @@ cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, u
   if (le__) return le__;
   cudaError_t e = cudaGetLastError();
   if (e) return e;
-  unsigned grid = ceil_div(max_victims ? max_victims : 1, 512);
+  unsigned grid = ceil_div(max_victims ? max_victims : 1, 1024);   // one pass of 4 victims per thread
   if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
   le__ = launch_pdl(k_victims_apply, dim3(grid), dim3(256), 0, s, T, evict_mode);
   if (le__) return le__;
