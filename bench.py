@@ -331,7 +331,7 @@ def _hbm_peak():
         return 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
 
 
-def state_bench(torch, um, mem, budget, arena_bytes, seed=0):
+def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
     """State-kernel microbench (SURVEY §8(d) last row): C3-64K-sized tables (64 KiB blocks
     over the same frame budget / 1.5x arena), each op on a cold L2 (the previous op's
     zero-fill streams GBs through it):
@@ -348,7 +348,7 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0):
       directive per block 4 sk rd + 8 DISC slot; per G block + 8 (sk wr, map wr)"""
     import numpy as np
     import tracegen as tg
-    B = 64 * 1024
+    B = block
     nb = arena_bytes // B
     n = 1 << 21
     cfg = mem.config(arena_bytes, budget, um.UM_F_TIMING)
@@ -515,7 +515,13 @@ def main_ours(args):
     # the TMA kernel path (K4) on the same step, for comparison with the auto path
     k4 = run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=um.UM_F_COPY_KERNEL) \
         if not args.no_compare else None
-    state = state_bench(torch, um, mem, budget, arena_bytes) if not args.no_state_bench else None
+    state = None
+    if not args.no_state_bench:
+        # two runs on fresh arenas over the same memory; the second is reported (the first
+        # pays first-touch costs of the workspace pages and kernel images: 47 vs 30 us)
+        state_bench(torch, um, mem, budget, arena_bytes, seed=1)
+        state = state_bench(torch, um, mem, budget, arena_bytes, seed=0)
+        state["reps"] = "second of two runs (first = warm-up)"
     e2e_s = None
     if not args.no_e2e:
         e2e_s = run_e2e(torch, um, harness, mem, trace, 1, min(K, 3))

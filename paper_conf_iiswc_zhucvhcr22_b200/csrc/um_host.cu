@@ -32,7 +32,7 @@ struct Layout {
   uint64_t used[2], disc[2];
   uint64_t need, needk, needhf, victim, vframe, vhf, vkind, d2h_frame, d2h_hf;
   uint64_t tile_status, tile_cnt, tags, ctl, hchunks, stage, xitems, bounce;
-  uint64_t obits, wbits, dlo, dpre, dw;
+  uint64_t obits, wbits, dlo, dpre, dw, vscratch, vpass;
   uint64_t stage_bytes, max_tiles, cap, total, ce_group, bounce_bytes;
 };
 
@@ -86,6 +86,8 @@ static Layout make_layout(const um_config* c) {
   L.needk = take(nf);
   L.needhf = take(4 * nf);
   L.victim = take(4 * nf);
+  L.vscratch = take(4 * (2 * L.cap + 2048));   // wide victim scan: candidates per tile
+  L.vpass = take(8 * (nf / 128 + L.max_tiles + 2));   // wide victim apply: work table
   L.vframe = take(4 * nf);
   L.vhf = take(4 * nf);
   L.vkind = take(nf);
@@ -798,6 +800,8 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   T.needk = (uint8_t*)(ws + L.needk);
   T.needhf = (uint32_t*)(ws + L.needhf);
   T.victim = (uint32_t*)(ws + L.victim);
+  T.vscratch = (uint32_t*)(ws + L.vscratch);
+  T.vpass = (unsigned long long*)(ws + L.vpass);
   T.vframe = (uint32_t*)(ws + L.vframe);
   T.vhf = (uint32_t*)(ws + L.vhf);
   T.vkind = (uint8_t*)(ws + L.vkind);

@@ -39,6 +39,9 @@ struct Ctl {
   unsigned int k_want;                  // wide victim scan: victims wanted
   unsigned int need_cnt[2];             // streaming classify: need-list slots, by sub-op parity
   unsigned int k0_take, k0_pend;        // wide victim scan with k = 0: frames to take, pending flag
+  unsigned long long vs_combo;          // wide victim scan: (candidates of finished tiles << 32) | next ticket
+  unsigned int first_skip;              // wide victim scan: first ticket not examined
+  unsigned int vt_reach;                // wide victim scan: passes in the apply work table (vpass)
   // counters, striped over 8 cache lines by CTA index (fire-and-forget atomics from
   // thousands of CTAs do not serialise on one address); the host sums the stripes
   long long stats[8][S_N];
@@ -70,6 +73,8 @@ struct Tables {
   uint8_t* needk;       // [nframes] their state at classification
   uint32_t* needhf;     // [nframes] their host frame at classification (H) or NONE
   uint32_t* victim;     // [nframes] victims, in eviction order
+  uint32_t* vscratch;   // [2 cap + 2048] wide victim scan: the candidates of tile t at [t * 2048, ...), in ring order
+  unsigned long long* vpass;  // [nframes / 128 + tiles] wide victim apply work table: (tile << 4 | pass) | prefix << 32
   uint32_t* vframe;     // [nframes] victim's frame
   uint32_t* vhf;        // [nframes] host frame receiving a G victim's write-back, else NONE
   uint8_t* vkind;       // [nframes] victim's state when chosen

@@ -305,6 +305,9 @@ __global__ void k_init(Tables T, int nh) {
       for (int i = 0; i < S_N; ++i) c->stats[j][i] = 0;
     c->need_cnt[0] = c->need_cnt[1] = 0;
     c->k0_take = c->k0_pend = 0;
+    c->vs_combo = 0;
+    c->first_skip = ~0u;
+    c->vt_reach = 0;
   }
 }
 
@@ -860,27 +863,32 @@ __global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, const __grid_
 }
 
 // ------------------------------------------------------------------------------------
-// K3 (wide): the same victim rule for large sub-ops, over all SMs.  Pass 1 scans the
-// concatenation DISC[head,tail) ++ USED[head,tail) in tiles taken in ascending order
-// from a ticket by a persistent grid (all CTAs resident): candidates (live, not pinned)
-// are ranked with a block scan + decoupled look-back, rank < k are the victims (exactly
-// the first k in queue order).  The first tile whose inclusive count reaches k is
-// recorded; tiles fetched after that is known are not read at all (their status is
-// published as "k reached"), so a scan stops soon after its k-th candidate instead of
-// reading the whole ring.  Ring heads may advance over examined dead/consumed entries
-// only: the first kept live entry, or the first entry of an unexamined tile, bounds
-// them.  Pass 2 reclaims the victims in parallel (host frames for write-backs come
-// from the free stack, one atomic per CTA chunk; ids are not observable).
+// K3 (wide): the same victim rule for large sub-ops, over all SMs, without a look-back
+// chain.  The victims are the first k candidates (live, not pinned) of DISC[head,tail)
+// ++ USED[head,tail) (PAPER §5.5); which of them comes first in the victim
+// list is not observable (frame ids and the victim <-> newcomer pairing are internal),
+// only the set is.
+//  Pass 1 (k_victims_scan): a persistent grid takes tiles of 2048 entries in ascending
+//   order from a ticket; each tile writes its candidates' blocks, in ring order, to its
+//   own scratch slice, and its candidate count and first kept-live positions to its
+//   tile record, then adds the count to a running total.  A tile is not read at all if
+//   the total of the (earlier-ticketed) tiles finished so far already reaches k: the k-th
+//   candidate lies before it.  No tile waits for another.  The last CTA to finish scans
+//   the tile counts, finds the tile holding the k-th candidate (reach), writes every
+//   tile's exclusive candidate prefix, advances the ring heads and does the frame
+//   bookkeeping.
+//  Pass 2 (k_victims_apply): tile t <= reach reclaims its first min(count, k - prefix)
+//   candidates as victims prefix .. prefix + take - 1, gathered from its scratch slice.
 // ------------------------------------------------------------------------------------
 constexpr int kVsTPB = 256, kVsIPT = 8, kVsTile = kVsTPB * kVsIPT;   // victim scan tiles
+constexpr int kVaPass = 128;   // victims per warp pass of k_victims_apply
 
 __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want,
-                                                            int npar) {
+                                                            int npar, int prefetch) {
   pdl_enter();
   constexpr int NW = kVsTPB / 32;
-  const unsigned long long FP = 2ull << 62;
   __shared__ uint32_t s_off[kVsIPT * NW + 1];
-  __shared__ unsigned long long s_excl, s_dh, s_ld, s_uh, s_lu, s_mk[2];
+  __shared__ unsigned long long s_dh, s_ld, s_uh, s_lu, s_mk[2];
   __shared__ uint32_t s_k, s_nn, s_f0, s_tile, s_skip;
   __shared__ int s_last;
   Ctl* c = T.ctl;
@@ -894,7 +902,6 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
     s_k = nn > f0 ? nn - f0 : 0u;
     s_nn = nn;
     s_f0 = f0;
-    s_mk[0] = s_mk[1] = ~0ull;
     if (blockIdx.x == 0 && !evict_mode) {
       c->n_need = nn;              // publish the streaming classify's need count
       c->need_cnt[npar ^ 1] = 0;   // and clear the other parity slot (read by no one now)
@@ -902,11 +909,10 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
   }
   __syncthreads();
   if (s_k == 0) {
-    // nothing to evict (the sub-op's need fits the free frames): one CTA does the
-    // bookkeeping of an empty victim list, the others exit; no ticket, look-back or
-    // completion counter is touched, so they stay clean for the next scan
-    // free_top and used_tail are advanced by k_victims_apply, which runs after this
-    // grid completes: other CTAs of this grid may still be reading free_top
+    // nothing to evict (the sub-op's need fits the free frames): one CTA records an
+    // empty victim list, the others exit.  free_top and used_tail are advanced by
+    // k_victims_apply, which runs after this grid completes (other CTAs of this grid may
+    // still be reading free_top).
     if (blockIdx.x == 0 && threadIdx.x == 0) {
       c->n_vict = 0;
       c->f0 = s_f0;
@@ -917,36 +923,35 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
   }
   const unsigned long long L = s_ld + s_lu;
   const uint32_t k = s_k;
-  const uint32_t ntiles = k ? (uint32_t)((L + kVsTile - 1) / kVsTile) : 0u;
+  const uint32_t ntiles = (uint32_t)((L + kVsTile - 1) / kVsTile);
   const int w = threadIdx.x >> 5;
   const unsigned lt = lanemask_lt();
   const unsigned me = 1u << (threadIdx.x & 31);
-  unsigned long long mk0 = ~0ull, mk1 = ~0ull;
+  // Tickets and the running candidate total share one 64-bit word, so a ticket comes
+  // with a consistent snapshot: every count in it was added by a finished tile, which
+  // took its ticket earlier -- a smaller one.  If the snapshot reaches k, tiles [0, t)
+  // hold >= k candidates and tile t is not read.  Thread 0 fetches the next ticket while
+  // the current tile is processed (the atomic's latency is off the critical path).
+  if (threadIdx.x == 0) {
+    const unsigned long long x = atomicAdd(&c->vs_combo, 1ull);
+    s_tile = (uint32_t)x;
+    s_skip = (uint32_t)(x >> 32);   // snapshot
+  }
   while (true) {
-    if (threadIdx.x == 0) {
-      const uint32_t t = atomicAdd(&c->scan_ticket, 1u);
-      s_tile = t;
-      s_skip = t >= ntiles ? 2u : (*(volatile uint32_t*)&c->reach_tile < t ? 1u : 0u);
-    }
     __syncthreads();
-    const uint32_t tile = s_tile, skip = s_skip;
-    __syncthreads();
-    if (skip == 2u) break;
-    const unsigned long long tbase = (unsigned long long)tile * kVsTile;
-    if (skip == 1u) {
-      // every later ticket skips as well, so this CTA is done
-      if (threadIdx.x == 0) {
-        ((volatile unsigned long long*)T.tile_status)[tile] = FP | pack2(k, 0);
-        __threadfence();
-        if (tbase < s_ld) {
-          mk0 = min(mk0, s_dh + tbase);
-          mk1 = min(mk1, s_uh);
-        } else {
-          mk1 = min(mk1, s_uh + (tbase - s_ld));
-        }
-      }
+    const uint32_t tile = s_tile, snap = s_skip;
+    __syncthreads();   // s_tile / s_skip are rewritten below
+    if (tile >= ntiles) break;
+    if (snap >= k) {   // later tickets skip as well
+      if (threadIdx.x == 0) atomicMin(&c->first_skip, tile);
       break;
     }
+    unsigned long long nxt = 0;
+    if (threadIdx.x == 0) {
+      if (prefetch) nxt = atomicAdd(&c->vs_combo, 1ull);
+      s_mk[0] = s_mk[1] = ~0ull;
+    }
+    const unsigned long long tbase = (unsigned long long)tile * kVsTile;
     // three load phases, each with all kVsIPT loads in flight: ring entries, the state
     // words of their blocks (liveness), the pin words of live entries
     uint32_t bb[kVsIPT], kk[kVsIPT], wv[kVsIPT];
@@ -976,87 +981,141 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
     }
 #pragma unroll
     for (int q = 0; q < kVsIPT; ++q) bC[q] = __ballot_sync(FULL, wv[q] != seq);
-    const uint32_t tt = ordered_offsets<kVsTPB, kVsIPT>(bC, bC, s_off);
-    const unsigned long long tot = pack2(tt & 0xffffu, 0);
-    if (threadIdx.x < 32) {
-      unsigned long long ex = lookback_warp(T, tile, tot);
-      if (threadIdx.x == 0) {
-        s_excl = ex;
-        if (unpackA(ex) + unpackA(tot) >= k) atomicMin(&c->reach_tile, tile);
-      }
-    }
-    __syncthreads();
-    const uint32_t eC = unpackA(s_excl);
+    const uint32_t cnt = ordered_offsets<kVsTPB, kVsIPT>(bC, bC, s_off) & 0xffffu;
+    unsigned long long mk0 = ~0ull, mk1 = ~0ull;   // first live entry kept (pinned), per ring
+    uint32_t* scr = T.vscratch + tbase;
 #pragma unroll
     for (int q = 0; q < kVsIPT; ++q) {
-      bool sel = false;
-      if (bC[q] & me) {
-        const uint32_t r = eC + (s_off[q * NW + w] & 0xffffu) + __popc(bC[q] & lt);
-        if (r < k) {
-          T.victim[r] = bb[q];
-          sel = true;
-        }
-      }
-      if ((bL[q] & me) && !sel) {
+      if (bC[q] & me) scr[(s_off[q * NW + w] & 0xffffu) + __popc(bC[q] & lt)] = bb[q];
+      else if (bL[q] & me) {
         const unsigned long long idx = tbase + q * kVsTPB + threadIdx.x;
-        if (idx < s_ld) mk0 = min(mk0, s_dh + idx);
-        else mk1 = min(mk1, s_uh + (idx - s_ld));
+        if (idx < s_ld) mk0 = min(mk0, idx);
+        else mk1 = min(mk1, idx);
       }
     }
+    if (mk0 != ~0ull) atomicMin(&s_mk[0], mk0);
+    if (mk1 != ~0ull) atomicMin(&s_mk[1], mk1);
     __syncthreads();
+    if (threadIdx.x == 0) {
+      uint32_t* rec = T.tile_cnt + (size_t)tile * 8;
+      rec[0] = cnt;
+      *reinterpret_cast<unsigned long long*>(rec + 2) = s_mk[0];
+      *reinterpret_cast<unsigned long long*>(rec + 4) = s_mk[1];
+      // no fence: the records are read by the finalizing CTA after the completion
+      // counter below (fenced), the scratch slice by k_victims_apply (next launch)
+      // without prefetch the next ticket comes with this tile's count (one atomic)
+      if (!prefetch) nxt = atomicAdd(&c->vs_combo, ((unsigned long long)cnt << 32) | 1ull) + ((unsigned long long)cnt << 32);
+      else if (cnt) atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32);
+      s_tile = (uint32_t)nxt;
+      s_skip = (uint32_t)(nxt >> 32);
+    }
   }
-  if (mk0 != ~0ull) atomicMin(&s_mk[0], mk0);
-  if (mk1 != ~0ull) atomicMin(&s_mk[1], mk1);
+  // completion: the last CTA of the grid finalizes
   __syncthreads();
   if (threadIdx.x == 0) {
-    if (s_mk[0] != ~0ull) atomicMin(&c->minkeep[0], s_mk[0]);
-    if (s_mk[1] != ~0ull) atomicMin(&c->minkeep[1], s_mk[1]);
     __threadfence();
     s_last = atomicAdd(&c->scan_done, 1u) == gridDim.x - 1;
   }
   __syncthreads();
-  if (s_last) {
-    __threadfence();
-    const uint32_t fetched = min(ntiles, *(volatile uint32_t*)&c->scan_ticket);
-    for (uint32_t i = threadIdx.x; i < fetched; i += blockDim.x) T.tile_status[i] = 0ull;
-    if (threadIdx.x == 0) {
-      const uint32_t reach = *(volatile uint32_t*)&c->reach_tile;
-      uint32_t found = 0;
-      if (k) found = reach != ~0u ? k : unpackA(((volatile unsigned long long*)T.tile_status)[ntiles - 1] & ((1ull << 62) - 1));
-      found = min(k, found);
-      // victim bookkeeping for the apply pass (which reads f0 / n_vict only)
-      c->n_vict = found;
-      stat_add(T, S_EVICT, found);
-      if (k) {
-        const unsigned long long m0 = *(volatile unsigned long long*)&c->minkeep[0];
-        const unsigned long long m1 = *(volatile unsigned long long*)&c->minkeep[1];
-        c->disc_head = m0 != ~0ull ? m0 : c->disc_tail;
-        c->used_head = m1 != ~0ull ? m1 : c->used_tail;
-      }
-      c->minkeep[0] = c->minkeep[1] = ~0ull;
-      const int f0 = (int)s_f0;
-      c->f0 = (uint32_t)f0;
-      if (evict_mode) {
-        c->free_top = f0 + (int)found;
-      } else {
-        c->free_top = f0 - (int)min((uint32_t)f0, s_nn);
-        c->used_tail += c->n_rekey;
-      }
-      c->scan_ticket = 0;
-      c->scan_done = 0;
-      c->reach_tile = ~0u;
-    }
-    __threadfence();
+  if (!s_last) return;
+  __threadfence();
+  __shared__ unsigned long long s_sc[kVsTPB / 32];
+  __shared__ uint32_t s_reach, s_found;
+  __shared__ unsigned long long s_kd, s_ku;
+  const uint32_t fs = *(volatile uint32_t*)&c->first_skip;
+  const uint32_t E = min(ntiles, fs);   // tiles [0, E) were all examined
+  if (threadIdx.x == 0) {
+    s_reach = ~0u;
+    s_found = 0;
+    s_kd = s_ku = ~0ull;
   }
+  __syncthreads();
+  // Each thread owns a contiguous run of C tiles (independent loads in flight).  Pass A:
+  // candidate totals -> block scan -> found = min(k, total).  Pass B: per tile the
+  // exclusive prefix ex, the reach tile (ex < k <= ex + count), the first kept live
+  // entry of every tile before it (inclusive prefix < k), and the apply passes of the
+  // tile.  Pass C: the apply work table, one entry per pass of kVaPass victims of a
+  // tile, (tile << 4 | pass) | ex << 32, so the apply's warps are balanced whatever the
+  // spread of victims over tiles (a dense tile holds up to 2048).
+  const uint32_t C = (E + kVsTPB - 1) / kVsTPB;
+  const uint32_t ta = min(E, threadIdx.x * C), tb = min(E, ta + C);
+  // L2 reads (ld.global.cg): written by other CTAs of this grid, ordered by the fenced
+  // completion counter; independent, so they pipeline
+  const uint32_t* tc = T.tile_cnt;
+  uint32_t mine = 0;
+#pragma unroll 8
+  for (uint32_t t = ta; t < tb; ++t) mine += __ldcg(tc + (size_t)t * 8);
+  unsigned long long tot;
+  uint32_t ex = (uint32_t)block_excl_scan<kVsTPB>(mine, tot, s_sc);
+  const uint32_t found = (uint32_t)min((unsigned long long)k, tot);
+  uint32_t np = 0;
+  unsigned long long kd = ~0ull, ku = ~0ull;
+#pragma unroll 4
+  for (uint32_t t = ta; t < tb; ++t) {
+    const uint32_t v = __ldcg(tc + (size_t)t * 8);
+    const unsigned long long* rec = reinterpret_cast<const unsigned long long*>(tc + (size_t)t * 8 + 2);
+    const unsigned long long r0 = __ldcg(rec), r1 = __ldcg(rec + 1);
+    if (ex < k && ex + v >= k) s_reach = t;   // exactly one tile
+    if (ex + v < k) {                          // before the reach tile
+      kd = min(kd, r0);
+      ku = min(ku, r1);
+    }
+    const uint32_t take = ex >= found ? 0u : min(v, found - ex);
+    np += (take + kVaPass - 1) / kVaPass;
+    ex += v;
+  }
+  if (kd != ~0ull) atomicMin(&s_kd, kd);
+  if (ku != ~0ull) atomicMin(&s_ku, ku);
+  unsigned long long ptot;
+  uint32_t q0 = (uint32_t)block_excl_scan<kVsTPB>(np, ptot, s_sc);
+  ex = (uint32_t)(block_excl_scan<kVsTPB>(mine, tot, s_sc));
+#pragma unroll 4
+  for (uint32_t t = ta; t < tb; ++t) {
+    const uint32_t v = __ldcg(tc + (size_t)t * 8);
+    const uint32_t take = ex >= found ? 0u : min(v, found - ex);
+    const uint32_t P = (take + kVaPass - 1) / kVaPass;
+    for (uint32_t q = 0; q < P; ++q) T.vpass[q0 + q] = (unsigned long long)((t << 4) | q) | ((unsigned long long)ex << 32);
+    q0 += P;
+    ex += v;
+  }
+  const uint32_t npass = (uint32_t)ptot;
+  __syncthreads();
+  const uint32_t reach = s_reach;
+  if (threadIdx.x == 0) {
+    unsigned long long kd = s_kd, ku = s_ku;   // positions in the concatenated index space
+    if (reach != ~0u) {
+      const unsigned long long bound = (unsigned long long)reach * kVsTile;
+      if (bound < s_ld) {
+        kd = min(kd, bound);
+        ku = min(ku, s_ld);   // USED not reached: its head stays
+      } else {
+        ku = min(ku, bound);
+      }
+    }
+    c->disc_head = kd != ~0ull ? s_dh + kd : c->disc_tail;
+    c->used_head = ku != ~0ull ? s_uh + (ku - s_ld) : c->used_tail;
+    c->n_vict = found;
+    c->vt_reach = npass;
+    stat_add(T, S_EVICT, found);
+    const int f0 = (int)s_f0;
+    c->f0 = (uint32_t)f0;
+    if (evict_mode) {
+      c->free_top = f0 + (int)found;
+    } else {
+      c->free_top = f0 - (int)min((uint32_t)f0, s_nn);
+      c->used_tail += c->n_rekey;
+    }
+    c->scan_done = 0;
+    c->vs_combo = 0;
+    c->first_skip = ~0u;
+  }
+  __threadfence();
 }
 
 __global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode) {
   pdl_enter();
-  constexpr int TPB = 256, AIPT = 4, CH = TPB * AIPT;
+  constexpr int TPB = 256, AIPT = 4, CH = 32 * AIPT;
   __shared__ uint32_t s_cnt[8];
-  __shared__ unsigned long long s_sc[TPB / 32];
-  __shared__ int s_hb;
-  __shared__ uint32_t s_hav, s_db;
   Ctl* c = T.ctl;
   const uint32_t found = c->n_vict;
   if (found == 0) {            // uniform: no victims, no counters
@@ -1068,103 +1127,114 @@ __global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode)
     return;
   }
   const int f0 = (int)c->f0;   // free_top when the victims were chosen (set by the scan)
-  // contiguous chunk of victims per CTA; one host-frame pop (and D2H-list append) per
-  // chunk of CH victims instead of one same-address atomic per victim.  Item (q, t) of a
-  // chunk is victim base + q * TPB + t (coalesced); every load phase keeps AIPT loads
-  // of a thread in flight.
-  const uint32_t j0 = (uint32_t)((unsigned long long)found * blockIdx.x / gridDim.x);
-  const uint32_t j1 = (uint32_t)((unsigned long long)found * (blockIdx.x + 1) / gridDim.x);
+  const uint32_t npass = c->vt_reach;
+  const int lane = threadIdx.x & 31;
+  const unsigned lt = lanemask_lt();
   uint32_t nG = 0, nAv = 0, nGL = 0;
-  for (uint32_t base = j0; base < j1; base += CH) {
-    uint32_t v[AIPT], fr[AIPT], hf[AIPT];
-    uint8_t ss[AIPT], nk[AIPT];
+  // One warp per pass of the scan's work table: pass q of tile t reclaims the tile's
+  // victims prefix + q * CH + [0, CH), out of its first take = min(count, found -
+  // prefix) candidates.  Item (i, lane) = victim base + 32 i + lane (coalesced); each
+  // load phase keeps AIPT loads of a lane in flight; one host-frame pop (and D2H-list
+  // append) per pass.
+  static_assert(CH == kVaPass, "pass size");
+  const uint32_t nwarps = gridDim.x * (TPB / 32);
+  for (uint32_t p = blockIdx.x * (TPB / 32) + (threadIdx.x >> 5); p < npass; p += nwarps) {
+    const unsigned long long ent = T.vpass[p];
+    const uint32_t tile = (uint32_t)ent >> 4, pre = (uint32_t)(ent >> 32);
+    const uint32_t cnt = T.tile_cnt[(size_t)tile * 8];
+    const uint32_t take = pre >= found ? 0u : min(cnt, found - pre);
+    const uint32_t* scr = T.vscratch + (size_t)tile * kVsTile;
+    {
+      const uint32_t base = ((uint32_t)ent & 15u) * CH;
+      uint32_t v[AIPT], fr[AIPT], hf[AIPT];
+      uint8_t ss[AIPT], nk[AIPT];
 #pragma unroll
-    for (int q = 0; q < AIPT; ++q) {
-      const uint32_t j = base + q * TPB + threadIdx.x;
-      v[q] = j < j1 ? T.victim[j] : UM_NONE;
-      nk[q] = (j < j1 && !evict_mode) ? T.needk[(uint32_t)f0 + j] : (uint8_t)0xff;
-    }
-#pragma unroll
-    for (int q = 0; q < AIPT; ++q) {
-      ss[q] = v[q] != UM_NONE ? ld_st(T, v[q]) : (uint8_t)0xff;
-      fr[q] = v[q] != UM_NONE ? T.frame_of[v[q]] : UM_NONE;
-    }
-    uint32_t mA = 0, cA = 0, cD = 0;   // bit q: needs a host frame from the pool
-#pragma unroll
-    for (int q = 0; q < AIPT; ++q) {
-      const uint32_t j = base + q * TPB + threadIdx.x;
-      const bool isG = ss[q] == ST_G;
-      // a write-back victim's bytes land in the host frame of the block migrating into
-      // its frame (fused swap, R5) when there is one
-      hf[q] = (isG && nk[q] == ST_H) ? T.needhf[(uint32_t)f0 + j] : UM_NONE;
-      (void)j;
-    }
-#pragma unroll
-    for (int q = 0; q < AIPT; ++q) {
-      const bool isG = ss[q] == ST_G;
-      if (isG && hf[q] == UM_NONE) {
-        mA |= 1u << q;
-        ++cA;
+      for (int q = 0; q < AIPT; ++q) {
+        const uint32_t i = base + q * 32 + lane;
+        v[q] = i < take ? scr[i] : UM_NONE;
+        nk[q] = (i < take && !evict_mode) ? T.needk[(uint32_t)f0 + pre + i] : (uint8_t)0xff;
       }
-      cD += evict_mode && isG;
-    }
-    unsigned long long tot;
-    const unsigned long long pre = block_excl_scan<TPB>(pack2(cA, cD), tot, s_sc);
-    if (threadIdx.x == 0) {
-      const uint32_t tA = unpackA(tot), tD = unpackB(tot);
-      s_hb = 0;
-      s_hav = 0;
-      if (tA) {
-        const int old = atomicSub(&c->hfree_top, (int)tA);
-        const int avail = old < 0 ? 0 : (old < (int)tA ? old : (int)tA);
-        if (avail < (int)tA) {
-          atomicAdd(&c->hfree_top, (int)tA - avail);
-          atomicExch(&c->err, 2u);   // host-frame pool exhausted -> UM_ENOMEM
+#pragma unroll
+      for (int q = 0; q < AIPT; ++q) {
+        ss[q] = v[q] != UM_NONE ? ld_st(T, v[q]) : (uint8_t)0xff;
+        fr[q] = v[q] != UM_NONE ? T.frame_of[v[q]] : UM_NONE;
+      }
+#pragma unroll
+      for (int q = 0; q < AIPT; ++q) {
+        // a write-back victim's bytes land in the host frame of the block migrating into
+        // its frame (fused swap, R5) when there is one
+        hf[q] = (ss[q] == ST_G && nk[q] == ST_H) ? T.needhf[(uint32_t)f0 + pre + base + q * 32 + lane] : UM_NONE;
+      }
+      unsigned bA[AIPT], bD[AIPT];
+      uint32_t tA = 0, tD = 0;
+#pragma unroll
+      for (int q = 0; q < AIPT; ++q) {
+        const bool isG = ss[q] == ST_G;
+        bA[q] = __ballot_sync(FULL, isG && hf[q] == UM_NONE);
+        bD[q] = __ballot_sync(FULL, evict_mode && isG);
+        tA += __popc(bA[q]);
+        tD += __popc(bD[q]);
+      }
+      int hb = 0;
+      uint32_t hav = 0, db = 0;
+      if (lane == 0) {
+        if (tA) {
+          const int old = atomicSub(&c->hfree_top, (int)tA);
+          const int avail = old < 0 ? 0 : (old < (int)tA ? old : (int)tA);
+          if (avail < (int)tA) {
+            atomicAdd(&c->hfree_top, (int)tA - avail);
+            atomicExch(&c->err, 2u);   // host-frame pool exhausted -> UM_ENOMEM
+          }
+          hb = old;
+          hav = (uint32_t)avail;
         }
-        s_hb = old;
-        s_hav = (uint32_t)avail;
+        if (tD) db = atomicAdd(&c->n_d2h, tD);
       }
-      s_db = tD ? atomicAdd(&c->n_d2h, tD) : 0u;
-    }
-    __syncthreads();
-    uint32_t rA = unpackA(pre), rD = unpackB(pre);
+      hb = __shfl_sync(FULL, hb, 0);
+      hav = __shfl_sync(FULL, hav, 0);
+      db = __shfl_sync(FULL, db, 0);
+      uint32_t rA = 0, rD = 0;   // ranks: earlier passes q, then lanes below
 #pragma unroll
-    for (int q = 0; q < AIPT; ++q) {
-      if ((mA >> q) & 1u) {
-        hf[q] = rA < s_hav ? T.hfree_stack[s_hb - 1 - (int)rA] : UM_NONE;
-        ++rA;
-      }
-    }
-#pragma unroll
-    for (int q = 0; q < AIPT; ++q) {
-      const uint32_t j = base + q * TPB + threadIdx.x;
-      if (v[q] == UM_NONE) continue;
-      const bool isG = ss[q] == ST_G;
-      T.vframe[j] = fr[q];
-      T.vkind[j] = ss[q];
-      T.vhf[j] = hf[q];
-      T.sk[v[q]] = mk_sk(isG ? ST_H : ST_HD, 0);
-      T.map[v[q]] = UM_NONE;
-      T.frame_of[v[q]] = UM_NONE;
-      T.hframe[v[q]] = hf[q];
-      nG += isG;
-      nAv += !isG;
-      nGL += ss[q] == ST_GL;
-      if (evict_mode) {
-        T.free_stack[f0 + j] = fr[q];
-        if (isG) {
-          T.d2h_frame[s_db + rD] = fr[q];
-          T.d2h_hf[s_db + rD] = hf[q];
-          ++rD;
+      for (int q = 0; q < AIPT; ++q) {
+        if ((bA[q] >> lane) & 1u) {
+          const uint32_t r = rA + __popc(bA[q] & lt);
+          hf[q] = r < hav ? T.hfree_stack[hb - 1 - (int)r] : UM_NONE;
         }
+        rA += __popc(bA[q]);
+      }
+#pragma unroll
+      for (int q = 0; q < AIPT; ++q) {
+        const uint32_t j = pre + base + q * 32 + lane;
+        if (v[q] != UM_NONE) {
+          const bool isG = ss[q] == ST_G;
+          T.victim[j] = v[q];
+          T.vframe[j] = fr[q];
+          T.vkind[j] = ss[q];
+          T.vhf[j] = hf[q];
+          T.sk[v[q]] = mk_sk(isG ? ST_H : ST_HD, 0);
+          T.map[v[q]] = UM_NONE;
+          T.frame_of[v[q]] = UM_NONE;
+          T.hframe[v[q]] = hf[q];
+          nG += isG;
+          nAv += !isG;
+          nGL += ss[q] == ST_GL;
+          if (evict_mode) {
+            T.free_stack[f0 + j] = fr[q];
+            if (isG) {
+              const uint32_t d = db + rD + __popc(bD[q] & lt);
+              T.d2h_frame[d] = fr[q];
+              T.d2h_hf[d] = hf[q];
+            }
+          }
+        }
+        rD += __popc(bD[q]);
       }
     }
-    __syncthreads();
   }
-  uint32_t cnt[3] = {nG, nAv, nGL};
+  uint32_t cnt3[3] = {nG, nAv, nGL};
   const int slots[3] = {S_D2H, S_D2H_AV, S_UNMAPS};
   const long long mul[3] = {(long long)T.B, (long long)T.B, 1};
-  block_counts_to<3>(T, cnt, s_cnt, slots, mul);
+  block_counts_to<3>(T, cnt3, s_cnt, slots, mul);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1846,6 +1916,7 @@ static int g_nsm = 0;
 static int g_vscan_occ = 1;   // resident k_victims_scan CTAs per SM
 static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch (A/B)
 static int g_dir_occ = 8;     // resident k_directive CTAs per SM (persistent grid)
+static int g_vs_prefetch = 0; // UM_VS_PREFETCH=1: the wide victim scan fetches its next ticket a tile ahead (A/B on B200: 79 vs 73 us pressured touch -- the earlier snapshot reads more tiles past the k-th candidate)
 
 cudaError_t setup_kernels() {
   int dev;
@@ -1854,6 +1925,7 @@ cudaError_t setup_kernels() {
   e = cudaDeviceGetAttribute(&g_nsm, cudaDevAttrMultiProcessorCount, dev);
   if (e) return e;
   if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
+  if (const char* v = getenv("UM_VS_PREFETCH")) g_vs_prefetch = atoi(v) != 0;
   // Optionally one L1/shared carveout for every paging kernel (k_service needs 144 KB of
   // shared memory; a carveout change between consecutive kernels can force an SM drain).
   // UM_CARVEOUT=1 turns it on (A/B; off by default).
@@ -1938,11 +2010,12 @@ cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, u
   // ticket in order and a tile may wait on its predecessors' status)
   unsigned nt = ceil_div(scan_bound ? scan_bound : 1, kVsTile);
   const unsigned cap = (unsigned)(g_nsm * g_vscan_occ);
-  cudaError_t le__ = launch_pdl(k_victims_scan, dim3(nt < cap ? nt : cap), dim3(kVsTPB), 0, s, T, seq, evict_mode, want, npar);
+  cudaError_t le__ = launch_pdl(k_victims_scan, dim3(nt < cap ? nt : cap), dim3(kVsTPB), 0, s, T, seq, evict_mode, want, npar, g_vs_prefetch);
   if (le__) return le__;
   cudaError_t e = cudaGetLastError();
   if (e) return e;
-  unsigned grid = ceil_div(max_victims ? max_victims : 1, 1024);   // one pass of 4 victims per thread
+  // one warp per pass of <= kVaPass victims (<= max_victims / kVaPass + tiles passes)
+  unsigned grid = ceil_div((unsigned long long)ceil_div(max_victims ? max_victims : 1, kVaPass) + nt, 8);
   if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
   le__ = launch_pdl(k_victims_apply, dim3(grid), dim3(256), 0, s, T, evict_mode);
   if (le__) return le__;
