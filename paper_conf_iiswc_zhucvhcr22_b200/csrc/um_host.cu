@@ -684,7 +684,7 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     if (!iv.inl) {
       // per tile of this sub-op, the interval slice its items fall in: an index the
       // kernels would otherwise find by a dependent binary search over the staged list
-      const uint32_t tile = n <= kSmallPlan ? kSmallPlan : (uint32_t)kClsTile;
+      const uint32_t tile = n <= kSmallPlan ? kSmallPlan : classify_tile();
       const uint32_t nt = (n + tile - 1) / tile;
       uint64_t off;
       CK(a->stage.reserve(8ull * nt, &off));

@@ -123,11 +123,8 @@ constexpr int kScanIPT = 8;
 constexpr int kScanTile = kScanTPB * kScanIPT;
 // streaming state kernels (classify, directives): no inter-CTA ordering, one wave
 constexpr int kStTPB = 256;
-constexpr int kStIPT = 8;
-constexpr int kStTile = kStTPB * kStIPT;
-// multi-CTA classify: items per thread (two dependent gathers each)
-constexpr int kClsIPT = 4;
-constexpr int kClsTile = kStTPB * kClsIPT;
+// multi-CTA classify: items per thread (4, or 8 with UM_CLS_IPT=8); its tile in items
+uint32_t classify_tile();
 constexpr int kVictTPB = 1024;
 constexpr int kVictIPT = 4;
 constexpr int kXferStages = 4;

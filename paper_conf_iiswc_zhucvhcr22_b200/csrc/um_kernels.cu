@@ -548,19 +548,19 @@ __device__ bool grid_finish(const Tables& T, const int (&slots)[NC], const long 
   return true;
 }
 
-__global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
-                                                        uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
-                                                        int npar) {
-  pdl_enter();
-  constexpr int TPB = kStTPB, IPT = kClsIPT, TILE = kClsTile, NW = TPB / 32, NWORD = TILE / 32;
-  static_assert(NWORD <= 32, "one bitmap word per lane");
+template <int IPT>
+__device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
+                                              int touch, unsigned long long tail0, int npar) {
+  constexpr int TPB = kStTPB, TILE = TPB * IPT, NW = TPB / 32, NWORD = TILE / 32;
+  constexpr int PERL = (NWORD + 31) / 32;   // bitmap words per lane in the warp prefix
   // Interval lookup without a search: the tile's interval slice [ja, jb] is staged as
   // d[q] = lo - pre (block = rank + d), and the start of every slice interval but the
   // first sets one bit of a TILE-bit map at its in-tile position.  The interval of item
-  // i is then the number of set bits in [0, i] (a warp prefix of word popcounts plus one
+  // i is then the number of set bits in [0, i] (a prefix of word popcounts plus one
   // masked popc), so every item costs O(1) instead of a log2(TILE)-step dependent search.
   __shared__ uint32_t s_d[TILE];
   __shared__ uint32_t s_bits[NWORD];
+  __shared__ uint32_t s_wpre[NWORD];
   __shared__ uint32_t s_base;
   __shared__ uint32_t s_off[IPT * NW + 1];
   __shared__ uint32_t s_cnt[8];
@@ -577,7 +577,7 @@ __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_c
       qpre[r] = iv_pre(iv, ja + q);
     }
   }
-  if (threadIdx.x < NWORD) s_bits[threadIdx.x] = 0u;
+  for (int i = threadIdx.x; i < NWORD; i += TPB) s_bits[i] = 0u;
   __syncthreads();
 #pragma unroll
   for (int r = 0; r < IPT; ++r) {
@@ -592,8 +592,30 @@ __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_c
   }
   __syncthreads();
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  uint32_t wexcl;   // lane l: set bits in words [0, l)
-  {
+  if (PERL > 1 && w == 0) {
+    // one warp: exclusive prefix of the word popcounts (PERL consecutive words per lane)
+    uint32_t c[PERL], sum = 0;
+#pragma unroll
+    for (int i = 0; i < PERL; ++i) {
+      c[i] = lane * PERL + i < NWORD ? __popc(s_bits[lane * PERL + i]) : 0u;
+      sum += c[i];
+    }
+    uint32_t x = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    x -= sum;
+#pragma unroll
+    for (int i = 0; i < PERL; ++i) {
+      if (lane * PERL + i < NWORD) s_wpre[lane * PERL + i] = x;
+      x += c[i];
+    }
+  }
+  if (PERL > 1) __syncthreads();
+  uint32_t wexcl = 0;   // PERL == 1: lane l holds the set bits in words [0, l)
+  if (PERL == 1) {
     const uint32_t c = lane < NWORD ? __popc(s_bits[lane]) : 0u;
     uint32_t x = c;
 #pragma unroll
@@ -612,7 +634,8 @@ __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_c
   for (int k = 0; k < IPT; ++k) {
     const uint32_t idx = tbase + k * TPB + threadIdx.x;
     const int wi = k * NW + w;   // bitmap word of item (k, thread): in-tile position k*TPB + tid
-    const uint32_t j = __shfl_sync(FULL, wexcl, wi) + __popc(s_bits[wi] & le);
+    const uint32_t wp = PERL == 1 ? __shfl_sync(FULL, wexcl, wi & 31) : s_wpre[wi];
+    const uint32_t j = wp + __popc(s_bits[wi] & le);
     b[k] = g0 + idx + s_d[j];
   }
 #pragma unroll
@@ -681,6 +704,21 @@ __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_c
   const long long mul[6] = {1, 1, 1, B, B, B};
   block_counts_to<6>(T, v, s_cnt, touch ? slots_t : slots_p, mul);
   if (blockIdx.x == 0 && threadIdx.x == 0) T.ctl->n_rekey = n;   // USED slots appended
+}
+
+// 4 items per thread (8 CTAs/SM, 32 registers) or 8 (6 CTAs/SM, 40 registers);
+// UM_CLS_IPT selects (A/B)
+__global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
+                                                        uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
+                                                        int npar) {
+  pdl_enter();
+  classify_body<4>(T, iv, g0, n, seq, touch, tail0, npar);
+}
+__global__ void __launch_bounds__(kStTPB, 6) k_classify8(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
+                                                         uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
+                                                         int npar) {
+  pdl_enter();
+  classify_body<8>(T, iv, g0, n, seq, touch, tail0, npar);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1542,10 +1580,10 @@ __global__ void __launch_bounds__(256) k_app_stamp(Tables T, const __grid_consta
 // take one atomic per CTA (their order is not observable).  The last CTA publishes
 // disc_tail and the counters.
 // ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kStTPB, 6) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
-                                                         int discard_off, unsigned long long tail0) {
-  pdl_enter();
-  constexpr int TPB = kStTPB, IPT = kStIPT, TILE = kStTile;
+template <int IPT>
+__device__ __forceinline__ void directive_body(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
+                                               int discard_off, unsigned long long tail0) {
+  constexpr int TPB = kStTPB, TILE = TPB * IPT;
   __shared__ unsigned long long s_sc[TPB / 32];
   __shared__ int s_hb, s_fb;
   __shared__ uint32_t s_db, s_hav;
@@ -1675,6 +1713,19 @@ __global__ void __launch_bounds__(kStTPB, 6) k_directive(Tables T, int kind, uin
   block_counts_to<3>(T, v, s_cnt, slots, mul);
   // the host passes the exact tail; nothing in this launch reads c->disc_tail
   if (blockIdx.x == 0 && threadIdx.x == 0 && disc && active) c->disc_tail = tail0 + n;
+}
+
+// 8 blocks per thread (6 CTAs/SM) or 16 (4 CTAs/SM: 2^21 blocks in one round of 512
+// tiles, 16 state loads in flight per thread); UM_DIR_IPT selects (A/B)
+__global__ void __launch_bounds__(kStTPB, 6) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
+                                                         int discard_off, unsigned long long tail0) {
+  pdl_enter();
+  directive_body<8>(T, kind, lo, n, seq, discard_off, tail0);
+}
+__global__ void __launch_bounds__(kStTPB, 4) k_directive16(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
+                                                           int discard_off, unsigned long long tail0) {
+  pdl_enter();
+  directive_body<16>(T, kind, lo, n, seq, discard_off, tail0);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1916,6 +1967,9 @@ static int g_nsm = 0;
 static int g_vscan_occ = 1;   // resident k_victims_scan CTAs per SM
 static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch (A/B)
 static int g_dir_occ = 8;     // resident k_directive CTAs per SM (persistent grid)
+static int g_dir_occ16 = 4;   // ... of k_directive16
+static int g_dir_ipt = 8;     // UM_DIR_IPT=16: directives with 16 blocks per thread (A/B)
+static int g_cls_ipt = 4;     // UM_CLS_IPT=8: classify with 8 items per thread (A/B)
 static int g_vs_prefetch = 0; // UM_VS_PREFETCH=1: the wide victim scan fetches its next ticket a tile ahead (A/B on B200: 79 vs 73 us pressured touch -- the earlier snapshot reads more tiles past the k-th candidate)
 
 cudaError_t setup_kernels() {
@@ -1926,6 +1980,7 @@ cudaError_t setup_kernels() {
   if (e) return e;
   if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
   if (const char* v = getenv("UM_VS_PREFETCH")) g_vs_prefetch = atoi(v) != 0;
+  if (const char* v = getenv("UM_CLS_IPT")) g_cls_ipt = atoi(v) == 8 ? 8 : 4;
   // Optionally one L1/shared carveout for every paging kernel (k_service needs 144 KB of
   // shared memory; a carveout change between consecutive kernels can force an SM drain).
   // UM_CARVEOUT=1 turns it on (A/B; off by default).
@@ -1949,6 +2004,10 @@ cudaError_t setup_kernels() {
   if (e) return e;
   if (g_dir_occ < 1) g_dir_occ = 1;
   if (const char* v = getenv("UM_DIR_OCC")) g_dir_occ = std::max(1, atoi(v));
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_dir_occ16, k_directive16, kStTPB, 0);
+  if (e) return e;
+  if (g_dir_occ16 < 1) g_dir_occ16 = 1;
+  if (const char* v = getenv("UM_DIR_IPT")) g_dir_ipt = atoi(v) == 16 ? 16 : 8;
   int smem = (int)(kXferChunk * (1 + 2 * kXferStages));
   return cudaFuncSetAttribute(k_service, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
 }
@@ -1983,10 +2042,13 @@ cudaError_t launch_poison(const Tables& T, cudaStream_t s) {
   return cudaGetLastError();
 }
 
+uint32_t classify_tile() { return (uint32_t)kStTPB * (uint32_t)g_cls_ipt; }
+
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
                             unsigned long long tail0, int npar, cudaStream_t s) {
-  unsigned nt = n ? ceil_div(n, kClsTile) : 1;
-  cudaError_t le__ = launch_pdl(k_classify, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar);
+  unsigned nt = n ? ceil_div(n, classify_tile()) : 1;
+  cudaError_t le__ = launch_pdl(g_cls_ipt == 8 ? k_classify8 : k_classify, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n,
+                                seq, touch, tail0, npar);
   if (le__) return le__;
   return cudaGetLastError();
 }
@@ -2045,9 +2107,12 @@ cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, 
 
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq, int discard_off,
                              unsigned long long tail0, cudaStream_t s) {
-  unsigned nt = n ? ceil_div(n, kStTile) : 1;
-  if (nt > (unsigned)(g_nsm * g_dir_occ)) nt = (unsigned)(g_nsm * g_dir_occ);   // persistent
-  cudaError_t le__ = launch_pdl(k_directive, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq, discard_off, tail0);
+  const bool w16 = g_dir_ipt == 16;
+  unsigned nt = n ? ceil_div(n, kStTPB * (w16 ? 16 : 8)) : 1;
+  const int occ = w16 ? g_dir_occ16 : g_dir_occ;
+  if (nt > (unsigned)(g_nsm * occ)) nt = (unsigned)(g_nsm * occ);   // persistent
+  cudaError_t le__ = launch_pdl(w16 ? k_directive16 : k_directive, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq,
+                                discard_off, tail0);
   if (le__) return le__;
   return cudaGetLastError();
 }

@@ -1,8 +1,9 @@
 #!/bin/bash
-# A/B of an env toggle on bench.py's state microbench: VAR=name, runs 0 and 1
-for v in 1 0; do
-  echo "== $VAR=$v"
-  env $VAR=$v timeout 300 python tools/state_bench.py --reps 3 2>&1 | python -c "
+# A/B of env settings on bench.py's state microbench: CONFIGS="A=1 B=2;A=0" (';'-separated)
+IFS=';' read -ra CFG <<< "${CONFIGS:-X=0}"
+for c in "${CFG[@]}"; do
+  echo "== $c"
+  env $c timeout 300 python tools/state_bench.py --reps 3 2>&1 | python -c "
 import json,sys
 for l in sys.stdin:
   try: d=json.loads(l)
