@@ -706,19 +706,13 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
   if (blockIdx.x == 0 && threadIdx.x == 0) T.ctl->n_rekey = n;   // USED slots appended
 }
 
-// 4 items per thread (8 CTAs/SM, 32 registers) or 8 (6 CTAs/SM, 40 registers);
-// UM_CLS_IPT selects (A/B)
+// 4 items per thread, 8 CTAs/SM (A/B on B200: 8 items per thread at 6 CTAs/SM spills and
+// runs the 2^21-block touch in 42 vs 30 us)
 __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
                                                         uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
                                                         int npar) {
   pdl_enter();
   classify_body<4>(T, iv, g0, n, seq, touch, tail0, npar);
-}
-__global__ void __launch_bounds__(kStTPB, 6) k_classify8(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
-                                                         uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
-                                                         int npar) {
-  pdl_enter();
-  classify_body<8>(T, iv, g0, n, seq, touch, tail0, npar);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1715,17 +1709,12 @@ __device__ __forceinline__ void directive_body(const Tables& T, int kind, uint32
   if (blockIdx.x == 0 && threadIdx.x == 0 && disc && active) c->disc_tail = tail0 + n;
 }
 
-// 8 blocks per thread (6 CTAs/SM) or 16 (4 CTAs/SM: 2^21 blocks in one round of 512
-// tiles, 16 state loads in flight per thread); UM_DIR_IPT selects (A/B)
+// 8 blocks per thread, 6 CTAs/SM (A/B on B200: 16 per thread at 4 CTAs/SM, one round of
+// 512 tiles for 2^21 blocks, measured the same 14.3 us)
 __global__ void __launch_bounds__(kStTPB, 6) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
                                                          int discard_off, unsigned long long tail0) {
   pdl_enter();
   directive_body<8>(T, kind, lo, n, seq, discard_off, tail0);
-}
-__global__ void __launch_bounds__(kStTPB, 4) k_directive16(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
-                                                           int discard_off, unsigned long long tail0) {
-  pdl_enter();
-  directive_body<16>(T, kind, lo, n, seq, discard_off, tail0);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1967,9 +1956,6 @@ static int g_nsm = 0;
 static int g_vscan_occ = 1;   // resident k_victims_scan CTAs per SM
 static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch (A/B)
 static int g_dir_occ = 8;     // resident k_directive CTAs per SM (persistent grid)
-static int g_dir_occ16 = 4;   // ... of k_directive16
-static int g_dir_ipt = 8;     // UM_DIR_IPT=16: directives with 16 blocks per thread (A/B)
-static int g_cls_ipt = 4;     // UM_CLS_IPT=8: classify with 8 items per thread (A/B)
 static int g_vs_prefetch = 0; // UM_VS_PREFETCH=1: the wide victim scan fetches its next ticket a tile ahead (A/B on B200: 79 vs 73 us pressured touch -- the earlier snapshot reads more tiles past the k-th candidate)
 
 cudaError_t setup_kernels() {
@@ -1980,7 +1966,6 @@ cudaError_t setup_kernels() {
   if (e) return e;
   if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
   if (const char* v = getenv("UM_VS_PREFETCH")) g_vs_prefetch = atoi(v) != 0;
-  if (const char* v = getenv("UM_CLS_IPT")) g_cls_ipt = atoi(v) == 8 ? 8 : 4;
   // Optionally one L1/shared carveout for every paging kernel (k_service needs 144 KB of
   // shared memory; a carveout change between consecutive kernels can force an SM drain).
   // UM_CARVEOUT=1 turns it on (A/B; off by default).
@@ -2004,10 +1989,6 @@ cudaError_t setup_kernels() {
   if (e) return e;
   if (g_dir_occ < 1) g_dir_occ = 1;
   if (const char* v = getenv("UM_DIR_OCC")) g_dir_occ = std::max(1, atoi(v));
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_dir_occ16, k_directive16, kStTPB, 0);
-  if (e) return e;
-  if (g_dir_occ16 < 1) g_dir_occ16 = 1;
-  if (const char* v = getenv("UM_DIR_IPT")) g_dir_ipt = atoi(v) == 16 ? 16 : 8;
   int smem = (int)(kXferChunk * (1 + 2 * kXferStages));
   return cudaFuncSetAttribute(k_service, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
 }
@@ -2042,13 +2023,12 @@ cudaError_t launch_poison(const Tables& T, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-uint32_t classify_tile() { return (uint32_t)kStTPB * (uint32_t)g_cls_ipt; }
+uint32_t classify_tile() { return (uint32_t)kStTPB * 4u; }
 
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
                             unsigned long long tail0, int npar, cudaStream_t s) {
   unsigned nt = n ? ceil_div(n, classify_tile()) : 1;
-  cudaError_t le__ = launch_pdl(g_cls_ipt == 8 ? k_classify8 : k_classify, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n,
-                                seq, touch, tail0, npar);
+  cudaError_t le__ = launch_pdl(k_classify, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar);
   if (le__) return le__;
   return cudaGetLastError();
 }
@@ -2107,12 +2087,9 @@ cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, 
 
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq, int discard_off,
                              unsigned long long tail0, cudaStream_t s) {
-  const bool w16 = g_dir_ipt == 16;
-  unsigned nt = n ? ceil_div(n, kStTPB * (w16 ? 16 : 8)) : 1;
-  const int occ = w16 ? g_dir_occ16 : g_dir_occ;
-  if (nt > (unsigned)(g_nsm * occ)) nt = (unsigned)(g_nsm * occ);   // persistent
-  cudaError_t le__ = launch_pdl(w16 ? k_directive16 : k_directive, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq,
-                                discard_off, tail0);
+  unsigned nt = n ? ceil_div(n, kStTPB * 8) : 1;
+  if (nt > (unsigned)(g_nsm * g_dir_occ)) nt = (unsigned)(g_nsm * g_dir_occ);   // persistent
+  cudaError_t le__ = launch_pdl(k_directive, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq, discard_off, tail0);
   if (le__) return le__;
   return cudaGetLastError();
 }
