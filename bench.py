@@ -315,8 +315,20 @@ def c1_rate(torch, um, harness):
         e1.synchronize()
         wall = time.perf_counter() - w0
         n = len(t) - 500
+        # device-only rate: 150 ops queued behind a device sleep (host enqueue off the
+        # critical path), so the span holds the GPU's own per-op time
+        um.um_get_stats(arena.handle)
+        with torch.cuda.stream(ps):
+            torch.cuda._sleep(200_000_000)
+        g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        g0.record(ps)
+        harness.issue(arena, t, "eager", 0, 150)
+        g1.record(ps)
+        g1.synchronize()
         return {"ops": n, "ops_per_s": n / wall, "us_per_op_wall": wall / n * 1e6,
-                "us_per_op_device": e0.elapsed_time(e1) * 1e3 / n}
+                "us_per_op_device": e0.elapsed_time(e1) * 1e3 / n,
+                "us_per_op_device_only": g0.elapsed_time(g1) * 1e3 / 150,
+                "device_only_note": "ops 0-150 replayed again on the same arena behind a device sleep"}
     finally:
         arena.close()
 

@@ -411,7 +411,6 @@ __device__ __forceinline__ void classify_single(const Tables& T, const OpIv& iv,
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint32_t idx = k * TPB + threadIdx.x;
-    bool nd = false;
     b[k] = 0;
     s[k] = 0xff;
     if (idx < n) {
@@ -422,14 +421,19 @@ __device__ __forceinline__ void classify_single(const Tables& T, const OpIv& iv,
         if (s_pre[mid] <= g) lo = mid; else hi = mid;
       }
       jlo = lo;
-      const uint32_t bb = s_lo[lo] + (g - s_pre[lo]);
-      const uint8_t ss = ld_st(T, bb);
-      T.pin[bb] = seq;
-      T.used_ring[(tail0 + idx) & T.cap_mask] = kseq | bb;
-      b[k] = bb;
-      s[k] = ss;
-      nd = ss <= ST_HD;
-      cls += 1u << (4 * ss);
+      b[k] = s_lo[lo] + (g - s_pre[lo]);
+      s[k] = ld_st(T, b[k]);   // all state loads before any store (stores could alias them)
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < IPT; ++k) {
+    const uint32_t idx = k * TPB + threadIdx.x;
+    bool nd = false;
+    if (idx < n) {
+      T.pin[b[k]] = seq;
+      T.used_ring[(tail0 + idx) & T.cap_mask] = kseq | b[k];
+      nd = s[k] <= ST_HD;
+      cls += 1u << (4 * s[k]);
     }
     bN[k] = __ballot_sync(FULL, nd);
   }
@@ -745,22 +749,32 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
     while (found < k && pos < tail) {
       const uint32_t w = (uint32_t)min((unsigned long long)W, tail - pos);
       const uint32_t first = threadIdx.x * kVictIPT;
-      uint32_t bb[kVictIPT];
+      // three load phases (ring entries, their state words, pins of live entries), each
+      // with all kVictIPT loads of a thread in flight
+      uint32_t bb[kVictIPT], kk[kVictIPT], wv[kVictIPT];
       unsigned candm = 0, livem = 0;
       uint32_t cc = 0;
 #pragma unroll
       for (int q = 0; q < kVictIPT; ++q) {
-        bb[q] = 0;
-        if (first + q < w) {
-          unsigned long long e = R[(pos + first + q) & T.cap_mask];
-          uint32_t blk = (uint32_t)e, kk = (uint32_t)(e >> 32);
-          bool live = entry_live(T, ring == RING_DISC, blk, kk);
-          bool cand = live && T.pin[blk] != seq;
-          bb[q] = blk;
-          livem |= (unsigned)live << q;
-          candm |= (unsigned)cand << q;
-          cc += cand;
-        }
+        const unsigned long long e = first + q < w ? R[(pos + first + q) & T.cap_mask] : ~0ull;
+        bb[q] = (uint32_t)e;
+        kk[q] = (uint32_t)(e >> 32);
+      }
+#pragma unroll
+      for (int q = 0; q < kVictIPT; ++q) wv[q] = bb[q] != UM_NONE ? T.sk[bb[q]] : 0u;
+#pragma unroll
+      for (int q = 0; q < kVictIPT; ++q) {
+        const uint8_t ss = st_of(wv[q]);
+        const bool live = bb[q] != UM_NONE && (ring == RING_DISC ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) &&
+                          key_of(wv[q]) == kk[q];
+        livem |= (unsigned)live << q;
+        wv[q] = live ? T.pin[bb[q]] : seq;
+      }
+#pragma unroll
+      for (int q = 0; q < kVictIPT; ++q) {
+        const bool cand = wv[q] != seq;
+        candm |= (unsigned)cand << q;
+        cc += cand;
       }
       unsigned long long tot;
       uint32_t rank = (uint32_t)block_excl_scan<kVictTPB>(cc, tot, s_scan);
@@ -811,13 +825,11 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
     uint32_t isG = 0, needA = 0;
     if (j < found) {
       v = T.victim[j];
+      const uint8_t nk = evict_mode ? (uint8_t)0xff : T.needk[(uint32_t)f0 + j];   // independent of v
       ss = ld_st(T, v);
       fr = T.frame_of[v];
       isG = ss == ST_G;
-      if (isG && !evict_mode) {
-        const uint32_t i = (uint32_t)f0 + j;
-        if (T.needk[i] == ST_H) swap_hf = T.needhf[i];
-      }
+      if (isG && nk == ST_H) swap_hf = T.needhf[(uint32_t)f0 + j];
       needA = isG && swap_hf == UM_NONE;
     }
     unsigned long long tot, totA;
