@@ -40,7 +40,8 @@ class Oracle:
     GPU frames (A15: oversubscription = arena / budget, L383)."""
 
     def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int,
-                 discard_off: bool = False, record: bool = False, host_release: bool = True):
+                 discard_off: bool = False, record: bool = False, host_release: bool = True,
+                 overlap: int = 0):
         if arena_bytes % block_bytes:
             raise ValueError("arena_bytes must be a multiple of block_bytes")
         self.B = block_bytes
@@ -56,6 +57,14 @@ class Oracle:
         # observable difference is the stale value a discarded block reads back, and
         # §4.1 (L160) allows zeros there.  host_release=False is the paper-literal model.
         self.host_release = host_release
+        # overlap (reading R7 / SURVEY NEXT-2): the application kernel of a
+        # GPU sub-op may still run while the next sub-ops are serviced, as the paper's
+        # asynchronous API calls overlap compute (L146, L166).  Victim selection then
+        # also skips the blocks of the last `overlap` GPU sub-ops -- the longest suffix
+        # of them that still leaves the current sub-op satisfiable (sizes summing with
+        # |S| to at most nframes).  overlap = 0 is the sequential model of SURVEY §8(c).
+        self.overlap = overlap
+        self.window: list = []                  # (blocks, count) of recent GPU sub-ops, oldest first
         n = self.nblocks
         self.st = [U] * n
         self.key = [0] * n
@@ -155,6 +164,19 @@ class Oracle:
         S: ascending distinct blocks, len(S) <= nframes."""
         st = self.st
         pinned = set(S)
+        if self.overlap:
+            # R7: protect the blocks of the in-flight application kernels of the previous
+            # GPU sub-ops; a window member is dropped (its kernel waited for) when keeping
+            # it could leave fewer than k candidates
+            keep, tot = [], len(S)
+            for blocks, cnt in reversed(self.window[-self.overlap:]):
+                if tot + cnt > self.nframes:
+                    break
+                tot += cnt
+                keep.append(blocks)
+            for blocks in keep:
+                pinned |= blocks
+            self.window = (self.window + [(frozenset(S), len(S))])[-self.overlap:]
         # steps 1-3: classify; blocks with no GPU frame need one
         need = [b for b in S if st[b] in (U, H, HD)]
         k = max(0, len(need) - self.free)
@@ -398,12 +420,12 @@ def apply_op(o: Oracle, op: tuple, mode: str):
 
 
 def replay(trace, mode: str = "eager", record: bool = False, stop: int | None = None,
-           host_release: bool = True) -> Oracle:
+           host_release: bool = True, overlap: int = 0) -> Oracle:
     """Replay a tracegen.Trace (optionally only its first `stop` ops) in one mode."""
     if mode not in MODES:
         raise ValueError(mode)
     o = Oracle(trace.block_bytes, trace.arena_bytes, trace.budget_bytes,
-               discard_off=(mode == "base"), record=record, host_release=host_release)
+               discard_off=(mode == "base"), record=record, host_release=host_release, overlap=overlap)
     for i, op in enumerate(trace.iter_ops()):
         if stop is not None and i >= stop:
             break

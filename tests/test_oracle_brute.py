@@ -62,8 +62,10 @@ class _DList:
 class LinkedModel:
     """Independent re-statement of the transition table."""
 
-    def __init__(self, B, nblocks, nframes, mode, host_release=True):
+    def __init__(self, B, nblocks, nframes, mode, host_release=True, overlap=0):
         self.B, self.n, self.F, self.mode, self.rel = B, nblocks, nframes, mode, host_release
+        # R7 window: block lists of the previous GPU sub-ops, newest first
+        self.W, self.recent = overlap, []
         self.state = ["U"] * nblocks
         self.gpu = [0] * nblocks
         self.host = [0] * nblocks
@@ -104,6 +106,16 @@ class LinkedModel:
     def gpu_sub(self, blocks, touch, writes):
         t = self.tick()
         excl = set(blocks)
+        if self.W:
+            # protect previous sub-ops newest first while the frames they could hold,
+            # plus this sub-op's, fit in the budget (R7)
+            room = self.F - len(blocks)
+            for prev in self.recent[:self.W]:
+                room -= len(prev)
+                if room < 0:
+                    break
+                excl.update(prev)
+            self.recent.insert(0, list(blocks))
         while sum(1 for b in blocks if self.state[b] in ("U", "H", "HD")) > self.nfree:
             # one victim at a time, each time re-scanning from the queue heads
             self.reclaim(self.evict_one(excl))
@@ -227,11 +239,12 @@ class LinkedModel:
                 "stats": dict(self.c), "contents": content}
 
 
-def _compare(trace, mode, host_release=True):
-    o = replay(trace, mode, host_release=host_release)
+def _compare(trace, mode, host_release=True, overlap=0):
+    o = replay(trace, mode, host_release=host_release, overlap=overlap)
     o.check_conservation()
     d = o.dump()
-    m = LinkedModel(trace.block_bytes, trace.nblocks, trace.nframes, mode, host_release).run(trace).result()
+    m = LinkedModel(trace.block_bytes, trace.nblocks, trace.nframes, mode, host_release,
+                    overlap).run(trace).result()
     assert [ST_NAMES[s] for s in d["st"]] == m["st"]
     assert d["used_order"] == m["used_order"]
     assert d["disc_order"] == m["disc_order"]
@@ -269,14 +282,15 @@ def _mk(seq, nframes):
     return tb.build()
 
 
+@pytest.mark.parametrize("overlap", [0, 2])
 @pytest.mark.parametrize("nframes", [1, 2])
 @pytest.mark.parametrize("length", [1, 2, 3])
-def test_exhaustive_vs_linked_model(nframes, length):
+def test_exhaustive_vs_linked_model(nframes, length, overlap):
     n = 0
     for seq in itertools.product(_ALPHA, repeat=length):
         t = _mk(seq, nframes)
         for mode in ("base", "eager", "lazy"):
-            _compare(t, mode)
+            _compare(t, mode, overlap=overlap)
         n += 1
     assert n == len(_ALPHA) ** length
 
@@ -517,3 +531,37 @@ def test_next3_radix_hashjoin_invariants(ov):
             assert mv["eager"] == mv["base"]
         else:
             assert mv["eager"] <= mv["base"]
+
+
+# ------------------------------------------------------------------ R7 (UM_F_OVERLAP)
+@settings(max_examples=150, deadline=None, suppress_health_check=[HealthCheck.too_slow])
+@given(seed=hst.integers(0, 10**6), nblocks=hst.integers(1, 10), nframes=hst.integers(1, 5),
+       overlap=hst.integers(1, 3))
+def test_overlap_vs_linked_model(seed, nblocks, nframes, overlap):
+    """The window rule (reading R7) restated independently in the linked-list model; its
+    victim loop fails if the window ever leaves fewer candidates than k."""
+    t = tg.gen_small(seed, nblocks=nblocks, nframes=nframes, n_ops=40)
+    for mode in ("base", "eager", "lazy"):
+        _compare(t, mode, overlap=overlap)
+
+
+@settings(max_examples=60, deadline=None)
+@given(seed=hst.integers(0, 10**6), nblocks=hst.integers(2, 10), nframes=hst.integers(1, 4))
+def test_overlap_keeps_semantics(seed, nblocks, nframes):
+    """R7 changes which block is evicted, never what a program reads: the flat-memory
+    check (iii)/(iv) and the no-writeback-of-discarded invariant (ii) hold with the
+    window, and without memory pressure the window changes nothing at all."""
+    t = tg.gen_small(seed, nblocks=nblocks, nframes=nframes, n_ops=40)
+    for mode in ("base", "eager", "lazy"):
+        o = replay(t, mode, overlap=2, record=True)
+        o.check_conservation()
+        got = o.contents()
+        val, dc, hist = FlatMemory(t, mode).run()
+        for b in range(t.nblocks):
+            assert got[b] == val[b] if not dc[b] else got[b] in hist[b], (mode, b)
+        for (_s, kind, _b, prev) in o.log:
+            if kind == "D2H":
+                assert ST_NAMES[prev] == "G"
+    roomy = tg.gen_small(seed, nblocks=nblocks, nframes=nblocks, n_ops=40)   # arena <= budget
+    for mode in ("base", "eager", "lazy"):
+        assert replay(roomy, mode, overlap=2).dump() == replay(roomy, mode).dump()
