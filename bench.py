@@ -48,6 +48,10 @@ def parse():
     p.add_argument("--pin-threads", type=int, default=8)
     p.add_argument("--no-compare", action="store_true")
     p.add_argument("--no-state-bench", action="store_true")
+    p.add_argument("--app-overlap", default="off", choices=["on", "off"],
+                   help="UM_F_OVERLAP (reading R7) for the headline modes: app kernels pipelined with the "
+                        "next sub-ops (measured no faster on C3: the step is transfer-bound and a write-"
+                        "saturating app kernel slows the latency-bound planning kernels)")
     return p.parse_args()
 
 
@@ -169,6 +173,7 @@ def run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=None, flags_extr
         evs[0].record(ps)
         for j in range(K):
             harness.issue(arena, trace, mode, *bounds[W + j])
+            um.um_join(arena.handle)                # the iteration ends with its app kernels
             evs[j + 1].record(ps)
         evs[-1].synchronize()
         wall = time.perf_counter() - wall0
@@ -184,12 +189,12 @@ def run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=None, flags_extr
         arena.close()
 
 
-def run_e2e(torch, um, harness, mem, trace, W, K):
+def run_e2e(torch, um, harness, mem, trace, W, K, flags_extra=0):
     """End to end through the public API: the trace WITH the host-side data generation
     (prefetch(data,HOST); host_write; prefetch(data,GPU): the step's inputs cross
     host->device), plus a device->host read of the step's counters each step; host
     wall-clock per step."""
-    arena = harness.make_arena(trace, "eager", mem=mem, flags=um.UM_F_APP_STAMP)
+    arena = harness.make_arena(trace, "eager", mem=mem, flags=um.UM_F_APP_STAMP | flags_extra)
     try:
         harness.alloc_buffers(arena, trace)
         bounds = harness.iteration_bounds(trace)
@@ -522,11 +527,18 @@ def main_ours(args):
 
     res = {}
     clocks = Clocks(dev.index)
+    ovf = um.UM_F_OVERLAP if args.app_overlap == "on" else 0
     for mode in args.modes.split(","):
-        res[mode] = run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=clocks if mode == "eager" else None)
-    # the TMA kernel path (K4) on the same step, for comparison with the auto path
-    k4 = run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=um.UM_F_COPY_KERNEL) \
+        res[mode] = run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=clocks if mode == "eager" else None,
+                             flags_extra=ovf)
+    # the TMA kernel path (K4) on the same step, for comparison with the auto path, and the
+    # same step with the app kernels serialized on the paging stream (no R7 window)
+    k4 = run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=um.UM_F_COPY_KERNEL | ovf) \
         if not args.no_compare else None
+    # the other app-kernel schedule on the same step (R7 overlap <-> sequential)
+    other = run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=um.UM_F_OVERLAP ^ ovf) \
+        if not args.no_compare else None
+    ovl_r, seq_r = (res.get("eager"), other) if ovf else (other, res.get("eager"))
     state = None
     if not args.no_state_bench:
         # two runs on fresh arenas over the same memory; the second is reported (the first
@@ -536,7 +548,7 @@ def main_ours(args):
         state["reps"] = "second of two runs (first = warm-up)"
     e2e_s = None
     if not args.no_e2e:
-        e2e_s = run_e2e(torch, um, harness, mem, trace, 1, min(K, 3))
+        e2e_s = run_e2e(torch, um, harness, mem, trace, 1, min(K, 3), flags_extra=ovf)
 
     head = res.get("eager") or next(iter(res.values()))
     t_iter_ms = head["iter_ms"]
@@ -571,7 +583,9 @@ def main_ours(args):
                    "layers": trace.meta["layers"], "ops_per_iter": trace.meta["ops_per_iter"],
                    "host_pool_bytes": host_pool, "budget_requested_bytes": int(args.budget_gib * GiB), "parallelism": f"independent arenas x{ws}",
                    "l2": "working set 255 GiB >> 126 MB L2 (no flush needed)",
-                   "headline_mode": "eager (UvmDiscard)"},
+                   "headline_mode": "eager (UvmDiscard)",
+                   "app_overlap": ("UM_F_OVERLAP: app kernels pipelined with the next 2 GPU sub-ops (reading R7), "
+                                   "every mode" if ovf else "off: app kernels serialized on the paging stream")},
         "iter_ms": {m: r["iter_ms"] for m, r in res.items()},
         "speedup_vs_discard_off": (base["iter_ms"] / t_iter_ms) if base else None,
         "gb_avoided_per_iter": avoided,
@@ -593,6 +607,14 @@ def main_ours(args):
                      "launches_per_iter": tm["xfer_launches"] / K, "xfer_share_of_step": tm["ms_xfer"] / (t_iter_ms * K)},
         "link_peak": link,
         "transfer_paths": _paths(res.get("eager"), k4, link),
+        "app_overlap": ({"eager_overlap_iter_ms": ovl_r["iter_ms"], "eager_sequential_iter_ms": seq_r["iter_ms"],
+                         "speedup": seq_r["iter_ms"] / ovl_r["iter_ms"],
+                         "plan_ms_per_iter": {"overlap": ovl_r["timing"]["ms_plan"] / K,
+                                              "sequential": seq_r["timing"]["ms_plan"] / K},
+                         "same_link_bytes": seq_r["stats_per_iter"]["h2d_bytes"] == ovl_r["stats_per_iter"]["h2d_bytes"]
+                         and seq_r["stats_per_iter"]["d2h_bytes"] == ovl_r["stats_per_iter"]["d2h_bytes"],
+                         "headline": "overlap" if ovf else "sequential"}
+                        if (ovl_r and seq_r) else None),
         "roofline_state": state,
         "c1_directives": c1,
         "c4_sweep": c4,

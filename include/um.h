@@ -69,8 +69,17 @@ enum {
                             every UM_ACC_WRITE block (simulated application kernel)    */
   UM_F_TIMING = 16u,     /* record CUDA events around the planning and transfer kernels
                             of every op (read with um_timing)                          */
-  UM_F_COPY_KERNEL = 32u /* always move data with the TMA kernel (K4).  Default (neither
+  UM_F_COPY_KERNEL = 32u,/* always move data with the TMA kernel (K4).  Default (neither
                             flag): sub-ops moving >= 16 MiB use K4-CE, smaller ones K4  */
+  UM_F_OVERLAP = 64u     /* pipelined application kernels (reading R7; the
+                            paper's async API calls overlap compute):
+                            the UM_F_APP_STAMP kernel of a touch sub-op runs on an
+                            arena-internal app stream and overlaps the next sub-ops;
+                            victim selection skips the blocks of the last 2 GPU sub-ops
+                            (the longest suffix that leaves k satisfiable).  Ops that
+                            move data out or free frames (prefetch HOST, evict) wait for
+                            every app kernel.  An op's completion on the caller's stream
+                            covers the paging work only: use um_join for the app work. */
 };
 
 /* One GPU access record of a batch (16 bytes).  Covers every block overlapping
@@ -152,6 +161,11 @@ um_status um_host_write(um_arena *a, uint64_t off, uint64_t len, void *stream);
  * that application kernels translate through: addr = frames + map[b]*block + off%block.
  * G and GL blocks are mapped; U/H/HD/GE are not (an eager discard unmaps). */
 um_status um_block_table(um_arena *a, const uint32_t **dev_map);
+
+/* Make `stream` wait for all work the arena has enqueued so far, including the
+ * UM_F_OVERLAP application kernels (without that flag it equals an empty op's
+ * hand-off).  Enqueues only; never blocks the host. */
+um_status um_join(um_arena *a, void *stream);
 
 /* The arena's internal paging stream (work enqueued on it needs no event hand-off). */
 um_status um_stream(um_arena *a, void **stream);

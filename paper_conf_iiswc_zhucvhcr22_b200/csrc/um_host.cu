@@ -161,6 +161,22 @@ struct Stager {
     pos = hi;
     return cudaSuccess;
   }
+  // Keep [off, off+bytes) reserved until the work enqueued on stream s so far is done
+  // (an application kernel on another stream still reading staged intervals, R7).
+  cudaError_t fence(uint64_t off, uint64_t bytes, cudaStream_t s) {
+    cudaEvent_t ev;
+    cudaError_t e;
+    if (pool.empty()) {
+      e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+      if (e) return e;
+    } else {
+      ev = pool.back();
+      pool.pop_back();
+    }
+    e = cudaEventRecord(ev, s);
+    fly.push_back({off, off + bytes, ev});
+    return e;
+  }
   cudaError_t push(uint64_t off, uint64_t bytes, cudaStream_t s) {
     cudaError_t e = cudaMemcpyAsync(dev + off, host + off, bytes, cudaMemcpyHostToDevice, s);
     if (e) return e;
@@ -215,7 +231,7 @@ struct um_arena {
   Ctl* hctl = nullptr;  // pinned mirror for reads
   std::vector<Iv> ivs;
   // UM_F_TIMING: event pairs around planning / transfer launches
-  struct Span { cudaEvent_t a, b; int xfer; };
+  struct Span { cudaEvent_t a, b; int xfer; uint32_t seq; };
   std::vector<Span> spans;
   std::vector<cudaEvent_t> evpool;
   double ms_plan = 0, ms_xfer = 0;
@@ -229,6 +245,21 @@ struct um_arena {
   char* bounce = nullptr;
   uint64_t ce_min_bytes = 16ull << 20;  // auto mode: sub-ops moving >= this use the copy engines
   uint64_t n_ce = 0;
+  // UM_F_OVERLAP (reading R7): application kernels run on their own stream `as`; the
+  // last kOverlapW GPU sub-ops form the victim-exclusion window; `pend` holds the app
+  // kernels the paging stream has not waited for yet (ascending seq)
+  cudaStream_t as = nullptr;
+  cudaEvent_t ev_app_in = nullptr;
+  // the app kernel's CTAs per SM while it overlaps paging work: its grid-stride CTAs
+  // live for the whole kernel, so a full-occupancy grid would keep the paging and
+  // zero-fill kernels off the SMs until it ends (UM_APP_CTAS overrides)
+  int app_ctas = 1;
+  struct WinE { uint32_t seq, n; };
+  WinE win[kOverlapW] = {};
+  int nwin = 0;
+  struct Pend { uint32_t seq; cudaEvent_t ev; };
+  std::deque<Pend> pend;
+  std::vector<cudaEvent_t> apool;
 };
 
 namespace {
@@ -307,7 +338,47 @@ static void span_close(um_arena* a, cudaEvent_t open, int xfer) {
   if (!open) return;
   cudaEvent_t e = tev(a);
   cudaEventRecord(e, a->ps);
-  a->spans.push_back({open, e, xfer});
+  a->spans.push_back({open, e, xfer, a->clock});
+}
+
+// ---- UM_F_OVERLAP (reading R7) ----------------------------------------------------
+static inline bool overlap_on(const um_arena* a) { return (a->cfg.flags & UM_F_OVERLAP) != 0; }
+
+// The paging stream waits for every application kernel of a sub-op with seq < floor
+// (the app stream runs them in order, so waiting for the newest of them suffices).
+static um_status app_wait_below(um_arena* a, uint32_t floor) {
+  cudaEvent_t last = nullptr;
+  while (!a->pend.empty() && a->pend.front().seq < floor) {
+    if (last) a->apool.push_back(last);
+    last = a->pend.front().ev;
+    a->pend.pop_front();
+  }
+  if (last) {
+    CK(cudaStreamWaitEvent(a->ps, last, 0));
+    a->apool.push_back(last);
+  }
+  return UM_OK;
+}
+static um_status app_wait_all(um_arena* a) { return app_wait_below(a, UM_NONE); }
+
+// Victim floor of GPU sub-op `seq` with n distinct blocks: the longest suffix of the last
+// kOverlapW GPU sub-ops whose block counts, added to n, stay <= nframes is protected
+// (so k = need - free stays satisfiable); the floor is the seq of its oldest member, or
+// seq itself when nothing is protected.  Identical to oracle.sim's window rule.
+static uint32_t window_floor(um_arena* a, uint32_t seq, uint32_t n) {
+  uint64_t tot = n;
+  uint32_t floor = seq;
+  for (int i = a->nwin - 1; i >= 0; --i) {
+    if (tot + a->win[i].n > a->nframes) break;
+    tot += a->win[i].n;
+    floor = a->win[i].seq;
+  }
+  if (a->nwin == kOverlapW) {
+    for (int i = 1; i < kOverlapW; ++i) a->win[i - 1] = a->win[i];
+    a->nwin--;
+  }
+  a->win[a->nwin++] = {seq, n};
+  return floor;
 }
 
 // K7 trigger: the host keeps an upper bound of each ring's occupancy (appends are
@@ -628,9 +699,11 @@ static um_status run_gpu_op(um_arena* a, int touch) {
   if (total == 0) {
     a->clock++;
     a->subops++;
+    if (overlap_on(a)) window_floor(a, a->clock, 0);
     return UM_OK;
   }
   const uint32_t m = dev ? a->dev_m : (uint32_t)a->ivs.size();
+  uint64_t iv_off = 0, iv_bytes = 0;   // staged interval arrays (read by the app kernels)
   OpIv iv{};
   iv.m = m;
   if (dev) {
@@ -656,6 +729,8 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     const uint64_t bytes = o_w + bytes_w;
     uint64_t off;
     CK(a->stage.reserve(bytes, &off));
+    iv_off = off;
+    iv_bytes = (bytes + 15) & ~15ull;
     uint32_t* hlo = (uint32_t*)(a->stage.host + off + o_lo);
     uint32_t* hpre = (uint32_t*)(a->stage.host + off + o_pre);
     uint8_t* hw = a->stage.host + off + o_w;
@@ -681,6 +756,14 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     a->subops++;
     um_status st = ensure_ring_room(a, RING_USED, n);
     if (st) return st;
+    if (overlap_on(a)) {
+      a->T.pfloor = window_floor(a, seq, n);
+      st = app_wait_below(a, a->T.pfloor);   // app kernels outside the window finish first
+      if (st) return st;
+    } else {
+      a->T.pfloor = seq;
+    }
+    uint64_t tj_off = 0, tj_bytes = 0;
     if (!iv.inl) {
       // per tile of this sub-op, the interval slice its items fall in: an index the
       // kernels would otherwise find by a dependent binary search over the staged list
@@ -688,6 +771,8 @@ static um_status run_gpu_op(um_arena* a, int touch) {
       const uint32_t nt = (n + tile - 1) / tile;
       uint64_t off;
       CK(a->stage.reserve(8ull * nt, &off));
+      tj_off = off;
+      tj_bytes = (8ull * nt + 15) & ~15ull;
       uint32_t* tj = (uint32_t*)(a->stage.host + off);
       auto seek = [&](uint64_t g) {
         while (hp[jcur + 1] <= g) ++jcur;
@@ -730,7 +815,26 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     }
     a->n_xfer++;
     if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP)) {
-      CK(launch_app_stamp(a->T, iv, (uint32_t)g0, n, seq, a->ps));
+      if (overlap_on(a) && !getenv("UM_OVERLAP_SERIAL")) {   // (diagnostic: window rule only)
+        // R7: the application kernel runs on its own stream after this sub-op's
+        // transfers and overlaps the next sub-ops' planning and transfers
+        CK(cudaEventRecord(a->ev_app_in, a->ps));
+        CK(cudaStreamWaitEvent(a->as, a->ev_app_in, 0));
+        CK(launch_app_stamp(a->T, iv, (uint32_t)g0, n, seq, a->app_ctas, a->as));
+        cudaEvent_t e;
+        if (a->apool.empty()) {
+          CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        } else {
+          e = a->apool.back();
+          a->apool.pop_back();
+        }
+        CK(cudaEventRecord(e, a->as));
+        a->pend.push_back({seq, e});
+        if (iv_bytes) CK(a->stage.fence(iv_off, iv_bytes, a->as));
+        if (tj_bytes) CK(a->stage.fence(tj_off, tj_bytes, a->as));
+      } else {
+        CK(launch_app_stamp(a->T, iv, (uint32_t)g0, n, seq, 8, a->ps));
+      }
       a->n_launch++;
     }
   }
@@ -843,14 +947,24 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
     uint32_t z = T.zero_hf;
     memset((char*)cfg->host_chunks[z / hpc] + (size_t)(z % hpc) * a->B, 0, a->B);
   }
-  if ((e = cudaStreamCreateWithFlags(&a->ps, cudaStreamNonBlocking))) return fail(e);
+  // UM_F_OVERLAP: the paging and copy streams take the highest priority and the app
+  // stream the lowest, so queued paging CTAs are scheduled ahead of app CTAs
+  int prio_lo = 0, prio_hi = 0;
+  if ((cfg->flags & UM_F_OVERLAP) && !getenv("UM_NO_PRIO")) cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+  if ((e = cudaStreamCreateWithPriority(&a->ps, cudaStreamNonBlocking, prio_hi))) return fail(e);
+  if (cfg->flags & UM_F_OVERLAP) {
+    if ((e = cudaStreamCreateWithPriority(&a->as, cudaStreamNonBlocking, prio_lo))) return fail(e);
+    if ((e = cudaEventCreateWithFlags(&a->ev_app_in, cudaEventDisableTiming))) return fail(e);
+    if (const char* v = getenv("UM_APP_CTAS")) a->app_ctas = std::max(1, atoi(v));
+    if (const char* v = getenv("UM_APP_GRID")) a->app_ctas = -std::max(1, atoi(v));
+  }
   if ((e = cudaEventCreateWithFlags(&a->ev_in, cudaEventDisableTiming))) return fail(e);
   if ((e = cudaEventCreateWithFlags(&a->ev_out, cudaEventDisableTiming))) return fail(e);
   if ((e = cudaHostAlloc((void**)&a->hctl, sizeof(Ctl), cudaHostAllocDefault))) return fail(e);
   if ((e = cudaHostAlloc((void**)&a->hitems, sizeof(XItem) * a->nframes, cudaHostAllocDefault))) return fail(e);
   if ((e = cudaHostAlloc((void**)&a->hd2h, 8ull * a->nframes, cudaHostAllocDefault))) return fail(e);
   for (int i = 0; i < 2; ++i) {
-    if ((e = cudaStreamCreateWithFlags(&a->cs[i], cudaStreamNonBlocking))) return fail(e);
+    if ((e = cudaStreamCreateWithPriority(&a->cs[i], cudaStreamNonBlocking, prio_hi))) return fail(e);
     if ((e = cudaEventCreateWithFlags(&a->ev_cs[i], cudaEventDisableTiming))) return fail(e);
   }
   for (uint32_t i = 0; i < cfg->n_host_chunks; ++i) a->hhost.push_back((char*)cfg->host_chunks[i]);
@@ -871,7 +985,12 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
 UM_API um_status um_arena_destroy(um_arena* a) {
   if (!a) return UM_EINVAL;
   if (a->ps) cudaStreamSynchronize(a->ps);
+  if (a->as) cudaStreamSynchronize(a->as);
   a->stage.destroy();
+  for (auto& p : a->pend) cudaEventDestroy(p.ev);
+  for (auto e : a->apool) cudaEventDestroy(e);
+  if (a->ev_app_in) cudaEventDestroy(a->ev_app_in);
+  if (a->as) cudaStreamDestroy(a->as);
   for (auto& sp : a->spans) { cudaEventDestroy(sp.a); cudaEventDestroy(sp.b); }
   for (auto e : a->evpool) cudaEventDestroy(e);
   if (a->hctl) cudaFreeHost(a->hctl);
@@ -909,6 +1028,8 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
   // deduplicated on the device; otherwise the records (or the <= kIvInline records after a
   // 2n-event merge while they are packed into the kernel arguments) are the intervals
   if (n > kIvInline && a->nblocks < (1u << 31) && !sorted_disjoint(a, acc, n)) {
+    // the intake rewrites the device interval list that in-flight app kernels may read
+    if (overlap_on(a) && (s = app_wait_all(a))) return s;
     s = device_intake(a, acc, n);
     if (s) return s;
   } else {
@@ -934,6 +1055,8 @@ UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, v
     if (s) return s;
   } else {
     if ((s = seq_room(a, 1))) return s;
+    // moves data and frees frames: every in-flight application kernel finishes first (R7)
+    if (overlap_on(a) && (s = app_wait_all(a))) return s;
     a->ops++;
     a->subops++;
     const uint32_t seq = ++a->clock;
@@ -1006,6 +1129,8 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
   const uint32_t seq = ++a->clock;
   uint64_t want = (bytes + a->B - 1) / a->B;
   if (want > a->nframes) want = a->nframes;
+  a->T.pfloor = seq;   // no pinned blocks: every in-flight application kernel finishes first
+  if (overlap_on(a) && (s = app_wait_all(a))) return s;
   if (want) {
     cudaEvent_t sp = span_open(a);
     if (want > kVictWideMin)
@@ -1051,6 +1176,15 @@ UM_API um_status um_block_table(um_arena* a, const uint32_t** dev_map) {
   return UM_OK;
 }
 
+UM_API um_status um_join(um_arena* a, void* stream) {
+  ENTER(a);
+  if (overlap_on(a)) {
+    um_status s = app_wait_all(a);
+    if (s) return s;
+  }
+  return hand_out(a, stream);
+}
+
 UM_API um_status um_stream(um_arena* a, void** stream) {
   if (!a || !stream) return UM_EINVAL;
   *stream = (void*)a->ps;
@@ -1058,6 +1192,7 @@ UM_API um_status um_stream(um_arena* a, void** stream) {
 }
 
 static um_status sync_ctl(um_arena* a) {
+  if (a->as) CK(cudaStreamSynchronize(a->as));
   CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
   CK(cudaStreamSynchronize(a->ps));
   if (a->hctl->err == 1u) a->sticky = UM_EINVAL;
@@ -1117,6 +1252,10 @@ UM_API um_status um_dump(um_arena* a, uint8_t* st, uint32_t* used_order, uint32_
 UM_API um_status um_content_tags(um_arena* a, uint64_t* tags) {
   ENTER(a);
   if (!tags) return UM_EINVAL;
+  if (overlap_on(a)) {
+    um_status s = app_wait_all(a);
+    if (s) return s;
+  }
   CK(launch_tags(a->T, a->ps));
   CK(cudaMemcpyAsync(tags, a->T.tags, 8ull * a->nblocks, cudaMemcpyDeviceToHost, a->ps));
   CK(cudaStreamSynchronize(a->ps));
@@ -1127,14 +1266,19 @@ UM_API um_status um_timing(um_arena* a, double* ms_plan, double* ms_xfer, uint64
                            uint64_t* launches, int reset) {
   ENTER(a);
   CK(cudaStreamSynchronize(a->ps));
+  if (a->as) CK(cudaStreamSynchronize(a->as));
+  FILE* lg = nullptr;
+  if (const char* p = getenv("UM_SPAN_LOG")) lg = fopen(p, "a");   // diagnostics: one line per span
   for (auto& sp : a->spans) {
     float ms = 0;
     CK(cudaEventElapsedTime(&ms, sp.a, sp.b));
+    if (lg) fprintf(lg, "%u %d %.4f\n", sp.seq, sp.xfer, ms);
     (sp.xfer ? a->ms_xfer : a->ms_plan) += ms;
     a->evpool.push_back(sp.a);
     a->evpool.push_back(sp.b);
   }
   a->spans.clear();
+  if (lg) fclose(lg);
   if (ms_plan) *ms_plan = a->ms_plan;
   if (ms_xfer) *ms_xfer = a->ms_xfer;
   if (xfer_launches) *xfer_launches = a->n_xfer;

@@ -97,6 +97,10 @@ struct Tables {
   uint32_t B;               // block bytes
   uint32_t nblocks, nframes, nhframes;
   uint32_t zero_hf;         // host frame id of the zero page (never allocated)
+  // victim floor: a live ring entry is a candidate iff pin[b] < pfloor.  = seq of the
+  // current sub-op (its own blocks are never victims, A3), or with UM_F_OVERLAP the seq
+  // of the oldest GPU sub-op whose application kernel may still run (reading R7)
+  uint32_t pfloor;
 };
 
 // A GPU-destination op's distinct blocks as sorted disjoint intervals.  Interval j
@@ -105,6 +109,9 @@ struct Tables {
 // Small ops (m <= kIvInline) carry the list inline in the kernel parameters (no staging
 // copy); larger ones point at a staged device copy.
 constexpr uint32_t kIvInline = 24;
+// UM_F_OVERLAP: number of previous GPU sub-ops whose application kernels may still run
+// while a sub-op is serviced (reading R7; the oracle's `overlap` parameter)
+constexpr int kOverlapW = 2;
 struct OpIv {
   const uint32_t* lo;
   const uint32_t* pre;
@@ -151,7 +158,8 @@ cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, u
                                 uint64_t scan_bound, uint32_t max_victims, int npar, cudaStream_t s);
 constexpr uint32_t kVictWideMin = 8192;
 cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max_items, cudaStream_t s);
-cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, cudaStream_t s);
+cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int ctas_per_sm,
+                             cudaStream_t s);
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
                              int discard_off, unsigned long long tail0, cudaStream_t s);
 cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64_t cap_bound, cudaStream_t s);

@@ -768,11 +768,11 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
         const bool live = bb[q] != UM_NONE && (ring == RING_DISC ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) &&
                           key_of(wv[q]) == kk[q];
         livem |= (unsigned)live << q;
-        wv[q] = live ? T.pin[bb[q]] : seq;
+        wv[q] = live ? T.pin[bb[q]] : UM_NONE;
       }
 #pragma unroll
       for (int q = 0; q < kVictIPT; ++q) {
-        const bool cand = wv[q] != seq;
+        const bool cand = wv[q] < T.pfloor;   // live and not pinned by an in-flight sub-op
         candm |= (unsigned)cand << q;
         cc += cand;
       }
@@ -1020,11 +1020,11 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
       const uint8_t ss = st_of(wv[q]);
       const bool live = bb[q] != UM_NONE && (idx < s_ld ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) &&
                         key_of(wv[q]) == kk[q];
-      wv[q] = live ? T.pin[bb[q]] : seq;   // not a candidate unless live and unpinned
+      wv[q] = live ? T.pin[bb[q]] : UM_NONE;   // not a candidate unless live and unpinned
       bL[q] = __ballot_sync(FULL, live);
     }
 #pragma unroll
-    for (int q = 0; q < kVsIPT; ++q) bC[q] = __ballot_sync(FULL, wv[q] != seq);
+    for (int q = 0; q < kVsIPT; ++q) bC[q] = __ballot_sync(FULL, wv[q] < T.pfloor);
     const uint32_t cnt = ordered_offsets<kVsTPB, kVsIPT>(bC, bC, s_off) & 0xffffu;
     unsigned long long mk0 = ~0ull, mk1 = ~0ull;   // first live entry kept (pinned), per ring
     uint32_t* scr = T.vscratch + tbase;
@@ -1514,13 +1514,14 @@ __global__ void k_plan_commit(Tables T, uint32_t seq) {
 // flight, so the per-segment lookup latency is amortised over 256 KiB of writes.
 constexpr uint32_t kFillSeg = 256u << 10;
 
+template <int TPB = 256>
 __device__ __forceinline__ void fill_segment(uint4* dst, uint32_t n16, uint4 v) {
   uint32_t t = threadIdx.x;
-  for (; t + 7 * 256 < n16; t += 8 * 256) {
+  for (; t + 7 * TPB < n16; t += 8 * TPB) {
 #pragma unroll
-    for (int k = 0; k < 8; ++k) dst[t + k * 256] = v;
+    for (int k = 0; k < 8; ++k) dst[t + k * TPB] = v;
   }
-  for (; t < n16; t += 256) dst[t] = v;
+  for (; t < n16; t += TPB) dst[t] = v;
 }
 
 __global__ void __launch_bounds__(256) k_zero_items(Tables T, uint32_t i0, uint32_t i1) {
@@ -1545,7 +1546,11 @@ __global__ void __launch_bounds__(256) k_zero_items(Tables T, uint32_t i0, uint3
 // UM_ACC_WRITE access receives the content stamp s = (seq << 32) | block as the
 // 16-byte pattern {s, ~s}, written through its frame (G or GL blocks are mapped).
 // ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) k_app_stamp(Tables T, const __grid_constant__ OpIv iv, uint32_t g0, uint32_t n, uint32_t seq) {
+// TPB = 256 on the paging stream; TPB = 128 at one CTA per SM when it overlaps paging
+// work (UM_F_OVERLAP): its grid-stride CTAs live for the whole kernel, and a small
+// footprint leaves room on every SM for the 1024-thread planning CTAs.
+template <int TPB>
+__global__ void __launch_bounds__(TPB) k_app_stamp(Tables T, const __grid_constant__ OpIv iv, uint32_t g0, uint32_t n, uint32_t seq) {
   pdl_enter();
   __shared__ char* s_dst;
   __shared__ uint32_t s_blk;
@@ -1569,8 +1574,8 @@ __global__ void __launch_bounds__(256) k_app_stamp(Tables T, const __grid_consta
     char* d = s_dst;
     const unsigned long long sv = ((unsigned long long)seq << 32) | s_blk;
     __syncthreads();
-    if (d) fill_segment(reinterpret_cast<uint4*>(d), SEG / 16,
-                        make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32)));
+    if (d) fill_segment<TPB>(reinterpret_cast<uint4*>(d), SEG / 16,
+                             make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32)));
   }
 }
 
@@ -1986,7 +1991,7 @@ cudaError_t setup_kernels() {
   if (carve) {
     const void* ks[] = {(const void*)k_classify, (const void*)k_victims, (const void*)k_plan_small,
                         (const void*)k_victims_scan, (const void*)k_victims_apply, (const void*)k_service,
-                        (const void*)k_app_stamp, (const void*)k_directive, (const void*)k_ring_compact,
+                        (const void*)k_app_stamp<256>, (const void*)k_app_stamp<128>, (const void*)k_directive, (const void*)k_ring_compact,
                         (const void*)k_plan_commit, (const void*)k_zero_items, (const void*)k_mark,
                         (const void*)k_runs, (const void*)k_intake_clear};
     for (const void* k : ks) {
@@ -2087,12 +2092,17 @@ cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max
   return cudaGetLastError();
 }
 
-cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, cudaStream_t s) {
+cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int ctas_per_sm,
+                             cudaStream_t s) {
   const uint32_t SEG = T.B < kFillSeg ? T.B : kFillSeg;
   unsigned long long units = (unsigned long long)n * (T.B / SEG);
-  unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
+  // ctas_per_sm < 0: a grid of -ctas_per_sm CTAs in total (a bandwidth-capped background kernel)
+  const unsigned long long cap = ctas_per_sm < 0 ? (unsigned long long)(-ctas_per_sm)
+                                                 : (unsigned long long)g_nsm * ctas_per_sm;
+  unsigned grid = (unsigned)(units < cap ? units : cap);
   if (!grid) return cudaSuccess;
-  cudaError_t le__ = launch_pdl(k_app_stamp, dim3(grid), dim3(256), 0, s, T, iv, g0, n, seq);
+  cudaError_t le__ = ctas_per_sm >= 8 ? launch_pdl(k_app_stamp<256>, dim3(grid), dim3(256), 0, s, T, iv, g0, n, seq)
+                                      : launch_pdl(k_app_stamp<128>, dim3(grid), dim3(128), 0, s, T, iv, g0, n, seq);
   if (le__) return le__;
   return cudaGetLastError();
 }

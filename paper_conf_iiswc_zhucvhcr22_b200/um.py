@@ -21,6 +21,7 @@ UM_ACC_READ, UM_ACC_WRITE = 1, 2
 UM_ST_U, UM_ST_H, UM_ST_HD, UM_ST_G, UM_ST_GE, UM_ST_GL = range(6)
 ST_NAMES = ("U", "H", "HD", "G", "GE", "GL")
 UM_F_DISCARD_OFF, UM_F_COPY_CE, UM_F_CHECK, UM_F_APP_STAMP, UM_F_TIMING, UM_F_COPY_KERNEL = 1, 2, 4, 8, 16, 32
+UM_F_OVERLAP = 64
 UM_NONE = 0xFFFFFFFF
 
 
@@ -76,6 +77,7 @@ def lib():
             "um_host_write": [P, U64, U64, P],
             "um_block_table": [P, C.POINTER(P)],
             "um_stream": [P, C.POINTER(P)],
+            "um_join": [P, P],
             "um_get_stats": [P, C.POINTER(um_stats)],
             "um_dump": [P, P, P, C.POINTER(U32), P, C.POINTER(U32)],
             "um_content_tags": [P, P],
@@ -93,7 +95,7 @@ def lib():
 
 EXPORTS = ("um_workspace_size", "um_arena_create", "um_arena_destroy", "um_alloc", "um_prefetch", "um_discard",
            "um_discard_lazy", "um_touch_batch", "um_evict", "um_host_write", "um_block_table", "um_stream",
-           "um_get_stats", "um_dump", "um_content_tags", "um_timing", "um_strerror")
+           "um_join", "um_get_stats", "um_dump", "um_content_tags", "um_timing", "um_strerror")
 
 
 def _ck(fn, st):
@@ -158,6 +160,12 @@ def um_block_table(a) -> int:
     p = C.c_void_p()
     _ck("um_block_table", lib().um_block_table(a, C.byref(p)))
     return p.value
+
+
+def um_join(a, stream=None) -> None:
+    """Make `stream` (default: the arena's paging stream) wait for all enqueued work,
+    including UM_F_OVERLAP application kernels."""
+    _ck("um_join", lib().um_join(a, stream if stream is not None else um_stream(a)))
 
 
 def um_stream(a) -> int:

@@ -25,15 +25,18 @@ def _cuda():
 COPY_FLAGS = {"auto": 0, "kernel": 32, "ce": 2}   # UM_F_COPY_KERNEL / UM_F_COPY_CE
 
 
-def _gpu(trace, mode, copy="auto", **kw):
+def _gpu(trace, mode, copy="auto", overlap=False, **kw):
     from paper_conf_iiswc_zhucvhcr22_b200 import harness, um
-    flags = um.UM_F_APP_STAMP | um.UM_F_CHECK | COPY_FLAGS[copy]
+    flags = um.UM_F_APP_STAMP | um.UM_F_CHECK | COPY_FLAGS[copy] | (um.UM_F_OVERLAP if overlap else 0)
     return harness.run_trace(trace, mode, flags=flags, **kw)
 
 
-def assert_parity(trace, mode, g=None):
-    g = g if g is not None else _gpu(trace, mode)
-    o = oracle_replay(trace, mode).dump()
+OVERLAP_W = 2   # kOverlapW in csrc/um_internal.h (reading R7)
+
+
+def assert_parity(trace, mode, g=None, overlap=False):
+    g = g if g is not None else _gpu(trace, mode, overlap=overlap)
+    o = oracle_replay(trace, mode, overlap=OVERLAP_W if overlap else 0).dump()
     st_g = np.asarray(g["st"])
     st_o = np.asarray(o["st"])
     bad = np.nonzero(st_g != st_o)[0]
@@ -52,7 +55,9 @@ def assert_parity(trace, mode, g=None):
 def test_scenarios(name):
     sc = SCEN[name]
     trace, mode = scn.build(sc)
-    g, _ = assert_parity(trace, mode)
+    ov = sc.get("overlap", 0)
+    assert ov in (0, OVERLAP_W)
+    g, _ = assert_parity(trace, mode, overlap=bool(ov))
     for k, v in sc["expect"]["stats"].items():
         assert g["stats"][k] == v, k
     assert [scn.ST[x] for x in sc["expect"]["st"]] == list(g["st"])
@@ -286,3 +291,42 @@ def test_device_intake_wide(mode):
     t = tg.gen_random(7, block_bytes=4 << 10, arena_bytes=64 << 20, budget_bytes=24 << 20, n_ops=120,
                       max_ranges=1500, max_blocks=32, zipf_s=0.6)
     assert_parity(t, mode)
+
+
+# ------------------------------------------------------------------ R7: pipelined app kernels
+@pytest.mark.parametrize("seed", range(8))
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_overlap_small_random(seed, mode):
+    """UM_F_OVERLAP (reading R7): app kernels on their own stream, victim
+    selection skipping the last 2 GPU sub-ops' blocks; bit-exact against the oracle's
+    window rule, contents included (a hazard would show as a wrong content tag)."""
+    rng = np.random.default_rng(100 + seed)
+    nb, nf = int(rng.integers(2, 24)), int(rng.integers(1, 6))
+    t = tg.gen_small(100 + seed, nblocks=nb, nframes=nf, n_ops=300, max_ranges=4, max_blocks=6)
+    assert_parity(t, mode, overlap=True)
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_overlap_c1(mode):
+    assert_parity(tg.gen_c1(4), mode, overlap=True)
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_overlap_c3_small(mode):
+    """C3 with pipelined app kernels through every transfer path."""
+    t = tg.gen_c3(block_bytes=64 << 10, budget_bytes=192 << 20, iterations=2, workspace_bytes=4 << 20,
+                  layers=tg.scale_layers(tg.VGG16, 1.0 / 512, 1.0 / 64), batch=8)
+    for copy in ("auto", "kernel", "ce"):
+        assert_parity(t, mode, _gpu(t, mode, copy=copy, overlap=True), overlap=True)
+
+
+@pytest.mark.parametrize("mode", ["eager", "lazy"])
+def test_overlap_device_intake(mode):
+    """Unsorted batches (device intake rewrites the interval list: waits for app kernels)
+    and staged interval lists (stager fences) with pipelined app kernels."""
+    t = tg.gen_random(3, block_bytes=64 << 10, arena_bytes=32 << 20, budget_bytes=4 << 20, n_ops=400,
+                      max_ranges=200, max_blocks=8, zipf_s=0.8)
+    assert_parity(t, mode, overlap=True)
+    t = tg.gen_random(7, block_bytes=4 << 10, arena_bytes=64 << 20, budget_bytes=24 << 20, n_ops=120,
+                      max_ranges=1500, max_blocks=32, zipf_s=0.6)
+    assert_parity(t, mode, overlap=True)
