@@ -358,7 +358,8 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
                      discarded frames (victim scan + apply)
     Planning kernels are timed apart from the zero-fill (um_timing spans, CUDA events on
     the paging stream).  Algorithmic bytes per unit:
-      classify  per block 9 (interval record) + 4 sk rd + 4 pin wr + 8 USED slot;
+      classify  per block 4 (fault-list entry: the batch's runs average 2 blocks, so the
+                host stages it as one u32 per block) + 4 sk rd + 4 pin wr + 8 USED slot;
                 per need item + 9 (need, needk, needhf); per revive + 12 (frame_of rd,
                 sk wr, map wr); per H block + 4 (hframe rd)
       victims   per victim 12 (ring entry + sk) + 42 (apply: lists, sk/frame_of/map/hframe)
@@ -411,7 +412,7 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
 
         def cls_bytes(d):
             need = d["faults"] - d["remaps"]
-            return n * (9 + 4 + 4 + 8) + need * 9 + d["remaps"] * 12 + (d["h2d_bytes"] // B) * 4
+            return n * (4 + 4 + 4 + 8) + need * 9 + d["remaps"] * 12 + (d["h2d_bytes"] // B) * 4
         touch_bytes = cls_bytes(d0)
         pres_bytes = cls_bytes(d2) + d2["evictions"] * (12 + 42)
         dir_bytes = n * (4 + 8) + g_in * 8

@@ -722,6 +722,24 @@ static um_status run_gpu_op(um_arena* a, int touch) {
       acc += a->ivs[j].cnt;
     }
     iv.ipre[m] = acc;
+  } else if (total <= 3ull * m) {
+    // sparse batch (intervals average <= 3 blocks, e.g. a fault buffer of scattered
+    // pages): stage the distinct blocks themselves, bit 31 = write (argument marshalling;
+    // <= 12 B per interval against 9 B + the tile table, and the kernels then need no
+    // interval lookup)
+    const uint64_t bytes = 4ull * total;
+    uint64_t off;
+    CK(a->stage.reserve(bytes, &off));
+    iv_off = off;
+    iv_bytes = (bytes + 15) & ~15ull;
+    uint32_t* hb = (uint32_t*)(a->stage.host + off);
+    uint64_t g = 0;
+    for (uint32_t j = 0; j < m; ++j) {
+      const uint32_t wbit = a->ivs[j].w ? 0x80000000u : 0u;
+      for (uint32_t x = 0; x < a->ivs[j].cnt; ++x) hb[g++] = (a->ivs[j].lo + x) | wbit;
+    }
+    CK(a->stage.push(off, iv_bytes, a->ps));
+    iv.blist = (const uint32_t*)(a->stage.dev + off);
   } else {
     // stage lo[m], pre[m+1], w[m] through the pinned ring
     const uint64_t bytes_lo = 4ull * m, bytes_pre = 4ull * (m + 1), bytes_w = m;
@@ -764,7 +782,7 @@ static um_status run_gpu_op(um_arena* a, int touch) {
       a->T.pfloor = seq;
     }
     uint64_t tj_off = 0, tj_bytes = 0;
-    if (!iv.inl) {
+    if (!iv.inl && !iv.blist) {
       // per tile of this sub-op, the interval slice its items fall in: an index the
       // kernels would otherwise find by a dependent binary search over the staged list
       const uint32_t tile = n <= kSmallPlan ? kSmallPlan : classify_tile();

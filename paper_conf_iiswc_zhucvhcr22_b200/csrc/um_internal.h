@@ -116,6 +116,10 @@ struct OpIv {
   const uint32_t* lo;
   const uint32_t* pre;
   const uint8_t* wflag;
+  const uint32_t* blist; // "fault list" form (staged; null otherwise): the op's distinct blocks
+                         // in ascending order, one u32 per block, bit 31 = UM_ACC_WRITE.
+                         // Chosen by the host when intervals average <= 3 blocks (a sparse
+                         // batch): item g's block is one coalesced load, no interval lookup
   const uint32_t* tj;   // staged lists: per tile of the current sub-op, the interval slice
                         // [tj[2t], tj[2t+1]] its items fall in (host-computed, no search)
   uint32_t m;

@@ -389,19 +389,23 @@ __device__ __forceinline__ void classify_single(const Tables& T, const OpIv& iv,
   __shared__ uint32_t s_lo[TILE], s_pre[TILE + 1];
   __shared__ uint32_t s_j0, s_m;
   const int w = threadIdx.x >> 5;
-  if (threadIdx.x == 0) {
-    const uint32_t ja = iv.inl ? iv_find(iv, g0) : iv.tj[0];
-    const uint32_t jb = iv.inl ? iv_find(iv, g0 + n - 1) : iv.tj[1];
-    s_j0 = ja;
-    s_m = jb - ja + 1;
+  const bool list = iv.blist != nullptr;   // uniform: fault-list form, no interval lookup
+  if (!list) {
+    if (threadIdx.x == 0) {
+      const uint32_t ja = iv.inl ? iv_find(iv, g0) : iv.tj[0];
+      const uint32_t jb = iv.inl ? iv_find(iv, g0 + n - 1) : iv.tj[1];
+      s_j0 = ja;
+      s_m = jb - ja + 1;
+    }
+    __syncthreads();
+    const uint32_t j0 = s_j0, m = s_m;
+    for (uint32_t q = threadIdx.x; q <= m; q += blockDim.x) {
+      if (q < m) s_lo[q] = iv_lo(iv, j0 + q);
+      s_pre[q] = iv_pre(iv, j0 + q);
+    }
+    __syncthreads();
   }
-  __syncthreads();
-  const uint32_t j0 = s_j0, m = s_m;
-  for (uint32_t q = threadIdx.x; q <= m; q += blockDim.x) {
-    if (q < m) s_lo[q] = iv_lo(iv, j0 + q);
-    s_pre[q] = iv_pre(iv, j0 + q);
-  }
-  __syncthreads();
+  const uint32_t m = list ? 0u : s_m;
   const unsigned long long kseq = (unsigned long long)seq << 32;
   uint32_t b[IPT];
   uint8_t s[IPT];
@@ -415,13 +419,17 @@ __device__ __forceinline__ void classify_single(const Tables& T, const OpIv& iv,
     s[k] = 0xff;
     if (idx < n) {
       const uint32_t g = g0 + idx;
-      uint32_t lo = jlo, hi = m;  // largest j with s_pre[j] <= g (items ascend per thread)
-      while (hi - lo > 1) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (s_pre[mid] <= g) lo = mid; else hi = mid;
+      if (list) {
+        b[k] = iv.blist[g] & 0x7fffffffu;
+      } else {
+        uint32_t lo = jlo, hi = m;  // largest j with s_pre[j] <= g (items ascend per thread)
+        while (hi - lo > 1) {
+          const uint32_t mid = (lo + hi) >> 1;
+          if (s_pre[mid] <= g) lo = mid; else hi = mid;
+        }
+        jlo = lo;
+        b[k] = s_lo[lo] + (g - s_pre[lo]);
       }
-      jlo = lo;
-      b[k] = s_lo[lo] + (g - s_pre[lo]);
       s[k] = ld_st(T, b[k]);   // all state loads before any store (stores could alias them)
     }
   }
@@ -552,7 +560,7 @@ __device__ bool grid_finish(const Tables& T, const int (&slots)[NC], const long 
   return true;
 }
 
-template <int IPT>
+template <int IPT, bool LIST>
 __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
                                               int touch, unsigned long long tail0, int npar) {
   constexpr int TPB = kStTPB, TILE = TPB * IPT, NW = TPB / 32, NWORD = TILE / 32;
@@ -569,79 +577,88 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
   __shared__ uint32_t s_off[IPT * NW + 1];
   __shared__ uint32_t s_cnt[8];
   const uint32_t tile = blockIdx.x, tbase = tile * TILE, gt = g0 + tbase;
-  const uint32_t ja = iv.inl ? iv_find(iv, gt) : iv.tj[2 * tile];
-  const uint32_t jb = iv.inl ? iv_find(iv, g0 + min(n, tbase + TILE) - 1) : iv.tj[2 * tile + 1];
-  const uint32_t m = jb - ja + 1;   // <= TILE (every slice interval holds an item of the tile)
-  uint32_t qlo[IPT], qpre[IPT];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t b[IPT];
+  if constexpr (LIST) {
+    // fault-list form: one coalesced load per item, no interval slice, no barrier
 #pragma unroll
-  for (int r = 0; r < IPT; ++r) {
-    const uint32_t q = r * TPB + threadIdx.x;
-    if (q < m) {
-      qlo[r] = iv_lo(iv, ja + q);
-      qpre[r] = iv_pre(iv, ja + q);
+    for (int k = 0; k < IPT; ++k) {
+      const uint32_t idx = tbase + k * TPB + threadIdx.x;
+      b[k] = idx < n ? iv.blist[g0 + idx] & 0x7fffffffu : 0u;
     }
-  }
-  for (int i = threadIdx.x; i < NWORD; i += TPB) s_bits[i] = 0u;
-  __syncthreads();
+  } else {
+    const uint32_t ja = iv.inl ? iv_find(iv, gt) : iv.tj[2 * tile];
+    const uint32_t jb = iv.inl ? iv_find(iv, g0 + min(n, tbase + TILE) - 1) : iv.tj[2 * tile + 1];
+    const uint32_t m = jb - ja + 1;   // <= TILE (every slice interval holds an item of the tile)
+    uint32_t qlo[IPT], qpre[IPT];
 #pragma unroll
-  for (int r = 0; r < IPT; ++r) {
-    const uint32_t q = r * TPB + threadIdx.x;
-    if (q < m) {
-      s_d[q] = qlo[r] - qpre[r];
-      if (q) {
-        const uint32_t pos = qpre[r] - gt;   // in (0, TILE)
-        atomicOr(&s_bits[pos >> 5], 1u << (pos & 31));
+    for (int r = 0; r < IPT; ++r) {
+      const uint32_t q = r * TPB + threadIdx.x;
+      if (q < m) {
+        qlo[r] = iv_lo(iv, ja + q);
+        qpre[r] = iv_pre(iv, ja + q);
       }
     }
+    for (int i = threadIdx.x; i < NWORD; i += TPB) s_bits[i] = 0u;
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < IPT; ++r) {
+      const uint32_t q = r * TPB + threadIdx.x;
+      if (q < m) {
+        s_d[q] = qlo[r] - qpre[r];
+        if (q) {
+          const uint32_t pos = qpre[r] - gt;   // in (0, TILE)
+          atomicOr(&s_bits[pos >> 5], 1u << (pos & 31));
+        }
+      }
+    }
+    __syncthreads();
+    if (PERL > 1 && w == 0) {
+      // one warp: exclusive prefix of the word popcounts (PERL consecutive words per lane)
+      uint32_t c[PERL], sum = 0;
+#pragma unroll
+      for (int i = 0; i < PERL; ++i) {
+        c[i] = lane * PERL + i < NWORD ? __popc(s_bits[lane * PERL + i]) : 0u;
+        sum += c[i];
+      }
+      uint32_t x = sum;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += y;
+      }
+      x -= sum;
+#pragma unroll
+      for (int i = 0; i < PERL; ++i) {
+        if (lane * PERL + i < NWORD) s_wpre[lane * PERL + i] = x;
+        x += c[i];
+      }
+    }
+    if (PERL > 1) __syncthreads();
+    uint32_t wexcl = 0;   // PERL == 1: lane l holds the set bits in words [0, l)
+    if (PERL == 1) {
+      const uint32_t c = lane < NWORD ? __popc(s_bits[lane]) : 0u;
+      uint32_t x = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += y;
+      }
+      wexcl = x - c;
+    }
+    const unsigned le = lanemask_lt() | (1u << lane);
+#pragma unroll
+    for (int k = 0; k < IPT; ++k) {
+      const uint32_t idx = tbase + k * TPB + threadIdx.x;
+      const int wi = k * NW + w;   // bitmap word of item (k, thread): in-tile position k*TPB + tid
+      const uint32_t wp = PERL == 1 ? __shfl_sync(FULL, wexcl, wi & 31) : s_wpre[wi];
+      const uint32_t j = wp + __popc(s_bits[wi] & le);
+      b[k] = g0 + idx + s_d[j];
+    }
   }
-  __syncthreads();
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  if (PERL > 1 && w == 0) {
-    // one warp: exclusive prefix of the word popcounts (PERL consecutive words per lane)
-    uint32_t c[PERL], sum = 0;
-#pragma unroll
-    for (int i = 0; i < PERL; ++i) {
-      c[i] = lane * PERL + i < NWORD ? __popc(s_bits[lane * PERL + i]) : 0u;
-      sum += c[i];
-    }
-    uint32_t x = sum;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL, x, o);
-      if (lane >= o) x += y;
-    }
-    x -= sum;
-#pragma unroll
-    for (int i = 0; i < PERL; ++i) {
-      if (lane * PERL + i < NWORD) s_wpre[lane * PERL + i] = x;
-      x += c[i];
-    }
-  }
-  if (PERL > 1) __syncthreads();
-  uint32_t wexcl = 0;   // PERL == 1: lane l holds the set bits in words [0, l)
-  if (PERL == 1) {
-    const uint32_t c = lane < NWORD ? __popc(s_bits[lane]) : 0u;
-    uint32_t x = c;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL, x, o);
-      if (lane >= o) x += y;
-    }
-    wexcl = x - c;
-  }
-  const unsigned le = lanemask_lt() | (1u << lane);
   const unsigned long long kseq = (unsigned long long)seq << 32;
-  uint32_t b[IPT];
   uint8_t s[IPT];
   uint32_t cls = 0;   // per-class counts (<= IPT < 32 each), 5 bits per class U H HD G GE GL
-#pragma unroll
-  for (int k = 0; k < IPT; ++k) {
-    const uint32_t idx = tbase + k * TPB + threadIdx.x;
-    const int wi = k * NW + w;   // bitmap word of item (k, thread): in-tile position k*TPB + tid
-    const uint32_t wp = PERL == 1 ? __shfl_sync(FULL, wexcl, wi & 31) : s_wpre[wi];
-    const uint32_t j = wp + __popc(s_bits[wi] & le);
-    b[k] = g0 + idx + s_d[j];
-  }
 #pragma unroll
   for (int k = 0; k < IPT; ++k) {
     const uint32_t idx = tbase + k * TPB + threadIdx.x;
@@ -712,11 +729,12 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
 
 // 4 items per thread, 8 CTAs/SM (A/B on B200: 8 items per thread at 6 CTAs/SM spills and
 // runs the 2^21-block touch in 42 vs 30 us)
+template <bool LIST>
 __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
                                                         uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
                                                         int npar) {
   pdl_enter();
-  classify_body<4>(T, iv, g0, n, seq, touch, tail0, npar);
+  classify_body<4, LIST>(T, iv, g0, n, seq, touch, tail0, npar);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1560,10 +1578,18 @@ __global__ void __launch_bounds__(TPB) k_app_stamp(Tables T, const __grid_consta
   for (unsigned long long u = blockIdx.x; u < units; u += gridDim.x) {
     if (threadIdx.x == 0) {
       uint32_t g = g0 + (uint32_t)(u / spb);
-      uint32_t j = iv_find(iv, g);
       char* d = nullptr;
-      uint32_t bb = iv_lo(iv, j) + (g - iv_pre(iv, j));
-      if (iv_w(iv, j)) {
+      uint32_t bb, wr;
+      if (iv.blist) {
+        const uint32_t e = iv.blist[g];
+        bb = e & 0x7fffffffu;
+        wr = e >> 31;
+      } else {
+        const uint32_t j = iv_find(iv, g);
+        bb = iv_lo(iv, j) + (g - iv_pre(iv, j));
+        wr = iv_w(iv, j);
+      }
+      if (wr) {
         uint32_t fr = T.frame_of[bb];
         if (fr != UM_NONE) d = T.frames + (size_t)fr * T.B + (size_t)(u % spb) * SEG;
       }
@@ -1989,7 +2015,7 @@ cudaError_t setup_kernels() {
   bool carve = false;   // measured: no effect on the C1 small-op rate (B200, r01)
   if (const char* v = getenv("UM_CARVEOUT")) carve = atoi(v) != 0;
   if (carve) {
-    const void* ks[] = {(const void*)k_classify, (const void*)k_victims, (const void*)k_plan_small,
+    const void* ks[] = {(const void*)k_classify<false>, (const void*)k_classify<true>, (const void*)k_victims, (const void*)k_plan_small,
                         (const void*)k_victims_scan, (const void*)k_victims_apply, (const void*)k_service,
                         (const void*)k_app_stamp<256>, (const void*)k_app_stamp<128>, (const void*)k_directive, (const void*)k_ring_compact,
                         (const void*)k_plan_commit, (const void*)k_zero_items, (const void*)k_mark,
@@ -2045,7 +2071,8 @@ uint32_t classify_tile() { return (uint32_t)kStTPB * 4u; }
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
                             unsigned long long tail0, int npar, cudaStream_t s) {
   unsigned nt = n ? ceil_div(n, classify_tile()) : 1;
-  cudaError_t le__ = launch_pdl(k_classify, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar);
+  cudaError_t le__ = iv.blist ? launch_pdl(k_classify<true>, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar)
+                              : launch_pdl(k_classify<false>, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar);
   if (le__) return le__;
   return cudaGetLastError();
 }

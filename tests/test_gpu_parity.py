@@ -330,3 +330,16 @@ def test_overlap_device_intake(mode):
     t = tg.gen_random(7, block_bytes=4 << 10, arena_bytes=64 << 20, budget_bytes=24 << 20, n_ops=120,
                       max_ranges=1500, max_blocks=32, zipf_s=0.6)
     assert_parity(t, mode, overlap=True)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_sparse_fault_list(seed, mode):
+    """Sparse sorted fault batches (the state microbench's shape at test size): the host
+    stages them in the fault-list form (one u32 per block, bit 31 = write); batches span
+    many classify tiles, the wide victim scan and several sub-ops."""
+    t = tg.gen_sparse(seed)
+    assert_parity(t, mode)
+    if seed == 0:
+        assert_parity(t, mode, _gpu(t, mode, copy="ce"))
+        assert_parity(t, mode, overlap=True)

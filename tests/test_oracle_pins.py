@@ -189,3 +189,21 @@ def test_c4_closed_form(nb, p, pressure, mode):
         assert s["remaps"] == s["revalidations"] == 0
         assert s["unmaps"] == nb          # eager: at discard; lazy: at reclaim (§5.6)
         assert s["evictions"] == nb + k
+
+
+def test_sparse_trace_shape():
+    """gen_sparse must produce what the fault-list path needs (sorted, disjoint batches
+    of more than kIvInline = 24 records whose merged runs average <= 3 blocks), or the
+    GPU test of that path would silently exercise the interval form instead."""
+    t = tg.gen_sparse(0)
+    B = t.block_bytes
+    seen = 0
+    for (op, _fl, _off, _ln, accs) in t.iter_ops():
+        if op != tg.OP_TOUCH:
+            continue
+        lo = [a // B for (a, _l, _k) in accs]
+        assert lo == sorted(set(lo)) and len(lo) > 24
+        runs = 1 + sum(1 for x, y in zip(lo, lo[1:]) if y != x + 1)
+        assert len(lo) <= 3 * runs
+        seen += 1
+    assert seen >= 5

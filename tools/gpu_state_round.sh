@@ -13,4 +13,4 @@ for l in open("gpurun_out/state_bench.json"):
         print(l[:300]); continue
     print({k: (round(v["ms"] * 1000, 2), round(v["frac"], 3)) for k, v in d.items() if isinstance(v, dict)})
 PY
-[ -n "$TAG" ] && bash tools/ncu_state_micro.sh
+if [ -n "$TAG" ]; then bash tools/ncu_state_micro.sh; fi
