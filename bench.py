@@ -403,6 +403,19 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
             t = um.um_timing(h, reset=True)
             s1 = um.um_get_stats(h)
             return t, {k: s1[k] - s0[k] for k in s1}
+        # floor of the measurement: two events around one empty torch kernel on the same
+        # stream, behind the same device sleep (launch + event overhead, no work)
+        z = torch.zeros(1, device=mem.frames.device)
+        floor = []
+        for _ in range(3):
+            gate()
+            f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            with torch.cuda.stream(ps):
+                f0.record(ps)
+                z.add_(1)
+                f1.record(ps)
+            f1.synchronize()
+            floor.append(f0.elapsed_time(f1))
         t_touch, d0 = timed(lambda: um.um_touch_batch(h, acc0))
         t_disc, d1 = timed(lambda: um.um_discard(h, 0, n * B))
         t_pres, d2 = timed(lambda: um.um_touch_batch(h, acc1))
@@ -430,6 +443,7 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
                                           {"victims": d2["evictions"], "remaps": d2["remaps"]}),
                 "zero_fill_gbs": (n * B) / (t_touch["ms_xfer"] / 1e3) / 1e9 if t_touch["ms_xfer"] else None,
                 "peak_source": peak_src, "nblocks": nb, "nframes": budget // B,
+                "empty_kernel_span_us": min(floor) * 1e3,
                 "timing": "CUDA events around each op's planning launches on the paging stream; every launch "
                           "queued behind a device sleep; L2 cold (the previous op's zero-fill flushes it)"}
     finally:
