@@ -189,6 +189,51 @@ def run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=None, flags_extr
         arena.close()
 
 
+def c2_stream(torch, um, harness, mem, budget, pool_bytes):
+    """C2 streaming producer/consumer (BASELINE.json configs[1]):
+    2x oversubscription, 2 MiB blocks, chunks of 1 GiB, P = 2 passes, discard after
+    consume; F is the largest frame count whose host-resident half fits the pinned pool
+    this run already holds (the full-size F = 81,920 needs a 160 GiB pool).  One pass-pair
+    per mode on the same memory; checks the closed form."""
+    import tracegen as tg
+    B, c, P = mem.B, 512, 2
+    F = min(budget // B, (pool_bytes - 2 * GiB) // B) // 256 * 256
+    t = tg.gen_c2(F, c, P, block_bytes=B)
+    out = {"F": F, "buffer_gib": 2 * F * B / GiB, "budget_gib": F * B / GiB, "chunk_blocks": c, "passes": P,
+           "full_size_F": 81920}
+    ws_need = um.um_workspace_size(mem.config(t.arena_bytes, t.budget_bytes, 0))
+    assert ws_need <= mem.workspace.numel()
+    for mode in ("base", "eager", "lazy"):
+        arena = harness.make_arena(t, mode, mem=mem, flags=um.UM_F_APP_STAMP)
+        try:
+            harness.alloc_buffers(arena, t)
+            ps = torch.cuda.ExternalStream(arena.stream_ptr)
+            um.um_get_stats(arena.handle)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(ps)
+            harness.issue(arena, t, mode)
+            e1.record(ps)
+            e1.synchronize()
+            st = um.um_get_stats(arena.handle)
+            ms = e0.elapsed_time(e1)
+            link = st["h2d_bytes"] + st["d2h_bytes"]
+            out[mode] = {"ms": ms, "h2d_gb": st["h2d_bytes"] / 1e9, "d2h_gb": st["d2h_bytes"] / 1e9,
+                         "zf_gb": st["zf_bytes"] / 1e9,
+                         "serviced_gbs": (link + st["zf_bytes"]) / (ms / 1e3) / 1e9,
+                         "link_gbs": link / (ms / 1e3) / 1e9}
+            if mode == "base":
+                out[mode]["closed_form_ok"] = (st["h2d_bytes"], st["d2h_bytes"], st["zf_bytes"]) == (
+                    2 * (P - 1) * F * B, (2 * P - 1) * F * B, 2 * F * B)
+            else:
+                out[mode]["closed_form_ok"] = (st["h2d_bytes"], st["d2h_bytes"], st["zf_bytes"]) == (0, 0, 2 * P * F * B)
+        finally:
+            arena.close()
+    out["avoided_gb"] = (out["base"]["h2d_gb"] + out["base"]["d2h_gb"]) - (out["eager"]["h2d_gb"] + out["eager"]["d2h_gb"])
+    out["avoided_closed_form_gb"] = (4 * P - 3) * F * B / 1e9
+    out["speedup_eager_vs_base"] = out["base"]["ms"] / out["eager"]["ms"]
+    return out
+
+
 def run_e2e(torch, um, harness, mem, trace, W, K, flags_extra=0):
     """End to end through the public API: the trace WITH the host-side data generation
     (prefetch(data,HOST); host_write; prefetch(data,GPU): the step's inputs cross
@@ -561,6 +606,7 @@ def main_ours(args):
         state_bench(torch, um, mem, budget, arena_bytes, seed=1)
         state = state_bench(torch, um, mem, budget, arena_bytes, seed=0)
         state["reps"] = "second of two runs (first = warm-up)"
+    c2 = None if args.no_compare else c2_stream(torch, um, harness, mem, budget, host_pool)
     e2e_s = None
     if not args.no_e2e:
         e2e_s = run_e2e(torch, um, harness, mem, trace, 1, min(K, 3), flags_extra=ovf)
@@ -633,6 +679,7 @@ def main_ours(args):
         "roofline_state": state,
         "c1_directives": c1,
         "c4_sweep": c4,
+        "c2_streaming": c2,
         "clocks": head["clocks"],
         "gpu_launches": tm["launches"],
         "stats_per_iter_all_ranks": stats_all,
