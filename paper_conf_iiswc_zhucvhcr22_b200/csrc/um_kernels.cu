@@ -575,7 +575,7 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
   __shared__ uint32_t s_wpre[NWORD];
   __shared__ uint32_t s_base;
   __shared__ uint32_t s_off[IPT * NW + 1];
-  __shared__ uint32_t s_cnt[8];
+  __shared__ uint32_t s_cnt[2 * NW];
   const uint32_t tile = blockIdx.x, tbase = tile * TILE, gt = g0 + tbase;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   uint32_t b[IPT];
@@ -708,23 +708,44 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
       T.sk[bb] = mk_sk(ST_G, seq);   // refresh (G) / revalidate (GL -> G, L190)
     }
   }
-  // counters (classes: U H HD G GE GL)
-  const long long B = T.B;
-  const uint32_t c0 = cls & 31u, c1 = (cls >> 5) & 31u, c2 = (cls >> 10) & 31u, c3 = (cls >> 15) & 31u,
-                 c4 = (cls >> 20) & 31u, c5 = (cls >> 25) & 31u;
-  uint32_t v[6];
-  if (touch) {
-    // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE
-    v[0] = c0 + c1 + c2 + c4; v[1] = c3 + c5; v[2] = c4;
-  } else {
-    v[0] = c3; v[1] = c4; v[2] = c5;   // refreshes, remaps, revalidations
+  // counters (classes: U H HD G GE GL).  A thread's class counts (<= IPT each) are
+  // repacked 8 bits per class into two words and warp-summed (<= 32 * IPT = 128 per
+  // class); thread 0 sums the warps' words from shared memory and adds the counters:
+  // two reductions and one barrier instead of one reduction per counter
+  static_assert(32 * IPT < 256, "8-bit class lanes");
+  const uint32_t lo4 = (cls & 31u) | (((cls >> 5) & 31u) << 8) | (((cls >> 10) & 31u) << 16) |
+                       (((cls >> 15) & 31u) << 24);
+  const uint32_t hi2 = ((cls >> 20) & 31u) | (((cls >> 25) & 31u) << 8);
+  const uint32_t wl = __reduce_add_sync(FULL, lo4), wh = __reduce_add_sync(FULL, hi2);
+  if (lane == 0) {
+    s_cnt[w] = wl;          // s_cnt: 2 * NW words
+    s_cnt[NW + w] = wh;
   }
-  v[3] = c1; v[4] = c0 + c2; v[5] = c2;   // h2d, zf, h2d_avoided
-  const int slots_t[6] = {S_FAULTS, S_HITS, S_REMAPS, S_H2D, S_ZF, S_H2D_AV};
-  const int slots_p[6] = {S_REFRESH, S_REMAPS, S_REVAL, S_H2D, S_ZF, S_H2D_AV};
-  const long long mul[6] = {1, 1, 1, B, B, B};
-  block_counts_to<6>(T, v, s_cnt, touch ? slots_t : slots_p, mul);
-  if (blockIdx.x == 0 && threadIdx.x == 0) T.ctl->n_rekey = n;   // USED slots appended
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0, c4 = 0, c5 = 0;
+#pragma unroll
+    for (int i = 0; i < NW; ++i) {
+      const uint32_t a = s_cnt[i], e = s_cnt[NW + i];
+      c0 += a & 255u; c1 += (a >> 8) & 255u; c2 += (a >> 16) & 255u; c3 += a >> 24;
+      c4 += e & 255u; c5 += e >> 8;
+    }
+    const long long B = T.B;
+    if (touch) {
+      // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE
+      stat_add(T, S_FAULTS, c0 + c1 + c2 + c4);
+      stat_add(T, S_HITS, c3 + c5);
+      stat_add(T, S_REMAPS, c4);
+    } else {
+      stat_add(T, S_REFRESH, c3);   // refreshes, remaps, revalidations
+      stat_add(T, S_REMAPS, c4);
+      stat_add(T, S_REVAL, c5);
+    }
+    stat_add(T, S_H2D, (long long)c1 * B);          // h2d, zf, h2d_avoided
+    stat_add(T, S_ZF, (long long)(c0 + c2) * B);
+    stat_add(T, S_H2D_AV, (long long)c2 * B);
+    if (blockIdx.x == 0) T.ctl->n_rekey = n;   // USED slots appended
+  }
 }
 
 // 4 items per thread, 8 CTAs/SM (A/B on B200: 8 items per thread at 6 CTAs/SM spills and
