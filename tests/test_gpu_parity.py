@@ -343,3 +343,29 @@ def test_sparse_fault_list(seed, mode):
     if seed == 0:
         assert_parity(t, mode, _gpu(t, mode, copy="ce"))
         assert_parity(t, mode, overlap=True)
+
+
+def _sorted_batch_trace(runs, nblocks=4096, nframes=700, B=4 << 10, wfrac=0.5, seed=0):
+    """One arena, a few ops whose touch batches are the given lists of (first block,
+    run length) records (ascending, disjoint); W on a seeded subset of records."""
+    rng = np.random.default_rng(seed)
+    tb = tg.TraceBuilder(B, nblocks * B, nframes * B)
+    for batch in runs:
+        tb.touch([(lo * B, n * B, tg.ACC_WRITE if rng.random() < wfrac else tg.ACC_READ) for lo, n in batch])
+        tb.discard(0, (nblocks // 3) * B, lazy_ok=True)
+    return tb.build()
+
+
+@pytest.mark.parametrize("mode", ["eager", "lazy"])
+def test_fault_list_boundaries(mode):
+    """Edges of the staging choice: 24 records (inline), 25 (staged), runs of exactly 3
+    blocks (still the fault-list form) and of 4 (interval form), a list longer than
+    nframes (split into sub-ops inside the list), single-block records with alternating
+    W flags, adjacent single-block records that merge only where W agrees, and a repeat
+    of an earlier batch after a discard of its blocks (revives, revalidations)."""
+    gap = lambda n, run, step, base=0: [(base + i * step, run) for i in range(n)]
+    batches = [gap(24, 1, 3), gap(25, 1, 3), gap(300, 3, 5), gap(300, 4, 6), gap(1500, 1, 2, 1),
+               gap(2000, 1, 2), gap(1000, 1, 1, 2000), gap(25, 1, 3)]
+    t = _sorted_batch_trace(batches)
+    assert_parity(t, mode)
+    assert_parity(t, mode, _gpu(t, mode, copy="kernel"))
