@@ -137,6 +137,7 @@ constexpr int kStTPB = 256;
 // multi-CTA classify: items per thread (4, or 8 with UM_CLS_IPT=8); its tile in items
 uint32_t classify_tile();
 constexpr int kVictTPB = 1024;
+constexpr int kVaTPB = 512;   // k_victims_apply block size
 constexpr int kVictIPT = 4;
 constexpr int kXferStages = 4;
 constexpr uint32_t kXferChunk = 16384;

@@ -1195,9 +1195,11 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
   __threadfence();
 }
 
-__global__ void __launch_bounds__(256) k_victims_apply(Tables T, int evict_mode) {
+// 512-thread CTAs, 2 per SM (62 registers): the same resident warps as 4 x 256 in one
+// wave, and a quarter of the CTAs to dispatch when there is nothing to do (k = 0)
+__global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict_mode) {
   pdl_enter();
-  constexpr int TPB = 256, AIPT = 4, CH = 32 * AIPT;
+  constexpr int TPB = kVaTPB, AIPT = 4, CH = 32 * AIPT;
   __shared__ uint32_t s_cnt[8];
   Ctl* c = T.ctl;
   const uint32_t found = c->n_vict;
@@ -2122,9 +2124,9 @@ cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, u
   cudaError_t e = cudaGetLastError();
   if (e) return e;
   // one warp per pass of <= kVaPass victims (<= max_victims / kVaPass + tiles passes)
-  unsigned grid = ceil_div((unsigned long long)ceil_div(max_victims ? max_victims : 1, kVaPass) + nt, 8);
-  if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
-  le__ = launch_pdl(k_victims_apply, dim3(grid), dim3(256), 0, s, T, evict_mode);
+  unsigned grid = ceil_div((unsigned long long)ceil_div(max_victims ? max_victims : 1, kVaPass) + nt, kVaTPB / 32);
+  if (grid > (unsigned)g_nsm * 2) grid = g_nsm * 2;
+  le__ = launch_pdl(k_victims_apply, dim3(grid), dim3(kVaTPB), 0, s, T, evict_mode);
   if (le__) return le__;
   return cudaGetLastError();
 }
