@@ -722,7 +722,7 @@ static um_status run_gpu_op(um_arena* a, int touch) {
       acc += a->ivs[j].cnt;
     }
     iv.ipre[m] = acc;
-  } else if (total <= 3ull * m) {
+  } else if (total <= 3ull * m && 4ull * total <= a->L.stage_bytes / 2) {
     // sparse batch (intervals average <= 3 blocks, e.g. a fault buffer of scattered
     // pages): stage the distinct blocks themselves, bit 31 = write (argument marshalling;
     // <= 12 B per interval against 9 B + the tile table, and the kernels then need no
