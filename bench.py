@@ -234,6 +234,61 @@ def c2_stream(torch, um, harness, mem, budget, pool_bytes):
     return out
 
 
+class _MemView:
+    """The bench's frames and host pool seen at another block size, with its own
+    workspace (um.Arena needs .B, .frames and .config())."""
+
+    def __init__(self, torch, um, mem, B, arena_bytes, budget):
+        self.B, self.frames, self._mem = B, mem.frames, mem
+        probe = mem.config(arena_bytes, budget, 0)
+        probe.block_bytes = B
+        probe.workspace, probe.workspace_bytes = None, 0
+        self.workspace = torch.empty(um.um_workspace_size(probe), dtype=torch.uint8, device=mem.frames.device)
+
+    def config(self, arena_bytes, budget_bytes, flags):
+        c = self._mem.config(arena_bytes, budget_bytes, flags)
+        c.block_bytes = self.B
+        c.workspace, c.workspace_bytes = self.workspace.data_ptr(), self.workspace.numel()
+        return c
+
+
+def c3_64k(torch, um, harness, mem, budget, arena_bytes):
+    """The C3 64 KiB-block variant (~4.18 M blocks, ~2.79 M frames) on the
+    same frames and host pool: one warm-up and one timed iteration per mode (CUDA
+    events on the paging stream)."""
+    import tracegen as tg
+    B = 64 << 10
+    t = tg.gen_c3(block_bytes=B, budget_bytes=budget, oversub=arena_bytes / budget, iterations=2,
+                  with_host_data=True)
+    view = _MemView(torch, um, mem, B, t.arena_bytes, t.budget_bytes)
+    out = {"block_bytes": B, "nblocks": t.nblocks, "nframes": t.nframes}
+    for mode in ("base", "eager"):
+        arena = harness.make_arena(t, mode, mem=view, flags=um.UM_F_APP_STAMP | um.UM_F_TIMING)
+        try:
+            harness.alloc_buffers(arena, t)
+            bounds = harness.iteration_bounds(t)
+            ps = torch.cuda.ExternalStream(arena.stream_ptr)
+            harness.issue(arena, t, mode, *bounds[0])
+            s0 = um.um_get_stats(arena.handle)
+            um.um_timing(arena.handle, reset=True)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(ps)
+            harness.issue(arena, t, mode, *bounds[1])
+            e1.record(ps)
+            e1.synchronize()
+            s1 = um.um_get_stats(arena.handle)
+            tm = um.um_timing(arena.handle, reset=True)
+            d = {k: s1[k] - s0[k] for k in s1}
+            out[mode] = {"iter_ms": e0.elapsed_time(e1), "plan_ms": tm["ms_plan"], "xfer_ms": tm["ms_xfer"],
+                         "link_gb": (d["h2d_bytes"] + d["d2h_bytes"]) / 1e9, "zf_gb": d["zf_bytes"] / 1e9}
+        finally:
+            arena.close()
+    out["speedup_vs_discard_off"] = out["base"]["iter_ms"] / out["eager"]["iter_ms"]
+    out["gb_avoided_per_iter"] = out["base"]["link_gb"] - out["eager"]["link_gb"]
+    del view
+    return out
+
+
 def run_e2e(torch, um, harness, mem, trace, W, K, flags_extra=0):
     """End to end through the public API: the trace WITH the host-side data generation
     (prefetch(data,HOST); host_write; prefetch(data,GPU): the step's inputs cross
@@ -607,6 +662,7 @@ def main_ours(args):
         state = state_bench(torch, um, mem, budget, arena_bytes, seed=0)
         state["reps"] = "second of two runs (first = warm-up)"
     c2 = None if args.no_compare else c2_stream(torch, um, harness, mem, budget, host_pool)
+    c3k = None if args.no_compare else c3_64k(torch, um, harness, mem, budget, arena_bytes)
     e2e_s = None
     if not args.no_e2e:
         e2e_s = run_e2e(torch, um, harness, mem, trace, 1, min(K, 3), flags_extra=ovf)
@@ -680,6 +736,7 @@ def main_ours(args):
         "c1_directives": c1,
         "c4_sweep": c4,
         "c2_streaming": c2,
+        "c3_64k_blocks": c3k,
         "clocks": head["clocks"],
         "gpu_launches": tm["launches"],
         "stats_per_iter_all_ranks": stats_all,

@@ -239,15 +239,14 @@ def test_wide_victim_selection(mode):
         assert_parity(t, mode, _gpu(t, mode, copy=copy))
 
 
-def _full_size_trace(iterations=2):
+def _full_size_trace(iterations=2, B=2 << 20):
     import gc
     import torch
     gc.collect()
     torch.cuda.empty_cache()   # the previous full-size test's frames sit in torch's cache
     free, _ = torch.cuda.mem_get_info()
     GiB = 1 << 30
-    B = 2 << 20
-    budget = min(170 * GiB, free - 6 * GiB) // B * B
+    budget = min(170 * GiB, free - 8 * GiB) // (2 << 20) * (2 << 20)
     assert budget >= 160 * GiB, f"only {free / GiB:.1f} GiB free for the full-size case"
     return tg.gen_c3(block_bytes=B, budget_bytes=budget, oversub=1.5, iterations=iterations)
 
@@ -369,3 +368,15 @@ def test_fault_list_boundaries(mode):
     t = _sorted_batch_trace(batches)
     assert_parity(t, mode)
     assert_parity(t, mode, _gpu(t, mode, copy="kernel"))
+
+
+
+def test_c3_full_size_64k_blocks():
+    """The C3 64 KiB-block variant (~4.18 M blocks, ~2.79 M frames) at full
+    size, eager, default transfer selection: two iterations (the trace is periodic after
+    the first) bit-exact against the oracle, contents included."""
+    t = _full_size_trace(iterations=2, B=64 << 10)
+    assert t.nblocks > 4_000_000
+    pool = t.arena_bytes - t.budget_bytes + (2 << 30)
+    g = _gpu(t, "eager", host_pool_bytes=pool)
+    assert_parity(t, "eager", g)
