@@ -547,10 +547,33 @@ static um_status ce_subop(um_arena* a, uint32_t seq, uint32_t n) {
   const uint32_t nn = std::min<uint32_t>(a->hctl->n_need, n);
   const uint64_t G = a->L.ce_group, B = a->B;
   CopyList d2d, wb, h2d, sw;
+  // consecutive groups of zero-fill items only (no copy to order against) share one
+  // zero kernel instead of one launch per group
+  uint32_t zr0 = 0, zr1 = 0;
+  cudaStream_t zst = a->cs[0];
+  auto flush_zero = [&]() -> cudaError_t {
+    if (zr1 <= zr0) return cudaSuccess;
+    cudaError_t e = launch_zero_items(a->T, zr0, zr1, zst);
+    a->n_launch++;
+    zr0 = zr1 = 0;
+    return e;
+  };
   for (uint32_t g0 = 0, gi = 0; g0 < nn; g0 += (uint32_t)G, ++gi) {
     const uint32_t g1 = (uint32_t)std::min<uint64_t>(nn, g0 + G);
     cudaStream_t st = a->cs[gi & 1];
     char* bnc = a->bounce + (gi & 1) * G * B;
+    bool pure = true;
+    for (uint32_t i = g0; i < g1 && pure; ++i) pure = a->hitems[i].flags == XI_ZF;
+    if (pure) {
+      if (zr1 != g0 || zr1 <= zr0) {
+        CK(flush_zero());
+        zr0 = g0;
+        zst = st;
+      }
+      zr1 = g1;
+      continue;
+    }
+    CK(flush_zero());
     d2d.clear(); wb.clear(); h2d.clear(); sw.clear();
     bool anyzf = false;
     uint32_t k = 0;
@@ -576,6 +599,7 @@ static um_status ce_subop(um_arena* a, uint32_t seq, uint32_t n) {
     }
     CK(sw.issue(st));
   }
+  CK(flush_zero());
   for (int i = 0; i < 2; ++i) {
     CK(cudaEventRecord(a->ev_cs[i], a->cs[i]));
     CK(cudaStreamWaitEvent(a->ps, a->ev_cs[i], 0));
