@@ -20,5 +20,10 @@ independently written linked-list formulation on brute-forced inputs, and the
 invariants (i)-(vii) of SURVEY §8(c).  Parity unpinned: the exact byte totals of the
 C3 DNN trace (pinned only by the invariants), contents of GE/GL/HD blocks beyond
 readings A7/A9, all timings.
+
+`oracle.chunks.ChunkOracle` is the two-level model of SURVEY NEXT-1 (2 MiB chunks as the
+residency / eviction unit, page-granular partial discards), pinned in
+tests/test_oracle_chunks.py (hand-derived scenarios, reduction to oracle.sim, page-level
+invariants).  No CUDA path implements it yet.
 """
 from .sim import Oracle, replay, ST_NAMES, stamp  # noqa: F401
