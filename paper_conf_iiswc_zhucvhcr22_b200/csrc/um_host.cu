@@ -254,6 +254,7 @@ struct um_arena {
   // live for the whole kernel, so a full-occupancy grid would keep the paging and
   // zero-fill kernels off the SMs until it ends (UM_APP_CTAS overrides)
   int app_ctas = 1;
+  bool app_serial = false;   // UM_OVERLAP_SERIAL (diagnostic): window rule, app kernel on ps
   struct WinE { uint32_t seq, n; };
   WinE win[kOverlapW] = {};
   int nwin = 0;
@@ -857,7 +858,7 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     }
     a->n_xfer++;
     if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP)) {
-      if (overlap_on(a) && !getenv("UM_OVERLAP_SERIAL")) {   // (diagnostic: window rule only)
+      if (overlap_on(a) && !a->app_serial) {
         // R7: the application kernel runs on its own stream after this sub-op's
         // transfers and overlaps the next sub-ops' planning and transfers
         CK(cudaEventRecord(a->ev_app_in, a->ps));
@@ -999,6 +1000,7 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
     if ((e = cudaEventCreateWithFlags(&a->ev_app_in, cudaEventDisableTiming))) return fail(e);
     if (const char* v = getenv("UM_APP_CTAS")) a->app_ctas = std::max(1, atoi(v));
     if (const char* v = getenv("UM_APP_GRID")) a->app_ctas = -std::max(1, atoi(v));
+    a->app_serial = getenv("UM_OVERLAP_SERIAL") != nullptr;
   }
   if ((e = cudaEventCreateWithFlags(&a->ev_in, cudaEventDisableTiming))) return fail(e);
   if ((e = cudaEventCreateWithFlags(&a->ev_out, cudaEventDisableTiming))) return fail(e);
