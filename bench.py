@@ -656,11 +656,18 @@ def main_ours(args):
     ovl_r, seq_r = (res.get("eager"), other) if ovf else (other, res.get("eager"))
     state = None
     if not args.no_state_bench:
-        # two runs on fresh arenas over the same memory; the second is reported (the first
-        # pays first-touch costs of the workspace pages and kernel images: 47 vs 30 us)
+        # runs on fresh arenas over the same memory: one warm-up (first-touch costs of the
+        # workspace pages and kernel images), then three; per op the run with the median
+        # span is reported (single ~20 us spans vary by +-20 % from run to run)
         state_bench(torch, um, mem, budget, arena_bytes, seed=1)
-        state = state_bench(torch, um, mem, budget, arena_bytes, seed=0)
-        state["reps"] = "second of two runs (first = warm-up)"
+        runs = [state_bench(torch, um, mem, budget, arena_bytes, seed=s) for s in (0, 2, 3)]
+        state = dict(runs[0])
+        for op in ("touch_2^21_random", "discard_2^21", "touch_2^21_pressure"):
+            by = sorted(runs, key=lambda r: r[op]["ms"])
+            state[op] = dict(by[1][op])
+            state[op]["ms_runs"] = [r[op]["ms"] for r in runs]
+        state["empty_kernel_span_us"] = sorted(r["empty_kernel_span_us"] for r in runs)[1]
+        state["reps"] = "median of three runs (seeds 0, 2, 3) after one warm-up run"
     c2 = None if args.no_compare else c2_stream(torch, um, harness, mem, budget, host_pool)
     c3k = None if args.no_compare else c3_64k(torch, um, harness, mem, budget, arena_bytes)
     e2e_s = None
