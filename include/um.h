@@ -20,7 +20,7 @@
  * Execution.  All planning (state tables, victim selection, work-list compaction) runs
  * in sm_100a kernels on device-resident tables; data moves by a kernel-driven TMA copy
  * over mapped pinned host memory (K4, no host round trip) or, for large sub-ops, by the
- * copy engines from the device-made plan (K4-CE, one host sync per sub-op).  No CPU
+ * copy engines from the device-made plan (K4-CE, one host round trip per sub-op).  No CPU
  * fallback: the host never computes a state, a victim or a transfer list.
  *
  * Conventions (all functions):
@@ -63,7 +63,7 @@ enum { UM_ST_U = 0, UM_ST_H = 1, UM_ST_HD = 2, UM_ST_G = 3, UM_ST_GE = 4, UM_ST_
 enum {
   UM_F_DISCARD_OFF = 1u, /* "UVM-opt" baseline: discards are accepted no-ops */
   UM_F_COPY_CE = 2u,     /* always move data with the copy engines (K4-CE: device plan,
-                            one host sync per sub-op, cudaMemcpyBatchAsync on 2 streams)  */
+                            one host round trip per sub-op, cudaMemcpyBatchAsync on 2 streams)  */
   UM_F_CHECK = 4u,       /* poison frames with 0xA5 at creation; extra validation       */
   UM_F_APP_STAMP = 8u,   /* harness: after each touch sub-op, write the content stamp of
                             every UM_ACC_WRITE block (simulated application kernel)    */

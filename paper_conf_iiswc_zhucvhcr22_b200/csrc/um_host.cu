@@ -239,7 +239,8 @@ struct um_arena {
   // K4-CE path
   cudaStream_t cs[2] = {nullptr, nullptr};
   cudaEvent_t ev_cs[2] = {nullptr, nullptr};
-  XItem* hitems = nullptr;              // pinned mirror of xitems
+  XItem* hitems = nullptr;              // pinned mirror of xitems (written by k_plan_commit)
+  uint32_t* hflag = nullptr;            // pinned {seq, n_need} published by k_plan_commit
   uint32_t* hd2h = nullptr;             // pinned mirror of d2h_frame / d2h_hf
   std::vector<char*> hhost;             // host chunk pointers
   char* bounce = nullptr;
@@ -539,13 +540,33 @@ struct CopyList {
 //   kernel ; D2H bounce->host (fused swaps).
 // Stream order gives every frame its write-after-read order; alternating streams keep
 // both PCIe directions busy.  The paging stream waits for both copy streams.
+// Spin until k_plan_commit of sub-op `seq` has published its plan in mapped host memory
+// (no stream sync, no read-back copies).  Bounded: if the paging stream reports an error,
+// or goes idle without the flag, the op fails with UM_ECUDA instead of hanging.
+static um_status wait_plan(um_arena* a, uint32_t seq) {
+  volatile uint32_t* f = a->hflag;
+  for (uint64_t it = 1;; ++it) {
+    if (f[0] == seq) break;
+    if ((it & 255) == 0) {
+      const cudaError_t q = cudaStreamQuery(a->ps);
+      if (q == cudaSuccess) {
+        if (f[0] == seq) break;
+        a->sticky = UM_ECUDA;
+        return UM_ECUDA;
+      }
+      if (q != cudaErrorNotReady) CK(q);
+    }
+  }
+  std::atomic_thread_fence(std::memory_order_acquire);
+  return UM_OK;
+}
+
 static um_status ce_subop(um_arena* a, uint32_t seq, uint32_t n) {
   CK(launch_plan_commit(a->T, seq, n, a->ps));
   a->n_launch++;
-  CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
-  CK(cudaMemcpyAsync(a->hitems, a->T.xitems, sizeof(XItem) * n, cudaMemcpyDeviceToHost, a->ps));
-  CK(cudaStreamSynchronize(a->ps));
-  const uint32_t nn = std::min<uint32_t>(a->hctl->n_need, n);
+  um_status ws = wait_plan(a, seq);
+  if (ws) return ws;
+  const uint32_t nn = std::min<uint32_t>((uint32_t)((volatile uint32_t*)a->hflag)[1], n);
   const uint64_t G = a->L.ce_group, B = a->B;
   CopyList d2d, wb, h2d, sw;
   // consecutive groups of zero-fill items only (no copy to order against) share one
@@ -1005,7 +1026,11 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   if ((e = cudaEventCreateWithFlags(&a->ev_in, cudaEventDisableTiming))) return fail(e);
   if ((e = cudaEventCreateWithFlags(&a->ev_out, cudaEventDisableTiming))) return fail(e);
   if ((e = cudaHostAlloc((void**)&a->hctl, sizeof(Ctl), cudaHostAllocDefault))) return fail(e);
-  if ((e = cudaHostAlloc((void**)&a->hitems, sizeof(XItem) * a->nframes, cudaHostAllocDefault))) return fail(e);
+  if ((e = cudaHostAlloc((void**)&a->hitems, sizeof(XItem) * a->nframes, cudaHostAllocMapped))) return fail(e);
+  if ((e = cudaHostAlloc((void**)&a->hflag, 16, cudaHostAllocMapped))) return fail(e);
+  memset(a->hflag, 0, 16);
+  if ((e = cudaHostGetDevicePointer((void**)&a->T.hx, a->hitems, 0))) return fail(e);
+  if ((e = cudaHostGetDevicePointer((void**)&a->T.hflag, a->hflag, 0))) return fail(e);
   if ((e = cudaHostAlloc((void**)&a->hd2h, 8ull * a->nframes, cudaHostAllocDefault))) return fail(e);
   for (int i = 0; i < 2; ++i) {
     if ((e = cudaStreamCreateWithPriority(&a->cs[i], cudaStreamNonBlocking, prio_hi))) return fail(e);
@@ -1039,6 +1064,7 @@ UM_API um_status um_arena_destroy(um_arena* a) {
   for (auto e : a->evpool) cudaEventDestroy(e);
   if (a->hctl) cudaFreeHost(a->hctl);
   if (a->hitems) cudaFreeHost(a->hitems);
+  if (a->hflag) cudaFreeHost(a->hflag);
   if (a->hd2h) cudaFreeHost(a->hd2h);
   for (int i = 0; i < 2; ++i) {
     if (a->ev_cs[i]) cudaEventDestroy(a->ev_cs[i]);

@@ -42,6 +42,7 @@ struct Ctl {
   unsigned long long vs_combo;          // wide victim scan: (candidates of finished tiles << 32) | next ticket
   unsigned int first_skip;              // wide victim scan: first ticket not examined
   unsigned int vt_reach;                // wide victim scan: passes in the apply work table (vpass)
+  unsigned int pc_done;                 // k_plan_commit completion ticket (host read-back flag)
   // counters, striped over 8 cache lines by CTA index (fire-and-forget atomics from
   // thousands of CTAs do not serialise on one address); the host sums the stripes
   long long stats[8][S_N];
@@ -101,6 +102,11 @@ struct Tables {
   // current sub-op (its own blocks are never victims, A3), or with UM_F_OVERLAP the seq
   // of the oldest GPU sub-op whose application kernel may still run (reading R7)
   uint32_t pfloor;
+  // K4-CE read-back without a host stream sync: k_plan_commit also writes the plan into
+  // the pinned host mirror `hx` and its last CTA publishes {seq, n_need} in `hflag`
+  // (mapped pinned memory) after a system-scope fence; the host spins on hflag[0]
+  XItem* hx;
+  unsigned int* hflag;
 };
 
 // A GPU-destination op's distinct blocks as sorted disjoint intervals.  Interval j

@@ -1546,7 +1546,20 @@ __global__ void k_plan_commit(Tables T, uint32_t seq) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     XItem x = item_plan(T, i, f0, nfu);
     T.xitems[i] = x;
+    T.hx[i] = x;            // pinned host mirror (mapped)
     item_commit(T, i, x, seq);
+  }
+  // every thread's plan writes are performed system-wide before its CTA takes a ticket;
+  // the CTA with the last ticket publishes {n, seq} for the host's spin
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0 && atomicAdd(&T.ctl->pc_done, 1u) == gridDim.x - 1) {
+    T.ctl->pc_done = 0;
+    __threadfence_system();
+    volatile unsigned int* f = T.hflag;
+    f[1] = n;
+    __threadfence_system();
+    f[0] = seq;
   }
 }
 
