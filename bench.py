@@ -557,42 +557,115 @@ def _barrier(torch):
     torch.cuda.synchronize()
 
 
-def cpu_oracle_baseline(trace, W, budget_s=20.0):
-    """The oracle (oracle/sim.py, pure Python, 1 thread) replaying the same trace:
-    iterations after the first, until budget_s of CPU time."""
+def _gpu_node_cpus(dev_index):
+    """Host cores on the GPU's NUMA node (sysfs), intersected with this process's
+    affinity; all allowed cores if the node is unknown."""
+    allowed = sorted(os.sched_getaffinity(0))
+    try:
+        bus = subprocess.run(["nvidia-smi", "-i", str(dev_index), "--query-gpu=pci.bus_id", "--format=csv,noheader"],
+                             capture_output=True, text=True, timeout=30).stdout.strip().lower()
+        node = int(open(f"/sys/bus/pci/devices/{bus[-12:]}/numa_node").read())
+        cpus = set()
+        for part in open(f"/sys/devices/system/node/node{max(node, 0)}/cpulist").read().strip().split(","):
+            lo, _, hi = part.partition("-")
+            cpus.update(range(int(lo), int(hi or lo) + 1))
+        mine = [c for c in allowed if c in cpus]
+        return (mine or allowed), max(node, 0)
+    except Exception:
+        return allowed, None
+
+
+def _host_info():
+    model = None
+    try:
+        for line in subprocess.run(["lscpu"], capture_output=True, text=True, timeout=30).stdout.splitlines():
+            if line.startswith("Model name:"):
+                model = line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return {"nproc": os.cpu_count(), "lscpu_model": model}
+
+
+class _Pinned:
+    """Pin this process to one core on the GPU's NUMA node for the oracle's timing (the
+    oracle is single-threaded pure Python), restoring the affinity afterwards."""
+
+    def __init__(self, dev_index):
+        self.cpus, self.node = _gpu_node_cpus(dev_index)
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        self.core = self.cpus[-1]
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.old)
+
+    def info(self):
+        return {"cores": 1, "pinned_core": self.core, "numa_node": self.node, **_host_info()}
+
+
+def cpu_oracle_baseline(trace, W, dev_index=0, budget_s=20.0):
+    """The oracle (oracle/sim.py, pure Python, 1 thread pinned to one core of the GPU's
+    NUMA node) replaying the same trace: iterations after the first, until budget_s of
+    CPU time."""
     from oracle.sim import Oracle, apply_op
-    import tracegen as tg  # noqa: F401
     from paper_conf_iiswc_zhucvhcr22_b200 import harness
     bounds = harness.iteration_bounds(trace)
     o = Oracle(trace.block_bytes, trace.arena_bytes, trace.budget_bytes)
     ops = list(trace.iter_ops())
-    for op in ops[bounds[0][0]:bounds[0][1]]:
-        apply_op(o, op, "eager")
-    t0 = time.process_time()
-    n = 0
-    for (a, b) in bounds[1:]:
-        for op in ops[a:b]:
+    with _Pinned(dev_index) as pin:
+        for op in ops[bounds[0][0]:bounds[0][1]]:
             apply_op(o, op, "eager")
-        n += 1
-        if time.process_time() - t0 > budget_s:
-            break
-    dt = time.process_time() - t0
-    return {"value": n / dt, "unit": "iter/s", "cores": 1, "kind": "oracle",
+        t0 = time.process_time()
+        n = 0
+        for (a, b) in bounds[1:]:
+            for op in ops[a:b]:
+                apply_op(o, op, "eager")
+            n += 1
+            if time.process_time() - t0 > budget_s:
+                break
+        dt = time.process_time() - t0
+    return {"value": n / dt, "unit": "iter/s", "kind": "oracle", **pin.info(),
             "sample": f"C3 eager iterations 2..{n + 1} of the bench trace (iteration 1 replayed untimed)",
             "s_per_iter": dt / n}
 
 
-def _paths(auto, k4, link):
+def plan_sizes(args, free_bytes, lws):
+    """Frame budget, arena and host pool of the C3 run (both arms use this): the requested
+    budget, clamped to free HBM - 5 GiB, and to what host RAM can pin per local rank
+    ((arena - budget) + 2 GiB each).  Returns the sizes and the clamp applied, if any."""
+    B = args.block
+    want = int(args.budget_gib * GiB) // B * B
+    budget, why = want, []
+    if free_bytes is not None and free_bytes - 5 * GiB < budget:
+        budget = (free_bytes - 5 * GiB) // B * B
+        why.append("free HBM")
+    avail = _mem_available()
+    if avail:
+        fit = int((0.85 * avail / lws - 2 * GiB) / max(args.oversub - 1.0, 1e-9))
+        if fit < budget:
+            budget = max(B, fit // B * B)
+            why.append(f"host RAM ({avail / GiB:.0f} GiB available for {lws} local ranks)")
+    arena_bytes = int(budget * args.oversub) // B * B
+    return budget, arena_bytes, arena_bytes - budget + 2 * GiB, (", ".join(why) or None)
+
+
+def _paths(k4, ce, link):
     def one(r):
         if not r:
             return None
         sp = r["stats_per_iter"]
         lb = sp["h2d_bytes"] + sp["d2h_bytes"]
-        ach = lb * len(r["iter_ms_each"]) / (r["timing"]["ms_xfer"] / 1e3) / 1e9 if r["timing"]["ms_xfer"] else None
+        n = len(r["iter_ms_each"])
+        ach = lb * n / (r["timing"]["ms_xfer"] / 1e3) / 1e9 if r["timing"]["ms_xfer"] else None
         t_ideal = sp["h2d_bytes"] / (link["h2d_gbs"] * 1e9) + sp["d2h_bytes"] / (link["d2h_gbs"] * 1e9)
         pk = lb / t_ideal / 1e9 if t_ideal else None
-        return {"iter_ms": r["iter_ms"], "achieved_gbs": ach, "frac_of_link": (ach / pk) if (ach and pk) else None}
-    return {"auto (K4-CE >= 16 MiB)": one(auto), "k4_tma_kernel_only": one(k4)}
+        return {"iter_ms": r["iter_ms"], "iterations": n, "achieved_gbs": ach,
+                "frac_of_link": (ach / pk) if (ach and pk) else None}
+    return {"k4_tma_kernel (default engine)": one(k4),
+            "k4_ce (comparison: one cudaMemcpyAsync per coalesced run on 2 copy streams)": one(ce)}
 
 
 def build_trace(args, budget, with_host_data, iterations):
@@ -624,16 +697,8 @@ def main_ours(args):
     torch.cuda.empty_cache()
     free, total = torch.cuda.mem_get_info(dev)
     B = args.block
-    budget = min(int(args.budget_gib * GiB), free - 5 * GiB) // B * B
-    # host RAM guard: every local rank pins a pool of (arena - budget) + 2 GiB
     lws = int(os.environ.get("LOCAL_WORLD_SIZE", str(ws)))
-    avail = _mem_available()
-    if avail:
-        fit = int((0.85 * avail / lws - 2 * GiB) / max(args.oversub - 1.0, 1e-9))
-        if fit < budget:
-            budget = max(B, fit // B * B)
-    arena_bytes = int(budget * args.oversub) // B * B
-    host_pool = arena_bytes - budget + 2 * GiB
+    budget, arena_bytes, host_pool, clamp = plan_sizes(args, free, lws)
     trace = build_trace(args, budget, True, W + K)
     t_build = time.perf_counter()
     mem = um.Memory(B, arena_bytes, budget, host_pool_bytes=host_pool, device=dev.index,
@@ -646,12 +711,12 @@ def main_ours(args):
     for mode in args.modes.split(","):
         res[mode] = run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=clocks if mode == "eager" else None,
                              flags_extra=ovf)
-    # the TMA kernel path (K4) on the same step, for comparison with the auto path, and the
-    # same step with the app kernels serialized on the paging stream (no R7 window)
-    k4 = run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=um.UM_F_COPY_KERNEL | ovf) \
+    # comparison legs on the same step (at most 5 timed iterations each): the copy-engine
+    # transfer arm (K4-CE) and the other app-kernel schedule (R7 overlap <-> sequential)
+    Kc = min(K, 5)
+    ce = run_mode(torch, um, harness, mem, trace, "eager", W, Kc, flags_extra=um.UM_F_COPY_CE | ovf) \
         if not args.no_compare else None
-    # the other app-kernel schedule on the same step (R7 overlap <-> sequential)
-    other = run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=um.UM_F_OVERLAP ^ ovf) \
+    other = run_mode(torch, um, harness, mem, trace, "eager", W, Kc, flags_extra=um.UM_F_OVERLAP ^ ovf) \
         if not args.no_compare else None
     ovl_r, seq_r = (res.get("eager"), other) if ovf else (other, res.get("eager"))
     state = None
@@ -705,7 +770,8 @@ def main_ours(args):
         "config": {"workload": "C3 DNN activation trace, 1.5x oversubscription", "block_bytes": B_,
                    "budget_bytes": budget, "arena_bytes": arena_bytes, "batch": trace.meta["batch"],
                    "layers": trace.meta["layers"], "ops_per_iter": trace.meta["ops_per_iter"],
-                   "host_pool_bytes": host_pool, "budget_requested_bytes": int(args.budget_gib * GiB), "parallelism": f"independent arenas x{ws}",
+                   "host_pool_bytes": host_pool, "budget_requested_bytes": int(args.budget_gib * GiB),
+                   "budget_clamped_by": clamp, "parallelism": f"independent arenas x{ws}",
                    "l2": "working set 255 GiB >> 126 MB L2 (no flush needed)",
                    "headline_mode": "eager (UvmDiscard)",
                    "app_overlap": ("UM_F_OVERLAP: app kernels pipelined with the next 2 GPU sub-ops (reading R7), "
@@ -720,18 +786,19 @@ def main_ours(args):
         "serviced_gbs": (link_bytes + spi["zf_bytes"]) / (t_iter_ms / 1e3) / 1e9,
         "discard_us_per_gb": ({"eager": disc[-1]["eager"]["us_per_gb"], "lazy": disc[-1]["lazy"]["us_per_gb"],
                                "sweep": disc} if disc else None),
-        "roofline": {"kernel": "transfer engine: K4-CE (copy engines, device-made plan) for sub-ops >= 16 MiB, K4 TMA kernel below",
+        "roofline": {"kernel": "k_service (K4: TMA bulk-copy fused-swap kernel over mapped pinned host memory)",
                      "bound": "host_link",
                      "achieved": achieved, "peak": peak_eff, "unit": "GB/s",
                      "frac": (achieved / peak_eff) if achieved else None, "traffic": None,
-                     "traffic_note": "the dominant work is copy-engine transfers (not a kernel, invisible to ncu); the K4 TMA kernel's dram bytes per launch are in profiles/r01_ncu_summary.md",
+                     "traffic_note": "dram and PCIe bytes per k_service launch from one ncu --set full capture: profiles/r02_ncu_service.md",
                      "frac_vs_duplex": (achieved / link["duplex_gbs"]) if achieved else None,
                      "peak_source": "measured live in bench.py: pinned 1 GiB cudaMemcpyAsync (copy engines) H2D and D2H, best of 5, weighted by the step's H2D/D2H byte mix",
                      "algorithmic_bytes_per_launch": link_bytes_per_launch, "ms_per_launch": xfer_ms_per_launch,
                      "launches_per_iter": tm["xfer_launches"] / K, "xfer_share_of_step": tm["ms_xfer"] / (t_iter_ms * K)},
         "link_peak": link,
-        "transfer_paths": _paths(res.get("eager"), k4, link),
+        "transfer_paths": _paths(res.get("eager"), ce, link),
         "app_overlap": ({"eager_overlap_iter_ms": ovl_r["iter_ms"], "eager_sequential_iter_ms": seq_r["iter_ms"],
+                         "iterations": [len(ovl_r["iter_ms_each"]), len(seq_r["iter_ms_each"])],
                          "speedup": seq_r["iter_ms"] / ovl_r["iter_ms"],
                          "plan_ms_per_iter": {"overlap": ovl_r["timing"]["ms_plan"] / K,
                                               "sequential": seq_r["timing"]["ms_plan"] / K},
@@ -756,7 +823,7 @@ def main_ours(args):
                       "note": "host wall clock per step through the Python/C API incl. host data generation + counter readback"}
     out["plan_ms_per_iter"] = tm["ms_plan"] / K
     if not args.no_cpu:
-        cb = cpu_oracle_baseline(trace, W)
+        cb = cpu_oracle_baseline(trace, W, dev.index)
         cb["note"] = ("the oracle accounts bytes but moves none; compare its s_per_iter with plan_ms_per_iter "
                       "(the GPU's planning kernels for the same iteration), not with the transfer-bound step")
         cb["gpu_plan_speedup"] = cb["s_per_iter"] * 1e3 / out["plan_ms_per_iter"] if out["plan_ms_per_iter"] else None
@@ -767,31 +834,42 @@ def main_ours(args):
 def main_reference(args):
     """The base contract's reference arm for this tier: the CPU oracle, as it stands,
     replaying the same workload (one C3 iteration per step) on the host cores."""
-    rank, _, ws = dist_env()
+    rank, local, ws = dist_env()
     if rank != 0:
         return
     import tracegen as tg
     from oracle.sim import Oracle, apply_op
     W, K = args.warmup, args.steps
-    budget = int(args.budget_gib * GiB) // args.block * args.block
+    free = None
+    try:
+        import torch
+        if torch.cuda.is_available():
+            free = torch.cuda.mem_get_info(local)[0]
+    except Exception:
+        pass
+    lws = int(os.environ.get("LOCAL_WORLD_SIZE", str(ws)))
+    budget, arena_bytes, _, clamp = plan_sizes(args, free, lws)
     trace = tg.gen_c3(block_bytes=args.block, budget_bytes=budget, oversub=args.oversub, iterations=W + K)
     it = trace.meta["iterations"]
     per = len(trace.ops) // it
     ops = list(trace.iter_ops())
     o = Oracle(trace.block_bytes, trace.arena_bytes, trace.budget_bytes)
-    for op in ops[:W * per]:
-        apply_op(o, op, "eager")
-    t0 = time.process_time()
-    for op in ops[W * per:(W + K) * per]:
-        apply_op(o, op, "eager")
-    dt = (time.process_time() - t0) / K
+    with _Pinned(local) as pin:
+        for op in ops[:W * per]:
+            apply_op(o, op, "eager")
+        t0 = time.process_time()
+        for op in ops[W * per:(W + K) * per]:
+            apply_op(o, op, "eager")
+        dt = (time.process_time() - t0) / K
     v = 1.0 / dt
     print(json.dumps({
         "metric": METRIC, "impl": "reference", "value": v, "unit": "iter/s", "n_gpus": ws, "steps": K,
         "warmup": W, "ms_per_step": dt * 1e3, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-        "dtype": "u8", "data": "synthetic C3 trace", "config": {"workload": "C3 DNN activation trace, 1.5x oversubscription",
-                                                             "block_bytes": args.block, "budget_bytes": budget},
-        "cpu_baseline": {"value": v, "unit": "iter/s", "cores": 1, "kind": "oracle",
+        "dtype": "u8", "data": "synthetic C3 trace",
+        "config": {"workload": "C3 DNN activation trace, 1.5x oversubscription", "block_bytes": args.block,
+                   "budget_bytes": budget, "arena_bytes": arena_bytes,
+                   "budget_requested_bytes": int(args.budget_gib * GiB), "budget_clamped_by": clamp},
+        "cpu_baseline": {"value": v, "unit": "iter/s", "kind": "oracle", **pin.info(),
                          "sample": f"C3 eager iterations {W + 1}..{W + K} (state accounting only; moves no bytes)"},
         "e2e": {"value": v, "unit": "iter/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)

@@ -62,15 +62,17 @@ enum { UM_ST_U = 0, UM_ST_H = 1, UM_ST_HD = 2, UM_ST_G = 3, UM_ST_GE = 4, UM_ST_
 
 enum {
   UM_F_DISCARD_OFF = 1u, /* "UVM-opt" baseline: discards are accepted no-ops */
-  UM_F_COPY_CE = 2u,     /* always move data with the copy engines (K4-CE: device plan,
-                            one host round trip per sub-op, cudaMemcpyBatchAsync on 2 streams)  */
+  UM_F_COPY_CE = 2u,     /* comparison arm: move data with the copy engines (K4-CE:
+                            device plan, one host round trip per sub-op, one
+                            cudaMemcpyAsync per coalesced run on 2 copy streams)      */
   UM_F_CHECK = 4u,       /* poison frames with 0xA5 at creation; extra validation       */
   UM_F_APP_STAMP = 8u,   /* harness: after each touch sub-op, write the content stamp of
                             every UM_ACC_WRITE block (simulated application kernel)    */
   UM_F_TIMING = 16u,     /* record CUDA events around the planning and transfer kernels
                             of every op (read with um_timing)                          */
-  UM_F_COPY_KERNEL = 32u,/* always move data with the TMA kernel (K4).  Default (neither
-                            flag): sub-ops moving >= 16 MiB use K4-CE, smaller ones K4  */
+  UM_F_COPY_KERNEL = 32u,/* move data with the TMA kernel (K4).  This is also the default
+                            (neither flag); the flag only overrides the diagnostic
+                            UM_CE_MIN_BYTES environment threshold                      */
   UM_F_OVERLAP = 64u     /* pipelined application kernels (reading R7; the
                             paper's async API calls overlap compute):
                             the UM_F_APP_STAMP kernel of a touch sub-op runs on an

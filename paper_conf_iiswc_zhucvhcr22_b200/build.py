@@ -33,7 +33,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
         raise RuntimeError("nvcc failed building libum.so")
-    with open(os.path.join(PKG, "ptxas_info.txt"), "w") as f:
+    os.makedirs(os.path.join(ROOT, "build"), exist_ok=True)   # git-ignored
+    with open(os.path.join(ROOT, "build", "ptxas_info.txt"), "w") as f:
         f.write(r.stderr)
     if verbose:
         sys.stderr.write(r.stderr)

@@ -244,7 +244,7 @@ struct um_arena {
   uint32_t* hd2h = nullptr;             // pinned mirror of d2h_frame / d2h_hf
   std::vector<char*> hhost;             // host chunk pointers
   char* bounce = nullptr;
-  uint64_t ce_min_bytes = 16ull << 20;  // auto mode: sub-ops moving >= this use the copy engines
+  uint64_t ce_min_bytes = ~0ull;  // diagnostic auto mode (UM_CE_MIN_BYTES): sub-ops moving >= this use the copy engines
   uint64_t n_ce = 0;
   // UM_F_OVERLAP (reading R7): application kernels run on their own stream `as`; the
   // last kOverlapW GPU sub-ops form the victim-exclusion window; `pend` holds the app
@@ -473,6 +473,9 @@ static void build_intervals(um_arena* a, const um_access* acc, uint32_t n) {
   }
 }
 
+// The TMA kernel (K4) is the transfer engine; the copy engines (K4-CE) are the
+// comparison arm, selected with UM_F_COPY_CE (or, for A/B runs only, for sub-ops of at
+// least UM_CE_MIN_BYTES).
 static bool use_ce(um_arena* a, uint64_t n) {
   if (a->cfg.flags & UM_F_COPY_CE) return true;
   if (a->cfg.flags & UM_F_COPY_KERNEL) return false;
@@ -487,7 +490,7 @@ static inline char* frame_ptr(um_arena* a, uint32_t f) { return a->T.frames + (s
 // A copy list with run coalescing (adjacent items whose source and destination are
 // both contiguous AND inside the same host chunk allocation become one copy — a copy
 // may not span two pinned allocations even if they happen to be adjacent), issued as
-// one cudaMemcpyBatchAsync.
+// one copy call per run.
 struct CopyList {
   std::vector<void*> dst, src;
   std::vector<size_t> size;
@@ -504,30 +507,10 @@ struct CopyList {
     size.push_back(n);
     seg.push_back(chunk);
   }
+  // one cudaMemcpyAsync per coalesced run (the copy engines take 2 MiB+ runs at link rate)
   cudaError_t issue(cudaStream_t st) {
-    if (dst.empty()) return cudaSuccess;
-    if (dst.size() == 1) return cudaMemcpyAsync(dst[0], src[0], size[0], cudaMemcpyDefault, st);
-    cudaMemcpyAttributes attr{};
-    attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-    attr.flags = cudaMemcpyFlagPreferOverlapWithCompute;
-    size_t aidx = 0, fail = 0;
-    cudaError_t e = cudaMemcpyBatchAsync(dst.data(), src.data(), size.data(), dst.size(), &attr, &aidx, 1, &fail, st);
-    if (e == cudaSuccess) return e;
-    cudaGetLastError();
-    if (getenv("UM_DEBUG")) {
-      fprintf(stderr, "libum: cudaMemcpyBatchAsync(%zu copies) failed: %s (fail idx %zu); falling back\n", dst.size(),
-              cudaGetErrorString(e), fail);
-      for (size_t i = 0; i < dst.size() && i < 4; ++i) {
-        cudaPointerAttributes pa{}, pb{};
-        cudaPointerGetAttributes(&pa, dst[i]);
-        cudaPointerGetAttributes(&pb, src[i]);
-        cudaGetLastError();
-        fprintf(stderr, "  [%zu] dst %p (type %d) src %p (type %d) size %zu\n", i, dst[i], (int)pa.type, src[i],
-                (int)pb.type, size[i]);
-      }
-    }
     for (size_t i = 0; i < dst.size(); ++i) {
-      e = cudaMemcpyAsync(dst[i], src[i], size[i], cudaMemcpyDefault, st);
+      cudaError_t e = cudaMemcpyAsync(dst[i], src[i], size[i], cudaMemcpyDefault, st);
       if (e) return e;
     }
     return cudaSuccess;

@@ -22,10 +22,10 @@ def _cuda():
     build.build()
 
 
-COPY_FLAGS = {"auto": 0, "kernel": 32, "ce": 2}   # UM_F_COPY_KERNEL / UM_F_COPY_CE
+COPY_FLAGS = {"default": 0, "kernel": 32, "ce": 2}   # default = the TMA kernel K4; UM_F_COPY_KERNEL / UM_F_COPY_CE
 
 
-def _gpu(trace, mode, copy="auto", overlap=False, **kw):
+def _gpu(trace, mode, copy="default", overlap=False, **kw):
     from paper_conf_iiswc_zhucvhcr22_b200 import harness, um
     flags = um.UM_F_APP_STAMP | um.UM_F_CHECK | COPY_FLAGS[copy] | (um.UM_F_OVERLAP if overlap else 0)
     return harness.run_trace(trace, mode, flags=flags, **kw)
@@ -108,7 +108,7 @@ def test_c3_small(mode):
     t = tg.gen_c3(block_bytes=64 << 10, budget_bytes=192 << 20, iterations=2, workspace_bytes=4 << 20,
                   layers=tg.scale_layers(tg.VGG16, 1.0 / 512, 1.0 / 64), batch=8)
     assert t.arena_bytes > t.budget_bytes
-    for copy in ("auto", "kernel", "ce"):
+    for copy in ("default", "ce"):
         assert_parity(t, mode, _gpu(t, mode, copy=copy))
 
 
@@ -251,7 +251,7 @@ def _full_size_trace(iterations=2, B=2 << 20):
     return tg.gen_c3(block_bytes=B, budget_bytes=budget, oversub=1.5, iterations=iterations)
 
 
-@pytest.mark.parametrize("mode,copy", [("eager", "auto"), ("lazy", "kernel")])
+@pytest.mark.parametrize("mode,copy", [("eager", "default"), ("lazy", "ce"), ("base", "default")])
 def test_c3_full_size(mode, copy):
     """Parity at the bench's full size and launch configuration: C3 at 1.5x of a
     170 GiB frame budget (255 GiB arena, 2 MiB blocks), host pool = arena - budget +
@@ -315,7 +315,7 @@ def test_overlap_c3_small(mode):
     """C3 with pipelined app kernels through every transfer path."""
     t = tg.gen_c3(block_bytes=64 << 10, budget_bytes=192 << 20, iterations=2, workspace_bytes=4 << 20,
                   layers=tg.scale_layers(tg.VGG16, 1.0 / 512, 1.0 / 64), batch=8)
-    for copy in ("auto", "kernel", "ce"):
+    for copy in ("default", "ce"):
         assert_parity(t, mode, _gpu(t, mode, copy=copy, overlap=True), overlap=True)
 
 
@@ -371,12 +371,14 @@ def test_fault_list_boundaries(mode):
 
 
 
-def test_c3_full_size_64k_blocks():
+@pytest.mark.parametrize("copy", ["default", "ce"])
+def test_c3_full_size_64k_blocks(copy):
     """The C3 64 KiB-block variant (~4.18 M blocks, ~2.79 M frames) at full
-    size, eager, default transfer selection: two iterations (the trace is periodic after
-    the first) bit-exact against the oracle, contents included."""
+    size, eager, on the TMA kernel and on per-copy copy engines: two iterations (the trace
+    is periodic after the first) bit-exact against the oracle, contents
+    included."""
     t = _full_size_trace(iterations=2, B=64 << 10)
     assert t.nblocks > 4_000_000
     pool = t.arena_bytes - t.budget_bytes + (2 << 30)
-    g = _gpu(t, "eager", host_pool_bytes=pool)
+    g = _gpu(t, "eager", copy=copy, host_pool_bytes=pool)
     assert_parity(t, "eager", g)
