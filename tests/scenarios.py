@@ -49,6 +49,13 @@ def build(sc) -> tuple:
             tb.discard(int(w[1]), int(w[2]))
         elif op == "evict":
             tb.evict(int(w[1]) * B)
+        elif op == "evict_bytes":
+            tb.evict(int(w[1]))
+        elif op == "touch_bytes":
+            kind = {"R": tg.ACC_READ, "W": tg.ACC_WRITE, "RW": tg.ACC_READ | tg.ACC_WRITE}[w[3]]
+            tb.touch([(int(w[1]), int(w[2]), kind)])
+        elif op == "prefetch_bytes":
+            tb.prefetch(int(w[1]), int(w[2]), tg.DST_GPU if w[3] == "GPU" else tg.DST_HOST)
         elif op == "host_write":
             lo, hi = _blocks(w[1])
             tb.host_write(lo * B, (hi - lo + 1) * B)
