@@ -194,6 +194,22 @@ um_status um_content_tags(um_arena *a, uint64_t *tags);
 um_status um_timing(um_arena *a, double *ms_plan, double *ms_xfer, uint64_t *xfer_launches,
                     uint64_t *launches, int reset);
 
+/* Transfer log (parity and redundant-transfer accounting; PAPER
+ * L34 "overwritten before being read", Fig. 3 L125 required vs performed transfers).
+ * Attaches a caller-owned DEVICE buffer of cap_entries records of 16 bytes
+ * {uint32 seq, uint32 block, uint32 kind (0 = H2D, 1 = D2H, 2 = zero-fill), uint32
+ * state of the block before the move (UM_ST_*)} and restarts the count at zero.  From
+ * then on every block whose migration, write-back or zero-fill enters a work list the
+ * transfer engine executes appends one record, in no particular order (sort by seq).
+ * buf = NULL detaches.  The caller keeps the buffer alive until it detaches or
+ * destroys the arena.  Enqueued on the paging stream; UM_EINVAL if buf != NULL and
+ * cap_entries == 0. */
+um_status um_xlog_attach(um_arena *a, void *buf, uint64_t cap_entries);
+
+/* Synchronizes.  Number of records appended since the last attach; records beyond the
+ * capacity were counted but not written (*n > cap_entries means the log overflowed). */
+um_status um_xlog_count(um_arena *a, uint64_t *n);
+
 const char *um_strerror(um_status s);
 
 #ifdef __cplusplus

@@ -1315,6 +1315,25 @@ UM_API um_status um_content_tags(um_arena* a, uint64_t* tags) {
   return UM_OK;
 }
 
+UM_API um_status um_xlog_attach(um_arena* a, void* buf, uint64_t cap_entries) {
+  ENTER(a);
+  if (buf && cap_entries == 0) return UM_EINVAL;
+  // launches already enqueued carry their own copy of the tables: the reset is stream-ordered
+  CK(cudaMemsetAsync(&a->T.ctl->xlog_n, 0, sizeof(unsigned long long), a->ps));
+  a->T.xlog = (uint4*)buf;
+  a->T.xlog_cap = buf ? cap_entries : 0;
+  return UM_OK;
+}
+
+UM_API um_status um_xlog_count(um_arena* a, uint64_t* n) {
+  ENTER(a);
+  if (!n) return UM_EINVAL;
+  um_status s = sync_ctl(a);
+  if (s) return s;
+  *n = a->hctl->xlog_n;
+  return UM_OK;
+}
+
 UM_API um_status um_timing(um_arena* a, double* ms_plan, double* ms_xfer, uint64_t* xfer_launches,
                            uint64_t* launches, int reset) {
   ENTER(a);

@@ -43,6 +43,7 @@ struct Ctl {
   unsigned int first_skip;              // wide victim scan: first ticket not examined
   unsigned int vt_reach;                // wide victim scan: passes in the apply work table (vpass)
   unsigned int pc_done;                 // k_plan_commit completion ticket (host read-back flag)
+  unsigned long long xlog_n;            // transfer log: records appended (may exceed the capacity)
   // counters, striped over 8 cache lines by CTA index (fire-and-forget atomics from
   // thousands of CTAs do not serialise on one address); the host sums the stripes
   long long stats[8][S_N];
@@ -56,6 +57,10 @@ struct XItem {
   uint32_t flags;
 };
 enum { XI_H2D = 1u, XI_ZF = 2u, XI_D2H = 4u, XI_SWAP = 8u };
+
+// Transfer log record (um_xlog_attach): one per block moved or zero-filled, appended
+// where the work list that the transfer engine executes is fixed.
+enum { XL_H2D = 0u, XL_D2H = 1u, XL_ZF = 2u };
 
 // Everything a kernel needs, passed by value.
 struct Tables {
@@ -107,6 +112,9 @@ struct Tables {
   // (mapped pinned memory) after a system-scope fence; the host spins on hflag[0]
   XItem* hx;
   unsigned int* hflag;
+  // transfer log (null = off): {seq, block, XL_* kind, state before the move}
+  uint4* xlog;
+  unsigned long long xlog_cap;
 };
 
 // A GPU-destination op's distinct blocks as sorted disjoint intervals.  Interval j

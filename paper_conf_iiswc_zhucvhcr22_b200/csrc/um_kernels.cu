@@ -69,6 +69,14 @@ __device__ __forceinline__ void stat_add(const Tables& T, int slot, long long v)
   if (v) atomicAdd((unsigned long long*)&T.ctl->stats[blockIdx.x & 7][slot], (unsigned long long)v);
 }
 
+// Transfer log (um_xlog_attach; off when T.xlog is null): one record per block whose move
+// or zero-fill enters a work list the transfer engine executes.
+__device__ __forceinline__ void xlog_put(const Tables& T, uint32_t seq, uint32_t blk, uint32_t kind, uint32_t prev) {
+  if (!T.xlog) return;
+  const unsigned long long p = atomicAdd(&T.ctl->xlog_n, 1ull);
+  if (p < T.xlog_cap) T.xlog[p] = make_uint4(seq, blk, kind, prev);
+}
+
 // Exclusive block scan of a 64-bit value (two packed 31-bit counts add without carry).
 template <int TPB>
 __device__ __forceinline__ unsigned long long block_excl_scan(unsigned long long v, unsigned long long& total,
@@ -894,6 +902,7 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
         if (isG) {
           T.d2h_frame[gr] = fr;
           T.d2h_hf[gr] = hf;
+          xlog_put(T, seq, v, XL_D2H, ss);
         }
       }
     }
@@ -1197,7 +1206,7 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
 
 // 512-thread CTAs, 2 per SM (62 registers): the same resident warps as 4 x 256 in one
 // wave, and a quarter of the CTAs to dispatch when there is nothing to do (k = 0)
-__global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict_mode) {
+__global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict_mode, uint32_t seq) {
   pdl_enter();
   constexpr int TPB = kVaTPB, AIPT = 4, CH = 32 * AIPT;
   __shared__ uint32_t s_cnt[8];
@@ -1309,6 +1318,7 @@ __global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict
               const uint32_t d = db + rD + __popc(bD[q] & lt);
               T.d2h_frame[d] = fr[q];
               T.d2h_hf[d] = hf[q];
+              xlog_put(T, seq, v[q], XL_D2H, ss[q]);
             }
           }
         }
@@ -1410,6 +1420,14 @@ __device__ __forceinline__ void item_commit(const Tables& T, uint32_t i, const X
   }
 }
 
+// Transfer-log records of need item i: the newcomer's migration or zero-fill and, when
+// its frame comes from a valid victim, the victim's write-back.
+__device__ __forceinline__ void item_log(const Tables& T, uint32_t i, const XItem& x, uint32_t seq, uint32_t f0) {
+  if (!T.xlog) return;
+  xlog_put(T, seq, T.need[i], (x.flags & XI_H2D) ? XL_H2D : XL_ZF, T.needk[i]);
+  if (x.flags & XI_D2H) xlog_put(T, seq, T.victim[i - f0], XL_D2H, T.vkind[i - f0]);
+}
+
 struct Unit {
   char* frame;        // frame chunk (HBM)
   char* d2h_dst;      // host chunk receiving the old content, or null
@@ -1461,7 +1479,10 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
         x.d2h_dst = (p.flags & XI_D2H) ? hptr(T, p.dst_hf) + coff : nullptr;
         x.h2d_src = (p.flags & XI_H2D) ? hptr(T, p.src_hf) + coff : nullptr;
         x.zf = (p.flags & XI_ZF) != 0;
-        if (ch == 0 && (x.pure_zf() ? 1 : 2) == phase) item_commit(T, i, p, seq);
+        if (ch == 0 && (x.pure_zf() ? 1 : 2) == phase) {
+          item_log(T, i, p, seq, f0);
+          item_commit(T, i, p, seq);
+        }
       } else {
         uint32_t fr = T.d2h_frame[i], hf = T.d2h_hf[i];
         x.frame = T.frames + (size_t)fr * T.B + coff;
@@ -1547,6 +1568,7 @@ __global__ void k_plan_commit(Tables T, uint32_t seq) {
     XItem x = item_plan(T, i, f0, nfu);
     T.xitems[i] = x;
     T.hx[i] = x;            // pinned host mirror (mapped)
+    item_log(T, i, x, seq, f0);
     item_commit(T, i, x, seq);
   }
   // every thread's plan writes are performed system-wide before its CTA takes a ticket;
@@ -1763,6 +1785,7 @@ __device__ __forceinline__ void directive_body(const Tables& T, int kind, uint32
             T.d2h_frame[s_db + rA] = fr;
             T.d2h_hf[s_db + rA] = hf;
             T.hframe[bb] = hf;
+            xlog_put(T, seq, bb, XL_D2H, ss);
             ++rA;
             ++nD2H;
           } else {
@@ -2139,7 +2162,7 @@ cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, u
   // one warp per pass of <= kVaPass victims (<= max_victims / kVaPass + tiles passes)
   unsigned grid = ceil_div((unsigned long long)ceil_div(max_victims ? max_victims : 1, kVaPass) + nt, kVaTPB / 32);
   if (grid > (unsigned)g_nsm * 2) grid = g_nsm * 2;
-  le__ = launch_pdl(k_victims_apply, dim3(grid), dim3(kVaTPB), 0, s, T, evict_mode);
+  le__ = launch_pdl(k_victims_apply, dim3(grid), dim3(kVaTPB), 0, s, T, evict_mode, seq);
   if (le__) return le__;
   return cudaGetLastError();
 }

@@ -93,11 +93,39 @@ def result(arena: um.Arena) -> dict:
     return d
 
 
-def run_trace(trace, mode: str, **kw) -> dict:
+class XLog:
+    """A device buffer attached as the arena's transfer log (um_xlog_attach)."""
+
+    def __init__(self, arena: um.Arena, cap: int):
+        import torch
+        self.arena, self.cap = arena, cap
+        self.buf = torch.zeros((cap, 4), dtype=torch.int32, device=arena.frames.device)
+        um.um_xlog_attach(arena.handle, self.buf.data_ptr(), cap)
+
+    def records(self) -> list:
+        """(seq, kind, block, prev_state) tuples, sorted (the log's order is arbitrary)."""
+        n = um.um_xlog_count(self.arena.handle)
+        if n > self.cap:
+            raise RuntimeError(f"transfer log overflow: {n} records > capacity {self.cap}")
+        a = self.buf[:n].cpu().numpy().view(np.uint32).astype(np.int64)
+        return sorted((int(s), um.XL_KIND[k], int(b), int(p)) for s, b, k, p in a.tolist())
+
+    def detach(self):
+        um.um_xlog_attach(self.arena.handle, None, 0)
+
+
+def run_trace(trace, mode: str, xlog: int = 0, **kw) -> dict:
+    """Replay the whole trace on a fresh arena; xlog = capacity of a transfer log to
+    attach (its sorted records are returned under "xlog")."""
     arena = make_arena(trace, mode, **kw)
     try:
         alloc_buffers(arena, trace)
+        lg = XLog(arena, xlog) if xlog else None
         issue(arena, trace, mode)
-        return result(arena)
+        r = result(arena)
+        if lg:
+            r["xlog"] = lg.records()
+            lg.detach()
+        return r
     finally:
         arena.close()

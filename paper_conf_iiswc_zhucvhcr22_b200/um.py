@@ -82,6 +82,8 @@ def lib():
             "um_dump": [P, P, P, C.POINTER(U32), P, C.POINTER(U32)],
             "um_content_tags": [P, P],
             "um_timing": [P, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(U64), C.POINTER(U64), I],
+            "um_xlog_attach": [P, P, U64],
+            "um_xlog_count": [P, C.POINTER(U64)],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -95,7 +97,8 @@ def lib():
 
 EXPORTS = ("um_workspace_size", "um_arena_create", "um_arena_destroy", "um_alloc", "um_prefetch", "um_discard",
            "um_discard_lazy", "um_touch_batch", "um_evict", "um_host_write", "um_block_table", "um_stream",
-           "um_join", "um_get_stats", "um_dump", "um_content_tags", "um_timing", "um_strerror")
+           "um_join", "um_get_stats", "um_dump", "um_content_tags", "um_timing", "um_xlog_attach",
+           "um_xlog_count", "um_strerror")
 
 
 def _ck(fn, st):
@@ -200,6 +203,19 @@ def um_timing(a, reset: bool = False) -> dict:
     nx, nl = C.c_uint64(), C.c_uint64()
     _ck("um_timing", lib().um_timing(a, C.byref(p), C.byref(x), C.byref(nx), C.byref(nl), int(reset)))
     return {"ms_plan": p.value, "ms_xfer": x.value, "xfer_launches": nx.value, "launches": nl.value}
+
+
+XL_KIND = ("H2D", "D2H", "ZF")
+
+
+def um_xlog_attach(a, dev_ptr, cap_entries: int) -> None:
+    _ck("um_xlog_attach", lib().um_xlog_attach(a, dev_ptr, cap_entries))
+
+
+def um_xlog_count(a) -> int:
+    n = C.c_uint64()
+    _ck("um_xlog_count", lib().um_xlog_count(a, C.byref(n)))
+    return n.value
 
 
 # -------------------------------------------------------------------------------------

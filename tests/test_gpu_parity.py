@@ -25,18 +25,46 @@ def _cuda():
 COPY_FLAGS = {"default": 0, "kernel": 32, "ce": 2}   # default = the TMA kernel K4; UM_F_COPY_KERNEL / UM_F_COPY_CE
 
 
-def _gpu(trace, mode, copy="default", overlap=False, **kw):
+def xlog_bound(trace):
+    """Upper bound on the transfer-log records of a trace: every covered block of a GPU
+    op may bring one newcomer record and one victim write-back, every block of a
+    prefetch(HOST) or evict one write-back."""
+    B, F = trace.block_bytes, trace.budget_bytes // trace.block_bytes
+    n = 0
+    for kind, flags, off, ln, accs in trace.iter_ops():
+        if kind == tg.OP_TOUCH:
+            n += 2 * sum((o + m - 1) // B - o // B + 1 for (o, m, _k) in accs if m)
+        elif kind == tg.OP_PREFETCH:
+            n += (2 if flags == tg.DST_GPU else 1) * ((off + ln - 1) // B - off // B + 1 if ln else 0)
+        elif kind == tg.OP_EVICT:
+            n += min(F, ln // B + 1)
+    return n + 64
+
+
+def _gpu(trace, mode, copy="default", overlap=False, xlog=True, **kw):
+    """The CUDA path's result, with the transfer log attached (xlog_bound capacity)."""
     from paper_conf_iiswc_zhucvhcr22_b200 import harness, um
     flags = um.UM_F_APP_STAMP | um.UM_F_CHECK | COPY_FLAGS[copy] | (um.UM_F_OVERLAP if overlap else 0)
-    return harness.run_trace(trace, mode, flags=flags, **kw)
+    return harness.run_trace(trace, mode, flags=flags, xlog=xlog_bound(trace) if xlog else 0, **kw)
 
 
 OVERLAP_W = 2   # kOverlapW in csrc/um_internal.h (reading R7)
 
 
+def _first_diff(a, b):
+    for i, (x, y) in enumerate(zip(a, b)):
+        if x != y:
+            return f"transfer log differs at record {i}: gpu {x} oracle {y} (lengths {len(a)}, {len(b)})"
+    return f"transfer log lengths differ: gpu {len(a)} oracle {len(b)}"
+
+
 def assert_parity(trace, mode, g=None, overlap=False):
     g = g if g is not None else _gpu(trace, mode, overlap=overlap)
-    o = oracle_replay(trace, mode, overlap=OVERLAP_W if overlap else 0).dump()
+    orc = oracle_replay(trace, mode, overlap=OVERLAP_W if overlap else 0, record="xlog" in g)
+    o = orc.dump()
+    if "xlog" in g:
+        # every H2D / D2H / zero-fill, with its sub-op seq and the block's prior state
+        assert g["xlog"] == sorted(orc.log), _first_diff(g["xlog"], sorted(orc.log))
     st_g = np.asarray(g["st"])
     st_o = np.asarray(o["st"])
     bad = np.nonzero(st_g != st_o)[0]
