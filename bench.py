@@ -289,6 +289,44 @@ def c3_64k(torch, um, harness, mem, budget, arena_bytes):
     return out
 
 
+def rmt_leg(torch, um, harness, mem, budget, oversub, B):
+    """Redundant-transfer accounting of the CUDA path (PAPER L34 /
+    Fig. 3): two C3 iterations per mode with the transfer log attached
+    (um_xlog_attach), judged by paper_conf_iiswc_zhucvhcr22_b200/rmt.py over the second
+    (steady-state) iteration.  Two traces: Listing 6 as printed (never discards output_1
+    or data) and --discard-all-dead.  RMT_left should hold only blocks a discard covers
+    partly (A4: a discard ignores partial blocks, §5.4)."""
+    import tracegen as tg
+    from paper_conf_iiswc_zhucvhcr22_b200 import rmt
+    out = {"iteration": "second of two (steady state)",
+           "source": "CUDA-path transfer log (um_xlog_attach), judged by paper_conf_iiswc_zhucvhcr22_b200/rmt.py "
+                     "(pinned against oracle/rmt.py in tests/test_rmt_product.py)"}
+    for variant, dead in (("listing6_literal", False), ("discard_all_dead", True)):
+        t = tg.gen_c3(block_bytes=B, budget_bytes=budget, oversub=oversub, iterations=2, discard_all_dead=dead,
+                      with_host_data=True)
+        it2 = harness.iteration_bounds(t)[1]
+        res = {}
+        for mode in ("base", "eager"):
+            arena = harness.make_arena(t, mode, mem=mem, flags=um.UM_F_APP_STAMP)
+            try:
+                harness.alloc_buffers(arena, t)
+                lg = harness.XLog(arena, 8 << 20)
+                harness.issue(arena, t, mode)
+                log = lg.raw()
+                lg.detach()
+            finally:
+                arena.close()
+            res[mode] = rmt.analyze(t, log, op_range=it2)
+        b, e = res["base"], res["eager"]
+        out[variant] = {"rmt_base_gb": b["rmt_bytes"] / 1e9, "rmt_left_gb": e["rmt_bytes"] / 1e9,
+                        "link_gb": {"base": (b["h2d_bytes"] + b["d2h_bytes"]) / 1e9,
+                                    "eager": (e["h2d_bytes"] + e["d2h_bytes"]) / 1e9},
+                        "avoided_gb": (b["h2d_bytes"] + b["d2h_bytes"] - e["h2d_bytes"] - e["d2h_bytes"]) / 1e9,
+                        "rmt_base_split_gb": {"h2d": b["rmt_h2d_bytes"] / 1e9, "d2h": b["rmt_d2h_bytes"] / 1e9},
+                        "discarded_state_moves_eager": e["discarded_state_moves"]}
+    return out
+
+
 def run_e2e(torch, um, harness, mem, trace, W, K, flags_extra=0):
     """End to end through the public API: the trace WITH the host-side data generation
     (prefetch(data,HOST); host_write; prefetch(data,GPU): the step's inputs cross
@@ -733,6 +771,7 @@ def main_ours(args):
             state[op]["ms_runs"] = [r[op]["ms"] for r in runs]
         state["empty_kernel_span_us"] = sorted(r["empty_kernel_span_us"] for r in runs)[1]
         state["reps"] = "median of three runs (seeds 0, 2, 3) after one warm-up run"
+    rmt_r = None if args.no_compare else rmt_leg(torch, um, harness, mem, budget, args.oversub, B)
     c2 = None if args.no_compare else c2_stream(torch, um, harness, mem, budget, host_pool)
     c3k = None if args.no_compare else c3_64k(torch, um, harness, mem, budget, arena_bytes)
     e2e_s = None
@@ -807,6 +846,7 @@ def main_ours(args):
                          "headline": "overlap" if ovf else "sequential"}
                         if (ovl_r and seq_r) else None),
         "roofline_state": state,
+        "rmt": rmt_r,
         "c1_directives": c1,
         "c4_sweep": c4,
         "c2_streaming": c2,

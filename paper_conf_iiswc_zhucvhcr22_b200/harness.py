@@ -102,6 +102,13 @@ class XLog:
         self.buf = torch.zeros((cap, 4), dtype=torch.int32, device=arena.frames.device)
         um.um_xlog_attach(arena.handle, self.buf.data_ptr(), cap)
 
+    def raw(self) -> np.ndarray:
+        """The records as an int64 array of rows (seq, block, kind, prev_state)."""
+        n = um.um_xlog_count(self.arena.handle)
+        if n > self.cap:
+            raise RuntimeError(f"transfer log overflow: {n} records > capacity {self.cap}")
+        return self.buf[:n].cpu().numpy().view(np.uint32).astype(np.int64)
+
     def records(self) -> list:
         """(seq, kind, block, prev_state) tuples, sorted (the log's order is arbitrary)."""
         n = um.um_xlog_count(self.arena.handle)

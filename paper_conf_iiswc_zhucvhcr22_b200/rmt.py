@@ -103,11 +103,12 @@ def op_of_seq(trace, seqs):
     return np.searchsorted(starts, np.asarray(seqs, np.int64), side="right") - 1
 
 
-def analyze(trace, log):
+def analyze(trace, log, op_range=None):
     """log: (seq, kind, block, prev_state) records with kind in {"H2D", "D2H", "ZF"}, or
     an int array of rows (seq, block, kind 0/1/2, prev_state) as um_xlog records them.
     Returns byte totals, redundant bytes per direction, and the number of moves of
-    blocks that were discarded (HD, GE, GL) when they moved."""
+    blocks that were discarded (HD, GE, GL) when they moved.  op_range = (lo, hi) counts
+    only the moves made by ops lo..hi-1 (e.g. one steady-state iteration)."""
     B = trace.block_bytes
     if len(log) and isinstance(log[0], tuple) and isinstance(log[0][1], str):
         code = {"H2D": 0, "D2H": 1, "ZF": 2}
@@ -115,10 +116,13 @@ def analyze(trace, log):
     else:
         arr = np.asarray(log, np.int64).reshape(-1, 4)
     arr = arr[arr[:, 2] != 2]                       # zero-fills move nothing over the link
+    t = op_of_seq(trace, arr[:, 0])
+    if op_range is not None:
+        m = (t >= op_range[0]) & (t < op_range[1])
+        arr, t = arr[m], t[m]
     out = {"h2d_bytes": int((arr[:, 2] == 0).sum()) * B, "d2h_bytes": int((arr[:, 2] == 1).sum()) * B,
            "discarded_state_moves": int(np.isin(arr[:, 3], _STATE_DISCARDED).sum())}
     key, kind, T = events(trace)
-    t = op_of_seq(trace, arr[:, 0])
     b = arr[:, 1]
     # last WRITE/DEAD event at or before each event index (per block), forward-filled
     wd = np.where(kind != EV_READ, np.arange(len(kind)), -1)

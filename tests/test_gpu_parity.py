@@ -289,6 +289,11 @@ def test_c3_full_size(mode, copy):
     pool = t.arena_bytes - t.budget_bytes + (2 << 30)
     g = _gpu(t, mode, copy=copy, host_pool_bytes=pool)
     assert_parity(t, mode, g)
+    # north_star: no block moved while discarded (the CUDA path's own transfer log)
+    from paper_conf_iiswc_zhucvhcr22_b200 import rmt
+    r = rmt.analyze(t, g["xlog"])
+    assert r["discarded_state_moves"] == 0
+    assert r["h2d_bytes"] == g["stats"]["h2d_bytes"] and r["d2h_bytes"] == g["stats"]["d2h_bytes"]
 
 
 @pytest.mark.parametrize("pressure", [False, True])
