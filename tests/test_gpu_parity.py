@@ -413,5 +413,5 @@ def test_c3_full_size_64k_blocks(copy):
     t = _full_size_trace(iterations=2, B=64 << 10)
     assert t.nblocks > 4_000_000
     pool = t.arena_bytes - t.budget_bytes + (2 << 30)
-    g = _gpu(t, "eager", copy=copy, host_pool_bytes=pool)
+    g = _gpu(t, "eager", copy=copy, host_pool_bytes=pool, xlog=False)   # ~10 M records: counters only
     assert_parity(t, "eager", g)
