@@ -19,9 +19,10 @@
  *
  * Execution.  All planning (state tables, victim selection, work-list compaction) runs
  * in sm_100a kernels on device-resident tables; data moves by a kernel-driven TMA copy
- * over mapped pinned host memory (K4, no host round trip) or, for large sub-ops, by the
- * copy engines from the device-made plan (K4-CE, one host round trip per sub-op).  No CPU
- * fallback: the host never computes a state, a victim or a transfer list.
+ * over mapped pinned host memory (K4, no host round trip) or, as the comparison arm
+ * (UM_F_COPY_CE), by the copy engines from the device-made plan (K4-CE, one host round
+ * trip per sub-op).  No CPU fallback: the host never computes a state, a victim or a
+ * transfer list.
  *
  * Conventions (all functions):
  *  - Return um_status; UM_OK = 0.  No exceptions cross the ABI.
@@ -108,6 +109,18 @@ typedef struct {
   uint32_t n_host_chunks;
   uint64_t host_chunk_bytes;  /* multiple of block_bytes                                   */
   uint32_t flags;             /* UM_F_*                                                    */
+  uint32_t page_bytes;        /* 0 or block_bytes: single level.  Otherwise two-level
+                                 granularity (PAPER §5.3-5.4): a
+                                 block is a chunk of block_bytes/page_bytes <= 32 pages
+                                 (page_bytes a power of two >= 16384).  Chunks stay the
+                                 residency and eviction unit (L198, L209, L217-221); a
+                                 discard covering only some pages of a chunk marks them
+                                 dead without unmapping (L211); dead pages are not written
+                                 back and are zero-filled instead of migrated (L196-200)
+                                 until accessed again (a touch revives eagerly discarded
+                                 pages, a prefetch any, A8/A17).  Byte counters and
+                                 content tags are per page.  Not combinable with
+                                 UM_F_COPY_CE or UM_F_OVERLAP (UM_EINVAL).                */
 } um_config;
 
 /* Counters (int64, 16 slots).  Byte counters are multiples of block_bytes. */
@@ -181,10 +194,16 @@ um_status um_get_stats(um_arena *a, um_stats *out);
 um_status um_dump(um_arena *a, uint8_t *st, uint32_t *used_order, uint32_t *n_used,
                   uint32_t *disc_order, uint32_t *n_disc);
 
-/* Harness: synchronizes; content tag of every block (u64 per block): 0 = all-zero
- * block, stamp s = block filled with the 16-byte pattern {s, ~s}, UINT64_MAX = anything
- * else (corrupt).  Reads frames (G/GE/GL) or host frames (H; HD/U read as zero). */
+/* Harness: synchronizes; content tag of every block (u64 per block; per page, nblocks *
+ * block_bytes/page_bytes entries, at two levels): 0 = all-zero, stamp s = filled with
+ * the 16-byte pattern {s, ~s}, UINT64_MAX = anything else (corrupt).  Reads frames
+ * (G/GE/GL) or host frames (H; HD/U and the dead pages of an H chunk read as zero). */
 um_status um_content_tags(um_arena *a, uint64_t *tags);
+
+/* Two-level arenas (page_bytes < block_bytes): synchronizes; per chunk, the dead-page
+ * and lazily-discarded-page masks (bit p = page p).  Either pointer may be NULL.
+ * UM_EINVAL on a single-level arena. */
+um_status um_page_masks(um_arena *a, uint32_t *dead, uint32_t *lazy);
 
 /* Synchronizes.  Device time (ms) spent since the last reset in planning kernels
  * (classify, victim selection, directives, ring compaction) and in the transfer engine

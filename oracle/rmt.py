@@ -53,9 +53,10 @@ def _full(B, off, ln):
     return range(lo, max(lo, (off + ln) // B))
 
 
-def data_events(trace):
-    """Per block: the ascending op indices of its data events and the events."""
-    B = trace.block_bytes
+def data_events(trace, unit=None):
+    """Per block (per page of `unit` bytes at two levels): the ascending op indices of
+    its data events and the events."""
+    B = unit or trace.block_bytes
     idx, ev = {}, {}
 
     def add(b, t, e):
@@ -124,14 +125,15 @@ def redundant(idx, ev, t, b):
     return None
 
 
-def rmt_analyze(trace, log, by_op=False, detail=False):
+def rmt_analyze(trace, log, by_op=False, detail=False, page_bytes=None):
     """Redundant bytes of one run.  `log`: (seq, kind, block, prev_state) records (or
     (op, kind, block, prev_state) with by_op=True).  Returns byte totals, redundant
     bytes per direction and reason, and the moves of blocks that were in a discarded
     state (HD, GE, GL) when they moved — the north_star target is none in discard mode.
-    detail=True adds the redundant records (op, kind, block, reason)."""
-    B = trace.block_bytes
-    idx, ev = data_events(trace)
+    detail=True adds the redundant records (op, kind, block, reason).  page_bytes: the
+    log is per page (oracle.chunks); blocks in it are global page indices."""
+    B = page_bytes or trace.block_bytes
+    idx, ev = data_events(trace, B)
     recs = log if by_op else log_by_op(trace, log)
     out = {"h2d_bytes": 0, "d2h_bytes": 0, "rmt_h2d_bytes": 0, "rmt_d2h_bytes": 0,
            "reasons": {"dead": 0, "overwritten": 0, "discarded": 0}, "discarded_state_moves": 0}

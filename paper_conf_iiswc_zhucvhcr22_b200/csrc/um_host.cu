@@ -33,6 +33,7 @@ struct Layout {
   uint64_t need, needk, needhf, victim, vframe, vhf, vkind, d2h_frame, d2h_hf;
   uint64_t tile_status, tile_cnt, tags, ctl, hchunks, stage, xitems, bounce;
   uint64_t obits, wbits, dlo, dpre, dw, vscratch, vpass;
+  uint64_t pdead, plazy, phz, d2h_dmask;
   uint64_t stage_bytes, max_tiles, cap, total, ce_group, bounce_bytes;
 };
 
@@ -44,8 +45,19 @@ static uint64_t pow2_ceil(uint64_t x) {
 
 static bool is_pow2(uint64_t x) { return x && !(x & (x - 1)); }
 
+// Pages per chunk: 1 at single level (page_bytes 0 or = block_bytes).
+static uint32_t cfg_ppc(const um_config* c) {
+  return (c->page_bytes == 0 || c->page_bytes == c->block_bytes) ? 1u : c->block_bytes / c->page_bytes;
+}
+
 static um_status check_cfg(const um_config* c) {
   if (!c) return UM_EINVAL;
+  if (c->page_bytes && c->page_bytes != c->block_bytes) {   // two-level granularity (NEXT-1)
+    if (!is_pow2(c->page_bytes) || c->page_bytes < kXferChunk || c->page_bytes > c->block_bytes ||
+        c->block_bytes / c->page_bytes > 32)
+      return UM_EINVAL;
+    if (c->flags & (UM_F_COPY_CE | UM_F_OVERLAP)) return UM_EINVAL;
+  }
   if (!is_pow2(c->block_bytes) || c->block_bytes < 4096) return UM_EINVAL;
   if (c->arena_bytes == 0 || c->arena_bytes % c->block_bytes) return UM_EINVAL;
   if (c->arena_bytes / c->block_bytes >= 0xffffffffull) return UM_EINVAL;
@@ -66,7 +78,9 @@ static Layout make_layout(const um_config* c) {
   // tiles: classify/directive scan <= nblocks items, compaction <= cap, the wide victim
   // scan <= |DISC| + |USED| <= 2 * cap (its bound is also clamped to 2 * cap)
   L.max_tiles = (std::max(nb, 2 * L.cap) + 2048 - 1) / 2048 + 1;   // smallest scan tile: 2048 items
-  L.stage_bytes = std::min<uint64_t>(64ull << 20, 12 * nb + (1 << 20));
+  const uint64_t ppc = cfg_ppc(c);
+  // staged touch lists: 12 B per distinct block at two levels (chunk, cover, write masks)
+  L.stage_bytes = std::min<uint64_t>(64ull << 20, (ppc > 1 ? 24 : 12) * nb + (1 << 20));
   uint64_t o = 0;
   auto take = [&](uint64_t bytes) {
     uint64_t r = o;
@@ -95,7 +109,7 @@ static Layout make_layout(const um_config* c) {
   L.d2h_hf = take(4 * nf);
   L.tile_status = take(8 * L.max_tiles);
   L.tile_cnt = take(32 * L.max_tiles);
-  L.tags = take(8 * nb);
+  L.tags = take(8 * nb * ppc);   // content tags: per page
   L.ctl = take(sizeof(Ctl));
   L.hchunks = take(8ull * c->n_host_chunks);
   L.stage = take(L.stage_bytes);
@@ -111,6 +125,12 @@ static Layout make_layout(const um_config* c) {
   L.dlo = take(4 * nb);
   L.dpre = take(4 * (nb + 1));
   L.dw = take(nb);
+  L.d2h_dmask = take(4 * nf);
+  if (ppc > 1) {
+    L.pdead = take(4 * nb);
+    L.plazy = take(4 * nb);
+    L.phz = take(4 * nb);
+  }
   L.total = o;
   return L;
 }
@@ -199,6 +219,11 @@ struct Iv {
   uint8_t w;
 };
 
+// Two-level touch / prefetch list item: a chunk, the pages the op covers and writes.
+struct CItem {
+  uint32_t c, cm, wm;
+};
+
 }  // namespace
 
 struct um_arena {
@@ -230,6 +255,8 @@ struct um_arena {
   Stager stage;
   Ctl* hctl = nullptr;  // pinned mirror for reads
   std::vector<Iv> ivs;
+  std::vector<CItem> citems;   // two-level: the op's chunks with page masks
+  uint32_t ppc = 1, P = 0;     // pages per chunk, page bytes (single level: 1, B)
   // UM_F_TIMING: event pairs around planning / transfer launches
   struct Span { cudaEvent_t a, b; int xfer; uint32_t seq; };
   std::vector<Span> spans;
@@ -477,6 +504,7 @@ static void build_intervals(um_arena* a, const um_access* acc, uint32_t n) {
 // comparison arm, selected with UM_F_COPY_CE (or, for A/B runs only, for sub-ops of at
 // least UM_CE_MIN_BYTES).
 static bool use_ce(um_arena* a, uint64_t n) {
+  if (a->ppc > 1) return false;   // two-level: page-granular transfers run in K4 only
   if (a->cfg.flags & UM_F_COPY_CE) return true;
   if (a->cfg.flags & UM_F_COPY_KERNEL) return false;
   return n * a->B >= a->ce_min_bytes;
@@ -888,6 +916,115 @@ static um_status run_gpu_op(um_arena* a, int touch) {
   return UM_OK;
 }
 
+// ---- two-level granularity ------------------------------------------
+// Pages [p0, p1) (global page indices) of chunk c as the chunk's page mask.
+static uint32_t chunk_mask(const um_arena* a, uint64_t c, uint64_t p0, uint64_t p1) {
+  const uint64_t c0 = c * a->ppc;
+  const uint32_t lo = p0 > c0 ? (uint32_t)(p0 - c0) : 0u;
+  const uint32_t hi = p1 < c0 + a->ppc ? (uint32_t)(p1 - c0) : a->ppc;
+  return (hi >= 32 ? 0xffffffffu : ((1u << hi) - 1u)) & ~((1u << lo) - 1u);
+}
+
+// Append the chunks overlapping byte range [off, off+len) with their page masks.
+static void add_range(um_arena* a, uint64_t off, uint64_t len, bool w) {
+  if (!len) return;
+  const uint64_t p0 = off / a->P, p1 = (off + len - 1) / a->P + 1;
+  for (uint64_t c = p0 / a->ppc; c <= (p1 - 1) / a->ppc; ++c) {
+    const uint32_t m = chunk_mask(a, c, p0, p1);
+    a->citems.push_back({(uint32_t)c, m, w ? m : 0u});
+  }
+}
+
+// Sort by chunk and merge duplicates (argument marshalling: which pages the op names).
+static void finish_citems(um_arena* a) {
+  auto& v = a->citems;
+  std::sort(v.begin(), v.end(), [](const CItem& x, const CItem& y) { return x.c < y.c; });
+  size_t k = 0;
+  for (size_t i = 0; i < v.size(); ++i) {
+    if (k && v[k - 1].c == v[i].c) {
+      v[k - 1].cm |= v[i].cm;
+      v[k - 1].wm |= v[i].wm;
+    } else {
+      v[k++] = v[i];
+    }
+  }
+  v.resize(k);
+}
+
+// Two-level GPU-destination op over a->citems: the chunk-level chain of run_gpu_op in the
+// list form (classify / victims unchanged), the page-aware transfer kernel, then the page
+// revive of the op's cover masks, then the application kernel on the written pages.
+static um_status run_gpu_op2(um_arena* a, int touch) {
+  const uint64_t total = a->citems.size();
+  bool anyw = false;
+  for (const CItem& x : a->citems) anyw |= x.wm != 0;
+  {
+    um_status sr = seq_room(a, total ? (total + a->nframes - 1) / a->nframes : 1);
+    if (sr) return sr;
+  }
+  a->ops++;
+  if (total == 0) {
+    a->clock++;
+    a->subops++;
+    return UM_OK;
+  }
+  const uint64_t arr = (4 * total + 15) & ~15ull;
+  uint64_t off;
+  CK(a->stage.reserve(3 * arr, &off));
+  uint32_t* hb = (uint32_t*)(a->stage.host + off);
+  uint32_t* hc = (uint32_t*)(a->stage.host + off + arr);
+  uint32_t* hw = (uint32_t*)(a->stage.host + off + 2 * arr);
+  for (uint64_t g = 0; g < total; ++g) {
+    const CItem& x = a->citems[g];
+    hb[g] = x.c | (x.wm ? 0x80000000u : 0u);
+    hc[g] = x.cm;
+    hw[g] = x.wm;
+  }
+  CK(a->stage.push(off, 3 * arr, a->ps));
+  OpIv iv{};
+  iv.m = (uint32_t)total;
+  iv.blist = (const uint32_t*)(a->stage.dev + off);
+  iv.pcov = (const uint32_t*)(a->stage.dev + off + arr);
+  iv.pw = (const uint32_t*)(a->stage.dev + off + 2 * arr);
+  const uint32_t F = a->nframes;
+  for (uint64_t g0 = 0; g0 < total; g0 += F) {
+    const uint32_t n = (uint32_t)std::min<uint64_t>(F, total - g0);
+    const uint32_t seq = ++a->clock;
+    a->subops++;
+    um_status st = ensure_ring_room(a, RING_USED, n);
+    if (st) return st;
+    a->T.pfloor = seq;
+    cudaEvent_t sp = span_open(a);
+    const uint64_t tail0 = a->tail[RING_USED];
+    a->tail[RING_USED] += n;
+    if (n <= kSmallPlan) {
+      CK(launch_plan_small(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->ps));
+      a->n_launch += 1;
+    } else {
+      CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->npar, a->ps));
+      if (n > kVictWideMin)
+        CK(launch_victims_wide(a->T, seq, 0, 0, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), n,
+                               a->npar, a->ps));
+      else
+        CK(launch_victims(a->T, seq, 0, 0, a->npar, a->ps));
+      a->npar ^= 1;
+      a->n_launch += n > kVictWideMin ? 3 : 2;
+    }
+    span_close(a, sp, 0);
+    sp = span_open(a);
+    CK(launch_service(a->T, SVC_SUBOP, seq, n, a->ps));
+    span_close(a, sp, 1);
+    CK(launch_page_revive(a->T, iv, (uint32_t)g0, n, touch, a->ps));
+    a->n_launch += 2;
+    a->n_xfer++;
+    if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP)) {
+      CK(launch_app_stamp(a->T, iv, (uint32_t)g0, n, seq, 8, a->ps));
+      a->n_launch++;
+    }
+  }
+  return UM_OK;
+}
+
 }  // namespace
 
 // =====================================================================================
@@ -968,6 +1105,16 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   T.dlo = (uint32_t*)(ws + L.dlo);
   T.dpre = (uint32_t*)(ws + L.dpre);
   T.dw = (uint8_t*)(ws + L.dw);
+  T.d2h_dmask = (uint32_t*)(ws + L.d2h_dmask);
+  a->ppc = cfg_ppc(cfg);
+  a->P = cfg->block_bytes / a->ppc;
+  T.ppc = a->ppc;
+  T.P = a->P;
+  if (a->ppc > 1) {
+    T.pdead = (uint32_t*)(ws + L.pdead);
+    T.plazy = (uint32_t*)(ws + L.plazy);
+    T.phz = (uint32_t*)(ws + L.phz);
+  }
   a->bounce = ws + L.bounce;
   T.frames = (char*)cfg->frames;
   T.hpc = hpc;
@@ -1077,6 +1224,14 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
     if (!range_ok(a, acc[i].off, acc[i].len)) return UM_EINVAL;
   um_status s = hand_in(a, stream);
   if (s) return s;
+  if (a->ppc > 1) {   // two-level: the chunks with the pages each record covers / writes
+    a->citems.clear();
+    for (uint32_t i = 0; i < n; ++i) add_range(a, acc[i].off, acc[i].len, (acc[i].kind & UM_ACC_WRITE) != 0);
+    finish_citems(a);
+    s = run_gpu_op2(a, 1);
+    if (s) return s;
+    return hand_out(a, stream);
+  }
   // a batch of more records than fit inline that is not already sorted and disjoint is
   // deduplicated on the device; otherwise the records (or the <= kIvInline records after a
   // 2n-event merge while they are packed into the kernel arguments) are the intervals
@@ -1098,7 +1253,12 @@ UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, v
   if (!range_ok(a, off, len) || (dst != UM_DST_GPU && dst != UM_DST_HOST)) return UM_EINVAL;
   um_status s = hand_in(a, stream);
   if (s) return s;
-  if (dst == UM_DST_GPU) {
+  if (dst == UM_DST_GPU && a->ppc > 1) {
+    a->citems.clear();
+    add_range(a, off, len, false);
+    s = run_gpu_op2(a, 0);
+    if (s) return s;
+  } else if (dst == UM_DST_GPU) {
     a->ivs.clear();
     if (len) {
       uint64_t lo = off / a->B, hi = (off + len - 1) / a->B + 1;
@@ -1129,6 +1289,10 @@ UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, v
       span_close(a, sp, 1);
       a->n_launch += 2;
       a->n_xfer++;
+      if (a->ppc > 1) {   // revalidate the covered pages (A17); revived dead pages read zero
+        CK(launch_page_host_revive(a->T, lo, hi - lo, off / a->P, (off + len - 1) / a->P + 1, a->ps));
+        a->n_launch++;
+      }
     }
   }
   return hand_out(a, stream);
@@ -1159,6 +1323,27 @@ static um_status discard_common(um_arena* a, uint64_t off, uint64_t len, void* s
       CK(launch_directive(a->T, kind, (uint32_t)c0, n, seq, 0, tail0, a->ps));
       span_close(a, sp, 0);
       a->n_launch++;
+    }
+  }
+  if (a->ppc > 1 && !(a->cfg.flags & UM_F_DISCARD_OFF)) {
+    // pages fully inside the range whose chunk is not (at most the two edge chunks):
+    // marked dead without unmapping (§5.4)
+    const uint64_t pp0 = (off + a->P - 1) / a->P, pp1 = (off + len) / a->P;
+    if (pp1 > pp0) {
+      uint32_t ce[2] = {UM_NONE, UM_NONE}, me[2] = {0u, 0u};
+      int k = 0;
+      const uint64_t cand[2] = {pp0 / a->ppc, (pp1 - 1) / a->ppc};
+      for (int i = 0; i < 2; ++i) {
+        const uint64_t c = cand[i];
+        if ((i == 1 && c == cand[0]) || (c >= lo && c < hi)) continue;
+        ce[k] = (uint32_t)c;
+        me[k] = chunk_mask(a, c, pp0, pp1);
+        ++k;
+      }
+      if (k) {
+        CK(launch_page_discard(a->T, ce[0], me[0], ce[1], me[1], kind == DIR_DISCARD_LAZY, a->ps));
+        a->n_launch++;
+      }
     }
   }
   return hand_out(a, stream);
@@ -1215,9 +1400,8 @@ UM_API um_status um_host_write(um_arena* a, uint64_t off, uint64_t len, void* st
   a->ops++;
   a->subops++;
   const uint32_t seq = ++a->clock;
-  if (len) {
-    uint32_t lo = (uint32_t)(off / a->B), hi = (uint32_t)((off + len - 1) / a->B + 1);
-    CK(launch_host_write(a->T, lo, hi - lo, seq, a->ps));
+  if (len) {   // pages (= blocks at single level) overlapping the range
+    CK(launch_host_write(a->T, off / a->P, (off + len - 1) / a->P + 1, seq, a->ps));
     a->n_launch += 2;
   }
   return hand_out(a, stream);
@@ -1310,8 +1494,18 @@ UM_API um_status um_content_tags(um_arena* a, uint64_t* tags) {
     if (s) return s;
   }
   CK(launch_tags(a->T, a->ps));
-  CK(cudaMemcpyAsync(tags, a->T.tags, 8ull * a->nblocks, cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaMemcpyAsync(tags, a->T.tags, 8ull * a->nblocks * a->ppc, cudaMemcpyDeviceToHost, a->ps));
   CK(cudaStreamSynchronize(a->ps));
+  return UM_OK;
+}
+
+UM_API um_status um_page_masks(um_arena* a, uint32_t* dead, uint32_t* lazy) {
+  ENTER(a);
+  if (a->ppc <= 1) return UM_EINVAL;
+  um_status s = sync_ctl(a);
+  if (s) return s;
+  if (dead) CK(cudaMemcpy(dead, a->T.pdead, 4ull * a->nblocks, cudaMemcpyDeviceToHost));
+  if (lazy) CK(cudaMemcpy(lazy, a->T.plazy, 4ull * a->nblocks, cudaMemcpyDeviceToHost));
   return UM_OK;
 }
 

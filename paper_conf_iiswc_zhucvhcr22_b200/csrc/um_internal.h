@@ -115,6 +115,19 @@ struct Tables {
   // transfer log (null = off): {seq, block, XL_* kind, state before the move}
   uint4* xlog;
   unsigned long long xlog_cap;
+  // Two-level granularity (null = single level): a block is
+  // a chunk of ppc pages of P bytes.  Per chunk, bit p = page p:
+  //   pdead  pages discarded while the chunk itself is not (G or H only): not written
+  //          back, zero-filled instead of migrated
+  //   plazy  the subset discarded lazily (revived by a prefetch only, A8 / A17)
+  //   phz    pages of an H chunk whose host content is logically zero (released or never
+  //          written host pages that became live again): migrated from the zero page
+  uint32_t* pdead;
+  uint32_t* plazy;
+  uint32_t* phz;
+  uint32_t* d2h_dmask;  // [nframes] dead-page mask of each D2H-only item (when it was listed)
+  uint32_t ppc;         // pages per chunk (1 = single level)
+  uint32_t P;           // page bytes (= B at single level)
 };
 
 // A GPU-destination op's distinct blocks as sorted disjoint intervals.  Interval j
@@ -136,6 +149,8 @@ struct OpIv {
                          // batch): item g's block is one coalesced load, no interval lookup
   const uint32_t* tj;   // staged lists: per tile of the current sub-op, the interval slice
                         // [tj[2t], tj[2t+1]] its items fall in (host-computed, no search)
+  const uint32_t* pcov; // two-level (with blist): per item, the chunk's pages the op covers
+  const uint32_t* pw;   // two-level (with blist): per item, the chunk's pages it writes
   uint32_t m;
   uint32_t inl;
   uint32_t ilo[kIvInline];
@@ -182,11 +197,21 @@ cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, 
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
                              int discard_off, unsigned long long tail0, cudaStream_t s);
 cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64_t cap_bound, cudaStream_t s);
-cudaError_t launch_host_write(const Tables& T, uint32_t lo, uint32_t n, uint32_t seq, cudaStream_t s);
+// Harness host write of pages [p0, p1) (global page indices; p = block at single level).
+cudaError_t launch_host_write(const Tables& T, uint64_t p0, uint64_t p1, uint32_t seq, cudaStream_t s);
 cudaError_t launch_tags(const Tables& T, cudaStream_t s);
 cudaError_t launch_plan_commit(const Tables& T, uint32_t seq, uint32_t max_items, cudaStream_t s);
 cudaError_t launch_zero_items(const Tables& T, uint32_t i0, uint32_t i1, cudaStream_t s);
 cudaError_t launch_poison(const Tables& T, cudaStream_t s);
+// Two-level page masks (NEXT-1).  After a GPU sub-op: revive the pages it covers
+// (touch: eagerly discarded pages only; prefetch: all, clearing lazy).  After a
+// prefetch(HOST) of chunks [lo, lo+n) covering pages [p0, p1) (global): revive, and mark
+// revived pages of host chunks zero.  A discard's partial edge chunk c: pages m.
+cudaError_t launch_page_revive(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, int touch, cudaStream_t s);
+cudaError_t launch_page_host_revive(const Tables& T, uint32_t lo, uint32_t n, uint64_t p0, uint64_t p1,
+                                    cudaStream_t s);
+cudaError_t launch_page_discard(const Tables& T, uint32_t c0, uint32_t m0, uint32_t c1, uint32_t m1, int lazy,
+                                cudaStream_t s);
 // Device intake: mark a staged record chunk into the op bitmaps; turn the bitmap words
 // [w0, w1) into sorted disjoint intervals (dlo/dpre/dw, ctl->iv_m / iv_d); clear them.
 // Records must not cover more than kMarkMaxBlocks blocks each (the host splits them).

@@ -77,6 +77,24 @@ __device__ __forceinline__ void xlog_put(const Tables& T, uint32_t seq, uint32_t
   if (p < T.xlog_cap) T.xlog[p] = make_uint4(seq, blk, kind, prev);
 }
 
+// A G block b entering the D2H-only list (prefetch HOST, evict) at position pos: its
+// dead pages (two-level) are recorded for the service kernel and not counted as moved.
+__device__ __forceinline__ void d2h_listed(const Tables& T, uint32_t seq, uint32_t b, uint32_t pos, uint32_t prev) {
+  uint32_t dm = 0u;
+  if (T.pdead) {
+    dm = T.pdead[b];
+    T.d2h_dmask[pos] = dm;
+    if (dm) {
+      const long long d = (long long)__popc(dm) * T.P;
+      stat_add(T, S_D2H, -d);
+      stat_add(T, S_D2H_AV, d);
+    }
+  }
+  if (T.xlog)
+    for (uint32_t p = 0; p < T.ppc; ++p)
+      if (!((dm >> p) & 1u)) xlog_put(T, seq, b * T.ppc + p, XL_D2H, prev);
+}
+
 // Exclusive block scan of a 64-bit value (two packed 31-bit counts add without carry).
 template <int TPB>
 __device__ __forceinline__ unsigned long long block_excl_scan(unsigned long long v, unsigned long long& total,
@@ -902,7 +920,7 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
         if (isG) {
           T.d2h_frame[gr] = fr;
           T.d2h_hf[gr] = hf;
-          xlog_put(T, seq, v, XL_D2H, ss);
+          d2h_listed(T, seq, v, gr, ss);
         }
       }
     }
@@ -1318,7 +1336,7 @@ __global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict
               const uint32_t d = db + rD + __popc(bD[q] & lt);
               T.d2h_frame[d] = fr[q];
               T.d2h_hf[d] = hf[q];
-              xlog_put(T, seq, v[q], XL_D2H, ss[q]);
+              d2h_listed(T, seq, v[q], d, ss[q]);
             }
           }
         }
@@ -1411,6 +1429,7 @@ __device__ __forceinline__ void item_commit(const Tables& T, uint32_t i, const X
   T.frame_of[bb] = x.fr;
   T.map[bb] = x.fr;
   const uint32_t hf = T.needhf[i];
+  if (T.phz && T.needk[i] == ST_H) T.phz[bb] = 0u;   // its pages now live in the frame
   if (T.needk[i] == ST_H && hf != UM_NONE) {
     T.hframe[bb] = UM_NONE;
     if (!(x.flags & XI_SWAP)) {
@@ -1420,12 +1439,55 @@ __device__ __forceinline__ void item_commit(const Tables& T, uint32_t i, const X
   }
 }
 
-// Transfer-log records of need item i: the newcomer's migration or zero-fill and, when
-// its frame comes from a valid victim, the victim's write-back.
-__device__ __forceinline__ void item_log(const Tables& T, uint32_t i, const XItem& x, uint32_t seq, uint32_t f0) {
+// Page masks of need item i (two-level, NEXT-1; all zero at single level): the
+// newcomer's dead pages (zero-filled instead of migrated) and zero-content
+// pages (migrated from the zero page) when it comes from the host, and the dead pages of
+// the victim whose frame it takes (not written back, L196-198).
+struct ItemPages { uint32_t ndead, nhz, vdead; };
+__device__ __forceinline__ ItemPages item_pages(const Tables& T, uint32_t i, const XItem& x, uint32_t f0) {
+  ItemPages m{0u, 0u, 0u};
+  if (!T.pdead) return m;
+  if (x.flags & XI_H2D) {
+    const uint32_t b = T.need[i];
+    m.ndead = T.pdead[b];
+    m.nhz = T.phz[b];
+  }
+  if (x.flags & XI_D2H) m.vdead = T.pdead[T.victim[i - f0]];
+  return m;
+}
+
+// Transfer-log records of need item i (one per page at two levels): the newcomer's
+// migration or zero-fill and, when its frame comes from a valid victim, the victim's
+// write-back of its live pages.
+__device__ __forceinline__ void item_log(const Tables& T, uint32_t i, const XItem& x, uint32_t seq, uint32_t f0,
+                                         const ItemPages& m) {
   if (!T.xlog) return;
-  xlog_put(T, seq, T.need[i], (x.flags & XI_H2D) ? XL_H2D : XL_ZF, T.needk[i]);
-  if (x.flags & XI_D2H) xlog_put(T, seq, T.victim[i - f0], XL_D2H, T.vkind[i - f0]);
+  const uint32_t b = T.need[i], k = T.needk[i];
+  for (uint32_t p = 0; p < T.ppc; ++p)
+    xlog_put(T, seq, b * T.ppc + p, ((x.flags & XI_H2D) && !((m.ndead >> p) & 1u)) ? XL_H2D : XL_ZF, k);
+  if (x.flags & XI_D2H) {
+    const uint32_t v = T.victim[i - f0];
+    for (uint32_t p = 0; p < T.ppc; ++p)
+      if (!((m.vdead >> p) & 1u)) xlog_put(T, seq, v * T.ppc + p, XL_D2H, T.vkind[i - f0]);
+  }
+}
+
+// Two-level byte counters: the planning kernels count whole chunks; dead pages of a
+// migrating newcomer are zero-filled instead (h2d -> zf + h2d_avoided) and dead pages
+// of a written-back victim are not moved (d2h -> d2h_avoided).
+__device__ __forceinline__ void item_page_stats(const Tables& T, const ItemPages& m) {
+  const long long P = T.P;
+  if (m.ndead) {
+    const long long d = (long long)__popc(m.ndead) * P;
+    stat_add(T, S_H2D, -d);
+    stat_add(T, S_ZF, d);
+    stat_add(T, S_H2D_AV, d);
+  }
+  if (m.vdead) {
+    const long long d = (long long)__popc(m.vdead) * P;
+    stat_add(T, S_D2H, -d);
+    stat_add(T, S_D2H_AV, d);
+  }
 }
 
 struct Unit {
@@ -1463,6 +1525,8 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
 
     uint32_t cached_i = UM_NONE;
     XItem cached;
+    ItemPages cpg{0u, 0u, 0u};
+    const uint32_t upp = T.P / CH;   // units per page (ppc = 1: one page = the block)
     // phase 1 commits pure zero-fill items, phase 2 all others (each exactly once)
     auto make = [&](unsigned long long t, int phase) -> Unit {
       unsigned long long u = ubeg + t;
@@ -1472,21 +1536,26 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
       if (mode == SVC_SUBOP) {
         if (i != cached_i) {
           cached = item_plan(T, i, f0, nfu);
+          cpg = item_pages(T, i, cached, f0);
           cached_i = i;
         }
         const XItem& p = cached;
+        const uint32_t pg = ch / upp;
         x.frame = T.frames + (size_t)p.fr * T.B + coff;
-        x.d2h_dst = (p.flags & XI_D2H) ? hptr(T, p.dst_hf) + coff : nullptr;
-        x.h2d_src = (p.flags & XI_H2D) ? hptr(T, p.src_hf) + coff : nullptr;
-        x.zf = (p.flags & XI_ZF) != 0;
+        x.d2h_dst = ((p.flags & XI_D2H) && !((cpg.vdead >> pg) & 1u)) ? hptr(T, p.dst_hf) + coff : nullptr;
+        const bool mig = (p.flags & XI_H2D) && !((cpg.ndead >> pg) & 1u);
+        x.h2d_src = mig ? hptr(T, ((cpg.nhz >> pg) & 1u) ? T.zero_hf : p.src_hf) + coff : nullptr;
+        x.zf = !mig;
         if (ch == 0 && (x.pure_zf() ? 1 : 2) == phase) {
-          item_log(T, i, p, seq, f0);
+          item_log(T, i, p, seq, f0, cpg);
+          item_page_stats(T, cpg);
           item_commit(T, i, p, seq);
         }
       } else {
         uint32_t fr = T.d2h_frame[i], hf = T.d2h_hf[i];
+        const uint32_t dm = T.pdead ? T.d2h_dmask[i] : 0u;
         x.frame = T.frames + (size_t)fr * T.B + coff;
-        x.d2h_dst = hf != UM_NONE ? hptr(T, hf) + coff : nullptr;
+        x.d2h_dst = (hf != UM_NONE && !((dm >> (ch / upp)) & 1u)) ? hptr(T, hf) + coff : nullptr;
         x.h2d_src = nullptr;
         x.zf = false;
       }
@@ -1568,7 +1637,7 @@ __global__ void k_plan_commit(Tables T, uint32_t seq) {
     XItem x = item_plan(T, i, f0, nfu);
     T.xitems[i] = x;
     T.hx[i] = x;            // pinned host mirror (mapped)
-    item_log(T, i, x, seq, f0);
+    item_log(T, i, x, seq, f0, ItemPages{0u, 0u, 0u});   // single level only
     item_commit(T, i, x, seq);
   }
   // every thread's plan writes are performed system-wide before its CTA takes a ticket;
@@ -1629,19 +1698,21 @@ template <int TPB>
 __global__ void __launch_bounds__(TPB) k_app_stamp(Tables T, const __grid_constant__ OpIv iv, uint32_t g0, uint32_t n, uint32_t seq) {
   pdl_enter();
   __shared__ char* s_dst;
-  __shared__ uint32_t s_blk;
-  const uint32_t SEG = T.B < kFillSeg ? T.B : kFillSeg;
-  const uint32_t spb = T.B / SEG;
+  __shared__ uint32_t s_q;
+  // segments never straddle a page (P = B at single level), so a segment has one stamp
+  const uint32_t SEG = T.P < kFillSeg ? T.P : kFillSeg;
+  const uint32_t spb = T.B / SEG, spp = T.P / SEG;
   const unsigned long long units = (unsigned long long)n * spb;
   for (unsigned long long u = blockIdx.x; u < units; u += gridDim.x) {
     if (threadIdx.x == 0) {
       uint32_t g = g0 + (uint32_t)(u / spb);
+      const uint32_t sg = (uint32_t)(u % spb), pg = sg / spp;
       char* d = nullptr;
       uint32_t bb, wr;
       if (iv.blist) {
         const uint32_t e = iv.blist[g];
         bb = e & 0x7fffffffu;
-        wr = e >> 31;
+        wr = iv.pw ? (iv.pw[g] >> pg) & 1u : e >> 31;   // two-level: the pages it writes
       } else {
         const uint32_t j = iv_find(iv, g);
         bb = iv_lo(iv, j) + (g - iv_pre(iv, j));
@@ -1649,18 +1720,78 @@ __global__ void __launch_bounds__(TPB) k_app_stamp(Tables T, const __grid_consta
       }
       if (wr) {
         uint32_t fr = T.frame_of[bb];
-        if (fr != UM_NONE) d = T.frames + (size_t)fr * T.B + (size_t)(u % spb) * SEG;
+        if (fr != UM_NONE) d = T.frames + (size_t)fr * T.B + (size_t)sg * SEG;
       }
       s_dst = d;
-      s_blk = bb;
+      s_q = bb * T.ppc + pg;   // content stamps are per page (= per block at single level)
     }
     __syncthreads();
     char* d = s_dst;
-    const unsigned long long sv = ((unsigned long long)seq << 32) | s_blk;
+    const unsigned long long sv = ((unsigned long long)seq << 32) | s_q;
     __syncthreads();
     if (d) fill_segment<TPB>(reinterpret_cast<uint4*>(d), SEG / 16,
                              make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32)));
   }
+}
+
+// ------------------------------------------------------------------------------------
+// Two-level page masks (oracle/chunks.py).  Chunks stay the
+// residency / eviction unit; pages discarded while their chunk is not are tracked in
+// pdead (plazy: the lazily discarded subset) and skipped by the transfer engine.
+// ------------------------------------------------------------------------------------
+// After a GPU sub-op: a touch revives the eagerly discarded pages it covers ("skip the
+// memory transfers ... until it gets accessed again", L196); a lazily discarded page
+// needs the prefetch (L186-190, A8); a prefetch revives every page it covers (A17).
+__global__ void __launch_bounds__(256) k_page_revive(Tables T, const __grid_constant__ OpIv iv, uint32_t g0, uint32_t n,
+                                                     int touch) {
+  pdl_enter();
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const uint32_t g = g0 + i, c = iv.blist[g] & 0x7fffffffu, cm = iv.pcov[g];
+    const uint32_t d = T.pdead[c];
+    if (!(d & cm)) continue;
+    if (touch) {
+      T.pdead[c] = d & ~(cm & ~T.plazy[c]);
+    } else {
+      T.pdead[c] = d & ~cm;
+      T.plazy[c] &= ~cm;
+    }
+  }
+}
+
+// After a prefetch(HOST) of chunks [lo, lo + n) covering global pages [p0, p1): every
+// chunk is now H; the pages covered are revalidated (A17), and a revalidated dead page
+// holds no data on the host (it was never written back, or its host copy was released:
+// R1), so it reads as zero and migrates from the zero page.
+__global__ void __launch_bounds__(256) k_page_host_revive(Tables T, uint32_t lo, uint32_t n, unsigned long long p0,
+                                                          unsigned long long p1) {
+  pdl_enter();
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const uint32_t c = lo + i;
+    const unsigned long long c0 = (unsigned long long)c * T.ppc;
+    const uint32_t a = p0 > c0 ? (uint32_t)(p0 - c0) : 0u;
+    const uint32_t e = p1 < c0 + T.ppc ? (uint32_t)(p1 - c0) : T.ppc;
+    const uint32_t cm = (e >= 32 ? 0xffffffffu : ((1u << e) - 1u)) & ~((1u << a) - 1u);
+    const uint32_t d = T.pdead[c];
+    if (!(d & cm)) continue;
+    T.pdead[c] = d & ~cm;
+    T.plazy[c] &= ~cm;
+    T.phz[c] |= d & cm;
+  }
+}
+
+// A discard covering only pages m of chunk c (its edge chunks; whole chunks are
+// handled at chunk level by k_directive): G or H chunks mark the pages dead without
+// unmapping or re-queueing ("avoid splitting 2MB GPU mappings", §5.4).
+__global__ void k_page_discard(Tables T, uint32_t c0, uint32_t m0, uint32_t c1, uint32_t m1, int lazy) {
+  pdl_enter();
+  const uint32_t c = threadIdx.x == 0 ? c0 : c1, m = threadIdx.x == 0 ? m0 : m1;
+  if (threadIdx.x > 1 || c == UM_NONE || !m) return;
+  const uint8_t ss = ld_st(T, c);
+  if (ss != ST_G && ss != ST_H) return;
+  const uint32_t d = T.pdead[c];
+  if (lazy) T.plazy[c] |= m & ~d;
+  else T.plazy[c] &= ~m;
+  T.pdead[c] = d | m;
 }
 
 // ------------------------------------------------------------------------------------
@@ -1759,6 +1890,7 @@ __device__ __forceinline__ void directive_body(const Tables& T, int kind, uint32
       const uint8_t ss = s[k];
       if (disc) {
         T.disc_ring[(tail0 + idx) & T.cap_mask] = kseq | bb;
+        if (T.pdead) T.pdead[bb] = T.plazy[bb] = T.phz[bb] = 0u;   // whole chunk: chunk level
         if (ss == ST_G) {
           T.sk[bb] = mk_sk(kind == DIR_DISCARD ? ST_GE : ST_GL, seq);
           if (kind == DIR_DISCARD) {
@@ -1785,7 +1917,7 @@ __device__ __forceinline__ void directive_body(const Tables& T, int kind, uint32
             T.d2h_frame[s_db + rA] = fr;
             T.d2h_hf[s_db + rA] = hf;
             T.hframe[bb] = hf;
-            xlog_put(T, seq, bb, XL_D2H, ss);
+            d2h_listed(T, seq, bb, s_db + rA, ss);
             ++rA;
             ++nD2H;
           } else {
@@ -1977,36 +2109,57 @@ __global__ void __launch_bounds__(256) k_intake_clear(Tables T, uint32_t w0, uin
 // ------------------------------------------------------------------------------------
 // Harness: host writes (Listing 6 "Generate data, labels").
 // ------------------------------------------------------------------------------------
-__global__ void k_hw_alloc(Tables T, uint32_t lo, uint32_t n) {
+// Pages [p0, p1) of chunk c (global page indices) as a mask of the chunk's pages.
+__device__ __forceinline__ uint32_t chunk_mask(const Tables& T, uint32_t c, unsigned long long p0, unsigned long long p1) {
+  const unsigned long long c0 = (unsigned long long)c * T.ppc;
+  const uint32_t a = p0 > c0 ? (uint32_t)(p0 - c0) : 0u;
+  const uint32_t e = p1 < c0 + T.ppc ? (uint32_t)(p1 - c0) : T.ppc;
+  return (e >= 32 ? 0xffffffffu : ((1u << e) - 1u)) & ~((1u << a) - 1u);
+}
+
+// Host write of pages [p0, p1): chunks [lo, lo + n) must be H; a chunk without a host
+// frame (zero content) gets one, and its pages the write does not cover stay logically
+// zero (phz).  The written pages become live (not dead, not zero).
+__global__ void k_hw_alloc(Tables T, uint32_t lo, uint32_t n, unsigned long long p0, unsigned long long p1) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
     uint32_t bb = lo + i;
     if (ld_st(T, bb) != ST_H) {
       atomicExch(&T.ctl->err, 1u);
       continue;
     }
+    const uint32_t m = T.pdead ? chunk_mask(T, bb, p0, p1) : 0u;
+    bool fresh = false;
     if (T.hframe[bb] == UM_NONE) {
       int idx = atomicSub(&T.ctl->hfree_top, 1) - 1;
       if (idx >= 0) {
         T.hframe[bb] = T.hfree_stack[idx];
+        fresh = true;
       } else {
         atomicAdd(&T.ctl->hfree_top, 1);
         atomicExch(&T.ctl->err, 2u);
       }
     }
+    if (T.pdead) {
+      const uint32_t full = T.ppc >= 32 ? 0xffffffffu : ((1u << T.ppc) - 1u);
+      T.phz[bb] = fresh ? (full & ~m) : (T.phz[bb] & ~m);
+      T.pdead[bb] &= ~m;
+      T.plazy[bb] &= ~m;
+    }
   }
 }
 
-__global__ void __launch_bounds__(256) k_hw_fill(Tables T, uint32_t lo, uint32_t n, uint32_t seq) {
-  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
-  const uint32_t cpb = T.B / CH;
-  const unsigned long long units = (unsigned long long)n * cpb;
+__global__ void __launch_bounds__(256) k_hw_fill(Tables T, unsigned long long p0, unsigned long long p1, uint32_t seq) {
+  const uint32_t CH = T.P < kXferChunk ? T.P : kXferChunk;
+  const uint32_t cpp = T.P / CH;
+  const unsigned long long units = (p1 - p0) * cpp;
   for (unsigned long long u = blockIdx.x; u < units; u += gridDim.x) {
-    uint32_t bb = lo + (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
+    const unsigned long long q = p0 + u / cpp;   // global page
+    const uint32_t bb = (uint32_t)(q / T.ppc), pg = (uint32_t)(q % T.ppc), ch = (uint32_t)(u % cpp);
     uint32_t hf = T.hframe[bb];
     if (hf == UM_NONE || ld_st(T, bb) != ST_H) continue;
-    unsigned long long sv = ((unsigned long long)seq << 32) | bb;
+    unsigned long long sv = ((unsigned long long)seq << 32) | (uint32_t)q;
     uint4 pat = make_uint4((uint32_t)sv, (uint32_t)(sv >> 32), ~(uint32_t)sv, ~(uint32_t)(sv >> 32));
-    uint4* dst = reinterpret_cast<uint4*>(hptr(T, hf) + (size_t)ch * CH);
+    uint4* dst = reinterpret_cast<uint4*>(hptr(T, hf) + (size_t)pg * T.P + (size_t)ch * CH);
     for (uint32_t t = threadIdx.x; t < CH / 16; t += blockDim.x) dst[t] = pat;
   }
 }
@@ -2015,24 +2168,28 @@ __global__ void __launch_bounds__(256) k_hw_fill(Tables T, uint32_t lo, uint32_t
 // Harness: content tag of every block (0 = zeros, s = uniform {s,~s}, ~0 = corrupt).
 // ------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(256) k_tags(Tables T) {
-  __shared__ int s_ok, s_zero;
-  for (uint32_t bb = blockIdx.x; bb < T.nblocks; bb += gridDim.x) {
+  // one tag per page (= per block at single level); dead pages and zero-content pages
+  // of an H chunk hold no data on the host and read as zero (R1)
+  const unsigned long long npages = (unsigned long long)T.nblocks * T.ppc;
+  for (unsigned long long q = blockIdx.x; q < npages; q += gridDim.x) {
+    const uint32_t bb = (uint32_t)(q / T.ppc), pg = (uint32_t)(q % T.ppc);
     uint8_t ss = ld_st(T, bb);
     const uint4* src = nullptr;
     if (ss == ST_G || ss == ST_GE || ss == ST_GL) {
       uint32_t fr = T.frame_of[bb];
-      if (fr != UM_NONE) src = reinterpret_cast<const uint4*>(T.frames + (size_t)fr * T.B);
+      if (fr != UM_NONE) src = reinterpret_cast<const uint4*>(T.frames + (size_t)fr * T.B + (size_t)pg * T.P);
     } else if (ss == ST_H) {
       uint32_t hf = T.hframe[bb];
-      if (hf != UM_NONE) src = reinterpret_cast<const uint4*>(hptr(T, hf));
+      const bool nodata = T.pdead && (((T.pdead[bb] | T.phz[bb]) >> pg) & 1u);
+      if (hf != UM_NONE && !nodata) src = reinterpret_cast<const uint4*>(hptr(T, hf) + (size_t)pg * T.P);
     }
     if (!src) {
-      if (threadIdx.x == 0) T.tags[bb] = (ss == ST_G || ss == ST_GE || ss == ST_GL) ? ~0ull : 0ull;
+      if (threadIdx.x == 0) T.tags[q] = (ss == ST_G || ss == ST_GE || ss == ST_GL) ? ~0ull : 0ull;
       continue;
     }
     uint4 v0 = src[0];
     bool ok = true;
-    for (uint32_t t = threadIdx.x; t < T.B / 16; t += blockDim.x) {
+    for (uint32_t t = threadIdx.x; t < T.P / 16; t += blockDim.x) {
       uint4 v = src[t];
       ok &= (v.x == v0.x) & (v.y == v0.y) & (v.z == v0.z) & (v.w == v0.w);
     }
@@ -2045,7 +2202,7 @@ __global__ void __launch_bounds__(256) k_tags(Tables T) {
       else if (s == 0 && ns == 0) tag = 0;
       else if (ns == ~s && s != 0) tag = s;
       else tag = ~0ull;
-      T.tags[bb] = tag;
+      T.tags[q] = tag;
     }
     __syncthreads();
   }
@@ -2180,7 +2337,7 @@ cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max
 
 cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int ctas_per_sm,
                              cudaStream_t s) {
-  const uint32_t SEG = T.B < kFillSeg ? T.B : kFillSeg;
+  const uint32_t SEG = T.P < kFillSeg ? T.P : kFillSeg;
   unsigned long long units = (unsigned long long)n * (T.B / SEG);
   // ctas_per_sm < 0: a grid of -ctas_per_sm CTAs in total (a bandwidth-capped background kernel)
   const unsigned long long cap = ctas_per_sm < 0 ? (unsigned long long)(-ctas_per_sm)
@@ -2209,13 +2366,41 @@ cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64
   return cudaGetLastError();
 }
 
-cudaError_t launch_host_write(const Tables& T, uint32_t lo, uint32_t n, uint32_t seq, cudaStream_t s) {
-  if (!n) return cudaSuccess;
-  k_hw_alloc<<<ceil_div(n, 256), 256, 0, s>>>(T, lo, n);
-  const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
-  unsigned long long units = (unsigned long long)n * (T.B / CH);
+cudaError_t launch_host_write(const Tables& T, uint64_t p0, uint64_t p1, uint32_t seq, cudaStream_t s) {
+  if (p1 <= p0) return cudaSuccess;
+  const uint32_t lo = (uint32_t)(p0 / T.ppc), n = (uint32_t)((p1 - 1) / T.ppc + 1 - lo);
+  k_hw_alloc<<<ceil_div(n, 256), 256, 0, s>>>(T, lo, n, p0, p1);
+  const uint32_t CH = T.P < kXferChunk ? T.P : kXferChunk;
+  unsigned long long units = (p1 - p0) * (T.P / CH);
   unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
-  k_hw_fill<<<grid, 256, 0, s>>>(T, lo, n, seq);
+  k_hw_fill<<<grid, 256, 0, s>>>(T, p0, p1, seq);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_page_revive(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, int touch, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  unsigned grid = ceil_div(n, 256);
+  if (grid > (unsigned)g_nsm * 4) grid = g_nsm * 4;
+  cudaError_t e = launch_pdl(k_page_revive, dim3(grid), dim3(256), 0, s, T, iv, g0, n, touch);
+  if (e) return e;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_page_host_revive(const Tables& T, uint32_t lo, uint32_t n, uint64_t p0, uint64_t p1,
+                                    cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  unsigned grid = ceil_div(n, 256);
+  if (grid > (unsigned)g_nsm * 4) grid = g_nsm * 4;
+  cudaError_t e = launch_pdl(k_page_host_revive, dim3(grid), dim3(256), 0, s, T, lo, n,
+                             (unsigned long long)p0, (unsigned long long)p1);
+  if (e) return e;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_page_discard(const Tables& T, uint32_t c0, uint32_t m0, uint32_t c1, uint32_t m1, int lazy,
+                                cudaStream_t s) {
+  cudaError_t e = launch_pdl(k_page_discard, dim3(1), dim3(32), 0, s, T, c0, m0, c1, m1, lazy);
+  if (e) return e;
   return cudaGetLastError();
 }
 
@@ -2236,7 +2421,8 @@ cudaError_t launch_zero_items(const Tables& T, uint32_t i0, uint32_t i1, cudaStr
 }
 
 cudaError_t launch_tags(const Tables& T, cudaStream_t s) {
-  unsigned grid = T.nblocks < (uint32_t)g_nsm * 16 ? T.nblocks : (unsigned)g_nsm * 16;
+  const unsigned long long np = (unsigned long long)T.nblocks * T.ppc;
+  unsigned grid = np < (unsigned long long)g_nsm * 16 ? (unsigned)np : (unsigned)g_nsm * 16;
   if (!grid) grid = 1;
   k_tags<<<grid, 256, 0, s>>>(T);
   return cudaGetLastError();

@@ -19,9 +19,11 @@ def mode_flags(mode: str) -> int:
 
 
 def make_arena(trace, mode: str, *, flags: int = um.UM_F_APP_STAMP | um.UM_F_CHECK, host_pool_bytes=None,
-               device: int = 0, mem=None) -> um.Arena:
+               device: int = 0, mem=None, page_bytes: int = 0) -> um.Arena:
+    """page_bytes < block_bytes: a two-level arena (chunks of block_bytes, pages of
+    page_bytes)."""
     return um.Arena(trace.block_bytes, trace.arena_bytes, trace.budget_bytes, flags=flags | mode_flags(mode),
-                    host_pool_bytes=host_pool_bytes, device=device, mem=mem)
+                    host_pool_bytes=host_pool_bytes, device=device, mem=mem, page_bytes=page_bytes)
 
 
 def alloc_buffers(arena: um.Arena, trace) -> None:
@@ -88,8 +90,11 @@ def result(arena: um.Arena) -> dict:
     """The observable result (same keys as the oracle's dump())."""
     d = um.um_dump(arena.handle, arena.nblocks, arena.nframes)
     d["stats"] = um.um_get_stats(arena.handle)
-    d["contents"] = um.um_content_tags(arena.handle, arena.nblocks)
+    d["contents"] = um.um_content_tags(arena.handle, arena.nblocks * arena.ppc)
     d["st"] = d["st"].astype(np.int64).tolist()
+    if arena.ppc > 1:
+        dead, lazy = um.um_page_masks(arena.handle, arena.nblocks)
+        d["dead"], d["lazy"] = dead.astype(np.int64).tolist(), lazy.astype(np.int64).tolist()
     return d
 
 

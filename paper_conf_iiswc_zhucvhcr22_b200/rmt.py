@@ -32,9 +32,10 @@ def _expand(lo, hi):
     return np.repeat(lo, n) + (np.arange(tot) - start), rep
 
 
-def events(trace):
-    """Sorted event keys (block, op, order) packed in one int64, and the event kinds."""
-    B = trace.block_bytes
+def events(trace, unit=None):
+    """Sorted event keys (block, op, order) packed in one int64, and the event kinds;
+    blocks are units of `unit` bytes (pages at two levels), default the trace's block."""
+    B = unit or trace.block_bytes
     ops = trace.ops
     T = len(ops) + 1
     blocks, times, kinds = [], [], []
@@ -103,13 +104,14 @@ def op_of_seq(trace, seqs):
     return np.searchsorted(starts, np.asarray(seqs, np.int64), side="right") - 1
 
 
-def analyze(trace, log, op_range=None):
+def analyze(trace, log, op_range=None, page_bytes=None):
     """log: (seq, kind, block, prev_state) records with kind in {"H2D", "D2H", "ZF"}, or
     an int array of rows (seq, block, kind 0/1/2, prev_state) as um_xlog records them.
     Returns byte totals, redundant bytes per direction, and the number of moves of
     blocks that were discarded (HD, GE, GL) when they moved.  op_range = (lo, hi) counts
-    only the moves made by ops lo..hi-1 (e.g. one steady-state iteration)."""
-    B = trace.block_bytes
+    only the moves made by ops lo..hi-1 (e.g. one steady-state iteration).  page_bytes:
+    a two-level arena's log (one record per page; blocks are global page indices)."""
+    B = page_bytes or trace.block_bytes
     if len(log) and isinstance(log[0], tuple) and isinstance(log[0][1], str):
         code = {"H2D": 0, "D2H": 1, "ZF": 2}
         arr = np.array([(s, b, code[k], p) for (s, k, b, p) in log], np.int64).reshape(-1, 4)
@@ -122,7 +124,7 @@ def analyze(trace, log, op_range=None):
         arr, t = arr[m], t[m]
     out = {"h2d_bytes": int((arr[:, 2] == 0).sum()) * B, "d2h_bytes": int((arr[:, 2] == 1).sum()) * B,
            "discarded_state_moves": int(np.isin(arr[:, 3], _STATE_DISCARDED).sum())}
-    key, kind, T = events(trace)
+    key, kind, T = events(trace, B)
     b = arr[:, 1]
     # last WRITE/DEAD event at or before each event index (per block), forward-filled
     wd = np.where(kind != EV_READ, np.arange(len(kind)), -1)

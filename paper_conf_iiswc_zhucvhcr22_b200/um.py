@@ -33,7 +33,8 @@ class um_config(C.Structure):
     _fields_ = [("device", C.c_int), ("block_bytes", C.c_uint32), ("arena_bytes", C.c_uint64),
                 ("budget_bytes", C.c_uint64), ("frames", C.c_void_p), ("workspace", C.c_void_p),
                 ("workspace_bytes", C.c_uint64), ("host_chunks", C.POINTER(C.c_void_p)),
-                ("n_host_chunks", C.c_uint32), ("host_chunk_bytes", C.c_uint64), ("flags", C.c_uint32)]
+                ("n_host_chunks", C.c_uint32), ("host_chunk_bytes", C.c_uint64), ("flags", C.c_uint32),
+                ("page_bytes", C.c_uint32)]
 
 
 STAT_FIELDS = ("h2d_bytes", "d2h_bytes", "zf_bytes", "h2d_avoided_bytes", "d2h_avoided_bytes", "faults",
@@ -84,6 +85,7 @@ def lib():
             "um_timing": [P, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(U64), C.POINTER(U64), I],
             "um_xlog_attach": [P, P, U64],
             "um_xlog_count": [P, C.POINTER(U64)],
+            "um_page_masks": [P, P, P],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -98,7 +100,7 @@ def lib():
 EXPORTS = ("um_workspace_size", "um_arena_create", "um_arena_destroy", "um_alloc", "um_prefetch", "um_discard",
            "um_discard_lazy", "um_touch_batch", "um_evict", "um_host_write", "um_block_table", "um_stream",
            "um_join", "um_get_stats", "um_dump", "um_content_tags", "um_timing", "um_xlog_attach",
-           "um_xlog_count", "um_strerror")
+           "um_xlog_count", "um_page_masks", "um_strerror")
 
 
 def _ck(fn, st):
@@ -192,6 +194,12 @@ def um_dump(a, nblocks: int, nframes: int) -> dict:
     return {"st": st, "used_order": used[:nu.value].tolist(), "disc_order": disc[:nd.value].tolist()}
 
 
+def um_page_masks(a, nblocks: int) -> tuple:
+    dead, lazy = np.zeros(nblocks, np.uint32), np.zeros(nblocks, np.uint32)
+    _ck("um_page_masks", lib().um_page_masks(a, dead.ctypes.data, lazy.ctypes.data))
+    return dead, lazy
+
+
 def um_content_tags(a, nblocks: int) -> np.ndarray:
     t = np.zeros(nblocks, np.uint64)
     _ck("um_content_tags", lib().um_content_tags(a, t.ctypes.data))
@@ -228,9 +236,10 @@ class Memory:
     (pinned host memory in chunks of <= 1 GiB, allocated from `threads` threads)."""
 
     def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, host_pool_bytes=None,
-                 host_chunk_bytes=None, device: int = 0, threads: int = 1):
+                 host_chunk_bytes=None, device: int = 0, threads: int = 1, page_bytes: int = 0):
         import torch
         self.B = block_bytes
+        self.page_bytes = page_bytes
         self.nframes = budget_bytes // block_bytes
         if host_pool_bytes is None:
             host_pool_bytes = arena_bytes          # every block can be host-resident
@@ -253,7 +262,7 @@ class Memory:
         probe = um_config(device=device, block_bytes=block_bytes, arena_bytes=arena_bytes,
                           budget_bytes=budget_bytes, frames=self.frames.data_ptr(), workspace=None,
                           workspace_bytes=0, host_chunks=C.cast(self._hc, C.POINTER(C.c_void_p)),
-                          n_host_chunks=nch, host_chunk_bytes=host_chunk_bytes, flags=0)
+                          n_host_chunks=nch, host_chunk_bytes=host_chunk_bytes, flags=0, page_bytes=page_bytes)
         ws = um_workspace_size(probe)
         self.workspace = torch.empty(ws, dtype=torch.uint8, device=dev)
         self.nch = nch
@@ -263,7 +272,7 @@ class Memory:
                          budget_bytes=budget_bytes, frames=self.frames.data_ptr(),
                          workspace=self.workspace.data_ptr(), workspace_bytes=self.workspace.numel(),
                          host_chunks=C.cast(self._hc, C.POINTER(C.c_void_p)), n_host_chunks=self.nch,
-                         host_chunk_bytes=self.host_chunk_bytes, flags=flags)
+                         host_chunk_bytes=self.host_chunk_bytes, flags=flags, page_bytes=self.page_bytes)
 
 
 class Arena:
@@ -271,13 +280,15 @@ class Arena:
 
     def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, flags: int = 0,
                  host_pool_bytes: int | None = None, host_chunk_bytes: int | None = None, device: int = 0,
-                 mem: Memory | None = None):
+                 mem: Memory | None = None, page_bytes: int = 0):
         self.B = block_bytes
         self.nblocks = arena_bytes // block_bytes
         self.nframes = budget_bytes // block_bytes
         self.mem = mem if mem is not None else Memory(block_bytes, arena_bytes, budget_bytes,
                                                       host_pool_bytes=host_pool_bytes,
-                                                      host_chunk_bytes=host_chunk_bytes, device=device)
+                                                      host_chunk_bytes=host_chunk_bytes, device=device,
+                                                      page_bytes=page_bytes)
+        self.ppc = block_bytes // page_bytes if page_bytes else 1
         self.frames = self.mem.frames
         self.cfg = self.mem.config(arena_bytes, budget_bytes, flags)
         self.handle = um_arena_create(self.cfg)

@@ -64,3 +64,26 @@ def test_workspace_size_and_config_validation_without_gpu():
     # arena_create rejects missing memory before touching the GPU
     out = C.c_void_p()
     assert um.lib().um_arena_create(C.byref(cfg), C.byref(out)) == um.UM_EINVAL
+
+
+def test_two_level_config_validation_without_gpu():
+    """page_bytes: 0 or block_bytes = single level; otherwise a power of
+    two >= 16 KiB with <= 32 pages per block, not with UM_F_COPY_CE / UM_F_OVERLAP."""
+    import ctypes as C
+    from paper_conf_iiswc_zhucvhcr22_b200 import um
+    hc = (C.c_void_p * 1)(1)
+    base = um.um_config(device=0, block_bytes=2 << 20, arena_bytes=64 << 20, budget_bytes=16 << 20, frames=None,
+                        workspace=None, workspace_bytes=0, host_chunks=C.cast(hc, C.POINTER(C.c_void_p)),
+                        n_host_chunks=1, host_chunk_bytes=64 << 20, flags=0, page_bytes=0)
+    ws1 = um.um_workspace_size(base)
+    ok = um.um_config.from_buffer_copy(base)
+    ok.page_bytes = 64 << 10
+    assert um.um_workspace_size(ok) > ws1          # page masks and per-page tags
+    same = um.um_config.from_buffer_copy(base)
+    same.page_bytes = 2 << 20
+    assert um.um_workspace_size(same) == ws1
+    for pb, fl in [(32 << 10, 0), (48 << 10, 0), (8 << 10, 0), (64 << 10, um.UM_F_COPY_CE), (64 << 10, 64)]:
+        bad = um.um_config.from_buffer_copy(base)
+        bad.page_bytes, bad.flags = pb, fl
+        with pytest.raises(um.UmError):
+            um.um_workspace_size(bad)

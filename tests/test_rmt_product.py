@@ -44,3 +44,30 @@ def test_op_of_seq(seed):
     seqs = np.arange(1, starts[-1] + 3)
     want = [max(i for i, s in enumerate(starts) if s <= q) for q in seqs]
     assert prmt.op_of_seq(t, seqs).tolist() == want
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_two_level_logs(mode):
+    """Per-page logs of the two-level oracle (oracle/chunks.py, NEXT-1)."""
+    from oracle.chunks import replay_chunks
+    P = 64 << 10
+    t = tg.gen_c3(block_bytes=2 << 20, budget_bytes=384 << 20, iterations=2, workspace_bytes=5 << 20,
+                  layers=tg.scale_layers(tg.VGG16, 1.0 / 64, 1.0 / 16), batch=6, discard_all_dead=True)
+    log = replay_chunks(t, P, mode, record=True).log
+    want = rmt_analyze(t, log, page_bytes=P)
+    got = prmt.analyze(t, log, page_bytes=P)
+    for k in ("h2d_bytes", "d2h_bytes", "rmt_h2d_bytes", "rmt_d2h_bytes", "rmt_bytes", "discarded_state_moves"):
+        assert got[k] == want[k], (k, got[k], want[k])
+    if mode != "base":
+        # what is left is only pages that a discard covers in part (A4 at page level),
+        # far less than the single-level run leaves (whole-chunk tails)
+        from oracle.sim import replay
+        single = rmt_analyze(t, replay(t, mode, record=True).log)
+        left = rmt_analyze(t, log, page_bytes=P, detail=True)["records"]
+        part, full = set(), set()
+        for kind, flags, off, ln, accs in t.iter_ops():
+            if kind == 2 and ln:
+                part.update(range(off // P, (off + ln - 1) // P + 1))
+                full.update(range(-(-off // P), (off + ln) // P))
+        assert all(q in part - full for (_t, _k, q, _r) in left)
+        assert got["rmt_bytes"] < single["rmt_bytes"]
