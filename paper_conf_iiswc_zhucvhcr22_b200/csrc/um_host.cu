@@ -1014,13 +1014,20 @@ static um_status run_gpu_op2(um_arena* a, int touch) {
     sp = span_open(a);
     CK(launch_service(a->T, SVC_SUBOP, seq, n, a->ps));
     span_close(a, sp, 1);
-    CK(launch_page_revive(a->T, iv, (uint32_t)g0, n, touch, a->ps));
-    a->n_launch += 2;
+    if (touch) {   // a touch revives the pages of each sub-op once it is serviced
+      CK(launch_page_revive(a->T, iv, (uint32_t)g0, n, 1, a->ps));
+      a->n_launch++;
+    }
+    a->n_launch++;
     a->n_xfer++;
     if (touch && anyw && (a->cfg.flags & UM_F_APP_STAMP)) {
       CK(launch_app_stamp(a->T, iv, (uint32_t)g0, n, seq, 8, a->ps));
       a->n_launch++;
     }
+  }
+  if (!touch) {   // a prefetch revalidates its pages when the whole op is done (oracle.chunks)
+    CK(launch_page_revive(a->T, iv, 0, (uint32_t)total, 0, a->ps));
+    a->n_launch++;
   }
   return UM_OK;
 }

@@ -1741,7 +1741,8 @@ __global__ void __launch_bounds__(TPB) k_app_stamp(Tables T, const __grid_consta
 // ------------------------------------------------------------------------------------
 // After a GPU sub-op: a touch revives the eagerly discarded pages it covers ("skip the
 // memory transfers ... until it gets accessed again", L196); a lazily discarded page
-// needs the prefetch (L186-190, A8); a prefetch revives every page it covers (A17).
+// needs the prefetch (L186-190, A8).  After a whole prefetch: it revives every page it
+// covers (A17).
 __global__ void __launch_bounds__(256) k_page_revive(Tables T, const __grid_constant__ OpIv iv, uint32_t g0, uint32_t n,
                                                      int touch) {
   pdl_enter();
@@ -1754,6 +1755,9 @@ __global__ void __launch_bounds__(256) k_page_revive(Tables T, const __grid_cons
     } else {
       T.pdead[c] = d & ~cm;
       T.plazy[c] &= ~cm;
+      // a chunk an earlier sub-op of this prefetch brought in and a later one evicted is
+      // on the host without its dead pages: revived, they read as zero
+      if (ld_st(T, c) == ST_H) T.phz[c] |= d & cm;
     }
   }
 }
