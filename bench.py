@@ -184,7 +184,7 @@ def run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=None, flags_extr
         per_iter = [evs[j].elapsed_time(evs[j + 1]) for j in range(K)]
         d = {k: s1[k] - s0[k] for k in s1}
         return {"mode": mode, "iter_ms": sum(per_iter) / K, "iter_ms_each": per_iter, "wall_s": wall,
-                "stats_per_iter": {k: v / K for k, v in d.items()}, "timing": tm, "clocks": ck}
+                "stats_per_iter": {k: v / K for k, v in d.items()}, "stats_total": d, "timing": tm, "clocks": ck}
     finally:
         arena.close()
 
@@ -737,6 +737,13 @@ def main_ours(args):
     B = args.block
     lws = int(os.environ.get("LOCAL_WORLD_SIZE", str(ws)))
     budget, arena_bytes, host_pool, clamp = plan_sizes(args, free, lws)
+    numa = None
+    if ws > 1:
+        # each rank's pinned host chunks on its GPU's NUMA node (first touch after binding)
+        from paper_conf_iiswc_zhucvhcr22_b200.dist import bind_to_gpu_numa_node
+        cpus, node = _gpu_node_cpus(dev.index)
+        bind_to_gpu_numa_node(cpus)
+        numa = {"node": node, "cpus": len(cpus)}
     trace = build_trace(args, budget, True, W + K)
     t_build = time.perf_counter()
     mem = um.Memory(B, arena_bytes, budget, host_pool_bytes=host_pool, device=dev.index,
@@ -782,7 +789,7 @@ def main_ours(args):
     t_iter_ms = head["iter_ms"]
     # max over ranks; the run's only collective: counters all-reduce (north_star)
     from paper_conf_iiswc_zhucvhcr22_b200.dist import reduce_run
-    stats_all, t_iter_ms = reduce_run(head["stats_per_iter"], t_iter_ms, device=dev)
+    stats_all, t_iter_ms = reduce_run(head["stats_total"], t_iter_ms, device=dev)   # int64 counters
     if rank != 0:
         return
     spi = head["stats_per_iter"]
@@ -810,7 +817,7 @@ def main_ours(args):
                    "budget_bytes": budget, "arena_bytes": arena_bytes, "batch": trace.meta["batch"],
                    "layers": trace.meta["layers"], "ops_per_iter": trace.meta["ops_per_iter"],
                    "host_pool_bytes": host_pool, "budget_requested_bytes": int(args.budget_gib * GiB),
-                   "budget_clamped_by": clamp, "parallelism": f"independent arenas x{ws}",
+                   "budget_clamped_by": clamp, "host_numa_binding": numa, "parallelism": f"independent arenas x{ws}",
                    "l2": "working set 255 GiB >> 126 MB L2 (no flush needed)",
                    "headline_mode": "eager (UvmDiscard)",
                    "app_overlap": ("UM_F_OVERLAP: app kernels pipelined with the next 2 GPU sub-ops (reading R7), "
@@ -853,7 +860,8 @@ def main_ours(args):
         "c3_64k_blocks": c3k,
         "clocks": head["clocks"],
         "gpu_launches": tm["launches"],
-        "stats_per_iter_all_ranks": stats_all,
+        "stats_all_ranks": {"counters": stats_all, "iterations_per_rank": K,
+                            "reduce": "NCCL all-reduce (int64 sum) of the counters, max of the iteration time"},
         "setup_s": {"pin_and_alloc": t_alloc},
     })
     if e2e_s is not None:

@@ -26,7 +26,8 @@ def _worker(rank, ws, port, q):
         assert world() == (rank, ws)
         # independent per-rank arenas: per-rank seed, no exchange during the replay
         t = tg.gen_c1(100 + rank).slice_ops(0, 1500)
-        s = replay(t, "eager").stats
+        s = dict(replay(t, "eager").stats)
+        s["big"] = (1 << 60) + 2 * rank + 1          # beyond 2^53: the reduce must be int64-exact
         red, tmax = reduce_run(s, 10.0 + rank)
         q.put((rank, s, red, tmax))
     finally:
@@ -50,6 +51,7 @@ def test_gloo_ws2_reduce_counters_and_max_time():
         assert tmax == 11.0
         for k in s0:
             assert red[k] == s0[k] + s1[k]
+        assert red["big"] == (1 << 61) + 4
 
 
 def test_reduce_run_single_process_is_identity():
