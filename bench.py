@@ -238,16 +238,16 @@ class _MemView:
     """The bench's frames and host pool seen at another block size, with its own
     workspace (um.Arena needs .B, .frames and .config())."""
 
-    def __init__(self, torch, um, mem, B, arena_bytes, budget):
-        self.B, self.frames, self._mem = B, mem.frames, mem
+    def __init__(self, torch, um, mem, B, arena_bytes, budget, page_bytes=0):
+        self.B, self.frames, self._mem, self.page_bytes = B, mem.frames, mem, page_bytes
         probe = mem.config(arena_bytes, budget, 0)
-        probe.block_bytes = B
+        probe.block_bytes, probe.page_bytes = B, page_bytes
         probe.workspace, probe.workspace_bytes = None, 0
         self.workspace = torch.empty(um.um_workspace_size(probe), dtype=torch.uint8, device=mem.frames.device)
 
     def config(self, arena_bytes, budget_bytes, flags):
         c = self._mem.config(arena_bytes, budget_bytes, flags)
-        c.block_bytes = self.B
+        c.block_bytes, c.page_bytes = self.B, self.page_bytes
         c.workspace, c.workspace_bytes = self.workspace.data_ptr(), self.workspace.numel()
         return c
 
@@ -294,36 +294,56 @@ def rmt_leg(torch, um, harness, mem, budget, oversub, B):
     Fig. 3): two C3 iterations per mode with the transfer log attached
     (um_xlog_attach), judged by paper_conf_iiswc_zhucvhcr22_b200/rmt.py over the second
     (steady-state) iteration.  Two traces: Listing 6 as printed (never discards output_1
-    or data) and --discard-all-dead.  RMT_left should hold only blocks a discard covers
-    partly (A4: a discard ignores partial blocks, §5.4)."""
+    or data) and --discard-all-dead, the latter also with 64 KiB pages (NEXT-1).  RMT_left
+    holds only blocks (pages) a discard covers partly (A4: a discard ignores partial
+    blocks, §5.4)."""
     import tracegen as tg
     from paper_conf_iiswc_zhucvhcr22_b200 import rmt
     out = {"iteration": "second of two (steady state)",
            "source": "CUDA-path transfer log (um_xlog_attach), judged by paper_conf_iiswc_zhucvhcr22_b200/rmt.py "
                      "(pinned against oracle/rmt.py in tests/test_rmt_product.py)"}
+    P = 64 << 10
     for variant, dead in (("listing6_literal", False), ("discard_all_dead", True)):
         t = tg.gen_c3(block_bytes=B, budget_bytes=budget, oversub=oversub, iterations=2, discard_all_dead=dead,
                       with_host_data=True)
         it2 = harness.iteration_bounds(t)[1]
         res = {}
-        for mode in ("base", "eager"):
-            arena = harness.make_arena(t, mode, mem=mem, flags=um.UM_F_APP_STAMP)
+        modes = [("base", mem, None), ("eager", mem, None)]
+        if dead:   # NEXT-1: the same run with 64 KiB pages in the 2 MiB chunks
+            modes.append(("eager_pages", _MemView(torch, um, mem, B, t.arena_bytes, t.budget_bytes, page_bytes=P), P))
+        for mode, m, pb in modes:
+            arena = harness.make_arena(t, mode.split("_")[0], mem=m, flags=um.UM_F_APP_STAMP, page_bytes=pb or 0)
             try:
                 harness.alloc_buffers(arena, t)
-                lg = harness.XLog(arena, 8 << 20)
-                harness.issue(arena, t, mode)
+                lg = harness.XLog(arena, (8 << 20) * (B // pb if pb else 1))
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                ps = torch.cuda.ExternalStream(arena.stream_ptr)
+                harness.issue(arena, t, mode.split("_")[0], 0, it2[0])
+                e0.record(ps)
+                harness.issue(arena, t, mode.split("_")[0], it2[0], it2[1])
+                e1.record(ps)
+                e1.synchronize()
                 log = lg.raw()
                 lg.detach()
             finally:
                 arena.close()
-            res[mode] = rmt.analyze(t, log, op_range=it2)
+            res[mode] = rmt.analyze(t, log, op_range=it2, page_bytes=pb)
+            res[mode]["iter_ms"] = e0.elapsed_time(e1)
         b, e = res["base"], res["eager"]
         out[variant] = {"rmt_base_gb": b["rmt_bytes"] / 1e9, "rmt_left_gb": e["rmt_bytes"] / 1e9,
                         "link_gb": {"base": (b["h2d_bytes"] + b["d2h_bytes"]) / 1e9,
                                     "eager": (e["h2d_bytes"] + e["d2h_bytes"]) / 1e9},
                         "avoided_gb": (b["h2d_bytes"] + b["d2h_bytes"] - e["h2d_bytes"] - e["d2h_bytes"]) / 1e9,
                         "rmt_base_split_gb": {"h2d": b["rmt_h2d_bytes"] / 1e9, "d2h": b["rmt_d2h_bytes"] / 1e9},
-                        "discarded_state_moves_eager": e["discarded_state_moves"]}
+                        "discarded_state_moves_eager": e["discarded_state_moves"],
+                        "iter_ms": {"base": b["iter_ms"], "eager": e["iter_ms"]}}
+        if "eager_pages" in res:
+            p_ = res["eager_pages"]
+            out[variant]["two_level_64k_pages"] = {
+                "rmt_left_gb": p_["rmt_bytes"] / 1e9, "link_gb": (p_["h2d_bytes"] + p_["d2h_bytes"]) / 1e9,
+                "avoided_gb": (b["h2d_bytes"] + b["d2h_bytes"] - p_["h2d_bytes"] - p_["d2h_bytes"]) / 1e9,
+                "discarded_state_moves": p_["discarded_state_moves"], "iter_ms": p_["iter_ms"],
+                "note": "NEXT-1: partial-chunk discards mark 64 KiB pages dead (no write-back, zero-fill on return)"}
     return out
 
 

@@ -288,9 +288,11 @@ class Arena:
                                                       host_pool_bytes=host_pool_bytes,
                                                       host_chunk_bytes=host_chunk_bytes, device=device,
                                                       page_bytes=page_bytes)
-        self.ppc = block_bytes // page_bytes if page_bytes else 1
         self.frames = self.mem.frames
         self.cfg = self.mem.config(arena_bytes, budget_bytes, flags)
+        if page_bytes:
+            self.cfg.page_bytes = page_bytes
+        self.ppc = block_bytes // self.cfg.page_bytes if self.cfg.page_bytes else 1
         self.handle = um_arena_create(self.cfg)
         self.stream_ptr = um_stream(self.handle)
 
