@@ -496,6 +496,18 @@ def c1_rate(torch, um, harness):
         arena.close()
 
 
+def _service_traffic():
+    """Per-launch traffic of k_service from the committed ncu capture of the bench's timed
+    iteration (tools/ncu_round.sh + tools/service_traffic.py); None if absent."""
+    path = os.path.join(ROOT, "profiles", "r02_service_traffic.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d, os.path.relpath(path, ROOT)
+    except Exception:
+        return None, None
+
+
 def _hbm_peak():
     """Measured HBM copy bandwidth (MEASURED_PEAKS.json, driver-written), else the
     profiling guide's fallback."""
@@ -814,6 +826,7 @@ def main_ours(args):
         return
     spi = head["stats_per_iter"]
     B_ = args.block
+    st_tr, st_tr_src = _service_traffic()
     link_bytes = spi["h2d_bytes"] + spi["d2h_bytes"]
     tm = head["timing"]
     xfer_ms_per_launch = tm["ms_xfer"] / max(1, tm["xfer_launches"])
@@ -855,8 +868,13 @@ def main_ours(args):
         "roofline": {"kernel": "k_service (K4: TMA bulk-copy fused-swap kernel over mapped pinned host memory)",
                      "bound": "host_link",
                      "achieved": achieved, "peak": peak_eff, "unit": "GB/s",
-                     "frac": (achieved / peak_eff) if achieved else None, "traffic": None,
-                     "traffic_note": "dram and PCIe bytes per k_service launch from one ncu --set full capture: profiles/r02_ncu_service.md",
+                     "frac": (achieved / peak_eff) if achieved else None,
+                     "traffic": (st_tr or {}).get("per_launch", {}).get("pcie_bytes"),
+                     "traffic_dram": (st_tr or {}).get("per_launch", {}).get("dram_bytes"),
+                     "traffic_ratio": (st_tr or {}).get("ratio"),
+                     "traffic_note": (f"pcie__read_bytes + pcie__write_bytes per k_service launch (the link-bound "
+                                      f"kernel's bytes; dram bytes beside) over every launch of the bench's timed "
+                                      f"iteration, from {st_tr_src}" if st_tr else "no committed ncu capture"),
                      "frac_vs_duplex": (achieved / link["duplex_gbs"]) if achieved else None,
                      "peak_source": "measured live in bench.py: pinned 1 GiB cudaMemcpyAsync (copy engines) H2D and D2H, best of 5, weighted by the step's H2D/D2H byte mix",
                      "algorithmic_bytes_per_launch": link_bytes_per_launch, "ms_per_launch": xfer_ms_per_launch,

@@ -164,6 +164,14 @@ um_status um_discard_lazy(um_arena *a, uint64_t off, uint64_t len, void *stream)
  * return (the caller may reuse it). */
 um_status um_touch_batch(um_arena *a, const um_access *acc, uint32_t n, void *stream);
 
+/* The application releases [off, off+len) (cudaFree of managed memory; reading R9 of
+ * DESIGN.md).  Every block FULLY inside the range returns to U (never populated: it
+ * reads as zeros) with no transfer: its GPU frame goes back to the pool the eviction
+ * process takes before any discarded or used page (the paper's unused queue, §5.5
+ * L217-221), a host copy is released.  The virtual range stays allocated (um_alloc is a
+ * bump allocator).  Consumes one sequence number. */
+um_status um_free(um_arena *a, uint64_t off, uint64_t len, void *stream);
+
 /* Make >= bytes of frames free by the eviction policy (PAPER §5.5). */
 um_status um_evict(um_arena *a, uint64_t bytes, void *stream);
 

@@ -258,6 +258,14 @@ class ChunkOracle(Oracle):
         self._chunk_level(off, ln)
         self._partial(off, ln, lazy=True)
 
+    def free_range(self, off: int, ln: int):
+        """um_free (R9) at chunk level: fully covered chunks return to U, page state with them."""
+        super().free_range(off, ln)
+        for c in self._full(off, ln):
+            self.dead[c] = self.lazy[c] = 0
+            for p in range(self.ppc):
+                self.gpu_ps[c * self.ppc + p] = self.host_ps[c * self.ppc + p] = 0
+
     def host_write(self, off: int, ln: int):
         self._check(off, ln)
         cover = self._by_chunk(self._pages_cover(off, ln))

@@ -12,7 +12,7 @@ path's, which must be equal).  Data events of block b, in trace order:
   READ   a touch whose records covering b include UM_ACC_READ;
   WRITE  a touch whose records covering b include UM_ACC_WRITE (after its READ, if the
          touch also reads b: the application reads, then writes), or a host_write of b;
-  DEAD   a discard (eager or lazy) that fully covers b (§5.4, A4).
+  DEAD   a discard (eager or lazy) that fully covers b (§5.4, A4), or a free of it.
 Prefetch, evict and the paging layer's own moves are not data events.
 
 A transfer (H2D or D2H) of b at op t moves b's value at that moment.  It is redundant iff
@@ -77,7 +77,7 @@ def data_events(trace, unit=None):
                     add(b, t, READ)
                 if b in wr:
                     add(b, t, WRITE)
-        elif kind == 2:                                 # discard / discard_lazy
+        elif kind in (2, 5):                            # discard / discard_lazy / free
             for b in _full(B, off, ln):
                 add(b, t, DEAD)
         elif kind == 4:                                 # host_write

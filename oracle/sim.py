@@ -348,6 +348,29 @@ class Oracle:
         for v in self._select_victims(want - self.free, ()):
             self._reclaim(v, seq)
 
+    def free_range(self, off: int, ln: int):
+        """um_free: the application releases [off, off+len) (cudaFree of managed memory).
+        Reading R9: every FULLY covered block returns to U ("never
+        populated", contents zero) with no transfer; a GPU frame it held goes to the
+        unused page queue, which the eviction process reclaims before the discarded
+        queue and without a transfer (§5.5) -- frames are anonymous, so it is
+        counted with the free frames; a host copy is released."""
+        self._check(off, ln)
+        self.stats["ops"] += 1
+        self._next_seq()
+        for b in self._full(off, ln):
+            s = self.st[b]
+            if s == G:
+                del self.used[b]
+                self.free += 1
+            elif s in (GE, GL):
+                del self.disc[b]
+                self.free += 1
+            self.st[b] = U
+            self.key[b] = 0
+            self.gpu_stamp[b] = 0
+            self.host_stamp[b] = 0
+
     def host_write(self, off: int, ln: int):
         """Harness op: the CPU writes new data into host-resident blocks ("Generate data,
         labels", Listing 6 L330).  Requires every covered block to be in H."""
@@ -415,6 +438,8 @@ def apply_op(o: Oracle, op: tuple, mode: str):
         o.evict(ln)
     elif kind == 4:
         o.host_write(off, ln)
+    elif kind == 5:
+        o.free_range(off, ln)
     else:
         raise ValueError(f"unknown op {kind}")
 

@@ -1364,6 +1364,25 @@ UM_API um_status um_discard_lazy(um_arena* a, uint64_t off, uint64_t len, void* 
   return discard_common(a, off, len, stream, DIR_DISCARD_LAZY);
 }
 
+UM_API um_status um_free(um_arena* a, uint64_t off, uint64_t len, void* stream) {
+  ENTER(a);
+  if (!range_ok(a, off, len)) return UM_EINVAL;
+  um_status s = hand_in(a, stream);
+  if (s) return s;
+  if ((s = seq_room(a, 1))) return s;
+  a->ops++;
+  a->subops++;
+  ++a->clock;
+  const uint64_t lo = (off + a->B - 1) / a->B, hi = (off + len) / a->B;   // fully covered blocks
+  if (hi > lo) {
+    cudaEvent_t sp = span_open(a);
+    CK(launch_free(a->T, (uint32_t)lo, (uint32_t)(hi - lo), a->ps));
+    span_close(a, sp, 0);
+    a->n_launch++;
+  }
+  return hand_out(a, stream);
+}
+
 UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
   ENTER(a);
   um_status s = hand_in(a, stream);

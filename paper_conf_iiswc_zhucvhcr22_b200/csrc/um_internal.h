@@ -197,6 +197,8 @@ cudaError_t launch_app_stamp(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, 
 cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
                              int discard_off, unsigned long long tail0, cudaStream_t s);
 cudaError_t launch_ring_compact(const Tables& T, int ring, uint64_t* dst, uint64_t cap_bound, cudaStream_t s);
+// um_free of blocks [lo, lo + n): back to U, frames and host frames released (R9).
+cudaError_t launch_free(const Tables& T, uint32_t lo, uint32_t n, cudaStream_t s);
 // Harness host write of pages [p0, p1) (global page indices; p = block at single level).
 cudaError_t launch_host_write(const Tables& T, uint64_t p0, uint64_t p1, uint32_t seq, cudaStream_t s);
 cudaError_t launch_tags(const Tables& T, cudaStream_t s);

@@ -2113,6 +2113,31 @@ __global__ void __launch_bounds__(256) k_intake_clear(Tables T, uint32_t w0, uin
 // ------------------------------------------------------------------------------------
 // Harness: host writes (Listing 6 "Generate data, labels").
 // ------------------------------------------------------------------------------------
+// um_free (reading R9): blocks [lo, lo + n) return to U with no transfer.  A GPU frame
+// goes back to the free pool (the paper's unused queue is reclaimed before the
+// discarded one and without a transfer, §5.5; frames are anonymous), a host
+// copy is released; the block's ring entries go stale by the liveness rule.
+__global__ void __launch_bounds__(256) k_free(Tables T, uint32_t lo, uint32_t n) {
+  pdl_enter();
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const uint32_t bb = lo + i;
+    const uint8_t ss = ld_st(T, bb);
+    if (ss == ST_U) continue;
+    if (ss == ST_G || ss == ST_GE || ss == ST_GL) {
+      const int idx = atomicAdd(&T.ctl->free_top, 1);
+      T.free_stack[idx] = T.frame_of[bb];
+      T.frame_of[bb] = UM_NONE;
+      T.map[bb] = UM_NONE;
+    } else if (T.hframe[bb] != UM_NONE) {   // H (HD holds none, R1)
+      const int idx = atomicAdd(&T.ctl->hfree_top, 1);
+      T.hfree_stack[idx] = T.hframe[bb];
+      T.hframe[bb] = UM_NONE;
+    }
+    T.sk[bb] = mk_sk(ST_U, 0);
+    if (T.pdead) T.pdead[bb] = T.plazy[bb] = T.phz[bb] = 0u;
+  }
+}
+
 // Pages [p0, p1) of chunk c (global page indices) as a mask of the chunk's pages.
 __device__ __forceinline__ uint32_t chunk_mask(const Tables& T, uint32_t c, unsigned long long p0, unsigned long long p1) {
   const unsigned long long c0 = (unsigned long long)c * T.ppc;
@@ -2378,6 +2403,15 @@ cudaError_t launch_host_write(const Tables& T, uint64_t p0, uint64_t p1, uint32_
   unsigned long long units = (p1 - p0) * (T.P / CH);
   unsigned grid = (unsigned)(units < (unsigned long long)g_nsm * 8 ? units : (unsigned long long)g_nsm * 8);
   k_hw_fill<<<grid, 256, 0, s>>>(T, p0, p1, seq);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_free(const Tables& T, uint32_t lo, uint32_t n, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  unsigned grid = ceil_div(n, 256);
+  if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
+  cudaError_t e = launch_pdl(k_free, dim3(grid), dim3(256), 0, s, T, lo, n);
+  if (e) return e;
   return cudaGetLastError();
 }
 

@@ -68,6 +68,8 @@ def _calls(trace, mode: str) -> list:
             out.append(("um_evict", L.um_evict, (ln,)))
         elif o == tg.OP_HOST_WRITE:
             out.append(("um_host_write", L.um_host_write, (off, ln)))
+        elif o == tg.OP_FREE:
+            out.append(("um_free", L.um_free, (off, ln)))
         else:
             raise ValueError(o)
     trace.meta[key] = out

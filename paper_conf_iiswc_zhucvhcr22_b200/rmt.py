@@ -6,7 +6,7 @@ record by record against the oracle's plain version (oracle/rmt.py).
 Definition (PAPER §1: a transfer is redundant when its data is "overwritten before
 being read"; Fig. 3; reading R8).  Data events of block b in op order:
 READ (a touch reading b), WRITE (a touch writing b, after its read if it also reads; a
-host_write), DEAD (a discard fully covering b, §5.4).  A move of b at op t is
+host_write), DEAD (a discard fully covering b, §5.4, or a free of it).  A move of b at op t is
 redundant iff b's last WRITE-or-DEAD event before t is DEAD (the value was discarded,
 §4.1), or b's first event at or after t is WRITE or DEAD.  The end of the trace
 reads every block.
@@ -61,7 +61,7 @@ def events(trace, unit=None):
             blocks.append(key // T)
             times.append(key % T)
             kinds.append(np.full(len(key), ev, np.int64))
-    for op, ev, full in ((tg.OP_DISCARD, EV_DEAD, True), (tg.OP_HOST_WRITE, EV_WRITE, False)):
+    for op, ev, full in ((tg.OP_DISCARD, EV_DEAD, True), (tg.OP_FREE, EV_DEAD, True), (tg.OP_HOST_WRITE, EV_WRITE, False)):
         idx = np.nonzero((ops["op"] == op) & (ops["len"] > 0))[0]
         off = ops["off"][idx].astype(np.int64)
         ln = ops["len"][idx].astype(np.int64)

@@ -75,6 +75,7 @@ def lib():
             "um_discard_lazy": [P, U64, U64, P],
             "um_touch_batch": [P, P, U32, P],
             "um_evict": [P, U64, P],
+            "um_free": [P, U64, U64, P],
             "um_host_write": [P, U64, U64, P],
             "um_block_table": [P, C.POINTER(P)],
             "um_stream": [P, C.POINTER(P)],
@@ -98,7 +99,7 @@ def lib():
 
 
 EXPORTS = ("um_workspace_size", "um_arena_create", "um_arena_destroy", "um_alloc", "um_prefetch", "um_discard",
-           "um_discard_lazy", "um_touch_batch", "um_evict", "um_host_write", "um_block_table", "um_stream",
+           "um_discard_lazy", "um_touch_batch", "um_evict", "um_free", "um_host_write", "um_block_table", "um_stream",
            "um_join", "um_get_stats", "um_dump", "um_content_tags", "um_timing", "um_xlog_attach",
            "um_xlog_count", "um_page_masks", "um_strerror")
 
@@ -155,6 +156,10 @@ def um_touch_batch(a, acc: np.ndarray, stream=None) -> None:
 
 def um_evict(a, nbytes: int, stream=None) -> None:
     _ck("um_evict", lib().um_evict(a, nbytes, stream))
+
+
+def um_free(a, off: int, ln: int, stream=None) -> None:
+    _ck("um_free", lib().um_free(a, off, ln, stream))
 
 
 def um_host_write(a, off: int, ln: int, stream=None) -> None:

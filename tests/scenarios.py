@@ -49,6 +49,9 @@ def build(sc) -> tuple:
             tb.discard(int(w[1]), int(w[2]))
         elif op == "evict":
             tb.evict(int(w[1]) * B)
+        elif op == "free":
+            lo, hi = _blocks(w[1])
+            tb.free(lo * B, (hi - lo + 1) * B)
         elif op == "evict_bytes":
             tb.evict(int(w[1]))
         elif op == "touch_bytes":

@@ -68,6 +68,8 @@ def _trace(P, ppc, nchunks, nframes, ops):
             tb.evict(op[1] * C)
         elif kind == "host_write":
             tb.host_write(op[1] * P, op[2] * P)
+        elif kind == "free":     # ("free", first chunk, n chunks)
+            tb.free(op[1] * C, op[2] * C)
         elif kind == "bytes":    # ("bytes", op, off, len[, extra]) raw byte ranges
             _, what, off, ln = op[:4]
             if what == "touch":
@@ -97,6 +99,8 @@ def test_hand_scenarios(mode):
                 ("evict", 2), ("touch", [(0, 8, "R")])]),
         (2, 1, [("touch", [(0, 8, "W")]), ("discard", 0, 4, False), ("discard", 4, 2, True),
                 ("prefetch", 0, 8, tg.DST_HOST), ("touch", [(0, 8, "R")])]),
+        (3, 2, [("touch", [(0, 8, "W")]), ("discard", 1, 2, False), ("free", 0, 1), ("touch", [(8, 4, "W")]),
+                ("prefetch", 4, 4, tg.DST_HOST), ("free", 1, 1), ("touch", [(0, 4, "R")])]),
     ]
     for nchunks, nframes, ops in cases:
         assert_page_parity(_trace(P16, 4, nchunks, nframes, ops), P16, mode)

@@ -238,7 +238,9 @@ def test_next3_radix_hashjoin(ov, mode):
     MiB = 1 << 20
     B = 64 * 1024
     for t in (tg.gen_radix(block_bytes=B, budget_bytes=int(64 * MiB / ov) // B * B, data_bytes=32 * MiB),
-              tg.gen_hashjoin(block_bytes=B, budget_bytes=int(72 * MiB / ov) // B * B, table_bytes=8 * MiB)):
+              tg.gen_hashjoin(block_bytes=B, budget_bytes=int(72 * MiB / ov) // B * B, table_bytes=8 * MiB),
+              tg.gen_hashjoin(block_bytes=B, budget_bytes=int(72 * MiB / ov) // B * B, table_bytes=8 * MiB,
+                              free_at_end=True)):
         assert_parity(t, mode)
 
 

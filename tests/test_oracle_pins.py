@@ -207,3 +207,25 @@ def test_sparse_trace_shape():
         assert len(lo) <= 3 * runs
         seen += 1
     assert seen >= 5
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_free_releases_without_transfers(mode):
+    """R9 (um_free): after the hash join frees its intermediates and outputs they are U
+    (contents zero); the frames they held are reused with no write-back, so freeing
+    never adds a transfer; conservation holds throughout."""
+    B = 64 << 10
+    kw = dict(block_bytes=B, budget_bytes=(36 << 20) // B * B, table_bytes=8 << 20)
+    a = replay(tg.gen_hashjoin(**kw), mode)
+    t = tg.gen_hashjoin(free_at_end=True, **kw)
+    b = replay(t, mode)
+    b.check_conservation()
+    for name, (off, ln) in t.buffers.items():
+        blocks = range(off // B, (off + ln) // B)
+        if name in ("R", "S"):
+            assert all(ST_NAMES[b.st[x]] != "U" for x in blocks)
+        else:
+            assert all(ST_NAMES[b.st[x]] == "U" and b.content(x) == 0 for x in blocks)
+    # the freed blocks' frames serve the final read of the tables: no more write-backs
+    # than the same run without the free and one more read
+    assert b.stats["d2h_bytes"] == a.stats["d2h_bytes"] and b.stats["evictions"] == a.stats["evictions"]

@@ -125,7 +125,7 @@ def _versioned_redundant(trace, recs):
                     reads_of[v] = t
             for b in wr:
                 ver[b] = ("w", next(nxt))
-        elif kind == 2:
+        elif kind in (2, 5):            # discard, free
             lo = -(-off // Bk)
             for b in range(lo, max(lo, (off + ln) // Bk)):
                 ver[b] = None
