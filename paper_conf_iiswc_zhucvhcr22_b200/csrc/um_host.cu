@@ -237,6 +237,10 @@ struct um_arena {
   // discard range takes a slot) and compaction keeps the tail, so the host passes the
   // tail to the appending kernels instead of having them read and publish it
   uint64_t tail[2] = {0, 0};
+  // upper bound of the frames held (G, GE, GL blocks): every GPU sub-op of n blocks may
+  // take n more; nothing is subtracted.  While bound + n <= nframes a sub-op cannot need
+  // a victim, and its victim kernels are not launched.
+  uint64_t used_ub = 0;
   int npar = 0;             // parity slot of the multi-CTA classify's need counter
   // device intake result for the current op (intervals in T.dlo/dpre/dw)
   bool dev_iv = false, dev_anyw = false;
@@ -863,18 +867,23 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     cudaEvent_t sp = span_open(a);
     const uint64_t tail0 = a->tail[RING_USED];
     a->tail[RING_USED] += n;
+    const uint64_t used_before = a->used_ub;
+    a->used_ub = std::min<uint64_t>(a->nframes, a->used_ub + n);
     if (n <= kSmallPlan) {
       CK(launch_plan_small(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->ps));
       a->n_launch += 1;
     } else {
-      CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->npar, a->ps));
-      if (n > kVictWideMin)
-        CK(launch_victims_wide(a->T, seq, 0, 0, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), n,
-                               a->npar, a->ps));
-      else
-        CK(launch_victims(a->T, seq, 0, 0, a->npar, a->ps));
+      const int k0 = used_before + n <= a->nframes;   // no victim possible: skip the victim kernels
+      CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->npar, k0, a->ps));
+      if (!k0) {
+        if (n > kVictWideMin)
+          CK(launch_victims_wide(a->T, seq, 0, 0, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap),
+                                 n, a->npar, a->ps));
+        else
+          CK(launch_victims(a->T, seq, 0, 0, a->npar, a->ps));
+      }
       a->npar ^= 1;
-      a->n_launch += n > kVictWideMin ? 3 : 2;
+      a->n_launch += k0 ? 1 : (n > kVictWideMin ? 3 : 2);
     }
     span_close(a, sp, 0);
     if (use_ce(a, n)) {
@@ -997,18 +1006,23 @@ static um_status run_gpu_op2(um_arena* a, int touch) {
     cudaEvent_t sp = span_open(a);
     const uint64_t tail0 = a->tail[RING_USED];
     a->tail[RING_USED] += n;
+    const uint64_t used_before = a->used_ub;
+    a->used_ub = std::min<uint64_t>(a->nframes, a->used_ub + n);
     if (n <= kSmallPlan) {
       CK(launch_plan_small(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->ps));
       a->n_launch += 1;
     } else {
-      CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->npar, a->ps));
-      if (n > kVictWideMin)
-        CK(launch_victims_wide(a->T, seq, 0, 0, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), n,
-                               a->npar, a->ps));
-      else
-        CK(launch_victims(a->T, seq, 0, 0, a->npar, a->ps));
+      const int k0 = used_before + n <= a->nframes;   // no victim possible: skip the victim kernels
+      CK(launch_classify(a->T, iv, (uint32_t)g0, n, seq, touch, tail0, a->npar, k0, a->ps));
+      if (!k0) {
+        if (n > kVictWideMin)
+          CK(launch_victims_wide(a->T, seq, 0, 0, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap),
+                                 n, a->npar, a->ps));
+        else
+          CK(launch_victims(a->T, seq, 0, 0, a->npar, a->ps));
+      }
       a->npar ^= 1;
-      a->n_launch += n > kVictWideMin ? 3 : 2;
+      a->n_launch += k0 ? 1 : (n > kVictWideMin ? 3 : 2);
     }
     span_close(a, sp, 0);
     sp = span_open(a);

@@ -44,6 +44,7 @@ struct Ctl {
   unsigned int vt_reach;                // wide victim scan: passes in the apply work table (vpass)
   unsigned int pc_done;                 // k_plan_commit completion ticket (host read-back flag)
   unsigned long long xlog_n;            // transfer log: records appended (may exceed the capacity)
+  unsigned int cls_done;                // k_classify with k = 0 guaranteed: completion ticket
   // counters, striped over 8 cache lines by CTA index (fire-and-forget atomics from
   // thousands of CTAs do not serialise on one address); the host sums the stripes
   long long stats[8][S_N];
@@ -180,8 +181,10 @@ cudaError_t setup_kernels();
 cudaError_t launch_init(const Tables& T, int nhframes_alloc, cudaStream_t s);
 // tail0: the ring tail before this sub-op's appends (host-tracked, exact); npar: parity
 // slot of the need counter for multi-CTA sub-ops (alternates per multi-CTA sub-op)
+// k0 != 0: the host guarantees that the sub-op needs no victim (its blocks fit the free
+// frames); classify then does the victim kernels' k = 0 bookkeeping and none is launched
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
-                            unsigned long long tail0, int npar, cudaStream_t s);
+                            unsigned long long tail0, int npar, int k0, cudaStream_t s);
 cudaError_t launch_victims(const Tables& T, uint32_t seq, int evict_mode, uint32_t want, int npar, cudaStream_t s);
 // K1+K2+K3 fused in one CTA for sub-ops of <= kSmallPlan blocks
 constexpr uint32_t kSmallPlan = 4096;

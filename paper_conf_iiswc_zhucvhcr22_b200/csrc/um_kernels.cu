@@ -779,9 +779,34 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
 template <bool LIST>
 __global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
                                                         uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
-                                                        int npar) {
+                                                        int npar, int k0) {
   pdl_enter();
   classify_body<4, LIST>(T, iv, g0, n, seq, touch, tail0, npar);
+  if (k0) {
+    // the host guarantees k = 0 (every block of the sub-op fits the free frames), so no
+    // victim kernel runs: the CTA that finishes last publishes the need count and does
+    // the k = 0 frame bookkeeping of the victim kernels
+    __shared__ int s_last;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      s_last = atomicAdd(&T.ctl->cls_done, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (s_last && threadIdx.x == 0) {
+      __threadfence();
+      Ctl* c = T.ctl;
+      const uint32_t nn = ((volatile unsigned int*)c->need_cnt)[npar];
+      const int f0 = c->free_top;
+      c->n_need = nn;
+      c->need_cnt[npar ^ 1] = 0;
+      c->n_vict = 0;
+      c->f0 = (uint32_t)f0;
+      c->free_top = f0 - (int)min((uint32_t)f0, nn);
+      c->used_tail += n;
+      c->cls_done = 0;
+    }
+  }
 }
 
 // ------------------------------------------------------------------------------------
@@ -2314,10 +2339,10 @@ cudaError_t launch_poison(const Tables& T, cudaStream_t s) {
 uint32_t classify_tile() { return (uint32_t)kStTPB * 4u; }
 
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
-                            unsigned long long tail0, int npar, cudaStream_t s) {
+                            unsigned long long tail0, int npar, int k0, cudaStream_t s) {
   unsigned nt = n ? ceil_div(n, classify_tile()) : 1;
-  cudaError_t le__ = iv.blist ? launch_pdl(k_classify<true>, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar)
-                              : launch_pdl(k_classify<false>, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar);
+  cudaError_t le__ = iv.blist ? launch_pdl(k_classify<true>, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar, k0)
+                              : launch_pdl(k_classify<false>, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar, k0);
   if (le__) return le__;
   return cudaGetLastError();
 }
