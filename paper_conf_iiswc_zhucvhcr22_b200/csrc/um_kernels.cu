@@ -936,6 +936,7 @@ __device__ __forceinline__ void victims_body(const Tables& T, uint32_t seq, int 
       T.vkind[j] = ss;
       T.vhf[j] = hf;
       T.sk[v] = mk_sk(isG ? ST_H : ST_HD, 0);
+      if (T.phz) T.phz[v] = 0u;   // written back whole (dead pages read as zero by rule)
       T.map[v] = UM_NONE;
       T.frame_of[v] = UM_NONE;
       T.hframe[v] = hf;
@@ -1349,6 +1350,7 @@ __global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict
           T.vkind[j] = ss[q];
           T.vhf[j] = hf[q];
           T.sk[v[q]] = mk_sk(isG ? ST_H : ST_HD, 0);
+          if (T.phz) T.phz[v[q]] = 0u;
           T.map[v[q]] = UM_NONE;
           T.frame_of[v[q]] = UM_NONE;
           T.hframe[v[q]] = hf[q];
@@ -1454,7 +1456,6 @@ __device__ __forceinline__ void item_commit(const Tables& T, uint32_t i, const X
   T.frame_of[bb] = x.fr;
   T.map[bb] = x.fr;
   const uint32_t hf = T.needhf[i];
-  if (T.phz && T.needk[i] == ST_H) T.phz[bb] = 0u;   // its pages now live in the frame
   if (T.needk[i] == ST_H && hf != UM_NONE) {
     T.hframe[bb] = UM_NONE;
     if (!(x.flags & XI_SWAP)) {
@@ -1523,121 +1524,158 @@ struct Unit {
   __device__ bool pure_zf() const { return zf && !d2h_dst; }
 };
 
+// One item's plan as the transfer loop needs it (block-base pointers and page masks).
+struct SPlan {
+  char* frame;          // the item's destination frame (HBM)
+  char* d2h;            // host frame receiving the victim's (or D2H-only block's) bytes, or null
+  const char* h2d;      // host frame holding the newcomer's bytes, or null (zero-fill)
+  uint32_t dmask;       // pages not written back (dead in the victim / D2H-only block)
+  uint32_t zmask;       // pages zero-filled instead of migrated (dead in the newcomer)
+  uint32_t hzmask;      // pages migrated from the zero page (zero content on the host)
+};
+
+// K4.  The CTA's warp walks a contiguous range of CH-byte units.  Plans are computed 32
+// items at a time, one per lane (coalesced, independent loads), into shared memory;
+// lane 0 issues the TMA operations from them, so the per-item lookups never sit between
+// two bulk copies.  Phase 1 stores the zero tile into every pure zero-fill unit; phase 2
+// runs the other units through an S-stage load -> store ring.  Items are committed
+// (state, mapping, host-frame release, counters, log) during phase 1's planning, by the
+// CTA holding the item's first unit; nothing the copies read is changed by a commit.
 __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t seq) {
   pdl_enter();
   extern __shared__ __align__(128) char smem[];
   __shared__ __align__(8) uint64_t bar[kXferStages];
+  __shared__ SPlan s_pl[32];
+  const uint32_t lane = threadIdx.x;
   const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
   const uint32_t cpb = T.B / CH;
+  const uint32_t upp = T.P / CH;   // units per page (single level: the whole block)
   char* zero = smem;
   char* stA = smem + CH;                      // S stages of CH (victim/old bytes)
   char* stB = smem + CH + kXferStages * CH;   // S stages of CH (new bytes)
-  for (uint32_t i = threadIdx.x * 16; i < CH; i += 32 * 16) *reinterpret_cast<uint4*>(zero + i) = make_uint4(0, 0, 0, 0);
+  for (uint32_t i = lane * 16; i < CH; i += 32 * 16) *reinterpret_cast<uint4*>(zero + i) = make_uint4(0, 0, 0, 0);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  __syncwarp();
   Ctl* c = T.ctl;
-  if (threadIdx.x == 0) {
-    const uint32_t n_items = mode == SVC_SUBOP ? c->n_need : c->n_d2h;
-    const uint32_t f0 = c->f0;
-    const uint32_t nfu = min(f0, n_items);
-    // each CTA takes a contiguous range of units, so consecutive units mostly share an
-    // item and its plan is looked up once (the lookups are dependent global loads)
-    const unsigned long long units = (unsigned long long)n_items * cpb;
-    const unsigned long long ubeg = units * blockIdx.x / gridDim.x;
-    const unsigned long long mine = units * (blockIdx.x + 1) / gridDim.x - ubeg;
+  const uint32_t n_items = mode == SVC_SUBOP ? c->n_need : c->n_d2h;
+  const uint32_t f0 = c->f0;
+  const uint32_t nfu = min(f0, n_items);
+  const unsigned long long units = (unsigned long long)n_items * cpb;
+  const unsigned long long ubeg = units * blockIdx.x / gridDim.x;
+  const unsigned long long uend = units * (blockIdx.x + 1) / gridDim.x;
+  if (lane == 0) {
     for (int s = 0; s < kXferStages; ++s) mbar_init(&bar[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-
-    uint32_t cached_i = UM_NONE;
-    XItem cached;
-    ItemPages cpg{0u, 0u, 0u};
-    const uint32_t upp = T.P / CH;   // units per page (ppc = 1: one page = the block)
-    // phase 1 commits pure zero-fill items, phase 2 all others (each exactly once)
-    auto make = [&](unsigned long long t, int phase) -> Unit {
-      unsigned long long u = ubeg + t;
-      uint32_t i = (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
-      size_t coff = (size_t)ch * CH;
-      Unit x;
+  }
+  __syncwarp();
+  // plans of items [b0, b0 + 32) (warp-collective); commit = phase 1 of a sub-op
+  uint32_t batch = UM_NONE;
+  auto plan_batch = [&](uint32_t b0, bool commit) {
+    __syncwarp();                       // every lane is done with the previous batch
+    const uint32_t i = b0 + lane;
+    if (i < n_items) {
+      SPlan q;
       if (mode == SVC_SUBOP) {
-        if (i != cached_i) {
-          cached = item_plan(T, i, f0, nfu);
-          cpg = item_pages(T, i, cached, f0);
-          cached_i = i;
-        }
-        const XItem& p = cached;
-        const uint32_t pg = ch / upp;
-        x.frame = T.frames + (size_t)p.fr * T.B + coff;
-        x.d2h_dst = ((p.flags & XI_D2H) && !((cpg.vdead >> pg) & 1u)) ? hptr(T, p.dst_hf) + coff : nullptr;
-        const bool mig = (p.flags & XI_H2D) && !((cpg.ndead >> pg) & 1u);
-        x.h2d_src = mig ? hptr(T, ((cpg.nhz >> pg) & 1u) ? T.zero_hf : p.src_hf) + coff : nullptr;
-        x.zf = !mig;
-        if (ch == 0 && (x.pure_zf() ? 1 : 2) == phase) {
-          item_log(T, i, p, seq, f0, cpg);
-          item_page_stats(T, cpg);
-          item_commit(T, i, p, seq);
+        const XItem x = item_plan(T, i, f0, nfu);
+        const ItemPages pg = item_pages(T, i, x, f0);
+        q.frame = T.frames + (size_t)x.fr * T.B;
+        q.d2h = (x.flags & XI_D2H) ? hptr(T, x.dst_hf) : nullptr;
+        q.h2d = (x.flags & XI_H2D) ? hptr(T, x.src_hf) : nullptr;
+        q.dmask = pg.vdead;
+        q.zmask = (x.flags & XI_H2D) ? pg.ndead : 0xffffffffu;
+        q.hzmask = pg.nhz;
+        if (commit && (unsigned long long)i * cpb >= ubeg && (unsigned long long)i * cpb < uend) {
+          item_log(T, i, x, seq, f0, pg);
+          item_page_stats(T, pg);
+          item_commit(T, i, x, seq);
         }
       } else {
-        uint32_t fr = T.d2h_frame[i], hf = T.d2h_hf[i];
-        const uint32_t dm = T.pdead ? T.d2h_dmask[i] : 0u;
-        x.frame = T.frames + (size_t)fr * T.B + coff;
-        x.d2h_dst = (hf != UM_NONE && !((dm >> (ch / upp)) & 1u)) ? hptr(T, hf) + coff : nullptr;
-        x.h2d_src = nullptr;
-        x.zf = false;
+        const uint32_t hf = T.d2h_hf[i];
+        q.frame = T.frames + (size_t)T.d2h_frame[i] * T.B;
+        q.d2h = hf != UM_NONE ? hptr(T, hf) : nullptr;
+        q.h2d = nullptr;
+        q.dmask = T.pdead ? T.d2h_dmask[i] : 0u;
+        q.zmask = 0u;
+        q.hzmask = 0u;
       }
-      return x;
-    };
-    // Phase 1: zero-fill units need no load: bulk-store the zeroed tile right away.
-    if (mode == SVC_SUBOP) {
-      uint32_t issued = 0;
-      for (unsigned long long t = 0; t < mine; ++t) {
-        Unit x = make(t, 1);
-        if (!x.pure_zf()) continue;
+      s_pl[lane] = q;
+    }
+    batch = b0;
+    __syncwarp();
+  };
+  // unit u of this CTA's range (warp-uniform: every lane builds the same unit)
+  auto make = [&](unsigned long long u, bool commit) -> Unit {
+    const uint32_t i = (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
+    if (batch == UM_NONE || i - batch >= 32u) plan_batch(i, commit);
+    const SPlan& q = s_pl[i - batch];
+    const size_t coff = (size_t)ch * CH;
+    const uint32_t pg = ch / upp;
+    Unit x;
+    x.frame = q.frame + coff;
+    x.d2h_dst = (q.d2h && !((q.dmask >> pg) & 1u)) ? q.d2h + coff : nullptr;
+    const bool mig = q.h2d && !((q.zmask >> pg) & 1u);
+    x.h2d_src = mig ? (((q.hzmask >> pg) & 1u) ? hptr(T, T.zero_hf) : q.h2d) + coff : nullptr;
+    x.zf = mode == SVC_SUBOP && !mig;
+    return x;
+  };
+  // Phase 1: zero-fill units need no load: bulk-store the zeroed tile right away (this
+  // pass also plans every item once with commit = true).
+  if (mode == SVC_SUBOP) {
+    uint32_t issued = 0;
+    for (unsigned long long u = ubeg; u < uend; ++u) {
+      const Unit x = make(u, true);
+      if (lane == 0 && x.pure_zf()) {
         bulk_s2g(x.frame, zero, CH);
         if ((++issued & 31) == 0) bulk_commit();
       }
-      bulk_commit();
     }
-    // Phase 2: transfer units through the S-stage TMA ring.
-    unsigned long long tn = 0;
-    auto next_xfer = [&](Unit& x) -> bool {
-      while (tn < mine) {
-        x = make(tn++, 2);
-        if (!x.pure_zf()) return true;
-      }
-      return false;
-    };
-    Unit U[kXferStages];
-    auto issue_loads = [&](int s, const Unit& x) {
-      uint32_t bytes = (x.d2h_dst ? CH : 0u) + (x.h2d_src ? CH : 0u);
-      mbar_expect_tx(&bar[s], bytes);
-      if (x.d2h_dst) bulk_g2s(stA + s * CH, x.frame, CH, &bar[s]);
-      if (x.h2d_src) bulk_g2s(stB + s * CH, x.h2d_src, CH, &bar[s]);
-    };
-    unsigned long long loaded = 0;
-    for (int s = 0; s < kXferStages; ++s) {
-      if (!next_xfer(U[s])) break;
-      issue_loads(s, U[s]);
-      ++loaded;
+    if (lane == 0) bulk_commit();
+    batch = UM_NONE;
+  }
+  // Phase 2: transfer units through the S-stage TMA ring.
+  unsigned long long tn = ubeg;
+  auto next_xfer = [&](Unit& x) -> bool {
+    while (tn < uend) {
+      x = make(tn++, false);
+      if (!x.pure_zf()) return true;
     }
-    for (unsigned long long k = 0; k < loaded; ++k) {
-      const int s = (int)(k % kXferStages);
+    return false;
+  };
+  Unit U[kXferStages];
+  auto issue_loads = [&](int s, const Unit& x) {
+    if (lane != 0) return;
+    const uint32_t bytes = (x.d2h_dst ? CH : 0u) + (x.h2d_src ? CH : 0u);
+    mbar_expect_tx(&bar[s], bytes);
+    if (x.d2h_dst) bulk_g2s(stA + s * CH, x.frame, CH, &bar[s]);
+    if (x.h2d_src) bulk_g2s(stB + s * CH, x.h2d_src, CH, &bar[s]);
+  };
+  unsigned long long loaded = 0;
+  for (int s = 0; s < kXferStages; ++s) {
+    if (!next_xfer(U[s])) break;
+    issue_loads(s, U[s]);
+    ++loaded;
+  }
+  for (unsigned long long k = 0; k < loaded; ++k) {
+    const int s = (int)(k % kXferStages);
+    if (lane == 0) {
       mbar_wait(&bar[s], (uint32_t)((k / kXferStages) & 1));
       const Unit& x = U[s];
       if (x.d2h_dst) bulk_s2g(x.d2h_dst, stA + s * CH, CH);
       if (x.h2d_src) bulk_s2g(x.frame, stB + s * CH, CH);
       else if (x.zf) bulk_s2g(x.frame, zero, CH);
       bulk_commit();
-      if (k >= 1 && loaded == k - 1 + kXferStages) {
-        const int sp = (int)((k - 1) % kXferStages);
-        Unit y;
-        if (next_xfer(y)) {
-          bulk_wait_read1();
-          U[sp] = y;
-          issue_loads(sp, U[sp]);
-          ++loaded;
-        }
+    }
+    if (k >= 1 && loaded == k - 1 + kXferStages) {
+      const int sp = (int)((k - 1) % kXferStages);
+      Unit y;
+      if (next_xfer(y)) {
+        if (lane == 0) bulk_wait_read1();
+        U[sp] = y;
+        issue_loads(sp, U[sp]);
+        ++loaded;
       }
     }
+  }
+  if (lane == 0) {
     bulk_wait_all();
     if (mode == SVC_D2H_ONLY) {
       __threadfence();
@@ -1958,7 +1996,10 @@ __device__ __forceinline__ void directive_body(const Tables& T, int kind, uint32
           T.frame_of[bb] = UM_NONE;
           T.map[bb] = UM_NONE;
         }
-        if (ss != ST_H) T.sk[bb] = mk_sk(ST_H, 0);
+        if (ss != ST_H) {
+          T.sk[bb] = mk_sk(ST_H, 0);
+          if (T.phz) T.phz[bb] = 0u;   // revived pages are marked by k_page_host_revive
+        }
       }
     }
   }
