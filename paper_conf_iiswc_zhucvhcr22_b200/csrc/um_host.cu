@@ -1514,6 +1514,7 @@ UM_API um_status um_dump(um_arena* a, uint8_t* st, uint32_t* used_order, uint32_
     for (unsigned long long p = head; p < tail; ++p) {
       uint64_t e = ring[p & (a->L.cap - 1)];
       uint32_t b = (uint32_t)e, k = (uint32_t)(e >> 32);
+      if (b == UM_NONE) continue;   // a slot whose block did not enter the ring
       uint8_t x = hst[b];
       bool live = (r == RING_USED ? x == ST_G : (x == ST_GE || x == ST_GL)) && (hsk[b] >> 3) == k;
       if (live) {

@@ -40,8 +40,11 @@ __device__ __forceinline__ uint8_t st_of(uint32_t w) { return (uint8_t)(w & 7u);
 __device__ __forceinline__ uint32_t key_of(uint32_t w) { return w >> 3; }
 __device__ __forceinline__ uint32_t mk_sk(uint8_t st, uint32_t key) { return (key << 3) | st; }
 __device__ __forceinline__ uint8_t ld_st(const Tables& T, uint32_t b) { return st_of(T.sk[b]); }
-// liveness of ring entry (key kk, block b) whose ring holds state set {G} (USED) or {GE, GL} (DISC)
+// liveness of ring entry (key kk, block b) whose ring holds state set {G} (USED) or {GE, GL} (DISC);
+// a slot whose block did not enter the ring holds kDeadSlot (block id NONE: no state gather)
+constexpr unsigned long long kDeadSlot = ~0ull;
 __device__ __forceinline__ bool entry_live(const Tables& T, bool disc, uint32_t blk, uint32_t kk) {
+  if (blk == UM_NONE) return false;
   const uint32_t w = T.sk[blk];
   const uint8_t ss = st_of(w);
   return (disc ? (ss == ST_GE || ss == ST_GL) : ss == ST_G) && key_of(w) == kk;
@@ -465,7 +468,8 @@ __device__ __forceinline__ void classify_single(const Tables& T, const OpIv& iv,
     bool nd = false;
     if (idx < n) {
       T.pin[b[k]] = seq;
-      T.used_ring[(tail0 + idx) & T.cap_mask] = kseq | b[k];
+      // a hit (touch of G / GL) keeps its key: its slot is dead from the start
+      T.used_ring[(tail0 + idx) & T.cap_mask] = (touch && (s[k] == ST_G || s[k] == ST_GL)) ? kDeadSlot : (kseq | b[k]);
       nd = s[k] <= ST_HD;
       cls += 1u << (4 * s[k]);
     }
@@ -705,7 +709,8 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
     const uint32_t idx = tbase + k * TPB + threadIdx.x;
     if (idx < n) {
       T.pin[b[k]] = seq;
-      T.used_ring[(tail0 + idx) & T.cap_mask] = kseq | b[k];
+      // a hit (touch of G / GL) keeps its key: its slot is dead from the start
+      T.used_ring[(tail0 + idx) & T.cap_mask] = (touch && (s[k] == ST_G || s[k] == ST_GL)) ? kDeadSlot : (kseq | b[k]);
       cls += 1u << (5 * s[k]);
     }
     bN[k] = __ballot_sync(FULL, s[k] <= ST_HD);   // 0xff (no item) is > ST_HD
@@ -1956,7 +1961,8 @@ __device__ __forceinline__ void directive_body(const Tables& T, int kind, uint32
       const uint32_t bb = lo + idx;
       const uint8_t ss = s[k];
       if (disc) {
-        T.disc_ring[(tail0 + idx) & T.cap_mask] = kseq | bb;
+        // only a G block enters DISC here (GL -> GE keeps its slot, A6; H -> HD has none)
+        T.disc_ring[(tail0 + idx) & T.cap_mask] = ss == ST_G ? (kseq | bb) : kDeadSlot;
         if (T.pdead) T.pdead[bb] = T.plazy[bb] = T.phz[bb] = 0u;   // whole chunk: chunk level
         if (ss == ST_G) {
           T.sk[bb] = mk_sk(kind == DIR_DISCARD ? ST_GE : ST_GL, seq);
