@@ -1607,13 +1607,25 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
     batch = b0;
     __syncwarp();
   };
-  // unit u of this CTA's range (warp-uniform: every lane builds the same unit)
-  auto make = [&](unsigned long long u, bool commit) -> Unit {
-    const uint32_t i = (uint32_t)(u / cpb), ch = (uint32_t)(u % cpb);
+  // Units are walked as (item, chunk) pairs with shifts (cpb and upp are powers of two):
+  // no 64-bit division per unit.  The warp walks them uniformly; lane 0 issues.
+  const uint32_t lcpb = 31 - __clz(cpb), lupp = 31 - __clz(upp);
+  const uint32_t i_lo = (uint32_t)(ubeg >> lcpb), i_end = (uint32_t)((uend + cpb - 1) >> lcpb);
+  const uint32_t ch_lo = (uint32_t)(ubeg & (cpb - 1));
+  const uint32_t ch_end_last = (uint32_t)(((uend - 1) & (cpb - 1)) + 1);
+  auto plan_of = [&](uint32_t i, bool commit) -> const SPlan& {
     if (batch == UM_NONE || i - batch >= 32u) plan_batch(i, commit);
-    const SPlan& q = s_pl[i - batch];
+    return s_pl[i - batch];
+  };
+  // pages of an item whose units only need the zero tile (nothing to load or write back)
+  auto pure_pages = [&](const SPlan& q) -> uint32_t {
+    const uint32_t zf = q.h2d ? q.zmask : 0xffffffffu;
+    const uint32_t wb = q.d2h ? ~q.dmask : 0u;
+    return mode == SVC_SUBOP ? (zf & ~wb) : 0u;
+  };
+  auto unit_of = [&](const SPlan& q, uint32_t ch) -> Unit {
     const size_t coff = (size_t)ch * CH;
-    const uint32_t pg = ch / upp;
+    const uint32_t pg = ch >> lupp;
     Unit x;
     x.frame = q.frame + coff;
     x.d2h_dst = (q.d2h && !((q.dmask >> pg) & 1u)) ? q.d2h + coff : nullptr;
@@ -1623,25 +1635,38 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
     return x;
   };
   // Phase 1: zero-fill units need no load: bulk-store the zeroed tile right away (this
-  // pass also plans every item once with commit = true).
-  if (mode == SVC_SUBOP) {
+  // pass also plans, and commits, every item of the range once).
+  if (mode == SVC_SUBOP && ubeg < uend) {
     uint32_t issued = 0;
-    for (unsigned long long u = ubeg; u < uend; ++u) {
-      const Unit x = make(u, true);
-      if (lane == 0 && x.pure_zf()) {
-        bulk_s2g(x.frame, zero, CH);
+    for (uint32_t i = i_lo; i < i_end; ++i) {
+      const SPlan& q = plan_of(i, true);
+      const uint32_t pm = pure_pages(q);
+      if (!pm || lane != 0) continue;
+      const uint32_t cb = i == i_lo ? ch_lo : 0u, ce = i + 1 == i_end ? ch_end_last : cpb;
+      for (uint32_t ch = cb; ch < ce; ++ch) {
+        if (!((pm >> (ch >> lupp)) & 1u)) continue;
+        bulk_s2g(q.frame + (size_t)ch * CH, zero, CH);
         if ((++issued & 31) == 0) bulk_commit();
       }
     }
     if (lane == 0) bulk_commit();
     batch = UM_NONE;
   }
-  // Phase 2: transfer units through the S-stage TMA ring.
-  unsigned long long tn = ubeg;
+  // Phase 2: the other units through the S-stage TMA ring (cursor: item ci, chunk cch)
+  uint32_t ci = i_lo, cch = ch_lo;
   auto next_xfer = [&](Unit& x) -> bool {
-    while (tn < uend) {
-      x = make(tn++, false);
-      if (!x.pure_zf()) return true;
+    while (ci < i_end) {
+      const SPlan& q = plan_of(ci, false);
+      const uint32_t ce = ci + 1 == i_end ? ch_end_last : cpb;
+      // pages with a load: not pure zero-fill (sub-op), live pages to write back (D2H-only)
+      const uint32_t keep = mode == SVC_SUBOP ? ~pure_pages(q) : (q.d2h ? ~q.dmask : 0u);
+      while (cch < ce && !((keep >> (cch >> lupp)) & 1u)) ++cch;
+      if (cch < ce) {
+        x = unit_of(q, cch++);
+        return true;
+      }
+      ++ci;
+      cch = 0;
     }
     return false;
   };
