@@ -48,6 +48,7 @@ def parse():
     p.add_argument("--pin-threads", type=int, default=8)
     p.add_argument("--no-compare", action="store_true")
     p.add_argument("--no-state-bench", action="store_true")
+    p.add_argument("--state-only", action="store_true", help="run only the state-kernel microbench")
     p.add_argument("--app-overlap", default="off", choices=["on", "off"],
                    help="UM_F_OVERLAP (reading R7) for the headline modes: app kernels pipelined with the "
                         "next sub-ops (measured no faster on C3: the step is transfer-bound and a write-"
@@ -621,6 +622,35 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
         del ws
 
 
+def state_runs(torch, um, mem, budget, arena_bytes):
+    """State microbench on fresh arenas over the same memory: one warm-up (first-touch
+    costs of the workspace pages and kernel images), then three; per op the run with the
+    median span is reported (single ~20 us spans vary by +-20 % from run to run)."""
+    state_bench(torch, um, mem, budget, arena_bytes, seed=1)
+    runs = [state_bench(torch, um, mem, budget, arena_bytes, seed=s) for s in (0, 2, 3)]
+    state = dict(runs[0])
+    for op in ("touch_2^21_random", "discard_2^21", "touch_2^21_pressure"):
+        by = sorted(runs, key=lambda r: r[op]["ms"])
+        state[op] = dict(by[1][op])
+        state[op]["ms_runs"] = [r[op]["ms"] for r in runs]
+    for k in ("empty_kernel_span_us", "zero_fill_gbs"):
+        state[k] = sorted(r[k] for r in runs)[1]
+    state["reps"] = "median of three runs (seeds 0, 2, 3) after one warm-up run"
+    return state
+
+
+def main_state_only(args):
+    """`--state-only`: the state-kernel microbench alone (for ncu launch lists and A/B)."""
+    import torch
+    from paper_conf_iiswc_zhucvhcr22_b200 import build, um
+    build.build()
+    torch.cuda.set_device(0)
+    free, _ = torch.cuda.mem_get_info(0)
+    budget, arena_bytes, _, _ = plan_sizes(args, free, 1)
+    mem = um.Memory(args.block, arena_bytes, budget, host_pool_bytes=2 * GiB)
+    print(json.dumps({"roofline_state": state_runs(torch, um, mem, budget, arena_bytes)}), flush=True)
+
+
 def _barrier(torch):
     from paper_conf_iiswc_zhucvhcr22_b200.dist import barrier
     barrier()
@@ -796,20 +826,7 @@ def main_ours(args):
     other = run_mode(torch, um, harness, mem, trace, "eager", W, Kc, flags_extra=um.UM_F_OVERLAP ^ ovf) \
         if not args.no_compare else None
     ovl_r, seq_r = (res.get("eager"), other) if ovf else (other, res.get("eager"))
-    state = None
-    if not args.no_state_bench:
-        # runs on fresh arenas over the same memory: one warm-up (first-touch costs of the
-        # workspace pages and kernel images), then three; per op the run with the median
-        # span is reported (single ~20 us spans vary by +-20 % from run to run)
-        state_bench(torch, um, mem, budget, arena_bytes, seed=1)
-        runs = [state_bench(torch, um, mem, budget, arena_bytes, seed=s) for s in (0, 2, 3)]
-        state = dict(runs[0])
-        for op in ("touch_2^21_random", "discard_2^21", "touch_2^21_pressure"):
-            by = sorted(runs, key=lambda r: r[op]["ms"])
-            state[op] = dict(by[1][op])
-            state[op]["ms_runs"] = [r[op]["ms"] for r in runs]
-        state["empty_kernel_span_us"] = sorted(r["empty_kernel_span_us"] for r in runs)[1]
-        state["reps"] = "median of three runs (seeds 0, 2, 3) after one warm-up run"
+    state = None if args.no_state_bench else state_runs(torch, um, mem, budget, arena_bytes)
     rmt_r = None if args.no_compare else rmt_leg(torch, um, harness, mem, budget, args.oversub, B)
     c2 = None if args.no_compare else c2_stream(torch, um, harness, mem, budget, host_pool)
     c3k = None if args.no_compare else c3_64k(torch, um, harness, mem, budget, arena_bytes)
@@ -965,5 +982,7 @@ if __name__ == "__main__":
     a = parse()
     if a.impl == "reference":
         main_reference(a)
+    elif a.state_only:
+        main_state_only(a)
     else:
         main_ours(a)
