@@ -590,10 +590,10 @@ __device__ bool grid_finish(const Tables& T, const int (&slots)[NC], const long 
   return true;
 }
 
-template <int IPT, bool LIST>
+template <int IPT, bool LIST, int TPB>
 __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
                                               int touch, unsigned long long tail0, int npar) {
-  constexpr int TPB = kStTPB, TILE = TPB * IPT, NW = TPB / 32, NWORD = TILE / 32;
+  constexpr int TILE = TPB * IPT, NW = TPB / 32, NWORD = TILE / 32;
   constexpr int PERL = (NWORD + 31) / 32;   // bitmap words per lane in the warp prefix
   // Interval lookup without a search: the tile's interval slice [ja, jb] is staged as
   // d[q] = lo - pre (block = rank + d), and the start of every slice interval but the
@@ -762,31 +762,35 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
       c4 += e & 255u; c5 += e >> 8;
     }
     const long long B = T.B;
+    // only non-zero counters (a uniform batch, e.g. all U, adds two instead of six)
+    auto add = [&](int slot, long long v) {
+      if (v) stat_add(T, slot, v);
+    };
     if (touch) {
       // faults: U+H+HD+GE ; hits: G+GL ; remaps: GE
-      stat_add(T, S_FAULTS, c0 + c1 + c2 + c4);
-      stat_add(T, S_HITS, c3 + c5);
-      stat_add(T, S_REMAPS, c4);
+      add(S_FAULTS, c0 + c1 + c2 + c4);
+      add(S_HITS, c3 + c5);
+      add(S_REMAPS, c4);
     } else {
-      stat_add(T, S_REFRESH, c3);   // refreshes, remaps, revalidations
-      stat_add(T, S_REMAPS, c4);
-      stat_add(T, S_REVAL, c5);
+      add(S_REFRESH, c3);   // refreshes, remaps, revalidations
+      add(S_REMAPS, c4);
+      add(S_REVAL, c5);
     }
-    stat_add(T, S_H2D, (long long)c1 * B);          // h2d, zf, h2d_avoided
-    stat_add(T, S_ZF, (long long)(c0 + c2) * B);
-    stat_add(T, S_H2D_AV, (long long)c2 * B);
+    add(S_H2D, (long long)c1 * B);          // h2d, zf, h2d_avoided
+    add(S_ZF, (long long)(c0 + c2) * B);
+    add(S_H2D_AV, (long long)c2 * B);
     if (blockIdx.x == 0) T.ctl->n_rekey = n;   // USED slots appended
   }
 }
 
 // 4 items per thread, 8 CTAs/SM (A/B on B200: 8 items per thread at 6 CTAs/SM spills and
 // runs the 2^21-block touch in 42 vs 30 us)
-template <bool LIST>
-__global__ void __launch_bounds__(kStTPB, 8) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
-                                                        uint32_t n, uint32_t seq, int touch, unsigned long long tail0,
-                                                        int npar, int k0) {
+template <bool LIST, int TPB>
+__global__ void __launch_bounds__(TPB, 2048 / TPB) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
+                                                              uint32_t n, uint32_t seq, int touch,
+                                                              unsigned long long tail0, int npar, int k0) {
   pdl_enter();
-  classify_body<4, LIST>(T, iv, g0, n, seq, touch, tail0, npar);
+  classify_body<4, LIST, TPB>(T, iv, g0, n, seq, touch, tail0, npar);
   if (k0) {
     // the host guarantees k = 0 (every block of the sub-op fits the free frames), so no
     // victim kernel runs: the CTA that finishes last publishes the need count and does
@@ -2338,6 +2342,9 @@ __global__ void __launch_bounds__(256) k_tags(Tables T) {
 // launch wrappers
 // ------------------------------------------------------------------------------------
 static int g_nsm = 0;
+// k_classify CTA size: 256 threads x 4 items (UM_CLS_TPB=512: 512 x 4, half the CTAs,
+// need-list atomics and counter reductions; A/B)
+static int g_cls_tpb = 256;
 static int g_vscan_occ = 1;   // resident k_victims_scan CTAs per SM
 static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch (A/B)
 static int g_dir_occ = 8;     // resident k_directive CTAs per SM (persistent grid)
@@ -2351,13 +2358,15 @@ cudaError_t setup_kernels() {
   if (e) return e;
   if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
   if (const char* v = getenv("UM_VS_PREFETCH")) g_vs_prefetch = atoi(v) != 0;
+  if (const char* v = getenv("UM_CLS_TPB")) g_cls_tpb = atoi(v) == 512 ? 512 : 256;
   // Optionally one L1/shared carveout for every paging kernel (k_service needs 144 KB of
   // shared memory; a carveout change between consecutive kernels can force an SM drain).
   // UM_CARVEOUT=1 turns it on (A/B; off by default).
   bool carve = false;   // measured: no effect on the C1 small-op rate (B200, r01)
   if (const char* v = getenv("UM_CARVEOUT")) carve = atoi(v) != 0;
   if (carve) {
-    const void* ks[] = {(const void*)k_classify<false>, (const void*)k_classify<true>, (const void*)k_victims, (const void*)k_plan_small,
+    const void* ks[] = {(const void*)k_classify<false, 256>, (const void*)k_classify<true, 256>,
+                        (const void*)k_classify<false, 512>, (const void*)k_classify<true, 512>, (const void*)k_victims, (const void*)k_plan_small,
                         (const void*)k_victims_scan, (const void*)k_victims_apply, (const void*)k_service,
                         (const void*)k_app_stamp<256>, (const void*)k_app_stamp<128>, (const void*)k_directive, (const void*)k_ring_compact,
                         (const void*)k_plan_commit, (const void*)k_zero_items, (const void*)k_mark,
@@ -2408,13 +2417,18 @@ cudaError_t launch_poison(const Tables& T, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-uint32_t classify_tile() { return (uint32_t)kStTPB * 4u; }
+uint32_t classify_tile() { return (uint32_t)g_cls_tpb * 4u; }
 
 cudaError_t launch_classify(const Tables& T, OpIv iv, uint32_t g0, uint32_t n, uint32_t seq, int touch,
                             unsigned long long tail0, int npar, int k0, cudaStream_t s) {
   unsigned nt = n ? ceil_div(n, classify_tile()) : 1;
-  cudaError_t le__ = iv.blist ? launch_pdl(k_classify<true>, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar, k0)
-                              : launch_pdl(k_classify<false>, dim3(nt), dim3(kStTPB), 0, s, T, iv, g0, n, seq, touch, tail0, npar, k0);
+  cudaError_t le__;
+  if (g_cls_tpb == 512)
+    le__ = iv.blist ? launch_pdl(k_classify<true, 512>, dim3(nt), dim3(512), 0, s, T, iv, g0, n, seq, touch, tail0, npar, k0)
+                    : launch_pdl(k_classify<false, 512>, dim3(nt), dim3(512), 0, s, T, iv, g0, n, seq, touch, tail0, npar, k0);
+  else
+    le__ = iv.blist ? launch_pdl(k_classify<true, 256>, dim3(nt), dim3(256), 0, s, T, iv, g0, n, seq, touch, tail0, npar, k0)
+                    : launch_pdl(k_classify<false, 256>, dim3(nt), dim3(256), 0, s, T, iv, g0, n, seq, touch, tail0, npar, k0);
   if (le__) return le__;
   return cudaGetLastError();
 }
