@@ -17,10 +17,13 @@ def launches(path):
     hi = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
     h = rows[hi]
     ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
+    mi = h.index("Metric Name") if "Metric Name" in h else None
     tot, cnt = collections.defaultdict(float), collections.Counter()
     scale = {"ns": 1e-6, "nsecond": 1e-6, "us": 1e-3, "usecond": 1e-3, "ms": 1.0, "msecond": 1.0}
     for r in rows[hi + 1:]:
         if len(r) <= vi or not r[vi]:
+            continue
+        if mi is not None and r[mi] != "gpu__time_duration.sum":
             continue
         name = r[ki].split("(")[0]
         tot[name] += float(r[vi].replace(",", "")) * scale.get(r[ui], 1.0)
