@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 #include <cstdio>
 #include <cstdint>
+#include <cstdlib>
 
 #define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) { printf("{\"error\":\"%s\",\"line\":%d}\n", cudaGetErrorString(e_), __LINE__); return 1; } } while (0)
 
@@ -46,11 +47,11 @@ __global__ void k_st(char* dst, unsigned long long units) {
 int main() {
   int nsm;
   CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0));
-  const size_t bytes = 32ull << 30;
+  const size_t bytes = (size_t)(getenv("ZF_GIB") ? atoi(getenv("ZF_GIB")) : 32) << 30;
   const unsigned long long units = bytes / CH;
   char* d;
   CK(cudaMalloc(&d, bytes));
-  CK(cudaFuncSetAttribute(k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)CH));
+  CK(cudaFuncSetAttribute(k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(9 * CH)));
   cudaEvent_t a, b;
   cudaEventCreate(&a);
   cudaEventCreate(&b);
@@ -76,6 +77,7 @@ int main() {
     run(nm, nsm, [&] { k_tma<<<nsm, 32 * W, CH>>>(d, units, W); });
   }
   run("tma1_2ctas", 2 * nsm, [&] { k_tma<<<2 * nsm, 32, CH>>>(d, units, 1); });
+  run("tma1_smem144k", nsm, [&] { k_tma<<<nsm, 32, 9 * CH>>>(d, units, 1); });
   for (int W : {4, 8, 16, 32}) {
     char nm[32];
     snprintf(nm, sizeof nm, "st_warps%d", W);
