@@ -22,8 +22,15 @@ C3 DNN trace (pinned only by the invariants), contents of GE/GL/HD blocks beyond
 readings A7/A9, all timings.
 
 `oracle.chunks.ChunkOracle` is the two-level model of SURVEY NEXT-1 (2 MiB chunks as the
-residency / eviction unit, page-granular partial discards), pinned in
-tests/test_oracle_chunks.py (hand-derived scenarios, reduction to oracle.sim, page-level
-invariants).  No CUDA path implements it yet.
+residency / eviction unit, page-granular partial discards, reading R10), pinned
+in tests/test_oracle_chunks.py (hand-derived scenarios, reduction to oracle.sim,
+page-level invariants); the CUDA path's two-level mode is compared with it in
+tests/test_gpu_pages.py.
+
+`oracle.rmt` is the redundant-transfer accounting of SURVEY §8(c) item 7 (DESIGN.md
+reading R8), pinned in tests/test_rmt.py (Fig. 2's two redundant transfers, the C2
+closed form, a versioned flat-memory second formulation).
+
+`Oracle.free_range` is um_free (reading R9), pinned by the hand-derived scenarios E13.
 """
 from .sim import Oracle, replay, ST_NAMES, stamp  # noqa: F401
