@@ -96,7 +96,7 @@ typedef struct {
 typedef struct {
   int device;                 /* CUDA device ordinal                                       */
   uint32_t block_bytes;       /* 65536 or 2097152 (any power of two >= 4096 is accepted)  */
-  uint64_t arena_bytes;       /* multiple of block_bytes; nblocks = arena/block < 2^32-1   */
+  uint64_t arena_bytes;       /* multiple of block_bytes; nblocks = arena/block < 2^31     */
   uint64_t budget_bytes;      /* nframes = budget/block >= 1                               */
   void *frames;               /* DEVICE, >= nframes*block_bytes, caller-owned              */
   void *workspace;            /* DEVICE, >= um_workspace_size(), caller-owned              */

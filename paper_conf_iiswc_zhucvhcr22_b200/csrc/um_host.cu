@@ -60,7 +60,9 @@ static um_status check_cfg(const um_config* c) {
   }
   if (!is_pow2(c->block_bytes) || c->block_bytes < 4096) return UM_EINVAL;
   if (c->arena_bytes == 0 || c->arena_bytes % c->block_bytes) return UM_EINVAL;
-  if (c->arena_bytes / c->block_bytes >= 0xffffffffull) return UM_EINVAL;
+  // block ids < 2^31: bit 31 of a staged list entry is the write flag (fault-list and
+  // two-level chunk-list forms)
+  if (c->arena_bytes / c->block_bytes >= 0x80000000ull) return UM_EINVAL;
   if (c->budget_bytes < c->block_bytes) return UM_EINVAL;
   if (c->budget_bytes / c->block_bytes >= 0x7fffffffull) return UM_EINVAL;
   if (c->host_chunk_bytes == 0 || c->host_chunk_bytes % c->block_bytes) return UM_EINVAL;
