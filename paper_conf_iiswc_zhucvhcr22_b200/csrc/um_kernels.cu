@@ -1543,26 +1543,32 @@ struct SPlan {
   uint32_t hzmask;      // pages migrated from the zero page (zero content on the host)
 };
 
-// K4.  The CTA's warp walks a contiguous range of CH-byte units.  Plans are computed 32
-// items at a time, one per lane (coalesced, independent loads), into shared memory;
-// lane 0 issues the TMA operations from them, so the per-item lookups never sit between
-// two bulk copies.  Phase 1 stores the zero tile into every pure zero-fill unit; phase 2
-// runs the other units through an S-stage load -> store ring.  Items are committed
-// (state, mapping, host-frame release, counters, log) during phase 1's planning, by the
-// CTA holding the item's first unit; nothing the copies read is changed by a commit.
-__global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t seq) {
+// K4.  Each CTA takes a contiguous range of CH-byte units.  Warp 0 moves data: it runs
+// the units that need a load (write-back, migration, or both: the fused swap) through an
+// S-stage load -> store ring driven by lane 0 (cp.async.bulk + mbarrier).  Warps 1-3
+// zero-fill: each takes a third of the range and bulk-stores a zeroed smem tile into its
+// pure zero-fill units, and commits (state, mapping, host-frame release, counters, log)
+// the items whose first unit lies in its third.  Zero-fill (HBM) and transfers (PCIe)
+// thus overlap inside every CTA.  Plans are computed 32 items at a time, one per lane
+// (independent loads), into the warp's shared-memory slots; a commit changes nothing a
+// plan reads.  D2H-only lists (prefetch HOST, evict) use warp 0 alone.
+constexpr int kSvcWarps = 4;
+
+__global__ void __launch_bounds__(32 * kSvcWarps, 1) k_service(Tables T, int mode, uint32_t seq) {
   pdl_enter();
   extern __shared__ __align__(128) char smem[];
   __shared__ __align__(8) uint64_t bar[kXferStages];
-  __shared__ SPlan s_pl[32];
-  const uint32_t lane = threadIdx.x;
+  __shared__ SPlan s_plw[kSvcWarps][32];
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  SPlan* s_pl = s_plw[warp];
   const uint32_t CH = T.B < kXferChunk ? T.B : kXferChunk;
   const uint32_t cpb = T.B / CH;
   const uint32_t upp = T.P / CH;   // units per page (single level: the whole block)
   char* zero = smem;
   char* stA = smem + CH;                      // S stages of CH (victim/old bytes)
   char* stB = smem + CH + kXferStages * CH;   // S stages of CH (new bytes)
-  for (uint32_t i = lane * 16; i < CH; i += 32 * 16) *reinterpret_cast<uint4*>(zero + i) = make_uint4(0, 0, 0, 0);
+  for (uint32_t i = threadIdx.x * 16; i < CH; i += 32 * kSvcWarps * 16)
+    *reinterpret_cast<uint4*>(zero + i) = make_uint4(0, 0, 0, 0);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   Ctl* c = T.ctl;
   const uint32_t n_items = mode == SVC_SUBOP ? c->n_need : c->n_d2h;
@@ -1571,14 +1577,16 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
   const unsigned long long units = (unsigned long long)n_items * cpb;
   const unsigned long long ubeg = units * blockIdx.x / gridDim.x;
   const unsigned long long uend = units * (blockIdx.x + 1) / gridDim.x;
-  if (lane == 0) {
+  if (threadIdx.x == 0) {
     for (int s = 0; s < kXferStages; ++s) mbar_init(&bar[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  __syncwarp();
-  // plans of items [b0, b0 + 32) (warp-collective); commit = phase 1 of a sub-op
+  __syncthreads();   // zero tile and barriers visible to every warp
+  const uint32_t lcpb = 31 - __clz(cpb), lupp = 31 - __clz(upp);
+  // plans of items [b0, b0 + 32) (warp-collective); commit items whose first unit is in
+  // [cb, ce) (a zero-fill warp's third of the range)
   uint32_t batch = UM_NONE;
-  auto plan_batch = [&](uint32_t b0, bool commit) {
+  auto plan_batch = [&](uint32_t b0, bool commit, unsigned long long cb, unsigned long long ce) {
     __syncwarp();                       // every lane is done with the previous batch
     const uint32_t i = b0 + lane;
     if (i < n_items) {
@@ -1592,7 +1600,8 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
         q.dmask = pg.vdead;
         q.zmask = (x.flags & XI_H2D) ? pg.ndead : 0xffffffffu;
         q.hzmask = pg.nhz;
-        if (commit && (unsigned long long)i * cpb >= ubeg && (unsigned long long)i * cpb < uend) {
+        const unsigned long long u0 = (unsigned long long)i << lcpb;
+        if (commit && u0 >= cb && u0 < ce) {
           item_log(T, i, x, seq, f0, pg);
           item_page_stats(T, pg);
           item_commit(T, i, x, seq);
@@ -1611,14 +1620,8 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
     batch = b0;
     __syncwarp();
   };
-  // Units are walked as (item, chunk) pairs with shifts (cpb and upp are powers of two):
-  // no 64-bit division per unit.  The warp walks them uniformly; lane 0 issues.
-  const uint32_t lcpb = 31 - __clz(cpb), lupp = 31 - __clz(upp);
-  const uint32_t i_lo = (uint32_t)(ubeg >> lcpb), i_end = (uint32_t)((uend + cpb - 1) >> lcpb);
-  const uint32_t ch_lo = (uint32_t)(ubeg & (cpb - 1));
-  const uint32_t ch_end_last = (uint32_t)(((uend - 1) & (cpb - 1)) + 1);
-  auto plan_of = [&](uint32_t i, bool commit) -> const SPlan& {
-    if (batch == UM_NONE || i - batch >= 32u) plan_batch(i, commit);
+  auto plan_of = [&](uint32_t i, bool commit, unsigned long long cb, unsigned long long ce) -> const SPlan& {
+    if (batch == UM_NONE || i - batch >= 32u) plan_batch(i, commit, cb, ce);
     return s_pl[i - batch];
   };
   // pages of an item whose units only need the zero tile (nothing to load or write back)
@@ -1627,6 +1630,39 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
     const uint32_t wb = q.d2h ? ~q.dmask : 0u;
     return mode == SVC_SUBOP ? (zf & ~wb) : 0u;
   };
+  if (warp != 0) {
+    // zero-fill warps: units [zb, ze) (a third of the CTA's range), walked as (item,
+    // chunk) pairs with shifts; lane 0 issues
+    if (mode != SVC_SUBOP) return;
+    const unsigned long long span = uend - ubeg;
+    const unsigned long long zb = ubeg + span * (warp - 1) / (kSvcWarps - 1);
+    const unsigned long long ze = ubeg + span * warp / (kSvcWarps - 1);
+    if (zb >= ze) return;
+    const uint32_t i_lo = (uint32_t)(zb >> lcpb), i_end = (uint32_t)((ze + cpb - 1) >> lcpb);
+    const uint32_t ch_lo = (uint32_t)(zb & (cpb - 1)), ch_end_last = (uint32_t)(((ze - 1) & (cpb - 1)) + 1);
+    uint32_t issued = 0;
+    for (uint32_t i = i_lo; i < i_end; ++i) {
+      const SPlan& q = plan_of(i, true, zb, ze);
+      const uint32_t pm = pure_pages(q);
+      if (!pm || lane != 0) continue;
+      const uint32_t cb = i == i_lo ? ch_lo : 0u, ce = i + 1 == i_end ? ch_end_last : cpb;
+      for (uint32_t ch = cb; ch < ce; ++ch) {
+        if (!((pm >> (ch >> lupp)) & 1u)) continue;
+        bulk_s2g(q.frame + (size_t)ch * CH, zero, CH);
+        if ((++issued & 31) == 0) bulk_commit();
+      }
+    }
+    if (lane == 0) {
+      bulk_commit();
+      bulk_wait_all();
+    }
+    return;
+  }
+  // warp 0: the units with a load, through the S-stage TMA ring (cursor: item ci, chunk cch)
+  if (ubeg >= uend) return;
+  const uint32_t i_lo = (uint32_t)(ubeg >> lcpb), i_end = (uint32_t)((uend + cpb - 1) >> lcpb);
+  const uint32_t ch_end_last = (uint32_t)(((uend - 1) & (cpb - 1)) + 1);
+  uint32_t ci = i_lo, cch = (uint32_t)(ubeg & (cpb - 1));
   auto unit_of = [&](const SPlan& q, uint32_t ch) -> Unit {
     const size_t coff = (size_t)ch * CH;
     const uint32_t pg = ch >> lupp;
@@ -1638,29 +1674,9 @@ __global__ void __launch_bounds__(32, 1) k_service(Tables T, int mode, uint32_t 
     x.zf = mode == SVC_SUBOP && !mig;
     return x;
   };
-  // Phase 1: zero-fill units need no load: bulk-store the zeroed tile right away (this
-  // pass also plans, and commits, every item of the range once).
-  if (mode == SVC_SUBOP && ubeg < uend) {
-    uint32_t issued = 0;
-    for (uint32_t i = i_lo; i < i_end; ++i) {
-      const SPlan& q = plan_of(i, true);
-      const uint32_t pm = pure_pages(q);
-      if (!pm || lane != 0) continue;
-      const uint32_t cb = i == i_lo ? ch_lo : 0u, ce = i + 1 == i_end ? ch_end_last : cpb;
-      for (uint32_t ch = cb; ch < ce; ++ch) {
-        if (!((pm >> (ch >> lupp)) & 1u)) continue;
-        bulk_s2g(q.frame + (size_t)ch * CH, zero, CH);
-        if ((++issued & 31) == 0) bulk_commit();
-      }
-    }
-    if (lane == 0) bulk_commit();
-    batch = UM_NONE;
-  }
-  // Phase 2: the other units through the S-stage TMA ring (cursor: item ci, chunk cch)
-  uint32_t ci = i_lo, cch = ch_lo;
   auto next_xfer = [&](Unit& x) -> bool {
     while (ci < i_end) {
-      const SPlan& q = plan_of(ci, false);
+      const SPlan& q = plan_of(ci, false, 0, 0);
       const uint32_t ce = ci + 1 == i_end ? ch_end_last : cpb;
       // pages with a load: not pure zero-fill (sub-op), live pages to write back (D2H-only)
       const uint32_t keep = mode == SVC_SUBOP ? ~pure_pages(q) : (q.d2h ? ~q.dmask : 0u);
@@ -2470,7 +2486,7 @@ cudaError_t launch_service(const Tables& T, int mode, uint32_t seq, uint32_t max
   unsigned grid = (unsigned)(units < (unsigned long long)g_nsm ? units : (unsigned long long)g_nsm);
   if (grid == 0) grid = 1;
   size_t smem = (size_t)CH * (1 + 2 * kXferStages);
-  cudaError_t le__ = launch_pdl(k_service, dim3(grid), dim3(32), smem, s, T, mode, seq);
+  cudaError_t le__ = launch_pdl(k_service, dim3(grid), dim3(32 * kSvcWarps), smem, s, T, mode, seq);
   if (le__) return le__;
   return cudaGetLastError();
 }
