@@ -570,8 +570,11 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
             s0 = um.um_get_stats(h)
             um.um_timing(h, reset=True)
             gate()
-            fn()
-            t = um.um_timing(h, reset=True)
+            h0 = time.perf_counter()
+            fn()                       # host: validation, record marshalling (A0/A1), enqueue
+            host_us = (time.perf_counter() - h0) * 1e6
+            t = dict(um.um_timing(h, reset=True))
+            t["host_us"] = host_us
             s1 = um.um_get_stats(h)
             return t, {k: s1[k] - s0[k] for k in s1}
         # floor of the measurement: two events around one empty torch kernel on the same
@@ -602,21 +605,25 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
         dir_bytes = n * (4 + 8) + g_in * 8
         peak, peak_src = _hbm_peak()
 
-        def rl(name, by, ms, extra=None):
+        def rl(name, by, ms, extra=None, host_us=None):
             a = by / (ms / 1e3) / 1e9 if ms else None
             r = {"kernel": name, "bound": "hbm", "achieved": a, "peak": peak, "unit": "GB/s",
-                 "frac": a / peak if a else None, "algorithmic_bytes": by, "ms": ms, "blocks": n}
+                 "frac": a / peak if a else None, "algorithmic_bytes": by, "ms": ms, "blocks": n,
+                 "host_api_us": host_us}
             r.update(extra or {})
             return r
-        return {"touch_2^21_random": rl("k_classify + k_victims_scan/apply (k = 0)", touch_bytes, t_touch["ms_plan"]),
-                "discard_2^21": rl("k_directive", dir_bytes, t_disc["ms_plan"]),
+        return {"touch_2^21_random": rl("k_classify (k = 0 is certain: no victim kernels)", touch_bytes,
+                                        t_touch["ms_plan"], host_us=t_touch["host_us"]),
+                "discard_2^21": rl("k_directive", dir_bytes, t_disc["ms_plan"], host_us=t_disc["host_us"]),
                 "touch_2^21_pressure": rl("k_classify + k_victims_scan + k_victims_apply", pres_bytes, t_pres["ms_plan"],
-                                          {"victims": d2["evictions"], "remaps": d2["remaps"]}),
+                                          {"victims": d2["evictions"], "remaps": d2["remaps"]}, host_us=t_pres["host_us"]),
                 "zero_fill_gbs": (n * B) / (t_touch["ms_xfer"] / 1e3) / 1e9 if t_touch["ms_xfer"] else None,
                 "peak_source": peak_src, "nblocks": nb, "nframes": budget // B,
                 "empty_kernel_span_us": min(floor) * 1e3,
                 "timing": "CUDA events around each op's planning launches on the paging stream; every launch "
-                          "queued behind a device sleep; L2 cold (the previous op's zero-fill flushes it)"}
+                          "queued behind a device sleep; L2 cold (the previous op's zero-fill flushes it); "
+                          "host_api_us = host time of the API call (validation, marshalling of the 2^21 records "
+                          "into the staged fault list, enqueue), which overlaps the device sleep"}
     finally:
         um.um_arena_destroy(h)
         del ws
