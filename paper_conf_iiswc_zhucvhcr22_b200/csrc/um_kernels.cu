@@ -1556,6 +1556,11 @@ constexpr int kSvcWarps = 4;
 
 __global__ void __launch_bounds__(32 * kSvcWarps, 1) k_service(Tables T, int mode, uint32_t seq) {
   pdl_enter();
+  // The frames were last written through the generic proxy (application kernel, an
+  // earlier sub-op's zero-fill commit path): order those writes before this kernel's
+  // bulk copies (async proxy).  The wait of programmatic dependent launch makes the
+  // predecessors' writes visible, but not to the async proxy.
+  asm volatile("fence.proxy.async.global;" ::: "memory");
   extern __shared__ __align__(128) char smem[];
   __shared__ __align__(8) uint64_t bar[kXferStages];
   __shared__ SPlan s_plw[kSvcWarps][32];
@@ -1655,6 +1660,7 @@ __global__ void __launch_bounds__(32 * kSvcWarps, 1) k_service(Tables T, int mod
     if (lane == 0) {
       bulk_commit();
       bulk_wait_all();
+      asm volatile("fence.proxy.async.global;" ::: "memory");   // bulk writes before generic readers
     }
     return;
   }
@@ -1727,6 +1733,7 @@ __global__ void __launch_bounds__(32 * kSvcWarps, 1) k_service(Tables T, int mod
   }
   if (lane == 0) {
     bulk_wait_all();
+    asm volatile("fence.proxy.async.global;" ::: "memory");   // bulk writes before generic readers
     if (mode == SVC_D2H_ONLY) {
       __threadfence();
       unsigned int d = atomicAdd(&c->app_units, 1u);
