@@ -1664,8 +1664,8 @@ __global__ void __launch_bounds__(32 * kSvcWarps, 1) k_service(Tables T, int mod
     }
     return;
   }
-  // warp 0: the units with a load, through the S-stage TMA ring (cursor: item ci, chunk cch)
-  if (ubeg >= uend) return;
+  // warp 0: the units with a load, through the S-stage TMA ring (cursor: item ci, chunk cch).
+  // A CTA with an empty range still reaches the D2H-only completion count below.
   const uint32_t i_lo = (uint32_t)(ubeg >> lcpb), i_end = (uint32_t)((uend + cpb - 1) >> lcpb);
   const uint32_t ch_end_last = (uint32_t)(((uend - 1) & (cpb - 1)) + 1);
   uint32_t ci = i_lo, cch = (uint32_t)(ubeg & (cpb - 1));
@@ -1681,7 +1681,7 @@ __global__ void __launch_bounds__(32 * kSvcWarps, 1) k_service(Tables T, int mod
     return x;
   };
   auto next_xfer = [&](Unit& x) -> bool {
-    while (ci < i_end) {
+    while (ubeg < uend && ci < i_end) {
       const SPlan& q = plan_of(ci, false, 0, 0);
       const uint32_t ce = ci + 1 == i_end ? ch_end_last : cpb;
       // pages with a load: not pure zero-fill (sub-op), live pages to write back (D2H-only)
