@@ -417,3 +417,25 @@ def test_c3_full_size_64k_blocks(copy):
     pool = t.arena_bytes - t.budget_bytes + (2 << 30)
     g = _gpu(t, "eager", copy=copy, host_pool_bytes=pool, xlog=False)   # ~10 M records: counters only
     assert_parity(t, "eager", g)
+
+
+@pytest.mark.parametrize("copy", ["default", "ce"])
+def test_sparse_d2h_lists(copy):
+    """D2H-only lists much shorter than their launch bound (prefetch HOST of mostly
+    non-resident ranges, evict of more than is queued): most transfer CTAs get no unit
+    and the list must still be reset for the next op (a stale entry would be written
+    back again over a reused host frame)."""
+    B = 4 << 10
+    tb = tg.TraceBuilder(B, 256 * B, 96 * B)
+    for r in range(6):
+        tb.touch([((r * 7) % 200 * B, 2 * B, tg.ACC_WRITE), ((r * 13 + 100) % 200 * B, B, tg.ACC_WRITE)])
+        tb.prefetch(0, 200 * B, tg.DST_HOST)          # 3 resident blocks among 200
+        tb.touch([(((r * 5) % 190) * B, 3 * B, tg.ACC_READ | tg.ACC_WRITE)])
+        tb.evict(96 * B)                               # more than is queued
+        if r == 0:
+            tb.prefetch(210 * B, 4 * B, tg.DST_HOST)
+            tb.host_write(210 * B, 4 * B)
+        tb.touch([(((r * 11) % 150) * B, 4 * B, tg.ACC_READ)])
+    t = tb.build()
+    for mode in ("base", "eager"):
+        assert_parity(t, mode, _gpu(t, mode, copy=copy))
