@@ -263,6 +263,7 @@ struct um_arena {
   std::vector<Iv> ivs;
   std::vector<CItem> citems;   // two-level: the op's chunks with page masks
   uint32_t ppc = 1, P = 0;     // pages per chunk, page bytes (single level: 1, B)
+  uint32_t lgB = 0, lgP = 0;   // log2 of block and page bytes (record -> block by shifts)
   // UM_F_TIMING: event pairs around planning / transfer launches
   struct Span { cudaEvent_t a, b; int xfer; uint32_t seq; };
   std::vector<Span> spans;
@@ -449,38 +450,44 @@ static bool range_ok(um_arena* a, uint64_t off, uint64_t len) {
   return off <= a->cfg.arena_bytes && len <= a->cfg.arena_bytes - off;
 }
 
-// Sorted disjoint intervals with constant write flag from access records.
-static void build_intervals(um_arena* a, const um_access* acc, uint32_t n) {
-  const uint64_t B = a->B;
-  // Fast path (linear): records already in ascending, non-overlapping block order —
-  // e.g. a fault batch sorted by address — are the intervals (adjacent equal-W records
-  // merge).  Anything else goes through the event sort below.
-  {
-    a->ivs.clear();
-    uint64_t prev_hi = 0;
-    bool ok = true;
-    for (uint32_t i = 0; i < n && ok; ++i) {
-      if (!acc[i].len) continue;
-      const uint64_t lo = acc[i].off / B, hi = (acc[i].off + acc[i].len - 1) / B + 1;
-      const uint8_t w = (acc[i].kind & UM_ACC_WRITE) ? 1 : 0;
-      if (!a->ivs.empty() && lo < prev_hi) {
-        ok = false;
-        break;
+// Records already in ascending, non-overlapping block order -- e.g. a fault batch sorted
+// by address -- are the intervals (adjacent equal-W records merge): one linear pass with
+// shifts (blocks are powers of two).  Returns false, with a->ivs unspecified, otherwise.
+static bool sorted_intervals(um_arena* a, const um_access* acc, uint32_t n) {
+  const uint32_t lg = a->lgB;
+  auto& v = a->ivs;
+  v.clear();
+  v.reserve(n);
+  uint64_t prev_hi = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    if (!acc[i].len) continue;
+    const uint64_t lo = acc[i].off >> lg, hi = ((acc[i].off + acc[i].len - 1) >> lg) + 1;
+    const uint8_t w = (acc[i].kind & UM_ACC_WRITE) ? 1 : 0;
+    if (!v.empty()) {
+      if (lo < prev_hi) return false;
+      if (prev_hi == lo && v.back().w == w) {
+        v.back().cnt += (uint32_t)(hi - lo);
+        prev_hi = hi;
+        continue;
       }
-      if (!a->ivs.empty() && prev_hi == lo && a->ivs.back().w == w)
-        a->ivs.back().cnt += (uint32_t)(hi - lo);
-      else
-        a->ivs.push_back({(uint32_t)lo, (uint32_t)(hi - lo), w});
-      prev_hi = hi;
     }
-    if (ok) return;
+    v.push_back({(uint32_t)lo, (uint32_t)(hi - lo), w});
+    prev_hi = hi;
   }
+  return true;
+}
+
+// Sorted disjoint intervals with constant write flag from any access records (the
+// <= kIvInline-record case that is not already sorted): a 2n-event sweep.
+static void build_intervals(um_arena* a, const um_access* acc, uint32_t n) {
+  if (sorted_intervals(a, acc, n)) return;
+  const uint32_t lg = a->lgB;
   struct Ev { uint64_t x; int dc, dw; };
   std::vector<Ev> ev;
   ev.reserve(2 * (size_t)n);
   for (uint32_t i = 0; i < n; ++i) {
     if (!acc[i].len) continue;
-    uint64_t lo = acc[i].off / B, hi = (acc[i].off + acc[i].len - 1) / B + 1;
+    uint64_t lo = acc[i].off >> lg, hi = ((acc[i].off + acc[i].len - 1) >> lg) + 1;
     int w = (acc[i].kind & UM_ACC_WRITE) ? 1 : 0;
     ev.push_back({lo, +1, w});
     ev.push_back({hi, -1, -w});
@@ -666,35 +673,20 @@ static um_status ce_d2h_only(um_arena* a, uint32_t nmax) {
   return UM_OK;
 }
 
-// True when the records are in ascending, non-overlapping block order (then they are the
-// intervals and no dedupe is needed).
-static bool sorted_disjoint(um_arena* a, const um_access* acc, uint32_t n) {
-  uint64_t prev_hi = 0;
-  bool any = false;
-  for (uint32_t i = 0; i < n; ++i) {
-    if (!acc[i].len) continue;
-    const uint64_t lo = acc[i].off / a->B, hi = (acc[i].off + acc[i].len - 1) / a->B + 1;
-    if (any && lo < prev_hi) return false;
-    prev_hi = hi;
-    any = true;
-  }
-  return true;
-}
-
 // Device intake: dedupe a batch of accesses on the GPU.  The host converts
 // each record to blocks and splits it into pieces of <= kMarkMaxBlocks (argument
 // marshalling), stages the pieces, and the kernels build the sorted disjoint interval
 // list in HBM.  One sync reads the interval count and the prefix array back: the host
 // needs them to number the sub-ops and index tiles, not to compute anything.
 static um_status device_intake(um_arena* a, const um_access* acc, uint32_t n) {
-  const uint64_t B = a->B;
+  const uint32_t lg = a->lgB;
   uint64_t bmin = ~0ull, bmax = 0;
   bool anyw = false;
   auto& mk = a->mark;
   mk.clear();
   for (uint32_t i = 0; i < n; ++i) {
     if (!acc[i].len) continue;
-    const uint64_t lo = acc[i].off / B, hi = (acc[i].off + acc[i].len - 1) / B + 1;
+    const uint64_t lo = acc[i].off >> lg, hi = ((acc[i].off + acc[i].len - 1) >> lg) + 1;
     const uint32_t w = (acc[i].kind & UM_ACC_WRITE) ? 1u : 0u;
     anyw |= w != 0;
     bmin = std::min(bmin, lo);
@@ -939,7 +931,7 @@ static uint32_t chunk_mask(const um_arena* a, uint64_t c, uint64_t p0, uint64_t 
 // Append the chunks overlapping byte range [off, off+len) with their page masks.
 static void add_range(um_arena* a, uint64_t off, uint64_t len, bool w) {
   if (!len) return;
-  const uint64_t p0 = off / a->P, p1 = (off + len - 1) / a->P + 1;
+  const uint64_t p0 = off >> a->lgP, p1 = ((off + len - 1) >> a->lgP) + 1;
   for (uint64_t c = p0 / a->ppc; c <= (p1 - 1) / a->ppc; ++c) {
     const uint32_t m = chunk_mask(a, c, p0, p1);
     a->citems.push_back({(uint32_t)c, m, w ? m : 0u});
@@ -1131,6 +1123,8 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   T.d2h_dmask = (uint32_t*)(ws + L.d2h_dmask);
   a->ppc = cfg_ppc(cfg);
   a->P = cfg->block_bytes / a->ppc;
+  a->lgB = 31 - __builtin_clz(a->B);
+  a->lgP = 31 - __builtin_clz(a->P);
   T.ppc = a->ppc;
   T.P = a->P;
   if (a->ppc > 1) {
@@ -1256,14 +1250,14 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
     return hand_out(a, stream);
   }
   // a batch of more records than fit inline that is not already sorted and disjoint is
-  // deduplicated on the device; otherwise the records (or the <= kIvInline records after a
-  // 2n-event merge while they are packed into the kernel arguments) are the intervals
-  if (n > kIvInline && a->nblocks < (1u << 31) && !sorted_disjoint(a, acc, n)) {
+  // deduplicated on the device; otherwise the records (one linear pass), or the <=
+  // kIvInline records after a 2n-event merge, are the intervals
+  if (n > kIvInline && !sorted_intervals(a, acc, n)) {
     // the intake rewrites the device interval list that in-flight app kernels may read
     if (overlap_on(a) && (s = app_wait_all(a))) return s;
     s = device_intake(a, acc, n);
     if (s) return s;
-  } else {
+  } else if (n <= kIvInline) {
     build_intervals(a, acc, n);
   }
   s = run_gpu_op(a, 1);
