@@ -232,6 +232,35 @@ def c2_stream(torch, um, harness, mem, budget, pool_bytes):
     out["avoided_gb"] = (out["base"]["h2d_gb"] + out["base"]["d2h_gb"]) - (out["eager"]["h2d_gb"] + out["eager"]["d2h_gb"])
     out["avoided_closed_form_gb"] = (4 * P - 3) * F * B / 1e9
     out["speedup_eager_vs_base"] = out["base"]["ms"] / out["eager"]["ms"]
+    # full size (F = 81,920 frames = 160 GiB, 320 GiB buffer) with discard: nothing is
+    # written back or migrated, so no host frame is needed; base mode at this size would
+    # need a 160 GiB pinned pool next to C3's and is reported at the F above
+    Ff = 81920
+    if Ff * B <= budget:
+        tf = tg.gen_c2(Ff, c, P, block_bytes=B)
+        view = _MemView(torch, um, mem, B, tf.arena_bytes, tf.budget_bytes)
+        full = {"F": Ff, "buffer_gib": 2 * Ff * B / GiB}
+        for mode in ("eager", "lazy"):
+            arena = harness.make_arena(tf, mode, mem=view, flags=um.UM_F_APP_STAMP)
+            try:
+                harness.alloc_buffers(arena, tf)
+                ps = torch.cuda.ExternalStream(arena.stream_ptr)
+                um.um_get_stats(arena.handle)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(ps)
+                harness.issue(arena, tf, mode)
+                e1.record(ps)
+                e1.synchronize()
+                st = um.um_get_stats(arena.handle)
+                ms = e0.elapsed_time(e1)
+                full[mode] = {"ms": ms, "zf_gb": st["zf_bytes"] / 1e9,
+                              "serviced_gbs": st["zf_bytes"] / (ms / 1e3) / 1e9,
+                              "closed_form_ok": (st["h2d_bytes"], st["d2h_bytes"], st["zf_bytes"]) == (0, 0, 2 * P * Ff * B),
+                              "avoided_closed_form_gb": (4 * P - 3) * Ff * B / 1e9}
+            finally:
+                arena.close()
+        del view
+        out["full_size_discard"] = full
     return out
 
 
