@@ -44,7 +44,7 @@ struct Ctl {
   unsigned int vt_reach;                // wide victim scan: passes in the apply work table (vpass)
   unsigned int pc_done;                 // k_plan_commit completion ticket (host read-back flag)
   unsigned long long xlog_n;            // transfer log: records appended (may exceed the capacity)
-  unsigned int cls_done;                // k_classify with k = 0 guaranteed: completion ticket
+  unsigned long long need_tk;           // k_classify with k = 0 certain: (need count << 32) | tickets
   // counters, striped over 8 cache lines by CTA index (fire-and-forget atomics from
   // thousands of CTAs do not serialise on one address); the host sums the stripes
   long long stats[8][S_N];

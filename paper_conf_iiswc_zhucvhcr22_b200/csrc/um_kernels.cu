@@ -592,7 +592,7 @@ __device__ bool grid_finish(const Tables& T, const int (&slots)[NC], const long 
 
 template <int IPT, bool LIST, int TPB>
 __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, uint32_t g0, uint32_t n, uint32_t seq,
-                                              int touch, unsigned long long tail0, int npar) {
+                                              int touch, unsigned long long tail0, int npar, int k0) {
   constexpr int TILE = TPB * IPT, NW = TPB / 32, NWORD = TILE / 32;
   constexpr int PERL = (NWORD + 31) / 32;   // bitmap words per lane in the warp prefix
   // Interval lookup without a search: the tile's interval slice [ja, jb] is staged as
@@ -718,7 +718,30 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
   // need-list slots: one atomic per CTA for the base, then warp-ballot ranks so that
   // consecutive lanes write consecutive slots (coalesced stores)
   const uint32_t tot = ordered_offsets<TPB, IPT>(bN, bN, s_off) & 0xffffu;
-  if (threadIdx.x == 0) s_base = tot ? atomicAdd(&T.ctl->need_cnt[npar], tot) : 0u;
+  if (threadIdx.x == 0) {
+    if (k0) {
+      // k = 0 is certain (the host's bound), so no victim kernel runs: one 64-bit atomic
+      // gives this CTA its need-list base (high word) and a ticket (low word); the CTA
+      // with the last ticket knows the sub-op's need count and does the victim kernels'
+      // k = 0 bookkeeping.  Nothing else in this launch reads what it writes.
+      Ctl* c = T.ctl;
+      const unsigned long long old = atomicAdd(&c->need_tk, ((unsigned long long)tot << 32) | 1ull);
+      s_base = (uint32_t)(old >> 32);
+      if ((uint32_t)old == gridDim.x - 1) {
+        const uint32_t nn = s_base + tot;
+        const int f0 = c->free_top;
+        c->n_need = nn;
+        c->need_cnt[npar ^ 1] = 0;   // the other parity slot, as the victim kernels do
+        c->n_vict = 0;
+        c->f0 = (uint32_t)f0;
+        c->free_top = f0 - (int)min((uint32_t)f0, nn);
+        c->used_tail += n;
+        c->need_tk = 0;
+      }
+    } else {
+      s_base = tot ? atomicAdd(&T.ctl->need_cnt[npar], tot) : 0u;
+    }
+  }
   __syncthreads();
   const uint32_t base = s_base;
   const unsigned lt = lanemask_lt();
@@ -790,32 +813,7 @@ __global__ void __launch_bounds__(TPB, 2048 / TPB) k_classify(Tables T, const __
                                                               uint32_t n, uint32_t seq, int touch,
                                                               unsigned long long tail0, int npar, int k0) {
   pdl_enter();
-  classify_body<4, LIST, TPB>(T, iv, g0, n, seq, touch, tail0, npar);
-  if (k0) {
-    // the host guarantees k = 0 (every block of the sub-op fits the free frames), so no
-    // victim kernel runs: the CTA that finishes last publishes the need count and does
-    // the k = 0 frame bookkeeping of the victim kernels
-    __shared__ int s_last;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      s_last = atomicAdd(&T.ctl->cls_done, 1u) == gridDim.x - 1;
-    }
-    __syncthreads();
-    if (s_last && threadIdx.x == 0) {
-      __threadfence();
-      Ctl* c = T.ctl;
-      const uint32_t nn = ((volatile unsigned int*)c->need_cnt)[npar];
-      const int f0 = c->free_top;
-      c->n_need = nn;
-      c->need_cnt[npar ^ 1] = 0;
-      c->n_vict = 0;
-      c->f0 = (uint32_t)f0;
-      c->free_top = f0 - (int)min((uint32_t)f0, nn);
-      c->used_tail += n;
-      c->cls_done = 0;
-    }
-  }
+  classify_body<4, LIST, TPB>(T, iv, g0, n, seq, touch, tail0, npar, k0);
 }
 
 // ------------------------------------------------------------------------------------
