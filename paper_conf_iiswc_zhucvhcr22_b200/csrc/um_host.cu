@@ -261,6 +261,8 @@ struct um_arena {
   Stager stage;
   Ctl* hctl = nullptr;  // pinned mirror for reads
   std::vector<Iv> ivs;
+  uint64_t iv_total = 0;       // blocks in ivs, and whether any interval is written
+  bool iv_anyw = false;
   std::vector<CItem> citems;   // two-level: the op's chunks with page masks
   uint32_t ppc = 1, P = 0;     // pages per chunk, page bytes (single level: 1, B)
   uint32_t lgB = 0, lgP = 0;   // log2 of block and page bytes (record -> block by shifts)
@@ -458,11 +460,14 @@ static bool sorted_intervals(um_arena* a, const um_access* acc, uint32_t n) {
   auto& v = a->ivs;
   v.clear();
   v.reserve(n);
-  uint64_t prev_hi = 0;
+  uint64_t prev_hi = 0, total = 0;
+  bool anyw = false;
   for (uint32_t i = 0; i < n; ++i) {
     if (!acc[i].len) continue;
     const uint64_t lo = acc[i].off >> lg, hi = ((acc[i].off + acc[i].len - 1) >> lg) + 1;
     const uint8_t w = (acc[i].kind & UM_ACC_WRITE) ? 1 : 0;
+    total += hi - lo;
+    anyw |= w != 0;
     if (!v.empty()) {
       if (lo < prev_hi) return false;
       if (prev_hi == lo && v.back().w == w) {
@@ -474,6 +479,8 @@ static bool sorted_intervals(um_arena* a, const um_access* acc, uint32_t n) {
     v.push_back({(uint32_t)lo, (uint32_t)(hi - lo), w});
     prev_hi = hi;
   }
+  a->iv_total = total;
+  a->iv_anyw = anyw;
   return true;
 }
 
@@ -510,6 +517,12 @@ static void build_intervals(um_arena* a, const um_access* acc, uint32_t n) {
       else
         a->ivs.push_back({(uint32_t)x, (uint32_t)(nx - x), w});
     }
+  }
+  a->iv_total = 0;
+  a->iv_anyw = false;
+  for (const Iv& x : a->ivs) {
+    a->iv_total += x.cnt;
+    a->iv_anyw |= x.w != 0;
   }
 }
 
@@ -738,13 +751,8 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     total = a->dev_total;
     anyw = a->dev_anyw;
   } else {
-    a->hpre.resize(a->ivs.size() + 1);
-    for (size_t j = 0; j < a->ivs.size(); ++j) {
-      a->hpre[j] = (uint32_t)total;
-      total += a->ivs[j].cnt;
-      anyw |= a->ivs[j].w;
-    }
-    a->hpre[a->ivs.size()] = (uint32_t)total;
+    total = a->iv_total;   // from the interval builder (hpre is made below only if needed)
+    anyw = a->iv_anyw;
   }
   {
     um_status sr = seq_room(a, total ? (total + a->nframes - 1) / a->nframes : 1);
@@ -808,13 +816,16 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     uint32_t* hpre = (uint32_t*)(a->stage.host + off + o_pre);
     uint8_t* hw = a->stage.host + off + o_w;
     uint32_t acc = 0;
+    a->hpre.resize((size_t)m + 1);   // host copy for the per-tile interval index below
     for (uint32_t j = 0; j < m; ++j) {
       hlo[j] = a->ivs[j].lo;
       hpre[j] = acc;
+      a->hpre[j] = acc;
       hw[j] = a->ivs[j].w;
       acc += a->ivs[j].cnt;
     }
     hpre[m] = acc;
+    a->hpre[m] = acc;
     CK(a->stage.push(off, (bytes + 15) & ~15ull, a->ps));
     iv.lo = (const uint32_t*)(a->stage.dev + off + o_lo);
     iv.pre = (const uint32_t*)(a->stage.dev + off + o_pre);
@@ -1277,9 +1288,12 @@ UM_API um_status um_prefetch(um_arena* a, uint64_t off, uint64_t len, int dst, v
     if (s) return s;
   } else if (dst == UM_DST_GPU) {
     a->ivs.clear();
+    a->iv_total = 0;
+    a->iv_anyw = false;
     if (len) {
-      uint64_t lo = off / a->B, hi = (off + len - 1) / a->B + 1;
+      uint64_t lo = off >> a->lgB, hi = ((off + len - 1) >> a->lgB) + 1;
       a->ivs.push_back({(uint32_t)lo, (uint32_t)(hi - lo), 0});
+      a->iv_total = hi - lo;
     }
     s = run_gpu_op(a, 0);
     if (s) return s;
