@@ -634,10 +634,18 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
         dir_bytes = n * (4 + 8) + g_in * 8
         peak, peak_src = _hbm_peak()
 
+        fl_ms = min(floor)
+
         def rl(name, by, ms, extra=None, host_us=None):
             a = by / (ms / 1e3) / 1e9 if ms else None
+            # the span includes the measurement floor (events around an empty kernel on the
+            # same stream, behind the same sleep); net of it, the span approximates the
+            # kernels' own duration (what ncu's gpu__time_duration measures)
+            net = ms - fl_ms if ms and ms > fl_ms else None
+            an = by / (net / 1e3) / 1e9 if net else None
             r = {"kernel": name, "bound": "hbm", "achieved": a, "peak": peak, "unit": "GB/s",
                  "frac": a / peak if a else None, "algorithmic_bytes": by, "ms": ms, "blocks": n,
+                 "net_of_floor": {"ms": net, "achieved": an, "frac": an / peak if an else None},
                  "host_api_us": host_us}
             r.update(extra or {})
             return r
