@@ -917,6 +917,7 @@ def main_ours(args):
                    "app_overlap": ("UM_F_OVERLAP: app kernels pipelined with the next 2 GPU sub-ops (reading R7), "
                                    "every mode" if ovf else "off: app kernels serialized on the paging stream")},
         "iter_ms": {m: r["iter_ms"] for m, r in res.items()},
+        "iter_ms_each": {m: r["iter_ms_each"] for m, r in res.items()},
         "speedup_vs_discard_off": (base["iter_ms"] / t_iter_ms) if base else None,
         "gb_avoided_per_iter": avoided,
         "link_gb_per_iter": {m: (r["stats_per_iter"]["h2d_bytes"] + r["stats_per_iter"]["d2h_bytes"]) / 1e9
