@@ -1394,6 +1394,8 @@ UM_API um_status um_free(um_arena* a, uint64_t off, uint64_t len, void* stream) 
   um_status s = hand_in(a, stream);
   if (s) return s;
   if ((s = seq_room(a, 1))) return s;
+  // frees frames an in-flight application kernel may still write: those finish first (R7)
+  if (overlap_on(a) && (s = app_wait_all(a))) return s;
   a->ops++;
   a->subops++;
   ++a->clock;
