@@ -274,6 +274,7 @@ class _MemView:
         probe.block_bytes, probe.page_bytes = B, page_bytes
         probe.workspace, probe.workspace_bytes = None, 0
         self.workspace = torch.empty(um.um_workspace_size(probe), dtype=torch.uint8, device=mem.frames.device)
+        torch.cuda.synchronize(mem.frames.device)   # handed to the arena's own streams
 
     def config(self, arena_bytes, budget_bytes, flags):
         c = self._mem.config(arena_bytes, budget_bytes, flags)
@@ -573,6 +574,7 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
     cfg.block_bytes = B
     ws_bytes = um.um_workspace_size(cfg)
     ws = torch.empty(ws_bytes, dtype=torch.uint8, device=mem.frames.device)
+    torch.cuda.synchronize(mem.frames.device)   # handed to the arena's own streams
     cfg.workspace, cfg.workspace_bytes = ws.data_ptr(), ws_bytes
     h = um.um_arena_create(cfg)
     try:

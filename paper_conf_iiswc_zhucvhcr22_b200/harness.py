@@ -106,7 +106,11 @@ class XLog:
     def __init__(self, arena: um.Arena, cap: int):
         import torch
         self.arena, self.cap = arena, cap
-        self.buf = torch.zeros((cap, 4), dtype=torch.int32, device=arena.frames.device)
+        # torch allocates on its current stream; the arena's paging stream does not wait for
+        # it, so the buffer is handed over only once torch's work on it is done (no zeroing:
+        # only the records appended are read)
+        self.buf = torch.empty((cap, 4), dtype=torch.int32, device=arena.frames.device)
+        torch.cuda.synchronize(arena.frames.device)
         um.um_xlog_attach(arena.handle, self.buf.data_ptr(), cap)
 
     def raw(self) -> np.ndarray:

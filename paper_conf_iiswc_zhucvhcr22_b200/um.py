@@ -271,6 +271,9 @@ class Memory:
         ws = um_workspace_size(probe)
         self.workspace = torch.empty(ws, dtype=torch.uint8, device=dev)
         self.nch = nch
+        # the arena's streams do not wait for torch's stream: hand the memory over only
+        # after any pending torch work on it (a previous owner's) is done
+        torch.cuda.synchronize(dev)
 
     def config(self, arena_bytes: int, budget_bytes: int, flags: int) -> um_config:
         return um_config(device=self.device, block_bytes=self.B, arena_bytes=arena_bytes,
