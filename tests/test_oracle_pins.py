@@ -229,3 +229,11 @@ def test_free_releases_without_transfers(mode):
     # the freed blocks' frames serve the final read of the tables: no more write-backs
     # than the same run without the free and one more read
     assert b.stats["d2h_bytes"] == a.stats["d2h_bytes"] and b.stats["evictions"] == a.stats["evictions"]
+
+
+def test_slice_ops_drops_private_meta():
+    """A sub-trace must not inherit a consumer's cache of its parent's op list."""
+    t = tg.gen_c1(0)
+    t.meta["_calls_eager"] = ["stale"]
+    s = t.slice_ops(0, 10)
+    assert "_calls_eager" not in s.meta and len(s) == 10 and s.meta["seed"] == 0
