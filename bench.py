@@ -648,6 +648,7 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
             r = {"kernel": name, "bound": "hbm", "achieved": a, "peak": peak, "unit": "GB/s",
                  "frac": a / peak if a else None, "algorithmic_bytes": by, "ms": ms, "blocks": n,
                  "net_of_floor": {"ms": net, "achieved": an, "frac": an / peak if an else None},
+                 "blocks_per_s": n / (ms / 1e3) if ms else None,
                  "host_api_us": host_us}
             r.update(extra or {})
             return r
@@ -773,9 +774,31 @@ def cpu_oracle_baseline(trace, W, dev_index=0, budget_s=20.0):
             if time.process_time() - t0 > budget_s:
                 break
         dt = time.process_time() - t0
+        # C1 (BASELINE configs[0]): the whole 10k-op trace, the small-op regime
+        import tracegen as tg
+        t1 = tg.gen_c1(0)
+        o1 = Oracle(t1.block_bytes, t1.arena_bytes, t1.budget_bytes)
+        c0 = time.process_time()
+        for op in t1.iter_ops():
+            apply_op(o1, op, "eager")
+        c1 = time.process_time() - c0
+    per = bounds[0][1] - bounds[0][0]
+    blocks = _blocks_per_iter(trace, bounds[1])
     return {"value": n / dt, "unit": "iter/s", "kind": "oracle", **pin.info(),
             "sample": f"C3 eager iterations 2..{n + 1} of the bench trace (iteration 1 replayed untimed)",
-            "s_per_iter": dt / n}
+            "s_per_iter": dt / n, "ops_per_s": n * per / dt, "block_events_per_s": n * blocks / dt,
+            "c1": {"ops": len(t1), "s": c1, "ops_per_s": len(t1) / c1}}
+
+
+def _blocks_per_iter(trace, bound):
+    """Blocks named by the ops of one iteration (record lengths in blocks; the unit of the
+    oracle's work)."""
+    B = trace.block_bytes
+    tot = 0
+    for kind, flags, off, ln, accs in list(trace.iter_ops())[bound[0]:bound[1]]:
+        rs = accs if accs is not None else [(off, ln, 0)]
+        tot += sum((o + m - 1) // B - o // B + 1 for (o, m, _k) in rs if m)
+    return tot
 
 
 def plan_sizes(args, free_bytes, lws):
