@@ -1,6 +1,6 @@
 """State-kernel microbench of bench.py's `state_bench` on C3-64K-sized tables without the
 170 GiB of frames: 4 KiB blocks, nblocks = 4,177,920, nframes = 2^21 + 2^20 (12 GiB of
-frames).  Ops: a touch of 2^21 distinct random blocks (all U, k = 0), a discard of blocks
+frames; 2,785,280 frames as in the bench).  Ops: a touch of 2^21 distinct random blocks (all U, k = 0), a discard of blocks
 [0, 2^21), a second random 2^21-block touch under pressure (revives, zero-fills, victims
 from DISC).  Prints per-op planning / transfer ms (CUDA-event spans).
 
@@ -21,7 +21,7 @@ from paper_conf_iiswc_zhucvhcr22_b200 import build, um  # noqa: E402
 build.build()
 B = 4096
 nb = 4177920
-nf = (1 << 21) + (1 << 20)
+nf = 2785280   # the bench's C3-64K frame count: the pressured touch needs ~356 k victims
 n = 1 << 21
 a = um.Arena(B, nb * B, nf * B, flags=um.UM_F_TIMING, host_pool_bytes=1 << 30)
 h = a.handle
