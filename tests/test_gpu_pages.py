@@ -191,3 +191,33 @@ def test_c3_two_level_removes_tail_rmt():
     assert r1["rmt_bytes"] > 0 and r1["discarded_state_moves"] == 0
     assert r2["rmt_bytes"] < r1["rmt_bytes"] and r2["discarded_state_moves"] == 0
     assert r2["h2d_bytes"] + r2["d2h_bytes"] < r1["h2d_bytes"] + r1["d2h_bytes"]
+
+
+def test_c3_full_size_two_level():
+    """NEXT-1 at the bench's full size: C3 (discard-all-dead) at 1.5x of a ~170 GiB budget,
+    2 MiB chunks of 64 KiB pages, two iterations; chunk states, queue orders, every counter,
+    the page masks and every page's content tag (4.2 M pages) against oracle/chunks.py.
+    (The per-page transfer log is compared at the smaller sizes above.)"""
+    import gc
+    import torch
+    from paper_conf_iiswc_zhucvhcr22_b200 import harness, um
+    gc.collect()
+    torch.cuda.empty_cache()
+    free, _ = torch.cuda.mem_get_info()
+    GiB = 1 << 30
+    budget = min(170 * GiB, free - 8 * GiB) // (2 << 20) * (2 << 20)
+    assert budget >= 160 * GiB, f"only {free / GiB:.1f} GiB free"
+    t = tg.gen_c3(block_bytes=2 << 20, budget_bytes=budget, oversub=1.5, iterations=2, discard_all_dead=True)
+    P = 64 << 10
+    pool = t.arena_bytes - t.budget_bytes + (2 << 30)
+    g = harness.run_trace(t, "eager", page_bytes=P, flags=um.UM_F_APP_STAMP | um.UM_F_CHECK, host_pool_bytes=pool)
+    d = replay_chunks(t, P, "eager").dump()
+    assert list(g["st"]) == d["st"]
+    assert g["stats"] == d["stats"], {k: (g["stats"][k], d["stats"][k]) for k in d["stats"] if g["stats"][k] != d["stats"][k]}
+    assert g["used_order"] == d["used_order"] and g["disc_order"] == d["disc_order"]
+    assert g["dead"] == d["dead"] and g["lazy"] == d["lazy"]
+    assert any(d["dead"])
+    cg = np.asarray(g["contents"], np.uint64)
+    co = np.asarray(d["contents"], np.uint64)
+    bad = np.nonzero(cg != co)[0]
+    assert len(bad) == 0, f"page contents differ at {bad[:8]}"
