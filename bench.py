@@ -698,6 +698,23 @@ def main_state_only(args):
     print(json.dumps({"roofline_state": state_runs(torch, um, mem, budget, arena_bytes)}), flush=True)
 
 
+_LEG_ERRORS = {}
+
+
+def _leg(torch, name, fn, *a, **kw):
+    """A side leg of the bench line: its failure is recorded in the line (leg_errors)
+    instead of losing the headline."""
+    try:
+        return fn(*a, **kw)
+    except Exception as e:   # noqa: BLE001 -- reported, not swallowed
+        import traceback
+        _LEG_ERRORS[name] = f"{type(e).__name__}: {e}"
+        traceback.print_exc()
+        torch.cuda.synchronize()
+        torch.cuda.empty_cache()
+        return None
+
+
 def _barrier(torch):
     from paper_conf_iiswc_zhucvhcr22_b200.dist import barrier
     barrier()
@@ -859,9 +876,9 @@ def main_ours(args):
     out = {"metric": METRIC, "impl": "ours", "n_gpus": ws, "steps": K, "warmup": W}
 
     link = measure_link_peak(torch, dev)
-    disc = None if args.no_discard_bench else discard_bench(torch, um)
-    c1 = None if args.no_discard_bench else c1_rate(torch, um, harness)
-    c4 = None if args.no_discard_bench else c4_sweep(torch, um, harness)
+    disc = None if args.no_discard_bench else _leg(torch, "discard_sweep", discard_bench, torch, um)
+    c1 = None if args.no_discard_bench else _leg(torch, "c1", c1_rate, torch, um, harness)
+    c4 = None if args.no_discard_bench else _leg(torch, "c4", c4_sweep, torch, um, harness)
 
     torch.cuda.empty_cache()
     free, total = torch.cuda.mem_get_info(dev)
@@ -890,18 +907,20 @@ def main_ours(args):
     # comparison legs on the same step (at most 5 timed iterations each): the copy-engine
     # transfer arm (K4-CE) and the other app-kernel schedule (R7 overlap <-> sequential)
     Kc = min(K, 5)
-    ce = run_mode(torch, um, harness, mem, trace, "eager", W, Kc, flags_extra=um.UM_F_COPY_CE | ovf) \
+    ce = _leg(torch, "ce_arm", run_mode, torch, um, harness, mem, trace, "eager", W, Kc,
+              flags_extra=um.UM_F_COPY_CE | ovf) \
         if not args.no_compare else None
-    other = run_mode(torch, um, harness, mem, trace, "eager", W, Kc, flags_extra=um.UM_F_OVERLAP ^ ovf) \
+    other = _leg(torch, "app_overlap", run_mode, torch, um, harness, mem, trace, "eager", W, Kc,
+                 flags_extra=um.UM_F_OVERLAP ^ ovf) \
         if not args.no_compare else None
     ovl_r, seq_r = (res.get("eager"), other) if ovf else (other, res.get("eager"))
-    state = None if args.no_state_bench else state_runs(torch, um, mem, budget, arena_bytes)
-    rmt_r = None if args.no_compare else rmt_leg(torch, um, harness, mem, budget, args.oversub, B)
-    c2 = None if args.no_compare else c2_stream(torch, um, harness, mem, budget, host_pool)
-    c3k = None if args.no_compare else c3_64k(torch, um, harness, mem, budget, arena_bytes)
+    state = None if args.no_state_bench else _leg(torch, "state", state_runs, torch, um, mem, budget, arena_bytes)
+    rmt_r = None if args.no_compare else _leg(torch, "rmt", rmt_leg, torch, um, harness, mem, budget, args.oversub, B)
+    c2 = None if args.no_compare else _leg(torch, "c2", c2_stream, torch, um, harness, mem, budget, host_pool)
+    c3k = None if args.no_compare else _leg(torch, "c3_64k", c3_64k, torch, um, harness, mem, budget, arena_bytes)
     e2e_s = None
     if not args.no_e2e:
-        e2e_s = run_e2e(torch, um, harness, mem, trace, 1, min(K, 3), flags_extra=ovf)
+        e2e_s = _leg(torch, "e2e", run_e2e, torch, um, harness, mem, trace, 1, min(K, 3), flags_extra=ovf)
 
     head = res.get("eager") or next(iter(res.values()))
     t_iter_ms = head["iter_ms"]
@@ -985,6 +1004,7 @@ def main_ours(args):
         "c3_64k_blocks": c3k,
         "clocks": head["clocks"],
         "gpu_launches": tm["launches"],
+        "leg_errors": _LEG_ERRORS or None,
         "stats_all_ranks": {"counters": stats_all, "iterations_per_rank": K,
                             "reduce": "NCCL all-reduce (int64 sum) of the counters, max of the iteration time"},
         "setup_s": {"pin_and_alloc": t_alloc},
