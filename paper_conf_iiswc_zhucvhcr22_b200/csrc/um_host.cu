@@ -15,6 +15,7 @@
 #include <cstring>
 #include <deque>
 #include <new>
+#include <chrono>
 #include <vector>
 
 #include "../../include/um.h"
@@ -266,6 +267,7 @@ struct um_arena {
   std::vector<CItem> citems;   // two-level: the op's chunks with page masks
   uint32_t ppc = 1, P = 0;     // pages per chunk, page bytes (single level: 1, B)
   uint32_t lgB = 0, lgP = 0;   // log2 of block and page bytes (record -> block by shifts)
+  bool host_prof = false;      // UM_HOST_PROFILE (diagnostic): host phases of a touch batch to stderr
   // UM_F_TIMING: event pairs around planning / transfer launches
   struct Span { cudaEvent_t a, b; int xfer; uint32_t seq; };
   std::vector<Span> spans;
@@ -1196,6 +1198,7 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   }
   for (uint32_t i = 0; i < cfg->n_host_chunks; ++i) a->hhost.push_back((char*)cfg->host_chunks[i]);
   if (const char* v = getenv("UM_CE_MIN_BYTES")) a->ce_min_bytes = strtoull(v, nullptr, 10);
+  a->host_prof = getenv("UM_HOST_PROFILE") != nullptr;
   if ((e = a->stage.init((uint8_t*)(ws + L.stage), L.stage_bytes))) return fail(e);
   // zero the whole workspace once: every table, ring slot and list starts defined (the
   // parity exports copy whole rings / lists; compute-sanitizer initcheck stays clean)
@@ -1248,8 +1251,11 @@ UM_API um_status um_alloc(um_arena* a, uint64_t bytes, uint64_t* off) {
 UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, void* stream) {
   ENTER(a);
   if (n && !acc) return UM_EINVAL;
+  using clk = std::chrono::steady_clock;
+  const auto t0 = clk::now();
   for (uint32_t i = 0; i < n; ++i)
     if (!range_ok(a, acc[i].off, acc[i].len)) return UM_EINVAL;
+  const auto t1 = clk::now();
   um_status s = hand_in(a, stream);
   if (s) return s;
   if (a->ppc > 1) {   // two-level: the chunks with the pages each record covers / writes
@@ -1271,8 +1277,15 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
   } else if (n <= kIvInline) {
     build_intervals(a, acc, n);
   }
+  const auto t2 = clk::now();
   s = run_gpu_op(a, 1);
   if (s) return s;
+  if (a->host_prof) {
+    const auto t3 = clk::now();
+    auto us = [](clk::duration d) { return std::chrono::duration<double, std::micro>(d).count(); };
+    fprintf(stderr, "libum touch_batch n=%u: range check %.1f us, intervals %.1f us, stage + launch %.1f us\n", n,
+            us(t1 - t0), us(t2 - t1), us(t3 - t2));
+  }
   return hand_out(a, stream);
 }
 
