@@ -264,6 +264,10 @@ struct um_arena {
   std::vector<Iv> ivs;
   uint64_t iv_total = 0;       // blocks in ivs, and whether any interval is written
   bool iv_anyw = false;
+  // sparse sorted batch, scanned once: the fault list (block | write << 31) ready to stage
+  std::vector<uint32_t> flist;
+  bool fl_ready = false;
+  uint32_t fl_m = 0;           // the batch's merged intervals (what decides the form)
   std::vector<CItem> citems;   // two-level: the op's chunks with page masks
   uint32_t ppc = 1, P = 0;     // pages per chunk, page bytes (single level: 1, B)
   uint32_t lgB = 0, lgP = 0;   // log2 of block and page bytes (record -> block by shifts)
@@ -483,6 +487,41 @@ static bool sorted_intervals(um_arena* a, const um_access* acc, uint32_t n) {
   }
   a->iv_total = total;
   a->iv_anyw = anyw;
+  return true;
+}
+
+// One pass over a batch that is already in ascending, non-overlapping block order (the
+// usual shape of a large fault batch): totals, the merged-interval count, and the fault
+// list itself (one u32 per block, bit 31 = write) -- no interval list is built.  Returns
+// false (nothing decided) if the records are not sorted and disjoint.
+static bool scan_sorted(um_arena* a, const um_access* acc, uint32_t n) {
+  const uint32_t lg = a->lgB;
+  auto& fl = a->flist;
+  fl.clear();
+  fl.reserve(n);
+  uint64_t prev_hi = 0, total = 0;
+  uint32_t m = 0;
+  uint8_t prev_w = 2;
+  bool anyw = false, fill = true;   // past 3 blocks per record the list form cannot be chosen
+  for (uint32_t i = 0; i < n; ++i) {
+    if (!acc[i].len) continue;
+    const uint64_t lo = acc[i].off >> lg, hi = ((acc[i].off + acc[i].len - 1) >> lg) + 1;
+    const uint8_t w = (acc[i].kind & UM_ACC_WRITE) ? 1 : 0;
+    if (m && lo < prev_hi) return false;
+    if (!(m && prev_hi == lo && prev_w == w)) ++m;   // a new merged interval
+    total += hi - lo;
+    fill = fill && total <= 3ull * n;
+    if (fill) {
+      const uint32_t wbit = w ? 0x80000000u : 0u;
+      for (uint64_t b = lo; b < hi; ++b) fl.push_back((uint32_t)b | wbit);
+    }
+    anyw |= w != 0;
+    prev_hi = hi;
+    prev_w = w;
+  }
+  a->iv_total = total;
+  a->iv_anyw = anyw;
+  a->fl_m = m;
   return true;
 }
 
@@ -767,11 +806,23 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     if (overlap_on(a)) window_floor(a, a->clock, 0);
     return UM_OK;
   }
-  const uint32_t m = dev ? a->dev_m : (uint32_t)a->ivs.size();
+  const bool fl = a->fl_ready;
+  a->fl_ready = false;
+  const uint32_t m = dev ? a->dev_m : (fl ? a->fl_m : (uint32_t)a->ivs.size());
   uint64_t iv_off = 0, iv_bytes = 0;   // staged interval arrays (read by the app kernels)
   OpIv iv{};
   iv.m = m;
-  if (dev) {
+  if (fl) {
+    // sparse sorted batch: the fault list made while scanning the records
+    const uint64_t bytes = 4ull * total;
+    uint64_t off;
+    CK(a->stage.reserve(bytes, &off));
+    iv_off = off;
+    iv_bytes = (bytes + 15) & ~15ull;
+    memcpy(a->stage.host + off, a->flist.data(), bytes);
+    CK(a->stage.push(off, iv_bytes, a->ps));
+    iv.blist = (const uint32_t*)(a->stage.dev + off);
+  } else if (dev) {
     // intervals made on the device by the intake kernels (already in HBM)
     iv.lo = a->T.dlo;
     iv.pre = a->T.dpre;
@@ -1269,12 +1320,17 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
   // a batch of more records than fit inline that is not already sorted and disjoint is
   // deduplicated on the device; otherwise the records (one linear pass), or the <=
   // kIvInline records after a 2n-event merge, are the intervals
-  if (n > kIvInline && !sorted_intervals(a, acc, n)) {
+  if (n > kIvInline && !scan_sorted(a, acc, n)) {
     // the intake rewrites the device interval list that in-flight app kernels may read
     if (overlap_on(a) && (s = app_wait_all(a))) return s;
     s = device_intake(a, acc, n);
     if (s) return s;
-  } else if (n <= kIvInline) {
+  } else if (n > kIvInline && a->fl_m > kIvInline && a->iv_total <= 3ull * a->fl_m &&
+             4ull * a->iv_total <= a->L.stage_bytes / 2) {
+    a->fl_ready = true;   // sparse batch: the fault list is already made
+  } else if (n > kIvInline) {
+    sorted_intervals(a, acc, n);   // sorted, but the interval forms fit it better
+  } else {
     build_intervals(a, acc, n);
   }
   const auto t2 = clk::now();
