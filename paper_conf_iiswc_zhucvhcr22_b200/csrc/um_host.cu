@@ -497,28 +497,34 @@ static bool sorted_intervals(um_arena* a, const um_access* acc, uint32_t n) {
 static bool scan_sorted(um_arena* a, const um_access* acc, uint32_t n) {
   const uint32_t lg = a->lgB;
   auto& fl = a->flist;
-  fl.clear();
-  fl.reserve(n);
-  uint64_t prev_hi = 0, total = 0;
-  uint32_t m = 0;
-  uint8_t prev_w = 2;
-  bool anyw = false, fill = true;   // past 3 blocks per record the list form cannot be chosen
+  size_t cap = (size_t)n + 1024, k = 0;
+  if (fl.size() < cap) fl.resize(cap);
+  uint32_t* out = fl.data();
+  uint64_t prev_hi = 0, total = 0, lim = 3ull * n;
+  uint32_t m = 0, prev_w = 2;
+  bool anyw = false, bad = false;
   for (uint32_t i = 0; i < n; ++i) {
-    if (!acc[i].len) continue;
-    const uint64_t lo = acc[i].off >> lg, hi = ((acc[i].off + acc[i].len - 1) >> lg) + 1;
-    const uint8_t w = (acc[i].kind & UM_ACC_WRITE) ? 1 : 0;
-    if (m && lo < prev_hi) return false;
-    if (!(m && prev_hi == lo && prev_w == w)) ++m;   // a new merged interval
-    total += hi - lo;
-    fill = fill && total <= 3ull * n;
-    if (fill) {
-      const uint32_t wbit = w ? 0x80000000u : 0u;
-      for (uint64_t b = lo; b < hi; ++b) fl.push_back((uint32_t)b | wbit);
-    }
+    const uint64_t off = acc[i].off, len = acc[i].len;
+    if (!len) continue;
+    const uint64_t lo = off >> lg, hi = ((off + len - 1) >> lg) + 1, cnt = hi - lo;
+    const uint32_t w = (acc[i].kind & UM_ACC_WRITE) ? 1u : 0u;
+    // branch-free on the data: order violations are collected and decided after the pass
+    bad |= (m != 0) & (lo < prev_hi);
+    m += 1u - (uint32_t)((m != 0) & (prev_hi == lo) & (prev_w == w));
+    total += cnt;
     anyw |= w != 0;
     prev_hi = hi;
     prev_w = w;
+    if (total > lim) continue;   // past 3 blocks per record the list form cannot be chosen
+    const uint32_t wbit = w << 31;
+    if (k + cnt > cap) {
+      cap = std::max<size_t>(2 * cap, k + cnt);
+      fl.resize(cap);
+      out = fl.data();
+    }
+    for (uint64_t x = 0; x < cnt; ++x) out[k++] = (uint32_t)(lo + x) | wbit;
   }
+  if (bad) return false;
   a->iv_total = total;
   a->iv_anyw = anyw;
   a->fl_m = m;
@@ -819,7 +825,7 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     CK(a->stage.reserve(bytes, &off));
     iv_off = off;
     iv_bytes = (bytes + 15) & ~15ull;
-    memcpy(a->stage.host + off, a->flist.data(), bytes);
+    memcpy(a->stage.host + off, a->flist.data(), bytes);   // flist holds exactly `total` entries
     CK(a->stage.push(off, iv_bytes, a->ps));
     iv.blist = (const uint32_t*)(a->stage.dev + off);
   } else if (dev) {
