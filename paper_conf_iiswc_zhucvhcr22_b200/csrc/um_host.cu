@@ -494,8 +494,10 @@ static bool sorted_intervals(um_arena* a, const um_access* acc, uint32_t n) {
 // usual shape of a large fault batch): totals, the merged-interval count, and the fault
 // list itself (one u32 per block, bit 31 = write) -- no interval list is built.  Returns
 // false (nothing decided) if the records are not sorted and disjoint.
-static bool scan_sorted(um_arena* a, const um_access* acc, uint32_t n) {
+static bool scan_sorted(um_arena* a, const um_access* acc, uint32_t n, bool* out_of_range) {
   const uint32_t lg = a->lgB;
+  const uint64_t arena = a->cfg.arena_bytes;
+  bool oor = false;
   auto& fl = a->flist;
   size_t cap = (size_t)n + 1024, k = 0;
   if (fl.size() < cap) fl.resize(cap);
@@ -505,6 +507,7 @@ static bool scan_sorted(um_arena* a, const um_access* acc, uint32_t n) {
   bool anyw = false, bad = false;
   for (uint32_t i = 0; i < n; ++i) {
     const uint64_t off = acc[i].off, len = acc[i].len;
+    oor |= (off > arena) | (len > arena - off);   // the API's range check, same pass
     if (!len) continue;
     const uint64_t lo = off >> lg, hi = ((off + len - 1) >> lg) + 1, cnt = hi - lo;
     const uint32_t w = (acc[i].kind & UM_ACC_WRITE) ? 1u : 0u;
@@ -524,6 +527,7 @@ static bool scan_sorted(um_arena* a, const um_access* acc, uint32_t n) {
     }
     for (uint64_t x = 0; x < cnt; ++x) out[k++] = (uint32_t)(lo + x) | wbit;
   }
+  *out_of_range = oor;
   if (bad) return false;
   a->iv_total = total;
   a->iv_anyw = anyw;
@@ -1310,8 +1314,17 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
   if (n && !acc) return UM_EINVAL;
   using clk = std::chrono::steady_clock;
   const auto t0 = clk::now();
-  for (uint32_t i = 0; i < n; ++i)
-    if (!range_ok(a, acc[i].off, acc[i].len)) return UM_EINVAL;
+  // a large single-level batch is scanned once here: range check, order check and (for a
+  // sorted one) totals and the fault list; anything else is range-checked on its own
+  bool scanned = false;
+  if (a->ppc == 1 && n > kIvInline) {
+    bool oor = false;
+    scanned = scan_sorted(a, acc, n, &oor);
+    if (oor) return UM_EINVAL;
+  } else {
+    for (uint32_t i = 0; i < n; ++i)
+      if (!range_ok(a, acc[i].off, acc[i].len)) return UM_EINVAL;
+  }
   const auto t1 = clk::now();
   um_status s = hand_in(a, stream);
   if (s) return s;
@@ -1326,7 +1339,7 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
   // a batch of more records than fit inline that is not already sorted and disjoint is
   // deduplicated on the device; otherwise the records (one linear pass), or the <=
   // kIvInline records after a 2n-event merge, are the intervals
-  if (n > kIvInline && !scan_sorted(a, acc, n)) {
+  if (n > kIvInline && !scanned) {
     // the intake rewrites the device interval list that in-flight app kernels may read
     if (overlap_on(a) && (s = app_wait_all(a))) return s;
     s = device_intake(a, acc, n);
@@ -1345,7 +1358,7 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
   if (a->host_prof) {
     const auto t3 = clk::now();
     auto us = [](clk::duration d) { return std::chrono::duration<double, std::micro>(d).count(); };
-    fprintf(stderr, "libum touch_batch n=%u: range check %.1f us, intervals %.1f us, stage + launch %.1f us\n", n,
+    fprintf(stderr, "libum touch_batch n=%u: scan %.1f us, intervals %.1f us, stage + launch %.1f us\n", n,
             us(t1 - t0), us(t2 - t1), us(t3 - t2));
   }
   return hand_out(a, stream);
