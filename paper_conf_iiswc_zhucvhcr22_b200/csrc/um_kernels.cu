@@ -1163,13 +1163,12 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
   if (!s_last) return;
   __threadfence();
   __shared__ unsigned long long s_sc[kVsTPB / 32];
-  __shared__ uint32_t s_reach, s_found;
+  __shared__ uint32_t s_reach;
   __shared__ unsigned long long s_kd, s_ku;
   const uint32_t fs = *(volatile uint32_t*)&c->first_skip;
   const uint32_t E = min(ntiles, fs);   // tiles [0, E) were all examined
   if (threadIdx.x == 0) {
     s_reach = ~0u;
-    s_found = 0;
     s_kd = s_ku = ~0ull;
   }
   __syncthreads();
