@@ -707,6 +707,8 @@ def _leg(torch, name, fn, *a, **kw):
     try:
         return fn(*a, **kw)
     except Exception as e:   # noqa: BLE001 -- reported, not swallowed
+        if dist_env()[2] > 1:
+            raise   # ranks would disagree on the barriers that follow: fail the whole run
         import traceback
         _LEG_ERRORS[name] = f"{type(e).__name__}: {e}"
         traceback.print_exc()
