@@ -865,13 +865,20 @@ def build_trace(args, budget, with_host_data, iterations):
 def main_ours(args):
     import torch
     rank, local, ws = dist_env()
+    # BENCH_SHARE_GPU=1 (testing the N>1 path on a one-GPU box): every rank on cuda:0,
+    # gloo for the collectives (NCCL refuses two ranks on one device)
+    share = os.environ.get("BENCH_SHARE_GPU") == "1"
+    gpu = 0 if share else local
     if ws > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        torch.cuda.set_device(gpu)
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", gpu))
     else:
         torch.cuda.set_device(0)
-    dev = torch.device("cuda", local if ws > 1 else 0)
+    dev = torch.device("cuda", gpu if ws > 1 else 0)
     from paper_conf_iiswc_zhucvhcr22_b200 import build, um, harness
     build.build()
     W, K = args.warmup, args.steps
@@ -928,7 +935,7 @@ def main_ours(args):
     t_iter_ms = head["iter_ms"]
     # max over ranks; the run's only collective: counters all-reduce (north_star)
     from paper_conf_iiswc_zhucvhcr22_b200.dist import reduce_run
-    stats_all, t_iter_ms = reduce_run(head["stats_total"], t_iter_ms, device=dev)   # int64 counters
+    stats_all, t_iter_ms = reduce_run(head["stats_total"], t_iter_ms, device=None if share else dev)   # int64 counters
     if rank != 0:
         return
     spi = head["stats_per_iter"]
