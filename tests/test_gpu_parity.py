@@ -439,3 +439,14 @@ def test_sparse_d2h_lists(copy):
     t = tb.build()
     for mode in ("base", "eager"):
         assert_parity(t, mode, _gpu(t, mode, copy=copy))
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_small_random_with_free(seed, mode):
+    """Random traces that also release ranges (um_free, reading R9)."""
+    rng = np.random.default_rng(300 + seed)
+    nb, nf = int(rng.integers(2, 24)), int(rng.integers(1, 6))
+    t = tg.gen_small(300 + seed, nblocks=nb, nframes=nf, n_ops=300, max_ranges=4, max_blocks=6,
+                     mix=[45, 12, 5, 10, 10, 3, 2, 13])
+    assert_parity(t, mode)

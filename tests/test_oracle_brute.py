@@ -13,7 +13,7 @@ import pytest
 from hypothesis import given, settings, strategies as hst, HealthCheck
 
 import tracegen as tg
-from oracle.sim import replay, ST_NAMES
+from oracle.sim import G, Oracle, apply_op, replay, ST_NAMES
 
 
 class _Node:
@@ -420,6 +420,12 @@ class FlatMemory:
                         lazy_pending[b] = True
             elif op == tg.OP_EVICT:
                 seq += 1
+            elif op == tg.OP_FREE:
+                # R9: fully covered blocks are released and read as never populated (zeros)
+                seq += 1
+                for b in range(-(-off // B), (off + ln) // B):
+                    val[b], dc[b], lazy_pending[b] = 0, False, False
+                    history[b].add(0)
             elif op == tg.OP_HOST_WRITE:
                 seq += 1
                 for b in (range(off // B, (off + ln - 1) // B + 1) if ln else []):
@@ -565,3 +571,26 @@ def test_overlap_keeps_semantics(seed, nblocks, nframes):
     roomy = tg.gen_small(seed, nblocks=nblocks, nframes=nblocks, n_ops=40)   # arena <= budget
     for mode in ("base", "eager", "lazy"):
         assert replay(roomy, mode, overlap=2).dump() == replay(roomy, mode).dump()
+
+
+@settings(max_examples=80, deadline=None)
+@given(seed=hst.integers(0, 10**6), nblocks=hst.integers(2, 10), nframes=hst.integers(1, 4),
+       host_release=hst.booleans())
+def test_free_flat_memory_and_conservation(seed, nblocks, nframes, host_release):
+    """R9 (um_free) inside random traces: conservation after every op, the flat-memory
+    contract with a free reading back as zeros, and no discarded block written back."""
+    t = tg.gen_small(seed, nblocks=nblocks, nframes=nframes, n_ops=50, mix=[45, 12, 5, 10, 10, 3, 2, 13])
+    for mode in ("base", "eager", "lazy"):
+        o = Oracle(t.block_bytes, t.arena_bytes, t.budget_bytes, discard_off=(mode == "base"),
+                   host_release=host_release, record=True)
+        for op in t.iter_ops():
+            apply_op(o, op, mode)
+            o.check_conservation()
+        assert all(k != "D2H" or p == G for (_s, k, _b, p) in o.log)
+        val, dc, hist = FlatMemory(t, mode).run()
+        got = o.contents()
+        for b in range(t.nblocks):
+            if not dc[b]:
+                assert got[b] == val[b], (mode, b)
+            else:
+                assert got[b] in hist[b], (mode, b)
