@@ -299,7 +299,8 @@ struct um_arena {
   int app_ctas = 1;
   bool app_serial = false;   // UM_OVERLAP_SERIAL (diagnostic): window rule, app kernel on ps
   struct WinE { uint32_t seq, n; };
-  WinE win[kOverlapW] = {};
+  WinE win[kOverlapWMax] = {};
+  int ovw = kOverlapW;      // window length (UM_OVERLAP_W overrides, 1..kOverlapWMax)
   int nwin = 0;
   struct Pend { uint32_t seq; cudaEvent_t ev; };
   std::deque<Pend> pend;
@@ -417,8 +418,8 @@ static uint32_t window_floor(um_arena* a, uint32_t seq, uint32_t n) {
     tot += a->win[i].n;
     floor = a->win[i].seq;
   }
-  if (a->nwin == kOverlapW) {
-    for (int i = 1; i < kOverlapW; ++i) a->win[i - 1] = a->win[i];
+  if (a->nwin == a->ovw) {
+    for (int i = 1; i < a->ovw; ++i) a->win[i - 1] = a->win[i];
     a->nwin--;
   }
   a->win[a->nwin++] = {seq, n};
@@ -1243,6 +1244,7 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
     if (const char* v = getenv("UM_APP_CTAS")) a->app_ctas = std::max(1, atoi(v));
     if (const char* v = getenv("UM_APP_GRID")) a->app_ctas = -std::max(1, atoi(v));
     a->app_serial = getenv("UM_OVERLAP_SERIAL") != nullptr;
+    if (const char* v = getenv("UM_OVERLAP_W")) a->ovw = std::min(kOverlapWMax, std::max(1, atoi(v)));
   }
   if ((e = cudaEventCreateWithFlags(&a->ev_in, cudaEventDisableTiming))) return fail(e);
   if ((e = cudaEventCreateWithFlags(&a->ev_out, cudaEventDisableTiming))) return fail(e);

@@ -140,6 +140,7 @@ constexpr uint32_t kIvInline = 24;
 // UM_F_OVERLAP: number of previous GPU sub-ops whose application kernels may still run
 // while a sub-op is serviced (reading R7; the oracle's `overlap` parameter)
 constexpr int kOverlapW = 2;
+constexpr int kOverlapWMax = 8;   // UM_OVERLAP_W (diagnostic A/B): another window length
 struct OpIv {
   const uint32_t* lo;
   const uint32_t* pre;
