@@ -2070,8 +2070,9 @@ __device__ __forceinline__ void directive_body(const Tables& T, int kind, uint32
 
 // 8 blocks per thread, 6 CTAs/SM (A/B on B200: 16 per thread at 4 CTAs/SM, one round of
 // 512 tiles for 2^21 blocks, measured the same 14.3 us)
-__global__ void __launch_bounds__(kStTPB, 6) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
-                                                         int discard_off, unsigned long long tail0) {
+template <int MINB>
+__global__ void __launch_bounds__(kStTPB, MINB) k_directive(Tables T, int kind, uint32_t lo, uint32_t n, uint32_t seq,
+                                                            int discard_off, unsigned long long tail0) {
   pdl_enter();
   directive_body<8>(T, kind, lo, n, seq, discard_off, tail0);
 }
@@ -2368,6 +2369,7 @@ static int g_cls_tpb = 256;
 static int g_vscan_occ = 1;   // resident k_victims_scan CTAs per SM
 static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch (A/B)
 static int g_dir_occ = 8;     // resident k_directive CTAs per SM (persistent grid)
+static int g_dir_minb = 6;    // k_directive CTAs/SM the registers allow: 6 (40 regs); UM_DIR_MINB=7/8 (36/32 regs: one wave for 2^21 blocks) for A/B
 static int g_vs_prefetch = 0; // UM_VS_PREFETCH=1: the wide victim scan fetches its next ticket a tile ahead (A/B on B200: 79 vs 73 us pressured touch -- the earlier snapshot reads more tiles past the k-th candidate)
 
 cudaError_t setup_kernels() {
@@ -2388,7 +2390,8 @@ cudaError_t setup_kernels() {
     const void* ks[] = {(const void*)k_classify<false, 256>, (const void*)k_classify<true, 256>,
                         (const void*)k_classify<false, 512>, (const void*)k_classify<true, 512>, (const void*)k_victims, (const void*)k_plan_small,
                         (const void*)k_victims_scan, (const void*)k_victims_apply, (const void*)k_service,
-                        (const void*)k_app_stamp<256>, (const void*)k_app_stamp<128>, (const void*)k_directive, (const void*)k_ring_compact,
+                        (const void*)k_app_stamp<256>, (const void*)k_app_stamp<128>, (const void*)k_directive<6>, (const void*)k_directive<7>, (const void*)k_directive<8>,
+                        (const void*)k_ring_compact,
                         (const void*)k_plan_commit, (const void*)k_zero_items, (const void*)k_mark,
                         (const void*)k_runs, (const void*)k_intake_clear};
     for (const void* k : ks) {
@@ -2399,7 +2402,11 @@ cudaError_t setup_kernels() {
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_vscan_occ, k_victims_scan, kVsTPB, 0);
   if (e) return e;
   if (g_vscan_occ < 1) g_vscan_occ = 1;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_dir_occ, k_directive, kStTPB, 0);
+  if (const char* v = getenv("UM_DIR_MINB")) g_dir_minb = std::min(8, std::max(6, atoi(v)));
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+      &g_dir_occ,
+      g_dir_minb == 8 ? (const void*)k_directive<8> : g_dir_minb == 7 ? (const void*)k_directive<7> : (const void*)k_directive<6>,
+      kStTPB, 0);
   if (e) return e;
   if (g_dir_occ < 1) g_dir_occ = 1;
   if (const char* v = getenv("UM_DIR_OCC")) g_dir_occ = std::max(1, atoi(v));
@@ -2514,7 +2521,10 @@ cudaError_t launch_directive(const Tables& T, int kind, uint32_t lo, uint32_t n,
                              unsigned long long tail0, cudaStream_t s) {
   unsigned nt = n ? ceil_div(n, kStTPB * 8) : 1;
   if (nt > (unsigned)(g_nsm * g_dir_occ)) nt = (unsigned)(g_nsm * g_dir_occ);   // persistent
-  cudaError_t le__ = launch_pdl(k_directive, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq, discard_off, tail0);
+  cudaError_t le__ =
+      g_dir_minb == 8   ? launch_pdl(k_directive<8>, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq, discard_off, tail0)
+      : g_dir_minb == 7 ? launch_pdl(k_directive<7>, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq, discard_off, tail0)
+                        : launch_pdl(k_directive<6>, dim3(nt), dim3(kStTPB), 0, s, T, kind, lo, n, seq, discard_off, tail0);
   if (le__) return le__;
   return cudaGetLastError();
 }
