@@ -104,7 +104,7 @@ static Layout make_layout(const um_config* c) {
   L.needhf = take(4 * nf);
   L.victim = take(4 * nf);
   L.vscratch = take(4 * (2 * L.cap + 2048));   // wide victim scan: candidates per tile
-  L.vpass = take(8 * (nf / 128 + L.max_tiles + 2));   // wide victim apply: work table
+  L.vpass = take(16 * (nf / 128 + L.max_tiles + 2));   // wide victim apply: work table
   L.vframe = take(4 * nf);
   L.vhf = take(4 * nf);
   L.vkind = take(nf);
@@ -1179,7 +1179,7 @@ UM_API um_status um_arena_create(const um_config* cfg, um_arena** out) {
   T.needhf = (uint32_t*)(ws + L.needhf);
   T.victim = (uint32_t*)(ws + L.victim);
   T.vscratch = (uint32_t*)(ws + L.vscratch);
-  T.vpass = (unsigned long long*)(ws + L.vpass);
+  T.vpass = (ulonglong2*)(ws + L.vpass);
   T.vframe = (uint32_t*)(ws + L.vframe);
   T.vhf = (uint32_t*)(ws + L.vhf);
   T.vkind = (uint8_t*)(ws + L.vkind);

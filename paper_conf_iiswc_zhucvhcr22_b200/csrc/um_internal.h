@@ -81,7 +81,7 @@ struct Tables {
   uint32_t* needhf;     // [nframes] their host frame at classification (H) or NONE
   uint32_t* victim;     // [nframes] victims, in eviction order
   uint32_t* vscratch;   // [2 cap + 2048] wide victim scan: the candidates of tile t at [t * 2048, ...), in ring order
-  unsigned long long* vpass;  // [nframes / 128 + tiles] wide victim apply work table: (tile << 4 | pass) | prefix << 32
+  ulonglong2* vpass;    // [nframes / 128 + tiles] wide victim apply work table, one entry per pass of <= 128 victims: {first victim index | tile << 32, offset in the tile's candidates | victims << 32}
   uint32_t* vframe;     // [nframes] victim's frame
   uint32_t* vhf;        // [nframes] host frame receiving a G victim's write-back, else NONE
   uint8_t* vkind;       // [nframes] victim's state when chosen

@@ -1024,11 +1024,30 @@ __global__ void __launch_bounds__(kVictTPB) k_plan_small(Tables T, const __grid_
 //   candidates as victims prefix .. prefix + take - 1, gathered from its scratch slice.
 // ------------------------------------------------------------------------------------
 constexpr int kVsTPB = 256, kVsIPT = 8, kVsTile = kVsTPB * kVsIPT;   // victim scan tiles
+#ifdef UM_VS_TRACE
+// Diagnostic build only (tools/vs_trace.py): per-CTA %globaltimer stamps of the victim
+// kernels.  [4b] start, [4b+1] end, [4b+2] tiles, [4b+3] end of the first tile of scan
+// CTA b; [6000 + 2b] apply CTA b; [8000], [8007], [8001] finalize start, after the tile
+// passes, end; [8002], [8003] examined tiles, k.
+__device__ unsigned long long g_vs_tr[8192];
+__device__ __forceinline__ unsigned long long vs_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define VS_TR(i, v) (g_vs_tr[(i)] = (unsigned long long)(v))
+#else
+#define VS_TR(i, v) ((void)0)
+#endif
 constexpr int kVaPass = 128;   // victims per warp pass of k_victims_apply
 
 __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t seq, int evict_mode, uint32_t want,
                                                             int npar, int prefetch) {
   pdl_enter();
+#ifdef UM_VS_TRACE
+  uint32_t tr_tiles = 0;
+  if (threadIdx.x == 0 && blockIdx.x < 1500) VS_TR(4 * blockIdx.x, vs_now());
+#endif
   constexpr int NW = kVsTPB / 32;
   __shared__ uint32_t s_off[kVsIPT * NW + 1];
   __shared__ unsigned long long s_dh, s_ld, s_uh, s_lu, s_mk[2];
@@ -1070,15 +1089,14 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
   const int w = threadIdx.x >> 5;
   const unsigned lt = lanemask_lt();
   const unsigned me = 1u << (threadIdx.x & 31);
-  // Tickets and the running candidate total share one 64-bit word, so a ticket comes
-  // with a consistent snapshot: every count in it was added by a finished tile, which
-  // took its ticket earlier -- a smaller one.  If the snapshot reaches k, tiles [0, t)
-  // hold >= k candidates and tile t is not read.  Thread 0 fetches the next ticket while
-  // the current tile is processed (the atomic's latency is off the critical path).
+  // CTA b starts on tile b (every grid CTA is resident); later tiles come from a ticket,
+  // tile gridDim.x + t.  Tickets and the running candidate total share one 64-bit word,
+  // so a ticket comes with a consistent snapshot: every count in it was added by a
+  // finished tile, which has a smaller index.  If the snapshot reaches k, tiles [0, t)
+  // hold >= k candidates and tile t is not read.
   if (threadIdx.x == 0) {
-    const unsigned long long x = atomicAdd(&c->vs_combo, 1ull);
-    s_tile = (uint32_t)x;
-    s_skip = (uint32_t)(x >> 32);   // snapshot
+    s_tile = blockIdx.x;
+    s_skip = 0;
   }
   while (true) {
     __syncthreads();
@@ -1090,6 +1108,9 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
       break;
     }
     unsigned long long nxt = 0;
+#ifdef UM_VS_TRACE
+    ++tr_tiles;
+#endif
     if (threadIdx.x == 0) {
       if (prefetch) nxt = atomicAdd(&c->vs_combo, 1ull);
       s_mk[0] = s_mk[1] = ~0ull;
@@ -1149,12 +1170,21 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
       // without prefetch the next ticket comes with this tile's count (one atomic)
       if (!prefetch) nxt = atomicAdd(&c->vs_combo, ((unsigned long long)cnt << 32) | 1ull) + ((unsigned long long)cnt << 32);
       else if (cnt) atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32);
-      s_tile = (uint32_t)nxt;
+      s_tile = gridDim.x + (uint32_t)nxt;
       s_skip = (uint32_t)(nxt >> 32);
+#ifdef UM_VS_TRACE
+      if (tr_tiles == 1 && blockIdx.x < 1500) VS_TR(4 * blockIdx.x + 3, vs_now());
+#endif
     }
   }
   // completion: the last CTA of the grid finalizes
   __syncthreads();
+#ifdef UM_VS_TRACE
+  if (threadIdx.x == 0 && blockIdx.x < 1500) {
+    VS_TR(4 * blockIdx.x + 1, vs_now());
+    VS_TR(4 * blockIdx.x + 2, tr_tiles);
+  }
+#endif
   if (threadIdx.x == 0) {
     __threadfence();
     s_last = atomicAdd(&c->scan_done, 1u) == gridDim.x - 1;
@@ -1162,6 +1192,9 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
   __syncthreads();
   if (!s_last) return;
   __threadfence();
+#ifdef UM_VS_TRACE
+  if (threadIdx.x == 0) VS_TR(8000, vs_now());
+#endif
   __shared__ unsigned long long s_sc[kVsTPB / 32];
   __shared__ uint32_t s_reach;
   __shared__ unsigned long long s_kd, s_ku;
@@ -1172,56 +1205,91 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
     s_kd = s_ku = ~0ull;
   }
   __syncthreads();
-  // Each thread owns a contiguous run of C tiles (independent loads in flight).  Pass A:
-  // candidate totals -> block scan -> found = min(k, total).  Pass B: per tile the
-  // exclusive prefix ex, the reach tile (ex < k <= ex + count), the first kept live
-  // entry of every tile before it (inclusive prefix < k), and the apply passes of the
-  // tile.  Pass C: the apply work table, one entry per pass of kVaPass victims of a
-  // tile, (tile << 4 | pass) | ex << 32, so the apply's warps are balanced whatever the
-  // spread of victims over tiles (a dense tile holds up to 2048).
-  const uint32_t C = (E + kVsTPB - 1) / kVsTPB;
-  const uint32_t ta = min(E, threadIdx.x * C), tb = min(E, ta + C);
+  // Tiles [0, E) in chunks of kFinS (one chunk up to 2048 tiles = 4M ring entries):
+  //  1. stage the chunk's candidate counts in shared memory (a strided load: all of a
+  //     thread's loads in flight, neighbouring lanes on neighbouring records);
+  //  2. each thread takes a contiguous run of kFinR tiles: block scan -> exclusive
+  //     candidate prefix ex (plus the carry of earlier chunks); per tile take = the
+  //     victims it supplies (ex >= k: none, else min(count, k - ex)), the reach tile (ex
+  //     < k <= ex + count), and its apply passes of <= kVaPass victims; a second block
+  //     scan places them in the work table, one 16-byte entry per pass {victim base,
+  //     tile, scratch offset, count}, so the apply's warps are balanced whatever the
+  //     spread of victims over tiles (a dense tile holds up to 2048);
+  //  3. inclusive prefixes back to shared memory; the first kept live entry of every
+  //     tile before the reach tile (inclusive prefix < k) is min-reduced with strided
+  //     loads again.
   // L2 reads (ld.global.cg): written by other CTAs of this grid, ordered by the fenced
-  // completion counter; independent, so they pipeline
+  // completion counter.
+  constexpr int kFinR = 8, kFinS = kFinR * kVsTPB;
+  __shared__ __align__(16) uint32_t s_fc[kFinS];
   const uint32_t* tc = T.tile_cnt;
-  uint32_t mine = 0;
-#pragma unroll 8
-  for (uint32_t t = ta; t < tb; ++t) mine += __ldcg(tc + (size_t)t * 8);
-  unsigned long long tot;
-  uint32_t ex = (uint32_t)block_excl_scan<kVsTPB>(mine, tot, s_sc);
-  const uint32_t found = (uint32_t)min((unsigned long long)k, tot);
-  uint32_t np = 0;
-  unsigned long long kd = ~0ull, ku = ~0ull;
-#pragma unroll 4
-  for (uint32_t t = ta; t < tb; ++t) {
-    const uint32_t v = __ldcg(tc + (size_t)t * 8);
-    const unsigned long long* rec = reinterpret_cast<const unsigned long long*>(tc + (size_t)t * 8 + 2);
-    const unsigned long long r0 = __ldcg(rec), r1 = __ldcg(rec + 1);
-    if (ex < k && ex + v >= k) s_reach = t;   // exactly one tile
-    if (ex + v < k) {                          // before the reach tile
-      kd = min(kd, r0);
-      ku = min(ku, r1);
+  unsigned long long carry = 0, pcarry = 0, kd = ~0ull, ku = ~0ull;
+  for (uint32_t c0 = 0; c0 < E; c0 += kFinS) {
+    const uint32_t ce = min((uint32_t)kFinS, E - c0);
+    {
+      uint32_t v[kFinR];
+#pragma unroll
+      for (int q = 0; q < kFinR; ++q) {
+        const uint32_t i = q * kVsTPB + threadIdx.x;
+        v[q] = i < ce ? __ldcg(tc + (size_t)(c0 + i) * 8) : 0u;
+      }
+#pragma unroll
+      for (int q = 0; q < kFinR; ++q) s_fc[q * kVsTPB + threadIdx.x] = v[q];
     }
-    const uint32_t take = ex >= found ? 0u : min(v, found - ex);
-    np += (take + kVaPass - 1) / kVaPass;
-    ex += v;
+    __syncthreads();
+    uint32_t v[kFinR], sum = 0;
+    {
+      const uint4* r = reinterpret_cast<const uint4*>(s_fc + threadIdx.x * kFinR);
+      const uint4 a = r[0], b = r[1];
+      v[0] = a.x; v[1] = a.y; v[2] = a.z; v[3] = a.w; v[4] = b.x; v[5] = b.y; v[6] = b.z; v[7] = b.w;
+    }
+#pragma unroll
+    for (int q = 0; q < kFinR; ++q) sum += v[q];
+    unsigned long long tot, ptot;
+    const unsigned long long ex0 = carry + block_excl_scan<kVsTPB>(sum, tot, s_sc);
+    uint32_t np = 0;
+    unsigned long long e = ex0;
+#pragma unroll
+    for (int q = 0; q < kFinR; ++q) {
+      const uint32_t take = e >= k ? 0u : (uint32_t)min((unsigned long long)v[q], k - e);
+      if (e < k && e + v[q] >= k) s_reach = c0 + threadIdx.x * kFinR + q;   // exactly one tile
+      np += (take + kVaPass - 1) / kVaPass;
+      e += v[q];
+    }
+    uint32_t q0 = (uint32_t)(pcarry + block_excl_scan<kVsTPB>(np, ptot, s_sc));
+    e = ex0;
+#pragma unroll
+    for (int q = 0; q < kFinR; ++q) {
+      const uint32_t take = e >= k ? 0u : (uint32_t)min((unsigned long long)v[q], k - e);
+      const uint32_t t = c0 + threadIdx.x * kFinR + q;
+      for (uint32_t off = 0; off < take; off += kVaPass)
+        T.vpass[q0++] = make_ulonglong2((unsigned long long)(e + off) | ((unsigned long long)t << 32),
+                                        (unsigned long long)off | ((unsigned long long)min((uint32_t)kVaPass, take - off) << 32));
+      e += v[q];
+      s_fc[threadIdx.x * kFinR + q] = (uint32_t)min(e, (unsigned long long)k);   // inclusive, clamped
+    }
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < kFinR; ++q) {
+      const uint32_t i = q * kVsTPB + threadIdx.x;
+      if (i < ce && s_fc[i] < k) {   // before the reach tile
+        const unsigned long long* rec = reinterpret_cast<const unsigned long long*>(tc + (size_t)(c0 + i) * 8 + 2);
+        kd = min(kd, __ldcg(rec));
+        ku = min(ku, __ldcg(rec + 1));
+      }
+    }
+    carry += tot;
+    pcarry += ptot;
+    __syncthreads();   // s_fc is restaged by the next chunk
   }
   if (kd != ~0ull) atomicMin(&s_kd, kd);
   if (ku != ~0ull) atomicMin(&s_ku, ku);
-  unsigned long long ptot;
-  uint32_t q0 = (uint32_t)block_excl_scan<kVsTPB>(np, ptot, s_sc);
-  ex = (uint32_t)(block_excl_scan<kVsTPB>(mine, tot, s_sc));
-#pragma unroll 4
-  for (uint32_t t = ta; t < tb; ++t) {
-    const uint32_t v = __ldcg(tc + (size_t)t * 8);
-    const uint32_t take = ex >= found ? 0u : min(v, found - ex);
-    const uint32_t P = (take + kVaPass - 1) / kVaPass;
-    for (uint32_t q = 0; q < P; ++q) T.vpass[q0 + q] = (unsigned long long)((t << 4) | q) | ((unsigned long long)ex << 32);
-    q0 += P;
-    ex += v;
-  }
-  const uint32_t npass = (uint32_t)ptot;
+  const uint32_t found = (uint32_t)min((unsigned long long)k, carry);
+  const uint32_t npass = (uint32_t)pcarry;
   __syncthreads();
+#ifdef UM_VS_TRACE
+  if (threadIdx.x == 0) VS_TR(8007, vs_now());
+#endif
   const uint32_t reach = s_reach;
   if (threadIdx.x == 0) {
     unsigned long long kd = s_kd, ku = s_ku;   // positions in the concatenated index space
@@ -1250,6 +1318,11 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
     c->scan_done = 0;
     c->vs_combo = 0;
     c->first_skip = ~0u;
+#ifdef UM_VS_TRACE
+    VS_TR(8001, vs_now());
+    VS_TR(8002, E);
+    VS_TR(8003, k);
+#endif
   }
   __threadfence();
 }
@@ -1281,22 +1354,25 @@ __global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict
   // load phase keeps AIPT loads of a lane in flight; one host-frame pop (and D2H-list
   // append) per pass.
   static_assert(CH == kVaPass, "pass size");
+#ifdef UM_VS_TRACE
+  if (threadIdx.x == 0 && blockIdx.x < 1000) VS_TR(6000 + 2 * blockIdx.x, vs_now());
+#endif
   const uint32_t nwarps = gridDim.x * (TPB / 32);
   for (uint32_t p = blockIdx.x * (TPB / 32) + (threadIdx.x >> 5); p < npass; p += nwarps) {
-    const unsigned long long ent = T.vpass[p];
-    const uint32_t tile = (uint32_t)ent >> 4, pre = (uint32_t)(ent >> 32);
-    const uint32_t cnt = T.tile_cnt[(size_t)tile * 8];
-    const uint32_t take = pre >= found ? 0u : min(cnt, found - pre);
-    const uint32_t* scr = T.vscratch + (size_t)tile * kVsTile;
+    // entry {victim index of the pass's first victim | tile << 32, offset in the tile's
+    // candidates | victims in the pass << 32}
+    const ulonglong2 ent = T.vpass[p];
+    const uint32_t j0 = (uint32_t)ent.x, tile = (uint32_t)(ent.x >> 32);
+    const uint32_t pn = (uint32_t)(ent.y >> 32);
+    const uint32_t* scr = T.vscratch + (size_t)tile * kVsTile + (uint32_t)ent.y;
     {
-      const uint32_t base = ((uint32_t)ent & 15u) * CH;
       uint32_t v[AIPT], fr[AIPT], hf[AIPT];
       uint8_t ss[AIPT], nk[AIPT];
 #pragma unroll
       for (int q = 0; q < AIPT; ++q) {
-        const uint32_t i = base + q * 32 + lane;
-        v[q] = i < take ? scr[i] : UM_NONE;
-        nk[q] = (i < take && !evict_mode) ? T.needk[(uint32_t)f0 + pre + i] : (uint8_t)0xff;
+        const uint32_t i = q * 32 + lane;
+        v[q] = i < pn ? scr[i] : UM_NONE;
+        nk[q] = (i < pn && !evict_mode) ? T.needk[(uint32_t)f0 + j0 + i] : (uint8_t)0xff;
       }
 #pragma unroll
       for (int q = 0; q < AIPT; ++q) {
@@ -1307,7 +1383,7 @@ __global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict
       for (int q = 0; q < AIPT; ++q) {
         // a write-back victim's bytes land in the host frame of the block migrating into
         // its frame (fused swap, R5) when there is one
-        hf[q] = (ss[q] == ST_G && nk[q] == ST_H) ? T.needhf[(uint32_t)f0 + pre + base + q * 32 + lane] : UM_NONE;
+        hf[q] = (ss[q] == ST_G && nk[q] == ST_H) ? T.needhf[(uint32_t)f0 + j0 + q * 32 + lane] : UM_NONE;
       }
       unsigned bA[AIPT], bD[AIPT];
       uint32_t tA = 0, tD = 0;
@@ -1348,7 +1424,7 @@ __global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict
       }
 #pragma unroll
       for (int q = 0; q < AIPT; ++q) {
-        const uint32_t j = pre + base + q * 32 + lane;
+        const uint32_t j = j0 + q * 32 + lane;
         if (v[q] != UM_NONE) {
           const bool isG = ss[q] == ST_G;
           T.victim[j] = v[q];
@@ -1381,6 +1457,9 @@ __global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict
   const int slots[3] = {S_D2H, S_D2H_AV, S_UNMAPS};
   const long long mul[3] = {(long long)T.B, (long long)T.B, 1};
   block_counts_to<3>(T, cnt3, s_cnt, slots, mul);
+#ifdef UM_VS_TRACE
+  if (threadIdx.x == 0 && blockIdx.x < 1000) VS_TR(6001 + 2 * blockIdx.x, vs_now());
+#endif
 }
 
 // ------------------------------------------------------------------------------------
@@ -2370,6 +2449,7 @@ static int g_vscan_occ = 1;   // resident k_victims_scan CTAs per SM
 static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch (A/B)
 static int g_dir_occ = 8;     // resident k_directive CTAs per SM (persistent grid)
 static int g_dir_minb = 6;    // k_directive CTAs/SM the registers allow: 6 (40 regs); UM_DIR_MINB=7/8 (36/32 regs: one wave for 2^21 blocks) for A/B
+static int g_vs_ctas = 0;     // UM_VS_CTAS=n caps the victim scan grid at n CTAs (test hook: small tables then take tiles by ticket and skip past the k-th candidate)
 static int g_vs_prefetch = 0; // UM_VS_PREFETCH=1: the wide victim scan fetches its next ticket a tile ahead (A/B on B200: 79 vs 73 us pressured touch -- the earlier snapshot reads more tiles past the k-th candidate)
 
 cudaError_t setup_kernels() {
@@ -2380,6 +2460,7 @@ cudaError_t setup_kernels() {
   if (e) return e;
   if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
   if (const char* v = getenv("UM_VS_PREFETCH")) g_vs_prefetch = atoi(v) != 0;
+  if (const char* v = getenv("UM_VS_CTAS")) g_vs_ctas = atoi(v) > 0 ? atoi(v) : 0;
   if (const char* v = getenv("UM_CLS_TPB")) g_cls_tpb = atoi(v) == 512 ? 512 : 256;
   // Optionally one L1/shared carveout for every paging kernel (k_service needs 144 KB of
   // shared memory; a carveout change between consecutive kernels can force an SM drain).
@@ -2478,7 +2559,7 @@ cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, u
   // persistent scan grid: never more CTAs than can be resident (tiles are taken from a
   // ticket in order and a tile may wait on its predecessors' status)
   unsigned nt = ceil_div(scan_bound ? scan_bound : 1, kVsTile);
-  const unsigned cap = (unsigned)(g_nsm * g_vscan_occ);
+  const unsigned cap = g_vs_ctas ? (unsigned)g_vs_ctas : (unsigned)(g_nsm * g_vscan_occ);
   cudaError_t le__ = launch_pdl(k_victims_scan, dim3(nt < cap ? nt : cap), dim3(kVsTPB), 0, s, T, seq, evict_mode, want, npar, g_vs_prefetch);
   if (le__) return le__;
   cudaError_t e = cudaGetLastError();
@@ -2633,3 +2714,9 @@ cudaError_t launch_intake_clear(const Tables& T, uint32_t w0, uint32_t w1, cudaS
 }
 
 }  // namespace um
+
+#ifdef UM_VS_TRACE
+extern "C" __attribute__((visibility("default"))) int um_debug_vs_trace(void* host, unsigned long long bytes) {
+  return (int)cudaMemcpyFromSymbol(host, um::g_vs_tr, bytes);
+}
+#endif

@@ -1,6 +1,8 @@
 """Parity of the CUDA path (libum.so, called through the C ABI) with the CPU oracle:
 per-block final state, USED/DISC order, every counter and every block's content tag
 must match bit-exactly.  Run with `pytest -m gpu` on a B200."""
+import os
+
 import numpy as np
 import pytest
 
@@ -267,6 +269,22 @@ def test_wide_victim_selection(mode):
     t = tb.build()
     for copy in ("kernel", "ce"):
         assert_parity(t, mode, _gpu(t, mode, copy=copy))
+
+
+@pytest.mark.parametrize("ctas", [1, 3])
+def test_wide_victim_scan_tickets(ctas):
+    """The same trace with the victim scan grid capped at 1 / 3 CTAs (UM_VS_CTAS, read
+    once per process, hence the subprocess): after its first tile every CTA takes tiles
+    by ticket and stops past the k-th candidate -- the path full-size tables take (more
+    tiles than resident CTAs), here at test size."""
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = ("import sys; sys.path[:0] = [%r, %r]; import test_gpu_parity as t\n"
+            "for m in ('base', 'eager', 'lazy'): t.test_wide_victim_selection(m)\nprint('ok')") % (root, os.path.join(root, "tests"))
+    env = dict(os.environ, UM_VS_CTAS=str(ctas))
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=900, cwd=root, env=env)
+    assert r.returncode == 0 and r.stdout.strip().endswith("ok"), r.stdout[-2000:] + r.stderr[-4000:]
 
 
 def _full_size_trace(iterations=2, B=2 << 20):
