@@ -41,7 +41,7 @@ class Oracle:
 
     def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int,
                  discard_off: bool = False, record: bool = False, host_release: bool = True,
-                 overlap: int = 0):
+                 overlap: int = 0, reserve: int = 0):
         if arena_bytes % block_bytes:
             raise ValueError("arena_bytes must be a multiple of block_bytes")
         self.B = block_bytes
@@ -64,6 +64,15 @@ class Oracle:
         # of them that still leaves the current sub-op satisfiable (sizes summing with
         # |S| to at most nframes).  overlap = 0 is the sequential model of SURVEY §8(c).
         self.overlap = overlap
+        # reserve (reading R12 / SURVEY NEXT-2, proactive eviction): the paper's
+        # eviction process starts only "when the GPU's free page queue is empty" (§5.5
+        # L219).  With reserve = R > 0 it also runs AHEAD of demand: after every GPU
+        # sub-op with at least one block, if fewer than R frames are free, it reclaims
+        # R - free more (best effort) in the same order (§5.5), skipping the
+        # blocks of that sub-op and, with overlap, of every sub-op in the window (their
+        # application kernels may still run).  Part of the sub-op: same seq, not an op.
+        # Its write-backs can then overlap the application kernel (L146, L166, L381).
+        self.reserve = reserve
         self.window: list = []                  # (blocks, count) of recent GPU sub-ops, oldest first
         n = self.nblocks
         self.st = [U] * n
@@ -232,6 +241,17 @@ class Oracle:
                     del self.disc[b]
                     self._to_used(b, seq)
 
+    def _evict_ahead(self, S: list, seq: int):
+        """R12 proactive eviction after GPU sub-op `seq` over blocks S (see __init__)."""
+        if self.reserve <= 0 or not S or self.free >= self.reserve:
+            return
+        pinned = set(S)
+        if self.overlap:
+            for blocks, _cnt in self.window:    # the last `overlap` GPU sub-ops, S included
+                pinned |= blocks
+        for v in self._select_victims(self.reserve - self.free, pinned):
+            self._reclaim(v, seq)
+
     # ------------------------------------------------------------------ API ops
     def touch(self, accesses):
         """um_touch_batch: a batch of GPU accesses ("faults").  Distinct blocks are
@@ -256,6 +276,7 @@ class Oracle:
                 if b in writes:
                     self.gpu_stamp[b] = stamp(seq, b)   # a write after a discard is
                                                         # visible (§4.1)
+            self._evict_ahead(chunk, seq)
 
     def prefetch(self, off: int, ln: int, dst: int):
         """um_prefetch (cudaMemPrefetchAsync, §2.1; Listing 2 L54-59)."""
@@ -268,7 +289,9 @@ class Oracle:
             F = self.nframes
             chunks = [S[i:i + F] for i in range(0, len(S), F)] or [[]]
             for chunk in chunks:
-                self._gpu_subop(chunk, self._next_seq(), touch=False)
+                seq = self._next_seq()
+                self._gpu_subop(chunk, seq, touch=False)
+                self._evict_ahead(chunk, seq)
             return
         seq = self._next_seq()
         st, sts = self.st, self.stats
@@ -445,12 +468,13 @@ def apply_op(o: Oracle, op: tuple, mode: str):
 
 
 def replay(trace, mode: str = "eager", record: bool = False, stop: int | None = None,
-           host_release: bool = True, overlap: int = 0) -> Oracle:
+           host_release: bool = True, overlap: int = 0, reserve: int = 0) -> Oracle:
     """Replay a tracegen.Trace (optionally only its first `stop` ops) in one mode."""
     if mode not in MODES:
         raise ValueError(mode)
     o = Oracle(trace.block_bytes, trace.arena_bytes, trace.budget_bytes,
-               discard_off=(mode == "base"), record=record, host_release=host_release, overlap=overlap)
+               discard_off=(mode == "base"), record=record, host_release=host_release, overlap=overlap,
+               reserve=reserve)
     for i, op in enumerate(trace.iter_ops()):
         if stop is not None and i >= stop:
             break

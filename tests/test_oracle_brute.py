@@ -594,3 +594,47 @@ def test_free_flat_memory_and_conservation(seed, nblocks, nframes, host_release)
                 assert got[b] == val[b], (mode, b)
             else:
                 assert got[b] in hist[b], (mode, b)
+
+
+# ------------------------------------------------------------------ R12 (proactive eviction)
+@settings(max_examples=80, deadline=None)
+@given(seed=hst.integers(0, 10**6), nblocks=hst.integers(2, 10), nframes=hst.integers(1, 5),
+       reserve=hst.integers(1, 4), overlap=hst.sampled_from([0, 2]))
+def test_reserve_keeps_semantics(seed, nblocks, nframes, reserve, overlap):
+    """R12 changes when a block is evicted, never what a program reads: the flat-memory
+    check (iii)/(iv), conservation after every op and the no-writeback-of-discarded
+    invariant (ii) hold; after a GPU op of at most nframes blocks without the window,
+    either `reserve` frames are free or every queued block belongs to that op (only the
+    op's own blocks are kept from early reclaim); with room to spare it changes nothing."""
+    t = tg.gen_small(seed, nblocks=nblocks, nframes=nframes, n_ops=40)
+    for mode in ("base", "eager", "lazy"):
+        o = Oracle(t.block_bytes, t.arena_bytes, t.budget_bytes, discard_off=(mode == "base"),
+                   record=True, overlap=overlap, reserve=reserve)
+        for op in t.iter_ops():
+            apply_op(o, op, mode)
+            o.check_conservation()
+            kind, flags, off, ln, accs = op
+            gpu = kind == 0 or (kind == 1 and flags == 0)
+            if gpu and not overlap:
+                cover = set()
+                for (a, n, _k) in (accs if kind == 0 else [(off, ln, 0)]):
+                    cover.update(o._cover(a, n))
+                if 0 < len(cover) <= nframes:
+                    others = [b for b in list(o.used) + list(o.disc) if b not in cover]
+                    assert o.free >= reserve or not others, (mode, o.free, others)
+        assert all(k != "D2H" or p == G for (_s, k, _b, p) in o.log)
+        val, dc, hist = FlatMemory(t, mode).run()
+        got = o.contents()
+        for b in range(t.nblocks):
+            assert got[b] == val[b] if not dc[b] else got[b] in hist[b], (mode, b)
+    roomy = tg.gen_small(seed, nblocks=nblocks, nframes=nblocks + reserve, n_ops=40)
+    for mode in ("base", "eager", "lazy"):
+        assert replay(roomy, mode, reserve=reserve).dump() == replay(roomy, mode).dump()
+
+
+def test_reserve_zero_is_the_paper_model():
+    """reserve = 0 (the default) is §5.5's on-demand eviction exactly."""
+    for seed in range(5):
+        t = tg.gen_c1(seed).slice_ops(0, 1500)
+        for mode in ("base", "eager", "lazy"):
+            assert replay(t, mode, reserve=0).dump() == replay(t, mode).dump()

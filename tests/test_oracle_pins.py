@@ -18,7 +18,7 @@ SCEN = scn.load()
 def test_scenario(name, host_release):
     sc = SCEN[name]
     trace, mode = scn.build(sc)
-    o = replay(trace, mode, host_release=host_release, overlap=sc.get("overlap", 0))
+    o = replay(trace, mode, host_release=host_release, overlap=sc.get("overlap", 0), reserve=sc.get("reserve", 0))
     o.check_conservation()
     d = o.dump()
     exp = sc["expect"]
