@@ -156,8 +156,9 @@ def measure_link_peak(torch, dev):
 
 
 # ------------------------------------------------------------------------------ ours
-def run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=None, flags_extra=0):
-    arena = harness.make_arena(trace, mode, mem=mem, flags=um.UM_F_APP_STAMP | um.UM_F_TIMING | flags_extra)
+def run_mode(torch, um, harness, mem, trace, mode, W, K, clocks=None, flags_extra=0, reserve=0):
+    arena = harness.make_arena(trace, mode, mem=mem, flags=um.UM_F_APP_STAMP | um.UM_F_TIMING | flags_extra,
+                               reserve_blocks=reserve)
     try:
         harness.alloc_buffers(arena, trace)
         bounds = harness.iteration_bounds(trace)

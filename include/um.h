@@ -121,6 +121,18 @@ typedef struct {
                                  pages, a prefetch any, A8/A17).  Byte counters and
                                  content tags are per page.  Not combinable with
                                  UM_F_COPY_CE or UM_F_OVERLAP (UM_EINVAL).                */
+  uint32_t reserve_blocks;    /* 0: evict on demand only (PAPER §5.5: "The eviction
+                                 process starts when the GPU's free page queue is empty").
+                                 R > 0: proactive eviction (reading R12, SURVEY
+                                 NEXT-2): after every GPU sub-op with >= 1 block, if fewer
+                                 than R frames are free, R - free more are reclaimed (best
+                                 effort) in the same order (discarded FIFO, then the LRU end
+                                 of USED, L219-221), skipping the sub-op's blocks and, with
+                                 UM_F_OVERLAP, the window's; valid victims are written back
+                                 on the paging stream, where they overlap the sub-op's
+                                 application kernel under UM_F_OVERLAP.  Same seq as the
+                                 sub-op.  Must be <= nframes; single level only (UM_EINVAL
+                                 with two-level page_bytes).                              */
 } um_config;
 
 /* Counters (int64, 16 slots).  Byte counters are multiples of block_bytes. */

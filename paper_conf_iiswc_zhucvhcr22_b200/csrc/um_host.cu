@@ -58,6 +58,7 @@ static um_status check_cfg(const um_config* c) {
         c->block_bytes / c->page_bytes > 32)
       return UM_EINVAL;
     if (c->flags & (UM_F_COPY_CE | UM_F_OVERLAP)) return UM_EINVAL;
+    if (c->reserve_blocks) return UM_EINVAL;
   }
   if (!is_pow2(c->block_bytes) || c->block_bytes < 4096) return UM_EINVAL;
   if (c->arena_bytes == 0 || c->arena_bytes % c->block_bytes) return UM_EINVAL;
@@ -66,6 +67,7 @@ static um_status check_cfg(const um_config* c) {
   if (c->arena_bytes / c->block_bytes >= 0x80000000ull) return UM_EINVAL;
   if (c->budget_bytes < c->block_bytes) return UM_EINVAL;
   if (c->budget_bytes / c->block_bytes >= 0x7fffffffull) return UM_EINVAL;
+  if (c->reserve_blocks > c->budget_bytes / c->block_bytes) return UM_EINVAL;
   if (c->host_chunk_bytes == 0 || c->host_chunk_bytes % c->block_bytes) return UM_EINVAL;
   if (c->n_host_chunks == 0) return UM_EINVAL;
   if ((uint64_t)c->n_host_chunks * (c->host_chunk_bytes / c->block_bytes) < 2) return UM_EINVAL;
@@ -793,6 +795,49 @@ static um_status device_intake(um_arena* a, const um_access* acc, uint32_t n) {
   return UM_OK;
 }
 
+// Evict mode of K3 (k = want - free on the device, clamped to the candidates: blocks
+// with pin >= T.pfloor are skipped), then the D2H-only list through the engine.  Used by
+// um_evict (R4) and by the proactive eviction after a GPU sub-op (R12).
+static um_status evict_enqueue(um_arena* a, uint32_t seq, uint32_t want) {
+  cudaEvent_t sp = span_open(a);
+  if (want > kVictWideMin)
+    CK(launch_victims_wide(a->T, seq, 1, want, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap),
+                           want, a->npar, a->ps));
+  else
+    CK(launch_victims(a->T, seq, 1, want, a->npar, a->ps));
+  a->n_launch += want > kVictWideMin ? 1 : 0;
+  span_close(a, sp, 0);
+  sp = span_open(a);
+  if (use_ce(a, want)) {
+    um_status s = ce_d2h_only(a, want);
+    if (s) return s;
+  } else {
+    CK(launch_service(a->T, SVC_D2H_ONLY, seq, want, a->ps));
+  }
+  span_close(a, sp, 1);
+  a->n_launch += 2;
+  a->n_xfer++;
+  return UM_OK;
+}
+
+// R12 proactive eviction after GPU sub-op `seq` (n >= 1 blocks): keep reserve_blocks
+// frames free, best effort.  Protected: the sub-op's blocks (pin == seq) and, with
+// UM_F_OVERLAP, every block of the window (the last ovw GPU sub-ops, this one included:
+// their application kernels may still run), i.e. pin >= the oldest member's seq; older
+// application kernels finish first (they wrote frames that may now be written back).
+static um_status evict_ahead(um_arena* a, uint32_t seq) {
+  const uint32_t R = a->cfg.reserve_blocks;
+  if (!R) return UM_OK;
+  uint32_t floor = seq;
+  if (overlap_on(a)) {
+    floor = a->nwin ? a->win[0].seq : seq;
+    um_status st = app_wait_below(a, floor);
+    if (st) return st;
+  }
+  a->T.pfloor = floor;
+  return evict_enqueue(a, seq, R);
+}
+
 // Enqueue the K1/K2 -> K3 -> K4/K5/K6 (-> K9) chain for every sub-op of a GPU op.
 static um_status run_gpu_op(um_arena* a, int touch) {
   uint64_t total = 0;
@@ -990,6 +1035,8 @@ static um_status run_gpu_op(um_arena* a, int touch) {
       }
       a->n_launch++;
     }
+    um_status ea = evict_ahead(a, seq);
+    if (ea) return ea;
   }
   return UM_OK;
 }
@@ -1511,25 +1558,7 @@ UM_API um_status um_evict(um_arena* a, uint64_t bytes, void* stream) {
   if (want > a->nframes) want = a->nframes;
   a->T.pfloor = seq;   // no pinned blocks: every in-flight application kernel finishes first
   if (overlap_on(a) && (s = app_wait_all(a))) return s;
-  if (want) {
-    cudaEvent_t sp = span_open(a);
-    if (want > kVictWideMin)
-      CK(launch_victims_wide(a->T, seq, 1, (uint32_t)want, std::min<uint64_t>(a->ub[RING_DISC] + a->ub[RING_USED], 2 * a->L.cap), (uint32_t)want, a->npar, a->ps));
-    else
-      CK(launch_victims(a->T, seq, 1, (uint32_t)want, a->npar, a->ps));
-    a->n_launch += want > kVictWideMin ? 1 : 0;
-    span_close(a, sp, 0);
-    sp = span_open(a);
-    if (use_ce(a, want)) {
-      s = ce_d2h_only(a, (uint32_t)want);
-      if (s) return s;
-    } else {
-      CK(launch_service(a->T, SVC_D2H_ONLY, seq, (uint32_t)want, a->ps));
-    }
-    span_close(a, sp, 1);
-    a->n_launch += 2;
-    a->n_xfer++;
-  }
+  if (want && (s = evict_enqueue(a, seq, (uint32_t)want))) return s;
   return hand_out(a, stream);
 }
 

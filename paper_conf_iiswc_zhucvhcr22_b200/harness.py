@@ -19,11 +19,12 @@ def mode_flags(mode: str) -> int:
 
 
 def make_arena(trace, mode: str, *, flags: int = um.UM_F_APP_STAMP | um.UM_F_CHECK, host_pool_bytes=None,
-               device: int = 0, mem=None, page_bytes: int = 0) -> um.Arena:
+               device: int = 0, mem=None, page_bytes: int = 0, reserve_blocks: int = 0) -> um.Arena:
     """page_bytes < block_bytes: a two-level arena (chunks of block_bytes, pages of
-    page_bytes)."""
+    page_bytes).  reserve_blocks > 0: proactive eviction (R12)."""
     return um.Arena(trace.block_bytes, trace.arena_bytes, trace.budget_bytes, flags=flags | mode_flags(mode),
-                    host_pool_bytes=host_pool_bytes, device=device, mem=mem, page_bytes=page_bytes)
+                    host_pool_bytes=host_pool_bytes, device=device, mem=mem, page_bytes=page_bytes,
+                    reserve_blocks=reserve_blocks)
 
 
 def alloc_buffers(arena: um.Arena, trace) -> None:

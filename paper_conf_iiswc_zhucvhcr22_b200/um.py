@@ -34,7 +34,7 @@ class um_config(C.Structure):
                 ("budget_bytes", C.c_uint64), ("frames", C.c_void_p), ("workspace", C.c_void_p),
                 ("workspace_bytes", C.c_uint64), ("host_chunks", C.POINTER(C.c_void_p)),
                 ("n_host_chunks", C.c_uint32), ("host_chunk_bytes", C.c_uint64), ("flags", C.c_uint32),
-                ("page_bytes", C.c_uint32)]
+                ("page_bytes", C.c_uint32), ("reserve_blocks", C.c_uint32)]
 
 
 STAT_FIELDS = ("h2d_bytes", "d2h_bytes", "zf_bytes", "h2d_avoided_bytes", "d2h_avoided_bytes", "faults",
@@ -288,7 +288,7 @@ class Arena:
 
     def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, flags: int = 0,
                  host_pool_bytes: int | None = None, host_chunk_bytes: int | None = None, device: int = 0,
-                 mem: Memory | None = None, page_bytes: int = 0):
+                 mem: Memory | None = None, page_bytes: int = 0, reserve_blocks: int = 0):
         self.B = block_bytes
         self.nblocks = arena_bytes // block_bytes
         self.nframes = budget_bytes // block_bytes
@@ -300,6 +300,7 @@ class Arena:
         self.cfg = self.mem.config(arena_bytes, budget_bytes, flags)
         if page_bytes:
             self.cfg.page_bytes = page_bytes
+        self.cfg.reserve_blocks = reserve_blocks   # R12 proactive eviction (0: on demand only)
         self.ppc = block_bytes // self.cfg.page_bytes if self.cfg.page_bytes else 1
         self.handle = um_arena_create(self.cfg)
         self.stream_ptr = um_stream(self.handle)

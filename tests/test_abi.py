@@ -87,3 +87,24 @@ def test_two_level_config_validation_without_gpu():
         bad.page_bytes, bad.flags = pb, fl
         with pytest.raises(um.UmError):
             um.um_workspace_size(bad)
+
+
+def test_reserve_config_validation_without_gpu():
+    """reserve_blocks (R12 proactive eviction): accepted up to nframes at single level;
+    above nframes, or with two-level page_bytes, UM_EINVAL."""
+    import ctypes as C
+    from paper_conf_iiswc_zhucvhcr22_b200 import um
+    hc = (C.c_void_p * 1)(1)
+    base = um.um_config(device=0, block_bytes=2 << 20, arena_bytes=64 << 20, budget_bytes=16 << 20, frames=None,
+                        workspace=None, workspace_bytes=0, host_chunks=C.cast(hc, C.POINTER(C.c_void_p)),
+                        n_host_chunks=1, host_chunk_bytes=64 << 20, flags=0, page_bytes=0)
+    ws = um.um_workspace_size(base)
+    for r in (1, 8):
+        ok = um.um_config.from_buffer_copy(base)
+        ok.reserve_blocks = r
+        assert um.um_workspace_size(ok) == ws
+    for r, pb in [(9, 0), (1, 64 << 10)]:
+        bad = um.um_config.from_buffer_copy(base)
+        bad.reserve_blocks, bad.page_bytes = r, pb
+        with pytest.raises(um.UmError):
+            um.um_workspace_size(bad)

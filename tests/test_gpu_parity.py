@@ -27,27 +27,32 @@ def _cuda():
 COPY_FLAGS = {"default": 0, "kernel": 32, "ce": 2}   # default = the TMA kernel K4; UM_F_COPY_KERNEL / UM_F_COPY_CE
 
 
-def xlog_bound(trace):
+def xlog_bound(trace, reserve=0):
     """Upper bound on the transfer-log records of a trace: every covered block of a GPU
     op may bring one newcomer record and one victim write-back, every block of a
-    prefetch(HOST) or evict one write-back."""
+    prefetch(HOST) or evict one write-back; with proactive eviction (R12) every GPU
+    sub-op may add `reserve` write-backs."""
     B, F = trace.block_bytes, trace.budget_bytes // trace.block_bytes
     n = 0
     for kind, flags, off, ln, accs in trace.iter_ops():
         if kind == tg.OP_TOUCH:
-            n += 2 * sum((o + m - 1) // B - o // B + 1 for (o, m, _k) in accs if m)
+            nb = sum((o + m - 1) // B - o // B + 1 for (o, m, _k) in accs if m)
+            n += 2 * nb + reserve * (nb // F + 1)
         elif kind == tg.OP_PREFETCH:
-            n += (2 if flags == tg.DST_GPU else 1) * ((off + ln - 1) // B - off // B + 1 if ln else 0)
+            nb = (off + ln - 1) // B - off // B + 1 if ln else 0
+            n += (2 if flags == tg.DST_GPU else 1) * nb + (reserve * (nb // F + 1) if flags == tg.DST_GPU else 0)
         elif kind == tg.OP_EVICT:
             n += min(F, ln // B + 1)
     return n + 64
 
 
-def _gpu(trace, mode, copy="default", overlap=False, xlog=True, **kw):
+def _gpu(trace, mode, copy="default", overlap=False, xlog=True, reserve=0, **kw):
     """The CUDA path's result, with the transfer log attached (xlog_bound capacity)."""
     from paper_conf_iiswc_zhucvhcr22_b200 import harness, um
     flags = um.UM_F_APP_STAMP | um.UM_F_CHECK | COPY_FLAGS[copy] | (um.UM_F_OVERLAP if overlap else 0)
-    return harness.run_trace(trace, mode, flags=flags, xlog=xlog_bound(trace) if xlog else 0, **kw)
+    if reserve:
+        kw["reserve_blocks"] = reserve
+    return harness.run_trace(trace, mode, flags=flags, xlog=xlog_bound(trace, reserve) if xlog else 0, **kw)
 
 
 OVERLAP_W = 2   # kOverlapW in csrc/um_internal.h (reading R7)
@@ -60,9 +65,9 @@ def _first_diff(a, b):
     return f"transfer log lengths differ: gpu {len(a)} oracle {len(b)}"
 
 
-def assert_parity(trace, mode, g=None, overlap=False):
-    g = g if g is not None else _gpu(trace, mode, overlap=overlap)
-    orc = oracle_replay(trace, mode, overlap=OVERLAP_W if overlap else 0, record="xlog" in g)
+def assert_parity(trace, mode, g=None, overlap=False, reserve=0):
+    g = g if g is not None else _gpu(trace, mode, overlap=overlap, reserve=reserve)
+    orc = oracle_replay(trace, mode, overlap=OVERLAP_W if overlap else 0, record="xlog" in g, reserve=reserve)
     o = orc.dump()
     if "xlog" in g:
         # every H2D / D2H / zero-fill, with its sub-op seq and the block's prior state
@@ -87,7 +92,7 @@ def test_scenarios(name):
     trace, mode = scn.build(sc)
     ov = sc.get("overlap", 0)
     assert ov in (0, OVERLAP_W)
-    g, _ = assert_parity(trace, mode, overlap=bool(ov))
+    g, _ = assert_parity(trace, mode, overlap=bool(ov), reserve=sc.get("reserve", 0))
     for k, v in sc["expect"]["stats"].items():
         assert g["stats"][k] == v, k
     assert [scn.ST[x] for x in sc["expect"]["st"]] == list(g["st"])
@@ -468,3 +473,50 @@ def test_small_random_with_free(seed, mode):
     t = tg.gen_small(300 + seed, nblocks=nb, nframes=nf, n_ops=300, max_ranges=4, max_blocks=6,
                      mix=[45, 12, 5, 10, 10, 3, 2, 13])
     assert_parity(t, mode)
+
+
+# ------------------------------------------------------------------ R12: proactive eviction
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+@pytest.mark.parametrize("overlap", [False, True])
+def test_reserve_small_random(seed, mode, overlap):
+    """um_config.reserve_blocks (reading R12): after every GPU sub-op the
+    engine reclaims frames ahead of demand; bit-exact against the oracle (state, queue
+    orders, counters, contents, transfer log), with and without the R7 window."""
+    rng = np.random.default_rng(200 + seed)
+    nb, nf = int(rng.integers(2, 24)), int(rng.integers(1, 6))
+    t = tg.gen_small(200 + seed, nblocks=nb, nframes=nf, n_ops=300, max_ranges=4, max_blocks=6)
+    assert_parity(t, mode, overlap=overlap, reserve=int(rng.integers(1, nf + 1)))
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_reserve_c1(mode):
+    t = tg.gen_c1(5).slice_ops(0, 5000)
+    assert_parity(t, mode, reserve=16)
+    assert_parity(t, mode, overlap=True, reserve=16)
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_reserve_c3_small(mode):
+    """C3 with proactive eviction through both transfer paths, sequential and pipelined."""
+    t = tg.gen_c3(block_bytes=64 << 10, budget_bytes=192 << 20, iterations=2, workspace_bytes=4 << 20,
+                  layers=tg.scale_layers(tg.VGG16, 1.0 / 512, 1.0 / 64), batch=8)
+    for copy in ("default", "ce"):
+        for ov in (False, True):
+            assert_parity(t, mode, _gpu(t, mode, copy=copy, overlap=ov, reserve=64), overlap=ov, reserve=64)
+
+
+@pytest.mark.parametrize("mode", ["eager", "lazy"])
+def test_reserve_wide(mode):
+    """A reserve above 8192 frames: the proactive eviction takes the wide victim scan."""
+    t = tg.gen_sparse(1, nframes=1 << 14)
+    assert_parity(t, mode, reserve=9000)
+
+
+def test_reserve_rejected():
+    """reserve_blocks > nframes, or with two-level granularity: UM_EINVAL."""
+    from paper_conf_iiswc_zhucvhcr22_b200 import um
+    with pytest.raises(Exception):
+        um.Arena(64 << 10, 8 << 20, 4 << 20, reserve_blocks=65, host_pool_bytes=8 << 20)
+    with pytest.raises(Exception):
+        um.Arena(2 << 20, 64 << 20, 16 << 20, page_bytes=64 << 10, reserve_blocks=1, host_pool_bytes=64 << 20)
