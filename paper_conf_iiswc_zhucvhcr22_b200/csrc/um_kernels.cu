@@ -807,9 +807,10 @@ __device__ __forceinline__ void classify_body(const Tables& T, const OpIv& iv, u
 }
 
 // 4 items per thread, 8 CTAs/SM (A/B on B200: 8 items per thread at 6 CTAs/SM spills and
-// runs the 2^21-block touch in 42 vs 30 us)
+// runs the 2^21-block touch in 42 vs 30 us); the interval form (bitmap prefix, one more
+// live array) runs 6 CTAs/SM (40 registers) so that it does not spill
 template <bool LIST, int TPB>
-__global__ void __launch_bounds__(TPB, 2048 / TPB) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
+__global__ void __launch_bounds__(TPB, (LIST ? 2048 : 1536) / TPB) k_classify(Tables T, const __grid_constant__ OpIv iv, uint32_t g0,
                                                               uint32_t n, uint32_t seq, int touch,
                                                               unsigned long long tail0, int npar, int k0) {
   pdl_enter();

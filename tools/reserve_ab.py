@@ -35,7 +35,11 @@ def main():
     for sched in a.schedules.split(","):
         fl = um.UM_F_OVERLAP if sched == "overlap" else 0
         for r in [int(x) for x in a.reserves.split(",")]:
-            res = bench.run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=fl, reserve=r)
+            try:
+                res = bench.run_mode(torch, um, harness, mem, trace, "eager", W, K, flags_extra=fl, reserve=r)
+            except um.UmError as e:   # e.g. the host-frame pool (arena - budget + 2 GiB) cannot hold the reserve
+                print(json.dumps({"schedule": sched, "reserve_blocks": r, "error": str(e)}), flush=True)
+                continue
             s = res["stats_per_iter"]
             print(json.dumps({"schedule": sched, "reserve_blocks": r, "reserve_gib": r * args.block / 2**30,
                               "iter_ms": res["iter_ms"], "iter_ms_each": res["iter_ms_each"],
