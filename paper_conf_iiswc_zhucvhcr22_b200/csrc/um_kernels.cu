@@ -336,7 +336,6 @@ __global__ void k_init(Tables T, int nh) {
     c->k0_take = c->k0_pend = 0;
     c->vs_combo = 0;
     c->first_skip = ~0u;
-    c->vs_bar = 0;
     c->vt_reach = 0;
   }
 }
@@ -1096,14 +1095,6 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
   // so a ticket comes with a consistent snapshot: every count in it was added by a
   // finished tile, which has a smaller index.  If the snapshot reaches k, tiles [0, t)
   // hold >= k candidates and tile t is not read.
-  // First wave: every CTA is resident (the grid is sized to the occupancy), so when
-  // tickets exist beyond it the CTAs meet at a grid barrier after their first tile and
-  // the first ticket's snapshot holds the whole wave's count: if the wave already holds
-  // k candidates (a pressured sub-op over a ring with few dead slots), no CTA reads a
-  // second tile (without it, CTAs that finish early take tickets before the wave's
-  // counts are in, about doubling the tiles read).
-  const bool wave_bar = !prefetch && ntiles > gridDim.x;
-  bool first = true;
   if (threadIdx.x == 0) {
     s_tile = blockIdx.x;
     s_skip = 0;
@@ -1178,25 +1169,14 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
       // no fence: the records are read by the finalizing CTA after the completion
       // counter below (fenced), the scratch slice by k_victims_apply (next launch)
       // without prefetch the next ticket comes with this tile's count (one atomic)
-      if (first && wave_bar) {
-        if (cnt) atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32);
-        __threadfence();
-        atomicAdd(&c->vs_bar, 1u);
-        while (*(volatile unsigned int*)&c->vs_bar < gridDim.x) __nanosleep(64);
-        __threadfence();
-        nxt = atomicAdd(&c->vs_combo, 1ull);
-      } else if (!prefetch) {
-        nxt = atomicAdd(&c->vs_combo, ((unsigned long long)cnt << 32) | 1ull) + ((unsigned long long)cnt << 32);
-      } else if (cnt) {
-        atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32);
-      }
+      if (!prefetch) nxt = atomicAdd(&c->vs_combo, ((unsigned long long)cnt << 32) | 1ull) + ((unsigned long long)cnt << 32);
+      else if (cnt) atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32);
       s_tile = gridDim.x + (uint32_t)nxt;
       s_skip = (uint32_t)(nxt >> 32);
 #ifdef UM_VS_TRACE
       if (tr_tiles == 1 && blockIdx.x < 1500) VS_TR(4 * blockIdx.x + 3, vs_now());
 #endif
     }
-    first = false;
   }
   // completion: the last CTA of the grid finalizes
   __syncthreads();
@@ -1339,7 +1319,6 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
     c->scan_done = 0;
     c->vs_combo = 0;
     c->first_skip = ~0u;
-    c->vs_bar = 0;
 #ifdef UM_VS_TRACE
     VS_TR(8001, vs_now());
     VS_TR(8002, E);
