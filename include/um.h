@@ -176,6 +176,15 @@ um_status um_discard_lazy(um_arena *a, uint64_t off, uint64_t len, void *stream)
  * return (the caller may reuse it). */
 um_status um_touch_batch(um_arena *a, const um_access *acc, uint32_t n, void *stream);
 
+/* The same batch with the records in DEVICE-accessible memory (the GPU's own fault
+ * buffer: faults are raised by the GPU): `acc` = n records, 16-byte
+ * aligned, written in stream order before this call on `stream`.  The GPU range-checks,
+ * expands and deduplicates them (op bitmap -> sorted distinct block list); the host only
+ * reads back the block count (one stream synchronization) to number the sub-ops, so the
+ * records have been consumed when the call returns.  A record outside the arena:
+ * UM_EINVAL with no state changed.  Single level only (UM_EINVAL with page_bytes). */
+um_status um_touch_batch_dev(um_arena *a, const um_access *acc, uint32_t n, void *stream);
+
 /* The application releases [off, off+len) (cudaFree of managed memory; reading R9 of
  * DESIGN.md).  Every block FULLY inside the range returns to U (never populated: it
  * reads as zeros) with no transfer: its GPU frame goes back to the pool the eviction

@@ -273,6 +273,7 @@ struct um_arena {
   std::vector<CItem> citems;   // two-level: the op's chunks with page masks
   uint32_t ppc = 1, P = 0;     // pages per chunk, page bytes (single level: 1, B)
   uint32_t lgB = 0, lgP = 0;   // log2 of block and page bytes (record -> block by shifts)
+  bool dev_list = false;       // run_gpu_op: the sorted block list is in T.dlo (um_touch_batch_dev)
   bool host_prof = false;      // UM_HOST_PROFILE (diagnostic): host phases of a touch batch to stderr
   // UM_F_TIMING: event pairs around planning / transfer launches
   struct Span { cudaEvent_t a, b; int xfer; uint32_t seq; };
@@ -842,9 +843,10 @@ static um_status evict_ahead(um_arena* a, uint32_t seq) {
 static um_status run_gpu_op(um_arena* a, int touch) {
   uint64_t total = 0;
   bool anyw = false;
-  const bool dev = a->dev_iv;
+  const bool dev = a->dev_iv, devl = a->dev_list;
   a->dev_iv = false;
-  if (dev) {
+  a->dev_list = false;
+  if (dev || devl) {
     total = a->dev_total;
     anyw = a->dev_anyw;
   } else {
@@ -864,7 +866,7 @@ static um_status run_gpu_op(um_arena* a, int touch) {
   }
   const bool fl = a->fl_ready;
   a->fl_ready = false;
-  const uint32_t m = dev ? a->dev_m : (fl ? a->fl_m : (uint32_t)a->ivs.size());
+  const uint32_t m = dev ? a->dev_m : (fl ? a->fl_m : (devl ? 0u : (uint32_t)a->ivs.size()));
   uint64_t iv_off = 0, iv_bytes = 0;   // staged interval arrays (read by the app kernels)
   OpIv iv{};
   iv.m = m;
@@ -878,6 +880,9 @@ static um_status run_gpu_op(um_arena* a, int touch) {
     memcpy(a->stage.host + off, a->flist.data(), bytes);   // flist holds exactly `total` entries
     CK(a->stage.push(off, iv_bytes, a->ps));
     iv.blist = (const uint32_t*)(a->stage.dev + off);
+  } else if (devl) {
+    // the distinct block list made on the device from device-resident records (HBM)
+    iv.blist = a->T.dlo;
   } else if (dev) {
     // intervals made on the device by the intake kernels (already in HBM)
     iv.lo = a->T.dlo;
@@ -1409,6 +1414,44 @@ UM_API um_status um_touch_batch(um_arena* a, const um_access* acc, uint32_t n, v
     auto us = [](clk::duration d) { return std::chrono::duration<double, std::micro>(d).count(); };
     fprintf(stderr, "libum touch_batch n=%u: scan %.1f us, intervals %.1f us, stage + launch %.1f us\n", n,
             us(t1 - t0), us(t2 - t1), us(t3 - t2));
+  }
+  return hand_out(a, stream);
+}
+
+UM_API um_status um_touch_batch_dev(um_arena* a, const um_access* acc, uint32_t n, void* stream) {
+  ENTER(a);
+  if ((n && !acc) || ((uintptr_t)acc & 15) || a->ppc > 1) return UM_EINVAL;
+  using clk = std::chrono::steady_clock;
+  const auto t0 = clk::now();
+  um_status s = hand_in(a, stream);
+  if (s) return s;
+  // the list rewrites T.dlo, which in-flight application kernels of earlier sub-ops may
+  // read (their block list)
+  if (overlap_on(a) && (s = app_wait_all(a))) return s;
+  cudaEvent_t sp = span_open(a);
+  CK(launch_mark_acc(a->T, acc, n, a->lgB, a->ps));
+  CK(launch_list(a->T, (a->nblocks + 31) / 32, a->ps));
+  span_close(a, sp, 0);
+  a->n_launch += (n ? 1 : 0) + 1;
+  // the host needs the distinct-block count to number the sub-ops (and learns of a
+  // range error before anything that changes state is enqueued)
+  CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
+  CK(cudaStreamSynchronize(a->ps));
+  const auto t1 = clk::now();
+  if (a->hctl->iv_err) {
+    CK(cudaMemsetAsync(&a->T.ctl->iv_err, 0, sizeof(unsigned int), a->ps));
+    return UM_EINVAL;
+  }
+  a->dev_list = true;
+  a->dev_total = a->hctl->iv_d;
+  a->dev_anyw = a->hctl->iv_m != 0;
+  s = run_gpu_op(a, 1);
+  if (s) return s;
+  if (a->host_prof) {
+    const auto t2 = clk::now();
+    auto us = [](clk::duration d) { return std::chrono::duration<double, std::micro>(d).count(); };
+    fprintf(stderr, "libum touch_batch_dev n=%u: intake + count read-back %.1f us, launch %.1f us\n", n,
+            us(t1 - t0), us(t2 - t1));
   }
   return hand_out(a, stream);
 }

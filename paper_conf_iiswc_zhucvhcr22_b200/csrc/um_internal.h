@@ -34,7 +34,8 @@ struct Ctl {
   unsigned int vict_done;               // wide victim apply completion counter
   unsigned int need_acc;                // streaming classify: need-list slots taken so far
   unsigned int reach_tile;              // wide victim scan: first tile whose inclusive count >= k
-  unsigned int iv_m, iv_d;              // device intake: intervals produced, distinct blocks
+  unsigned int iv_m, iv_d;              // device intake: intervals produced (list form: write blocks), distinct blocks
+  unsigned int iv_err;                  // device records: a record outside the arena (read and cleared by the host)
   unsigned long long minkeep[2];        // wide victim scan: first kept ring position
   unsigned int k_want;                  // wide victim scan: victims wanted
   unsigned int need_cnt[2];             // streaming classify: need-list slots, by sub-op parity
@@ -226,5 +227,11 @@ struct MarkRec { uint32_t lo, cnt, w, pad; };   // one staged (split) record, in
 cudaError_t launch_mark(const Tables& T, const MarkRec* rec, uint32_t n, cudaStream_t s);
 cudaError_t launch_runs(const Tables& T, uint32_t w0, uint32_t w1, cudaStream_t s);
 cudaError_t launch_intake_clear(const Tables& T, uint32_t w0, uint32_t w1, cudaStream_t s);
+// Device-resident records (um_touch_batch_dev): mark n um_access records (16-byte
+// aligned, device-accessible) into the op bitmaps (range errors set ctl->iv_err); turn
+// the bitmap's nwords words into the sorted distinct block list dlo (bit 31 = write),
+// ctl->iv_d = blocks, ctl->iv_m = write blocks, and clear the bitmaps.
+cudaError_t launch_mark_acc(const Tables& T, const void* acc, uint32_t n, uint32_t lg, cudaStream_t s);
+cudaError_t launch_list(const Tables& T, uint32_t nwords, cudaStream_t s);
 
 }  // namespace um

@@ -2313,6 +2313,111 @@ __global__ void __launch_bounds__(256) k_intake_clear(Tables T, uint32_t w0, uin
 }
 
 // ------------------------------------------------------------------------------------
+// Device-resident access records (um_touch_batch_dev; SURVEY A0/A1 on the device): the
+// GPU's own fault buffer analogue.  The records never visit the host.
+//   k_mark_acc  one thread per 16-byte record: the API's range check (a record outside
+//               the arena sets ctl->iv_err; the host then rejects the op), blocks
+//               [off/B, (off+len-1)/B] ORed into obits (and wbits for a WRITE access)
+//   k_list      one ordered pass over the bitmap words: the set bits, ascending, become
+//               the distinct block list (bit 31 = write) that the LIST classify reads
+//               (dlo), ranked by block scan + decoupled look-back; every word is zeroed
+//               once read (the bitmaps are clean for the next batch); the last tile
+//               publishes the block count (ctl->iv_d) and the write count (ctl->iv_m)
+// ------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_mark_acc(Tables T, const ulonglong2* acc, uint32_t n, uint32_t lg) {
+  pdl_enter();
+  const unsigned long long arena = (unsigned long long)T.nblocks << lg;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const ulonglong2 r = acc[i];   // {off, len | kind << 32} (um_access)
+    const unsigned long long off = r.x, len = (uint32_t)r.y;
+    const bool w = ((uint32_t)(r.y >> 32) & 2u) != 0;   // UM_ACC_WRITE (include/um.h)
+    if (off > arena || len > arena - off) {
+      T.ctl->iv_err = 1u;
+      continue;
+    }
+    if (!len) continue;
+    const uint32_t lo = (uint32_t)(off >> lg), hi = (uint32_t)((off + len - 1) >> lg) + 1u;
+    for (uint32_t wd = lo >> 5; wd <= (hi - 1) >> 5; ++wd) {
+      const uint32_t a = max(lo, wd << 5) - (wd << 5), b = min(hi, (wd + 1) << 5) - (wd << 5);   // bits [a, b)
+      const uint32_t mask = (b - a == 32) ? FULL : (((1u << (b - a)) - 1u) << a);
+      atomicOr(&T.obits[wd], mask);
+      if (w) atomicOr(&T.wbits[wd], mask);
+    }
+  }
+}
+
+constexpr int kListTPB = 512, kListIPT = 8, kListTile = kListTPB * kListIPT;   // words per tile
+
+__global__ void __launch_bounds__(kListTPB) k_list(Tables T, uint32_t nwords) {
+  pdl_enter();
+  __shared__ unsigned long long s_sc[kListTPB / 32];
+  __shared__ unsigned long long s_excl;
+  const uint32_t tile = blockIdx.x, ntiles = gridDim.x;
+  const uint32_t first = tile * kListTile + threadIdx.x * kListIPT;   // this thread's words
+  uint32_t o[kListIPT], wb[kListIPT];
+  uint32_t nB = 0, nW = 0;
+  if (first + kListIPT <= nwords) {
+    // two 32-byte loads per bitmap (8 words, 32-byte aligned: nwords-sized arrays from
+    // 256-byte aligned carves)
+    const uint4* po = reinterpret_cast<const uint4*>(T.obits + first);
+    const uint4* pw = reinterpret_cast<const uint4*>(T.wbits + first);
+    const uint4 a0 = po[0], a1 = po[1], b0 = pw[0], b1 = pw[1];
+    o[0] = a0.x; o[1] = a0.y; o[2] = a0.z; o[3] = a0.w; o[4] = a1.x; o[5] = a1.y; o[6] = a1.z; o[7] = a1.w;
+    wb[0] = b0.x; wb[1] = b0.y; wb[2] = b0.z; wb[3] = b0.w; wb[4] = b1.x; wb[5] = b1.y; wb[6] = b1.z; wb[7] = b1.w;
+  } else {
+#pragma unroll
+    for (int q = 0; q < kListIPT; ++q) {
+      o[q] = first + q < nwords ? T.obits[first + q] : 0u;
+      wb[q] = first + q < nwords ? T.wbits[first + q] : 0u;
+    }
+  }
+#pragma unroll
+  for (int q = 0; q < kListIPT; ++q) {
+    wb[q] &= o[q];
+    nB += __popc(o[q]);
+    nW += __popc(wb[q]);
+  }
+  unsigned long long tot;
+  const unsigned long long pre = block_excl_scan<kListTPB>(pack2(nB, nW), tot, s_sc);
+  if (threadIdx.x < 32) {
+    const unsigned long long ex = lookback_warp(T, tile, tot);
+    if (threadIdx.x == 0) s_excl = ex;
+  }
+  __syncthreads();
+  uint32_t R = unpackA(s_excl) + unpackA(pre);
+#pragma unroll
+  for (int q = 0; q < kListIPT; ++q) {
+    uint32_t m = o[q];
+    const uint32_t base = (first + q) * 32u;
+    while (m) {
+      const int i = __ffs(m) - 1;
+      m &= m - 1;
+      T.dlo[R++] = (base + (uint32_t)i) | (((wb[q] >> i) & 1u) << 31);
+    }
+  }
+  // clear the words read (each is read by this thread only)
+  if (first + kListIPT <= nwords) {
+    uint4* po = reinterpret_cast<uint4*>(T.obits + first);
+    uint4* pw = reinterpret_cast<uint4*>(T.wbits + first);
+    const uint4 z = make_uint4(0u, 0u, 0u, 0u);
+    if (nB) { po[0] = z; po[1] = z; }
+    if (nW) { pw[0] = z; pw[1] = z; }
+  } else {
+    for (int q = 0; q < kListIPT; ++q)
+      if (first + q < nwords) {
+        T.obits[first + q] = 0u;
+        T.wbits[first + q] = 0u;
+      }
+  }
+  if (tile == ntiles - 1 && threadIdx.x == 0) {
+    const unsigned long long all = s_excl + tot;
+    T.ctl->iv_d = unpackA(all);
+    T.ctl->iv_m = unpackB(all);
+  }
+  scan_finish(T, ntiles);
+}
+
+// ------------------------------------------------------------------------------------
 // Harness: host writes (Listing 6 "Generate data, labels").
 // ------------------------------------------------------------------------------------
 // um_free (reading R9): blocks [lo, lo + n) return to U with no transfer.  A GPU frame
@@ -2710,6 +2815,22 @@ cudaError_t launch_intake_clear(const Tables& T, uint32_t w0, uint32_t w1, cudaS
   unsigned grid = ceil_div(w1 - w0, 256);
   if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
   cudaError_t e = launch_pdl(k_intake_clear, dim3(grid), dim3(256), 0, s, T, w0, w1);
+  if (e) return e;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_mark_acc(const Tables& T, const void* acc, uint32_t n, uint32_t lg, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  unsigned grid = ceil_div(n, 256);
+  if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
+  cudaError_t e = launch_pdl(k_mark_acc, dim3(grid), dim3(256), 0, s, T, (const ulonglong2*)acc, n, lg);
+  if (e) return e;
+  return cudaGetLastError();
+}
+
+cudaError_t launch_list(const Tables& T, uint32_t nwords, cudaStream_t s) {
+  unsigned nt = nwords ? ceil_div(nwords, kListTile) : 1;
+  cudaError_t e = launch_pdl(k_list, dim3(nt), dim3(kListTPB), 0, s, T, nwords);
   if (e) return e;
   return cudaGetLastError();
 }

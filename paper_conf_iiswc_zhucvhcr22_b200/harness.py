@@ -41,10 +41,27 @@ def iteration_bounds(trace) -> list:
     return [(i * per, (i + 1) * per) for i in range(it)]
 
 
-def _calls(trace, mode: str) -> list:
+def _dev_records(trace, device: int = 0) -> int:
+    """The trace's access records copied once into device memory (the GPU's fault buffer
+    analogue for um_touch_batch_dev); returns its device address."""
+    import torch
+    key = f"_acc_dev{device}"
+    t = trace.meta.get(key)
+    if t is None:
+        acc = np.ascontiguousarray(trace.acc).view(np.uint8).reshape(-1)
+        t = torch.empty(max(16, acc.size), dtype=torch.uint8, device=torch.device("cuda", device))
+        if acc.size:
+            t[:acc.size].copy_(torch.from_numpy(acc))
+        torch.cuda.synchronize(device)   # the arena's streams do not wait for torch's
+        trace.meta[key] = t
+    return t.data_ptr()
+
+
+def _calls(trace, mode: str, dev_records: bool = False) -> list:
     """The trace as a list of (libum function, args-after-arena) tuples, built once per
-    (trace, mode): the issue loop then only makes the ctypes calls."""
-    key = "_calls_" + mode
+    (trace, mode): the issue loop then only makes the ctypes calls.  dev_records: touch
+    batches go through um_touch_batch_dev with the records in device memory."""
+    key = "_calls_" + mode + ("_dev" if dev_records else "")
     cached = trace.meta.get(key)
     if cached is not None:
         return cached
@@ -52,11 +69,14 @@ def _calls(trace, mode: str) -> list:
     acc = np.ascontiguousarray(trace.acc)
     trace.meta["_acc_keepalive"] = acc
     base = acc.ctypes.data
+    dbase = _dev_records(trace) if dev_records else 0
     lazy = mode == "lazy"
     out = []
     for r in trace.ops.tolist():          # (op, flags, n, off, len) as python ints
         o, fl, n, off, ln = r
-        if o == tg.OP_TOUCH:
+        if o == tg.OP_TOUCH and dev_records:
+            out.append(("um_touch_batch_dev", L.um_touch_batch_dev, (dbase + 16 * off if n else None, n)))
+        elif o == tg.OP_TOUCH:
             out.append(("um_touch_batch", L.um_touch_batch, (base + 16 * off if n else None, n)))
         elif o == tg.OP_PREFETCH:
             out.append(("um_prefetch", L.um_prefetch, (off, ln, fl)))
@@ -77,11 +97,12 @@ def _calls(trace, mode: str) -> list:
     return out
 
 
-def issue(arena: um.Arena, trace, mode: str, start: int = 0, stop: int | None = None, stream=None) -> None:
+def issue(arena: um.Arena, trace, mode: str, start: int = 0, stop: int | None = None, stream=None,
+          dev_records: bool = False) -> None:
     """Issue ops[start:stop] of the trace through the C ABI (no synchronization)."""
     a = arena.handle
     s = arena.stream_ptr if stream is None else stream
-    calls = _calls(trace, mode)
+    calls = _calls(trace, mode, dev_records)
     stop = len(calls) if stop is None else stop
     for name, fn, args in calls[start:stop]:
         st = fn(a, *args, s)
@@ -133,14 +154,15 @@ class XLog:
         um.um_xlog_attach(self.arena.handle, None, 0)
 
 
-def run_trace(trace, mode: str, xlog: int = 0, **kw) -> dict:
+def run_trace(trace, mode: str, xlog: int = 0, dev_records: bool = False, **kw) -> dict:
     """Replay the whole trace on a fresh arena; xlog = capacity of a transfer log to
-    attach (its sorted records are returned under "xlog")."""
+    attach (its sorted records are returned under "xlog"); dev_records: touch batches
+    from device memory (um_touch_batch_dev)."""
     arena = make_arena(trace, mode, **kw)
     try:
         alloc_buffers(arena, trace)
         lg = XLog(arena, xlog) if xlog else None
-        issue(arena, trace, mode)
+        issue(arena, trace, mode, dev_records=dev_records)
         r = result(arena)
         if lg:
             r["xlog"] = lg.records()

@@ -74,6 +74,7 @@ def lib():
             "um_discard": [P, U64, U64, P],
             "um_discard_lazy": [P, U64, U64, P],
             "um_touch_batch": [P, P, U32, P],
+            "um_touch_batch_dev": [P, P, U32, P],
             "um_evict": [P, U64, P],
             "um_free": [P, U64, U64, P],
             "um_host_write": [P, U64, U64, P],
@@ -99,7 +100,7 @@ def lib():
 
 
 EXPORTS = ("um_workspace_size", "um_arena_create", "um_arena_destroy", "um_alloc", "um_prefetch", "um_discard",
-           "um_discard_lazy", "um_touch_batch", "um_evict", "um_free", "um_host_write", "um_block_table", "um_stream",
+           "um_discard_lazy", "um_touch_batch", "um_touch_batch_dev", "um_evict", "um_free", "um_host_write", "um_block_table", "um_stream",
            "um_join", "um_get_stats", "um_dump", "um_content_tags", "um_timing", "um_xlog_attach",
            "um_xlog_count", "um_page_masks", "um_strerror")
 
@@ -152,6 +153,11 @@ def um_touch_batch(a, acc: np.ndarray, stream=None) -> None:
     acc = np.ascontiguousarray(acc)
     assert acc.dtype.itemsize == 16
     _ck("um_touch_batch", lib().um_touch_batch(a, acc.ctypes.data if len(acc) else None, len(acc), stream))
+
+
+def um_touch_batch_dev(a, acc_ptr: int, n: int, stream=None) -> None:
+    """acc_ptr: device address of n 16-byte um_access records (16-byte aligned)."""
+    _ck("um_touch_batch_dev", lib().um_touch_batch_dev(a, acc_ptr or None, n, stream))
 
 
 def um_evict(a, nbytes: int, stream=None) -> None:

@@ -520,3 +520,79 @@ def test_reserve_rejected():
         um.Arena(64 << 10, 8 << 20, 4 << 20, reserve_blocks=65, host_pool_bytes=8 << 20)
     with pytest.raises(Exception):
         um.Arena(2 << 20, 64 << 20, 16 << 20, page_bytes=64 << 10, reserve_blocks=1, host_pool_bytes=64 << 20)
+
+
+# ------------------------------------------------------------------ device-resident records
+def _gpu_dev(trace, mode, overlap=False, **kw):
+    return _gpu(trace, mode, overlap=overlap, dev_records=True, **kw)
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_dev_records_small_random(seed, mode):
+    """um_touch_batch_dev: the batch's records read from device memory, range-checked,
+    expanded and deduplicated on the GPU (op bitmap -> sorted block list); bit-exact
+    against the oracle's touch (state, queue orders, counters, contents, transfer log)."""
+    rng = np.random.default_rng(300 + seed)
+    nb, nf = int(rng.integers(2, 40)), int(rng.integers(1, 8))
+    t = tg.gen_small(300 + seed, nblocks=nb, nframes=nf, n_ops=300, max_ranges=6, max_blocks=6)
+    assert_parity(t, mode, _gpu_dev(t, mode))
+
+
+@pytest.mark.parametrize("mode", ["base", "eager", "lazy"])
+def test_dev_records_c1(mode):
+    t = tg.gen_c1(6).slice_ops(0, 5000)
+    assert_parity(t, mode, _gpu_dev(t, mode))
+    assert_parity(t, mode, _gpu_dev(t, mode, overlap=True), overlap=True)
+
+
+@pytest.mark.parametrize("mode", ["eager", "lazy"])
+def test_dev_records_unsorted_and_sparse(mode):
+    """Unsorted overlapping batches with mixed W flags (1-1500 records), and sparse sorted
+    batches spanning many tiles and several sub-ops (the state microbench's shape), over
+    arenas whose bitmap ends in a ragged word tile."""
+    t = tg.gen_random(3, block_bytes=64 << 10, arena_bytes=(32 << 20) + (37 << 16), budget_bytes=4 << 20,
+                      n_ops=400, max_ranges=200, max_blocks=8, zipf_s=0.8)
+    assert_parity(t, mode, _gpu_dev(t, mode))
+    t = tg.gen_random(7, block_bytes=4 << 10, arena_bytes=64 << 20, budget_bytes=24 << 20, n_ops=120,
+                      max_ranges=1500, max_blocks=32, zipf_s=0.6)
+    assert_parity(t, mode, _gpu_dev(t, mode))
+    t = tg.gen_sparse(2)
+    assert_parity(t, mode, _gpu_dev(t, mode))
+    assert_parity(t, mode, _gpu_dev(t, mode, overlap=True), overlap=True)
+
+
+def test_dev_records_range_error_changes_nothing():
+    """A device record outside the arena: UM_EINVAL, nothing changed, and the next batch
+    (whose bitmap words the rejected one had marked) is serviced exactly."""
+    import torch
+    from paper_conf_iiswc_zhucvhcr22_b200 import um
+    B, nb, nf = 64 << 10, 100, 20
+    a = um.Arena(B, nb * B, nf * B, flags=um.UM_F_CHECK, host_pool_bytes=nb * B)
+    try:
+        h = a.handle
+        def dev(recs):
+            arr = np.zeros(len(recs), dtype=tg.ACC_DTYPE)
+            for i, (o, l, k) in enumerate(recs):
+                arr[i] = (o, l, k)
+            t = torch.from_numpy(arr.view(np.uint8)).cuda()
+            torch.cuda.synchronize()
+            return t
+        ok = dev([(0, 3 * B, tg.ACC_WRITE), (10 * B, B, tg.ACC_READ)])
+        um.um_touch_batch_dev(h, ok.data_ptr(), 2)
+        before = um.um_dump(h, nb, nf), um.um_get_stats(h)
+        bad = dev([(50 * B, B, tg.ACC_READ), (nb * B - 10, 11, tg.ACC_READ)])
+        with pytest.raises(um.UmError) as e:
+            um.um_touch_batch_dev(h, bad.data_ptr(), 2)
+        assert e.value.status == um.UM_EINVAL
+        after = um.um_dump(h, nb, nf), um.um_get_stats(h)
+        assert np.array_equal(before[0]["st"], after[0]["st"]) and before[1] == after[1]
+        nxt = dev([(60 * B, 2 * B, tg.ACC_READ)])
+        um.um_touch_batch_dev(h, nxt.data_ptr(), 1)
+        d = um.um_dump(h, nb, nf)
+        st = np.asarray(d["st"])
+        assert list(np.nonzero(st == 3)[0]) == [0, 1, 2, 10, 60, 61]   # block 50 was never marked in
+        with pytest.raises(um.UmError):
+            um.um_touch_batch_dev(h, ok.data_ptr() + 8, 1)                # not 16-byte aligned
+    finally:
+        a.close()
