@@ -670,6 +670,64 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
         del ws
 
 
+def state_dev_records(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
+    """The state microbench's first touch (2^21 distinct random blocks, all U) with the
+    access records resident in HBM (the GPU's fault buffer analogue) through
+    um_touch_batch_dev: the GPU range-checks, expands and deduplicates them (k_mark_acc ->
+    op bitmap -> k_list), the host reads back only the block count, then the same LIST
+    classify runs.  Returns the intake span (k_mark_acc + k_list, behind a device sleep:
+    device time only), the host time of the whole API call on an idle device, and the
+    block count check.  Spans come from the library's own events (UM_SPAN_LOG)."""
+    import tempfile
+    import numpy as np
+    import tracegen as tg
+    B = block
+    nb = arena_bytes // B
+    n = 1 << 21
+    rng = np.random.default_rng(seed)
+    acc = np.zeros(n, dtype=tg.ACC_DTYPE)
+    acc["off"] = np.sort(rng.choice(nb, size=n, replace=False)).astype(np.uint64) * B
+    acc["len"] = B
+    acc["kind"] = tg.ACC_READ
+    dacc = torch.from_numpy(acc.view(np.uint8).reshape(-1)).to(mem.frames.device)
+    out = {}
+    for gated in (True, False):
+        cfg = mem.config(arena_bytes, budget, um.UM_F_TIMING)
+        cfg.block_bytes = B
+        ws_bytes = um.um_workspace_size(cfg)
+        ws = torch.empty(ws_bytes, dtype=torch.uint8, device=mem.frames.device)
+        torch.cuda.synchronize(mem.frames.device)
+        cfg.workspace, cfg.workspace_bytes = ws.data_ptr(), ws_bytes
+        h = um.um_arena_create(cfg)
+        fd, log = tempfile.mkstemp(suffix=".spans")
+        os.close(fd)
+        try:
+            ps = torch.cuda.ExternalStream(um.um_stream(h))
+            um.um_timing(h, reset=True)
+            if gated:
+                with torch.cuda.stream(ps):
+                    torch.cuda._sleep(100_000_000)
+            h0 = time.perf_counter()
+            um.um_touch_batch_dev(h, dacc.data_ptr(), n)
+            host_us = (time.perf_counter() - h0) * 1e6
+            os.environ["UM_SPAN_LOG"] = log
+            um.um_timing(h, reset=True)
+            del os.environ["UM_SPAN_LOG"]
+            spans = [(int(a), int(x), float(m)) for a, x, m in (ln.split() for ln in open(log))]
+            st = um.um_get_stats(h)
+            assert st["zf_bytes"] == n * B and st["faults"] == n
+            if gated:
+                out["intake_ms"] = spans[0][2]
+            else:
+                out["host_api_us"] = host_us
+                out["classify_span_ms_ungated"] = spans[1][2]
+        finally:
+            os.unlink(log)
+            um.um_arena_destroy(h)
+            del ws
+    return out
+
+
 def state_runs(torch, um, mem, budget, arena_bytes):
     """State microbench on fresh arenas over the same memory: one warm-up (first-touch
     costs of the workspace pages and kernel images), then three; per op the run with the
@@ -684,6 +742,28 @@ def state_runs(torch, um, mem, budget, arena_bytes):
     for k in ("empty_kernel_span_us", "zero_fill_gbs"):
         state[k] = sorted(r[k] for r in runs)[1]
     state["reps"] = "median of three runs (seeds 0, 2, 3) after one warm-up run"
+    # the same first touch from device-resident records (um_touch_batch_dev): the device
+    # path = intake (measured here) + the same LIST classify (the touch above)
+    state_dev_records(torch, um, mem, budget, arena_bytes, seed=1)
+    dr = [state_dev_records(torch, um, mem, budget, arena_bytes, seed=s) for s in (0, 2, 3)]
+    n, nb = 1 << 21, state["nblocks"]
+    intake_ms = sorted(d["intake_ms"] for d in dr)[1]
+    cls = state["touch_2^21_random"]
+    by = cls["algorithmic_bytes"] + 16 * n + 3 * (nb // 8) + 4 * n   # records, bitmap RMW + read of wbits, list write
+    ms = intake_ms + cls["ms"]
+    peak = cls["peak"]
+    state["touch_2^21_device_records"] = {
+        "kernel": "k_mark_acc + k_list (device intake) + k_classify", "bound": "hbm",
+        "achieved": by / (ms / 1e3) / 1e9, "peak": peak, "unit": "GB/s", "frac": by / (ms / 1e3) / 1e9 / peak,
+        "algorithmic_bytes": by, "ms": ms, "intake_ms": intake_ms, "classify_ms": cls["ms"],
+        "intake_ms_runs": [d["intake_ms"] for d in dr],
+        "host_api_us": sorted(d["host_api_us"] for d in dr)[1],
+        "host_api_us_runs": [d["host_api_us"] for d in dr],
+        "classify_span_ms_ungated": sorted(d["classify_span_ms_ungated"] for d in dr)[1],
+        "note": "records resident in HBM (16 B each); intake span behind a device sleep (device time); "
+                "classify = the LIST classify of touch_2^21_random (same list); host_api_us = the whole "
+                "API call on an idle device (intake launch, block-count read-back, classify and zero-fill "
+                "enqueue), against touch_2^21_random's host_api_us (host scan of the records)"}
     return state
 
 
