@@ -42,6 +42,7 @@ struct Ctl {
   unsigned int k0_take, k0_pend;        // wide victim scan with k = 0: frames to take, pending flag
   unsigned long long vs_combo;          // wide victim scan: (candidates of finished tiles << 32) | next ticket
   unsigned int first_skip;              // wide victim scan: first ticket not examined
+  unsigned int vs_fin;                  // wide victim scan: tiles finished (ticket pacing)
   unsigned int vt_reach;                // wide victim scan: passes in the apply work table (vpass)
   unsigned int pc_done;                 // k_plan_commit completion ticket (host read-back flag)
   unsigned long long xlog_n;            // transfer log: records appended (may exceed the capacity)

@@ -335,6 +335,7 @@ __global__ void k_init(Tables T, int nh) {
     c->need_cnt[0] = c->need_cnt[1] = 0;
     c->k0_take = c->k0_pend = 0;
     c->vs_combo = 0;
+    c->vs_fin = 0;
     c->first_skip = ~0u;
     c->vt_reach = 0;
   }
@@ -1169,9 +1170,36 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
       // no fence: the records are read by the finalizing CTA after the completion
       // counter below (fenced), the scratch slice by k_victims_apply (next launch)
       // without prefetch the next ticket comes with this tile's count (one atomic)
-      if (!prefetch) nxt = atomicAdd(&c->vs_combo, ((unsigned long long)cnt << 32) | 1ull) + ((unsigned long long)cnt << 32);
-      else if (cnt) atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32);
-      s_tile = gridDim.x + (uint32_t)nxt;
+      if (prefetch) {
+        if (cnt) atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32);
+      } else {
+        // Paced tickets: a CTA takes the next tile only while the tiles already handed
+        // out are not expected to hold the k-th candidate (estimate: the candidate
+        // density of the finished tiles); otherwise it waits until they finish (every
+        // grid CTA is resident, and tiles in flight depend on nothing) and takes a
+        // ticket then only if the count still falls short.  Without the pacing, CTAs
+        // that finish early take tickets before the wave's counts are in, about
+        // doubling the tiles read past the k-th candidate.
+        unsigned long long v = atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32) + ((unsigned long long)cnt << 32);
+        unsigned int fin = atomicAdd(&c->vs_fin, 1u) + 1u;
+        while (true) {
+          const unsigned long long tot = v >> 32;
+          const unsigned int issued = (unsigned int)min((unsigned long long)ntiles, (unsigned long long)gridDim.x + (uint32_t)v);
+          const unsigned int inflight = issued > fin ? issued - fin : 0u;
+          if (tot >= k || issued >= ntiles && inflight == 0) {
+            nxt = v | 0xffffffffull;   // stop: enough candidates, or every tile handed out
+            break;
+          }
+          if (!inflight || tot + (unsigned long long)inflight * tot / fin < k) {
+            nxt = atomicAdd(&c->vs_combo, 1ull);
+            break;
+          }
+          __nanosleep(128);
+          v = *(volatile unsigned long long*)&c->vs_combo;
+          fin = *(volatile unsigned int*)&c->vs_fin;
+        }
+      }
+      s_tile = (uint32_t)nxt == 0xffffffffu ? ntiles : gridDim.x + (uint32_t)nxt;
       s_skip = (uint32_t)(nxt >> 32);
 #ifdef UM_VS_TRACE
       if (tr_tiles == 1 && blockIdx.x < 1500) VS_TR(4 * blockIdx.x + 3, vs_now());
@@ -1200,7 +1228,10 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
   __shared__ uint32_t s_reach;
   __shared__ unsigned long long s_kd, s_ku;
   const uint32_t fs = *(volatile uint32_t*)&c->first_skip;
-  const uint32_t E = min(ntiles, fs);   // tiles [0, E) were all examined
+  // tiles [0, E) were all examined: below the first skipped ticket and below the first
+  // tile never handed out (paced tickets may stop short of both)
+  const unsigned long long handed = (unsigned long long)gridDim.x + (uint32_t)*(volatile unsigned long long*)&c->vs_combo;
+  const uint32_t E = (uint32_t)min(min((unsigned long long)ntiles, (unsigned long long)fs), handed);
   if (threadIdx.x == 0) {
     s_reach = ~0u;
     s_kd = s_ku = ~0ull;
@@ -1318,6 +1349,7 @@ __global__ void __launch_bounds__(kVsTPB, 4) k_victims_scan(Tables T, uint32_t s
     }
     c->scan_done = 0;
     c->vs_combo = 0;
+    c->vs_fin = 0;
     c->first_skip = ~0u;
 #ifdef UM_VS_TRACE
     VS_TR(8001, vs_now());
@@ -2324,91 +2356,106 @@ __global__ void __launch_bounds__(256) k_intake_clear(Tables T, uint32_t w0, uin
 //               once read (the bitmaps are clean for the next batch); the last tile
 //               publishes the block count (ctl->iv_d) and the write count (ctl->iv_m)
 // ------------------------------------------------------------------------------------
+constexpr int kMarkIPT = 4;   // records per thread per pass, all loads in flight
+
 __global__ void __launch_bounds__(256) k_mark_acc(Tables T, const ulonglong2* acc, uint32_t n, uint32_t lg) {
   pdl_enter();
   const unsigned long long arena = (unsigned long long)T.nblocks << lg;
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    const ulonglong2 r = acc[i];   // {off, len | kind << 32} (um_access)
-    const unsigned long long off = r.x, len = (uint32_t)r.y;
-    const bool w = ((uint32_t)(r.y >> 32) & 2u) != 0;   // UM_ACC_WRITE (include/um.h)
-    if (off > arena || len > arena - off) {
-      T.ctl->iv_err = 1u;
-      continue;
+  const int lane = threadIdx.x & 31;
+  const uint32_t step = gridDim.x * blockDim.x * kMarkIPT;
+  // warp-uniform trip count: every lane takes part in the shuffles below
+  for (uint32_t i0 = blockIdx.x * blockDim.x * kMarkIPT; i0 < n; i0 += step) {
+    ulonglong2 r[kMarkIPT];
+#pragma unroll
+    for (int q = 0; q < kMarkIPT; ++q) {
+      const uint32_t i = i0 + q * blockDim.x + threadIdx.x;
+      r[q] = i < n ? acc[i] : make_ulonglong2(0ull, 0ull);   // {off, len | kind << 32} (um_access); len 0 = nothing
     }
-    if (!len) continue;
-    const uint32_t lo = (uint32_t)(off >> lg), hi = (uint32_t)((off + len - 1) >> lg) + 1u;
-    for (uint32_t wd = lo >> 5; wd <= (hi - 1) >> 5; ++wd) {
-      const uint32_t a = max(lo, wd << 5) - (wd << 5), b = min(hi, (wd + 1) << 5) - (wd << 5);   // bits [a, b)
-      const uint32_t mask = (b - a == 32) ? FULL : (((1u << (b - a)) - 1u) << a);
-      atomicOr(&T.obits[wd], mask);
-      if (w) atomicOr(&T.wbits[wd], mask);
+#pragma unroll
+    for (int q = 0; q < kMarkIPT; ++q) {
+      const unsigned long long off = r[q].x, len = (uint32_t)r[q].y;
+      const bool w = ((uint32_t)(r[q].y >> 32) & 2u) != 0;   // UM_ACC_WRITE (include/um.h)
+      uint32_t wd = UM_NONE, m = 0u, mw = 0u, lo = 0u, hi = 0u;
+      bool multi = false;
+      if (off > arena || len > arena - off) {
+        T.ctl->iv_err = 1u;
+      } else if (len) {
+        lo = (uint32_t)(off >> lg);
+        hi = (uint32_t)((off + len - 1) >> lg) + 1u;
+        if ((lo >> 5) == ((hi - 1) >> 5)) {
+          wd = lo >> 5;
+          const uint32_t a = lo & 31u, b = a + (hi - lo);
+          m = (b - a == 32) ? FULL : (((1u << (b - a)) - 1u) << a);
+          mw = w ? m : 0u;
+        } else {
+          multi = true;
+        }
+      }
+      // records within one bitmap word: neighbouring lanes on the same word (a sorted
+      // fault batch puts ~16 records in a word) OR their bits together by a segmented
+      // suffix scan, and the first lane of each run issues the atomics (equal words that
+      // are not adjacent just issue one atomic per run: OR is idempotent)
+      uint32_t mo = m, mwo = mw;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t wo = __shfl_down_sync(FULL, wd, o);
+        const uint32_t x = __shfl_down_sync(FULL, mo, o), xw = __shfl_down_sync(FULL, mwo, o);
+        if (lane + o < 32 && wo == wd) {
+          mo |= x;
+          mwo |= xw;
+        }
+      }
+      const uint32_t prev = __shfl_up_sync(FULL, wd, 1);
+      if (wd != UM_NONE && (lane == 0 || prev != wd)) {
+        atomicOr(&T.obits[wd], mo);
+        if (mwo) atomicOr(&T.wbits[wd], mwo);
+      }
+      if (multi) {
+        for (uint32_t x = lo >> 5; x <= (hi - 1) >> 5; ++x) {
+          const uint32_t a = max(lo, x << 5) - (x << 5), b = min(hi, (x + 1) << 5) - (x << 5);   // bits [a, b)
+          const uint32_t mask = (b - a == 32) ? FULL : (((1u << (b - a)) - 1u) << a);
+          atomicOr(&T.obits[x], mask);
+          if (w) atomicOr(&T.wbits[x], mask);
+        }
+      }
     }
   }
 }
 
-constexpr int kListTPB = 512, kListIPT = 8, kListTile = kListTPB * kListIPT;   // words per tile
+// one bitmap word per thread; a tile's list entries are staged in shared memory (<= 32
+// per word) and written out coalesced
+constexpr int kListTPB = 256, kListTile = kListTPB;   // words per tile
 
 __global__ void __launch_bounds__(kListTPB) k_list(Tables T, uint32_t nwords) {
   pdl_enter();
   __shared__ unsigned long long s_sc[kListTPB / 32];
   __shared__ unsigned long long s_excl;
+  __shared__ uint32_t s_ent[kListTile * 32];
   const uint32_t tile = blockIdx.x, ntiles = gridDim.x;
-  const uint32_t first = tile * kListTile + threadIdx.x * kListIPT;   // this thread's words
-  uint32_t o[kListIPT], wb[kListIPT];
-  uint32_t nB = 0, nW = 0;
-  if (first + kListIPT <= nwords) {
-    // two 32-byte loads per bitmap (8 words, 32-byte aligned: nwords-sized arrays from
-    // 256-byte aligned carves)
-    const uint4* po = reinterpret_cast<const uint4*>(T.obits + first);
-    const uint4* pw = reinterpret_cast<const uint4*>(T.wbits + first);
-    const uint4 a0 = po[0], a1 = po[1], b0 = pw[0], b1 = pw[1];
-    o[0] = a0.x; o[1] = a0.y; o[2] = a0.z; o[3] = a0.w; o[4] = a1.x; o[5] = a1.y; o[6] = a1.z; o[7] = a1.w;
-    wb[0] = b0.x; wb[1] = b0.y; wb[2] = b0.z; wb[3] = b0.w; wb[4] = b1.x; wb[5] = b1.y; wb[6] = b1.z; wb[7] = b1.w;
-  } else {
-#pragma unroll
-    for (int q = 0; q < kListIPT; ++q) {
-      o[q] = first + q < nwords ? T.obits[first + q] : 0u;
-      wb[q] = first + q < nwords ? T.wbits[first + q] : 0u;
-    }
-  }
-#pragma unroll
-  for (int q = 0; q < kListIPT; ++q) {
-    wb[q] &= o[q];
-    nB += __popc(o[q]);
-    nW += __popc(wb[q]);
-  }
+  const uint32_t wd = tile * kListTile + threadIdx.x;
+  const uint32_t o = wd < nwords ? T.obits[wd] : 0u;
+  const uint32_t wb = (wd < nwords ? T.wbits[wd] : 0u) & o;
+  const uint32_t nB = __popc(o), nW = __popc(wb);
   unsigned long long tot;
   const unsigned long long pre = block_excl_scan<kListTPB>(pack2(nB, nW), tot, s_sc);
   if (threadIdx.x < 32) {
     const unsigned long long ex = lookback_warp(T, tile, tot);
     if (threadIdx.x == 0) s_excl = ex;
   }
-  __syncthreads();
-  uint32_t R = unpackA(s_excl) + unpackA(pre);
-#pragma unroll
-  for (int q = 0; q < kListIPT; ++q) {
-    uint32_t m = o[q];
-    const uint32_t base = (first + q) * 32u;
-    while (m) {
-      const int i = __ffs(m) - 1;
-      m &= m - 1;
-      T.dlo[R++] = (base + (uint32_t)i) | (((wb[q] >> i) & 1u) << 31);
-    }
+  uint32_t r = unpackA(pre), m = o;
+  while (m) {
+    const int i = __ffs(m) - 1;
+    m &= m - 1;
+    s_ent[r++] = (wd * 32u + (uint32_t)i) | (((wb >> i) & 1u) << 31);
   }
   // clear the words read (each is read by this thread only)
-  if (first + kListIPT <= nwords) {
-    uint4* po = reinterpret_cast<uint4*>(T.obits + first);
-    uint4* pw = reinterpret_cast<uint4*>(T.wbits + first);
-    const uint4 z = make_uint4(0u, 0u, 0u, 0u);
-    if (nB) { po[0] = z; po[1] = z; }
-    if (nW) { pw[0] = z; pw[1] = z; }
-  } else {
-    for (int q = 0; q < kListIPT; ++q)
-      if (first + q < nwords) {
-        T.obits[first + q] = 0u;
-        T.wbits[first + q] = 0u;
-      }
+  if (wd < nwords) {
+    if (o) T.obits[wd] = 0u;
+    if (wb) T.wbits[wd] = 0u;   // write bits are only ever set with their obits bit
   }
+  __syncthreads();
+  const uint32_t base = unpackA(s_excl), cnt = unpackA(tot);
+  for (uint32_t k = threadIdx.x; k < cnt; k += kListTPB) T.dlo[base + k] = s_ent[k];
   if (tile == ntiles - 1 && threadIdx.x == 0) {
     const unsigned long long all = s_excl + tot;
     T.ctl->iv_d = unpackA(all);
@@ -2821,7 +2868,7 @@ cudaError_t launch_intake_clear(const Tables& T, uint32_t w0, uint32_t w1, cudaS
 
 cudaError_t launch_mark_acc(const Tables& T, const void* acc, uint32_t n, uint32_t lg, cudaStream_t s) {
   if (!n) return cudaSuccess;
-  unsigned grid = ceil_div(n, 256);
+  unsigned grid = ceil_div(n, 256 * kMarkIPT);
   if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
   cudaError_t e = launch_pdl(k_mark_acc, dim3(grid), dim3(256), 0, s, T, (const ulonglong2*)acc, n, lg);
   if (e) return e;
