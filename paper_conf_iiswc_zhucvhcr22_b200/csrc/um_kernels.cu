@@ -2391,22 +2391,12 @@ __global__ void __launch_bounds__(256) k_mark_acc(Tables T, const ulonglong2* ac
           multi = true;
         }
       }
-      // records within one bitmap word: neighbouring lanes on the same word (a sorted
-      // fault batch puts ~16 records in a word) OR their bits together by a segmented
-      // suffix scan, and the first lane of each run issues the atomics (equal words that
-      // are not adjacent just issue one atomic per run: OR is idempotent)
-      uint32_t mo = m, mwo = mw;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t wo = __shfl_down_sync(FULL, wd, o);
-        const uint32_t x = __shfl_down_sync(FULL, mo, o), xw = __shfl_down_sync(FULL, mwo, o);
-        if (lane + o < 32 && wo == wd) {
-          mo |= x;
-          mwo |= xw;
-        }
-      }
-      const uint32_t prev = __shfl_up_sync(FULL, wd, 1);
-      if (wd != UM_NONE && (lane == 0 || prev != wd)) {
+      // records within one bitmap word (a sorted fault batch puts ~16 records in a
+      // word): the lanes on the same word OR their bits together (match + redux within
+      // each group) and the group's lowest lane issues the atomics
+      const unsigned peers = __match_any_sync(FULL, wd);
+      const uint32_t mo = __reduce_or_sync(peers, m), mwo = __reduce_or_sync(peers, mw);
+      if (wd != UM_NONE && lane == __ffs(peers) - 1) {
         atomicOr(&T.obits[wd], mo);
         if (mwo) atomicOr(&T.wbits[wd], mwo);
       }
@@ -2422,15 +2412,17 @@ __global__ void __launch_bounds__(256) k_mark_acc(Tables T, const ulonglong2* ac
   }
 }
 
-// one bitmap word per thread; a tile's list entries are staged in shared memory (<= 32
-// per word) and written out coalesced
-constexpr int kListTPB = 256, kListTile = kListTPB;   // words per tile
+// one bitmap word per thread, 1024 words per tile (few tiles: a short look-back); a
+// tile's list entries are staged in shared memory (<= 32 per word, 128 KB) and written
+// out coalesced
+constexpr int kListTPB = 1024, kListTile = kListTPB;   // words per tile
+constexpr int kListSmem = kListTile * 32 * 4;
 
 __global__ void __launch_bounds__(kListTPB) k_list(Tables T, uint32_t nwords) {
   pdl_enter();
   __shared__ unsigned long long s_sc[kListTPB / 32];
   __shared__ unsigned long long s_excl;
-  __shared__ uint32_t s_ent[kListTile * 32];
+  extern __shared__ uint32_t s_ent[];
   const uint32_t tile = blockIdx.x, ntiles = gridDim.x;
   const uint32_t wd = tile * kListTile + threadIdx.x;
   const uint32_t o = wd < nwords ? T.obits[wd] : 0u;
@@ -2644,6 +2636,8 @@ cudaError_t setup_kernels() {
   if (e) return e;
   if (g_dir_occ < 1) g_dir_occ = 1;
   if (const char* v = getenv("UM_DIR_OCC")) g_dir_occ = std::max(1, atoi(v));
+  e = cudaFuncSetAttribute(k_list, cudaFuncAttributeMaxDynamicSharedMemorySize, kListSmem);
+  if (e) return e;
   int smem = (int)(kXferChunk * (1 + 2 * kXferStages));
   return cudaFuncSetAttribute(k_service, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
 }
@@ -2877,7 +2871,7 @@ cudaError_t launch_mark_acc(const Tables& T, const void* acc, uint32_t n, uint32
 
 cudaError_t launch_list(const Tables& T, uint32_t nwords, cudaStream_t s) {
   unsigned nt = nwords ? ceil_div(nwords, kListTile) : 1;
-  cudaError_t e = launch_pdl(k_list, dim3(nt), dim3(kListTPB), 0, s, T, nwords);
+  cudaError_t e = launch_pdl(k_list, dim3(nt), dim3(kListTPB), (size_t)kListSmem, s, T, nwords);
   if (e) return e;
   return cudaGetLastError();
 }
