@@ -2356,51 +2356,46 @@ __global__ void __launch_bounds__(256) k_intake_clear(Tables T, uint32_t w0, uin
 //               once read (the bitmaps are clean for the next batch); the last tile
 //               publishes the block count (ctl->iv_d) and the write count (ctl->iv_m)
 // ------------------------------------------------------------------------------------
-constexpr int kMarkIPT = 4;   // records per thread per pass, all loads in flight
+constexpr int kMarkIPT = 8;   // consecutive records per thread, all loads in flight
 
+// Each thread takes kMarkIPT CONSECUTIVE records: in a sorted fault batch they fall in
+// one or two bitmap words, so the thread ORs their bits in a register and issues one
+// atomic per word it leaves (no cross-lane work; the ALU cost per record is a few
+// integer ops).  Unsorted records just flush more often.
 __global__ void __launch_bounds__(256) k_mark_acc(Tables T, const ulonglong2* acc, uint32_t n, uint32_t lg) {
   pdl_enter();
   const unsigned long long arena = (unsigned long long)T.nblocks << lg;
-  const int lane = threadIdx.x & 31;
-  const uint32_t step = gridDim.x * blockDim.x * kMarkIPT;
-  // warp-uniform trip count: every lane takes part in the shuffles below
-  for (uint32_t i0 = blockIdx.x * blockDim.x * kMarkIPT; i0 < n; i0 += step) {
+  const uint32_t stride = gridDim.x * blockDim.x * kMarkIPT;
+  for (uint32_t i0 = (blockIdx.x * blockDim.x + threadIdx.x) * kMarkIPT; i0 < n; i0 += stride) {
     ulonglong2 r[kMarkIPT];
 #pragma unroll
-    for (int q = 0; q < kMarkIPT; ++q) {
-      const uint32_t i = i0 + q * blockDim.x + threadIdx.x;
-      r[q] = i < n ? acc[i] : make_ulonglong2(0ull, 0ull);   // {off, len | kind << 32} (um_access); len 0 = nothing
-    }
+    for (int q = 0; q < kMarkIPT; ++q)   // {off, len | kind << 32} (um_access); len 0 = nothing
+      r[q] = i0 + q < n ? __ldg(acc + i0 + q) : make_ulonglong2(0ull, 0ull);
+    uint32_t cw = UM_NONE, cm = 0u, cmw = 0u;   // the word being accumulated
 #pragma unroll
     for (int q = 0; q < kMarkIPT; ++q) {
       const unsigned long long off = r[q].x, len = (uint32_t)r[q].y;
       const bool w = ((uint32_t)(r[q].y >> 32) & 2u) != 0;   // UM_ACC_WRITE (include/um.h)
-      uint32_t wd = UM_NONE, m = 0u, mw = 0u, lo = 0u, hi = 0u;
-      bool multi = false;
       if (off > arena || len > arena - off) {
         T.ctl->iv_err = 1u;
-      } else if (len) {
-        lo = (uint32_t)(off >> lg);
-        hi = (uint32_t)((off + len - 1) >> lg) + 1u;
-        if ((lo >> 5) == ((hi - 1) >> 5)) {
-          wd = lo >> 5;
-          const uint32_t a = lo & 31u, b = a + (hi - lo);
-          m = (b - a == 32) ? FULL : (((1u << (b - a)) - 1u) << a);
-          mw = w ? m : 0u;
-        } else {
-          multi = true;
+        continue;
+      }
+      if (!len) continue;
+      const uint32_t lo = (uint32_t)(off >> lg), hi = (uint32_t)((off + len - 1) >> lg) + 1u;
+      if ((lo >> 5) == ((hi - 1) >> 5)) {
+        const uint32_t wd = lo >> 5, a = lo & 31u, c = hi - lo;
+        const uint32_t m = (c == 32) ? FULL : (((1u << c) - 1u) << a);
+        if (wd != cw) {
+          if (cw != UM_NONE) {
+            atomicOr(&T.obits[cw], cm);
+            if (cmw) atomicOr(&T.wbits[cw], cmw);
+          }
+          cw = wd;
+          cm = cmw = 0u;
         }
-      }
-      // records within one bitmap word (a sorted fault batch puts ~16 records in a
-      // word): the lanes on the same word OR their bits together (match + redux within
-      // each group) and the group's lowest lane issues the atomics
-      const unsigned peers = __match_any_sync(FULL, wd);
-      const uint32_t mo = __reduce_or_sync(peers, m), mwo = __reduce_or_sync(peers, mw);
-      if (wd != UM_NONE && lane == __ffs(peers) - 1) {
-        atomicOr(&T.obits[wd], mo);
-        if (mwo) atomicOr(&T.wbits[wd], mwo);
-      }
-      if (multi) {
+        cm |= m;
+        if (w) cmw |= m;
+      } else {
         for (uint32_t x = lo >> 5; x <= (hi - 1) >> 5; ++x) {
           const uint32_t a = max(lo, x << 5) - (x << 5), b = min(hi, (x + 1) << 5) - (x << 5);   // bits [a, b)
           const uint32_t mask = (b - a == 32) ? FULL : (((1u << (b - a)) - 1u) << a);
@@ -2408,6 +2403,10 @@ __global__ void __launch_bounds__(256) k_mark_acc(Tables T, const ulonglong2* ac
           if (w) atomicOr(&T.wbits[x], mask);
         }
       }
+    }
+    if (cw != UM_NONE) {
+      atomicOr(&T.obits[cw], cm);
+      if (cmw) atomicOr(&T.wbits[cw], cmw);
     }
   }
 }
