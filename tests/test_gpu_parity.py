@@ -596,3 +596,44 @@ def test_dev_records_range_error_changes_nothing():
             um.um_touch_batch_dev(h, ok.data_ptr() + 8, 1)                # not 16-byte aligned
     finally:
         a.close()
+
+
+# ------------------------------------------------------------------ the state microbench's op sequence
+def _state_micro_parity(t, dev_records, pool=2 << 30):
+    g = _gpu(t, "eager", host_pool_bytes=pool, xlog=False, dev_records=dev_records)
+    assert_parity(t, "eager", g)
+    return g
+
+
+@pytest.mark.parametrize("dev_records", [False, True])
+def test_state_micro_medium(dev_records):
+    """bench.py's state microbench sequence at 1/4 size (1 M blocks of 4 KiB, 2/3 of them
+    framed, 2^19-record touches): host fault-list and device-record intake, the wide
+    victim scan with paced tickets; bit-exact against the oracle."""
+    nb = 1 << 20
+    t = tg.gen_state_micro(5, block_bytes=4 << 10, arena_bytes=nb * (4 << 10), budget_bytes=(2 * nb // 3) * (4 << 10),
+                           n=1 << 19)
+    g = _state_micro_parity(t, dev_records, pool=64 << 20)
+    assert g["stats"]["evictions"] > 8192
+
+
+@pytest.mark.parametrize("dev_records", [False, True])
+def test_state_micro_full_size(dev_records):
+    """The state microbench at its full size and launch configuration (SURVEY §8(d) last
+    row: 64 KiB blocks over the bench's 170 GiB budget at 1.5x -> 4.18 M blocks, 2.79 M
+    frames; a 2^21-record touch, a discard of 2^21 blocks, a second 2^21-record touch that
+    reclaims ~356 k discarded frames), through the host fault list and through
+    um_touch_batch_dev: every block's state, both queue orders, all counters and every
+    block's content tag against the oracle."""
+    import gc
+    import torch
+    gc.collect()
+    torch.cuda.empty_cache()
+    free, _ = torch.cuda.mem_get_info()
+    GiB = 1 << 30
+    budget = min(170 * GiB, free - 8 * GiB) // (2 << 20) * (2 << 20)
+    assert budget >= 160 * GiB, f"only {free / GiB:.1f} GiB free for the full-size case"
+    arena = int(budget * 1.5) // (2 << 20) * (2 << 20)
+    t = tg.gen_state_micro(0, block_bytes=64 << 10, arena_bytes=arena, budget_bytes=budget)
+    g = _state_micro_parity(t, dev_records)
+    assert g["stats"]["evictions"] > 300_000 and t.nblocks > 4_000_000
