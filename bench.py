@@ -579,17 +579,11 @@ def state_bench(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 1024):
     cfg.workspace, cfg.workspace_bytes = ws.data_ptr(), ws_bytes
     h = um.um_arena_create(cfg)
     try:
-        rng = np.random.default_rng(seed)
-
-        def records(blocks):
-            acc = np.zeros(len(blocks), dtype=tg.ACC_DTYPE)
-            acc["off"] = blocks.astype(np.uint64) * B
-            acc["len"] = B
-            acc["kind"] = tg.ACC_READ
-            return acc
-        b0 = np.sort(rng.choice(nb, size=n, replace=False))
-        b1 = np.sort(rng.choice(nb, size=n, replace=False))
-        acc0, acc1 = records(b0), records(b1)
+        # the op sequence's seeded records (tracegen.gen_state_micro: the GPU parity tests
+        # replay the same sequence at this size against the oracle)
+        tr = tg.gen_state_micro(seed, block_bytes=B, arena_bytes=arena_bytes, budget_bytes=budget, n=n)
+        acc0, acc1 = tr.acc[:n], tr.acc[n:]
+        b0 = (acc0["off"] // B).astype(np.int64)
         # a device sleep ahead of each op keeps the GPU behind the host, so every launch
         # of the op is queued before it runs and the spans hold device time only
         ps = torch.cuda.ExternalStream(um.um_stream(h))
@@ -684,11 +678,7 @@ def state_dev_records(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 10
     B = block
     nb = arena_bytes // B
     n = 1 << 21
-    rng = np.random.default_rng(seed)
-    acc = np.zeros(n, dtype=tg.ACC_DTYPE)
-    acc["off"] = np.sort(rng.choice(nb, size=n, replace=False)).astype(np.uint64) * B
-    acc["len"] = B
-    acc["kind"] = tg.ACC_READ
+    acc = tg.gen_state_micro(seed, block_bytes=B, arena_bytes=arena_bytes, budget_bytes=budget, n=n).acc[:n]
     dacc = torch.from_numpy(acc.view(np.uint8).reshape(-1)).to(mem.frames.device)
     out = {}
     for gated in (True, False):
