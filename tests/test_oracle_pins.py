@@ -237,3 +237,42 @@ def test_slice_ops_drops_private_meta():
     t.meta["_calls_eager"] = ["stale"]
     s = t.slice_ops(0, 10)
     assert "_calls_eager" not in s.meta and len(s) == 10 and s.meta["seed"] == 0
+
+
+# --------------------------------------------------------------------- state microbench closed form
+@pytest.mark.parametrize("nb,nf,n,seed", [(4096, 2730, 2048, 0), (4096, 2200, 2048, 1), (60000, 40000, 30000, 2)])
+def test_state_micro_closed_form(nb, nf, n, seed):
+    """The state microbench's sequence (tracegen.gen_state_micro: touch of n random blocks,
+    discard [0, n), touch of n other random blocks) derived by hand from §8(c)'s sub-op
+    algorithm with set arithmetic: the first touch zero-fills all n (free frames suffice);
+    the discard unmaps the G blocks inside [0, n) into DISC in ascending order (§5.1 L176);
+    the second touch revives the discarded blocks it covers (§5.7), hits the other
+    resident ones, zero-fills the rest, and reclaims k = need - free victims: the head of
+    DISC without a transfer, then (if DISC runs out) the LRU end of USED -- the first
+    touch's blocks outside [0, n), ascending -- written back (§5.5)."""
+    B = 4096
+    t = tg.gen_state_micro(seed, block_bytes=B, arena_bytes=nb * B, budget_bytes=nf * B, n=n)
+    b0 = set((t.acc["off"][:n] // B).tolist())
+    b1 = set((t.acc["off"][n:] // B).tolist())
+    ge = sorted(b for b in b0 if b < n)
+    need = len(b1 - b0)
+    free = nf - n
+    k = max(0, need - free)
+    cand = [b for b in ge if b not in b1]      # DISC head first, skipping the pinned sub-op
+    ucand = sorted(b0 - set(ge) - b1)          # then USED: (ukey = 1, block) ascending
+    vd = cand[:k]
+    vu = ucand[:k - len(vd)]
+    assert len(vd) + len(vu) == k
+    o = replay(t, "eager")
+    s = o.stats
+    assert s["zf_bytes"] == (n + need) * B
+    assert s["unmaps"] == len(ge)
+    assert s["remaps"] == len(b1 & set(ge))
+    assert s["hits"] == len(b1 & (b0 - set(ge)))
+    assert s["faults"] == n + need + len(b1 & set(ge))
+    assert s["evictions"] == k
+    assert s["d2h_avoided_bytes"] == len(vd) * B and s["d2h_bytes"] == len(vu) * B and s["h2d_bytes"] == 0
+    st = o.st
+    assert all(st[v] == 2 for v in vd) and all(st[v] == 1 for v in vu)        # HD, H
+    assert sorted(b for b in range(nb) if st[b] == 4) == sorted(set(cand) - set(vd))   # GE left
+    assert list(o.disc) == [b for b in cand if b not in set(vd)]
