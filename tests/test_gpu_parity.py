@@ -637,3 +637,29 @@ def test_state_micro_full_size(dev_records):
     t = tg.gen_state_micro(0, block_bytes=64 << 10, arena_bytes=arena, budget_bytes=budget)
     g = _state_micro_parity(t, dev_records)
     assert g["stats"]["evictions"] > 300_000 and t.nblocks > 4_000_000
+
+
+def test_dev_records_edge_cases():
+    """um_touch_batch_dev edge cases: an empty batch (still one sub-op: the oracle's touch
+    of no blocks consumes a seq), zero-length records mixed in, a record covering 100
+    blocks across four bitmap words, and UM_EINVAL on a two-level arena."""
+    import torch
+    from paper_conf_iiswc_zhucvhcr22_b200 import um
+    B = 64 << 10
+    tb = tg.TraceBuilder(B, 256 * B, 64 * B)
+    tb.touch([(5 * B, 0, tg.ACC_WRITE), (7 * B + 3, 10, tg.ACC_WRITE), (30 * B, 100 * B, tg.ACC_READ)])
+    tb.touch([])
+    tb.touch([(0, 0, tg.ACC_READ)])
+    tb.touch([(200 * B, 40 * B, tg.ACC_WRITE), (31 * B, 2 * B, tg.ACC_WRITE)])
+    t = tb.build()
+    for mode in ("base", "eager"):
+        assert_parity(t, mode, _gpu_dev(t, mode))
+    a = um.Arena(2 << 20, 64 << 20, 16 << 20, page_bytes=64 << 10, host_pool_bytes=64 << 20)
+    try:
+        rec = torch.zeros(16, dtype=torch.uint8, device="cuda")
+        torch.cuda.synchronize()
+        with pytest.raises(um.UmError) as e:
+            um.um_touch_batch_dev(a.handle, rec.data_ptr(), 1)
+        assert e.value.status == um.UM_EINVAL
+    finally:
+        a.close()
