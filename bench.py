@@ -29,6 +29,7 @@ sys.path.insert(0, ROOT)
 
 GiB = 1 << 30
 MiB = 1 << 20
+KiB = 1 << 10
 METRIC = "redundant H2D+D2H GB avoided; iter time at 1.5x oversub; discard us/GB"
 
 
@@ -444,6 +445,54 @@ def discard_bench(torch, um, reps=20):
         out.append(row)
     del mem
     torch.cuda.empty_cache()
+    return out
+
+
+def prefetch_sweep(torch, um, reps=10):
+    """Prefetch throughput vs transfer size (Figure 4 analogue, PAPER L205/L213:
+    cudaMemPrefetchAsync bandwidth grows with the transfer size).  An S-byte buffer is
+    moved to the GPU (um_prefetch GPU: H2D) and back (um_prefetch HOST: D2H), `reps`
+    times, on the TMA kernel (K4) and on the copy-engine arm, at 2 MiB and 64 KiB blocks;
+    GB/s = S / (CUDA-event span on the paging stream around the call: planning kernels,
+    transfer and launch latency), median over reps."""
+    out = {}
+    S_max = 1 * GiB
+    sizes = [64 * KiB, 256 * KiB, 1 * MiB, 4 * MiB, 16 * MiB, 64 * MiB, 256 * MiB, 1 * GiB]
+    for B in (2 * MiB, 64 * KiB):
+        mem = um.Memory(B, S_max, S_max, host_pool_bytes=S_max)
+        rows = {}
+        for eng, fl in (("k4", 0), ("ce", um.UM_F_COPY_CE)):
+            a = um.Arena(B, S_max, S_max, mem=mem, flags=fl)
+            try:
+                ps = torch.cuda.ExternalStream(a.stream_ptr)
+                um.um_prefetch(a.handle, 0, S_max, um.UM_DST_HOST, a.stream_ptr)   # U -> H, no transfer
+                r = []
+                for S in sizes:
+                    if S < B:
+                        continue
+                    up, down = [], []
+                    for _ in range(reps + 1):
+                        e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+                        e[0].record(ps)
+                        um.um_prefetch(a.handle, 0, S, um.UM_DST_GPU, a.stream_ptr)
+                        e[1].record(ps)
+                        um.um_prefetch(a.handle, 0, S, um.UM_DST_HOST, a.stream_ptr)
+                        e[2].record(ps)
+                        e[2].synchronize()
+                        up.append(e[0].elapsed_time(e[1]))
+                        down.append(e[1].elapsed_time(e[2]))
+                    up, down = statistics.median(up[1:]), statistics.median(down[1:])
+                    r.append({"bytes": S, "h2d_gbs": S / (up / 1e3) / 1e9, "d2h_gbs": S / (down / 1e3) / 1e9,
+                              "h2d_us": up * 1e3, "d2h_us": down * 1e3})
+                st = um.um_get_stats(a.handle)
+                moved = sum(x["bytes"] for x in r) * (reps + 1)
+                assert st["h2d_bytes"] == moved and st["d2h_bytes"] == moved
+                rows[eng] = r
+            finally:
+                a.close()
+        out[f"{B // KiB}KiB_blocks"] = rows
+        del mem
+        torch.cuda.empty_cache()
     return out
 
 
@@ -959,6 +1008,7 @@ def main_ours(args):
     disc = None if args.no_discard_bench else _leg(torch, "discard_sweep", discard_bench, torch, um)
     c1 = None if args.no_discard_bench else _leg(torch, "c1", c1_rate, torch, um, harness)
     c4 = None if args.no_discard_bench else _leg(torch, "c4", c4_sweep, torch, um, harness)
+    pfs = None if args.no_discard_bench else _leg(torch, "prefetch_sweep", prefetch_sweep, torch, um)
 
     torch.cuda.empty_cache()
     free, total = torch.cuda.mem_get_info(dev)
@@ -1091,6 +1141,7 @@ def main_ours(args):
         "rmt": rmt_r,
         "c1_directives": c1,
         "c4_sweep": c4,
+        "prefetch_sweep": pfs,
         "c2_streaming": c2,
         "c3_64k_blocks": c3k,
         "clocks": head["clocks"],
