@@ -544,6 +544,8 @@ def test_dev_records_c1(mode):
     t = tg.gen_c1(6).slice_ops(0, 5000)
     assert_parity(t, mode, _gpu_dev(t, mode))
     assert_parity(t, mode, _gpu_dev(t, mode, overlap=True), overlap=True)
+    assert_parity(t, mode, _gpu_dev(t, mode, copy="ce"))
+    assert_parity(t, mode, _gpu_dev(t, mode, reserve=8), reserve=8)
 
 
 @pytest.mark.parametrize("mode", ["eager", "lazy"])
