@@ -1428,30 +1428,18 @@ UM_API um_status um_touch_batch_dev(um_arena* a, const um_access* acc, uint32_t 
   // the list rewrites T.dlo, which in-flight application kernels of earlier sub-ops may
   // read (their block list)
   if (overlap_on(a) && (s = app_wait_all(a))) return s;
-  // sorted block-disjoint records (the usual shape) expand straight into the block
-  // list; anything else is deduplicated through the op bitmap
   cudaEvent_t sp = span_open(a);
-  CK(launch_expand(a->T, acc, n, a->lgB, a->ps));
+  CK(launch_mark_acc(a->T, acc, n, a->lgB, a->ps));
+  CK(launch_list(a->T, (a->nblocks + 31) / 32, a->ps));
   span_close(a, sp, 0);
-  a->n_launch++;
+  a->n_launch += (n ? 1 : 0) + 1;
   // the host needs the distinct-block count to number the sub-ops (and learns of a
   // range error before anything that changes state is enqueued)
   CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
   CK(cudaStreamSynchronize(a->ps));
-  if (!a->hctl->iv_err && a->hctl->iv_unsorted) {
-    CK(cudaMemsetAsync(&a->T.ctl->iv_unsorted, 0, sizeof(unsigned int), a->ps));
-    sp = span_open(a);
-    CK(launch_mark_acc(a->T, acc, n, a->lgB, a->ps));
-    CK(launch_list(a->T, (a->nblocks + 31) / 32, a->ps));
-    span_close(a, sp, 0);
-    a->n_launch += 2;
-    CK(cudaMemcpyAsync(a->hctl, a->T.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, a->ps));
-    CK(cudaStreamSynchronize(a->ps));
-  }
   const auto t1 = clk::now();
   if (a->hctl->iv_err) {
     CK(cudaMemsetAsync(&a->T.ctl->iv_err, 0, sizeof(unsigned int), a->ps));
-    if (a->hctl->iv_unsorted) CK(cudaMemsetAsync(&a->T.ctl->iv_unsorted, 0, sizeof(unsigned int), a->ps));
     return UM_EINVAL;
   }
   a->dev_list = true;

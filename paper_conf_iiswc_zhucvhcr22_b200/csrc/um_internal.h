@@ -36,7 +36,6 @@ struct Ctl {
   unsigned int reach_tile;              // wide victim scan: first tile whose inclusive count >= k
   unsigned int iv_m, iv_d;              // device intake: intervals produced (list form: write blocks), distinct blocks
   unsigned int iv_err;                  // device records: a record outside the arena (read and cleared by the host)
-  unsigned int iv_unsorted;             // device records: not ascending block-disjoint (read and cleared by the host)
   unsigned long long minkeep[2];        // wide victim scan: first kept ring position
   unsigned int k_want;                  // wide victim scan: victims wanted
   unsigned int need_cnt[2];             // streaming classify: need-list slots, by sub-op parity
@@ -235,8 +234,5 @@ cudaError_t launch_intake_clear(const Tables& T, uint32_t w0, uint32_t w1, cudaS
 // ctl->iv_d = blocks, ctl->iv_m = write blocks, and clear the bitmaps.
 cudaError_t launch_mark_acc(const Tables& T, const void* acc, uint32_t n, uint32_t lg, cudaStream_t s);
 cudaError_t launch_list(const Tables& T, uint32_t nwords, cudaStream_t s);
-// Sorted block-disjoint records straight to the block list (dlo), no bitmap; sets
-// ctl->iv_unsorted if the records are not in that shape (the list is then invalid).
-cudaError_t launch_expand(const Tables& T, const void* acc, uint32_t n, uint32_t lg, cudaStream_t s);
 
 }  // namespace um

@@ -2356,89 +2356,6 @@ __global__ void __launch_bounds__(256) k_intake_clear(Tables T, uint32_t w0, uin
 //               once read (the bitmaps are clean for the next batch); the last tile
 //               publishes the block count (ctl->iv_d) and the write count (ctl->iv_m)
 // ------------------------------------------------------------------------------------
-// Sorted, block-disjoint records (the usual fault-buffer shape: ascending addresses, no
-// block covered twice) need no bitmap: the block list is the records' blocks in order,
-// record i's at the exclusive prefix of the block counts.  k_expand ranks them by block
-// scan + decoupled look-back and writes them (bit 31 = write); a record that starts
-// below its predecessor's end sets ctl->iv_unsorted and the host falls back to
-// k_mark_acc + k_list.  Range errors set ctl->iv_err as in k_mark_acc.
-constexpr int kExpTPB = 512, kExpIPT = 8, kExpTile = kExpTPB * kExpIPT;   // records per tile
-
-__global__ void __launch_bounds__(kExpTPB) k_expand(Tables T, const ulonglong2* acc, uint32_t n, uint32_t lg) {
-  pdl_enter();
-  __shared__ unsigned long long s_sc[kExpTPB / 32];
-  __shared__ unsigned long long s_excl;
-  const unsigned long long arena = (unsigned long long)T.nblocks << lg;
-  const uint32_t tile = blockIdx.x, ntiles = gridDim.x;
-  const uint32_t i0 = tile * kExpTile + threadIdx.x * kExpIPT;   // this thread's consecutive records
-  ulonglong2 r[kExpIPT];
-#pragma unroll
-  for (int q = 0; q < kExpIPT; ++q) r[q] = i0 + q < n ? __ldg(acc + i0 + q) : make_ulonglong2(0ull, 0ull);
-  // the last block of the record before this thread's first (a neighbour's: L1 / L2)
-  unsigned long long prev_end = 0ull;   // one past the previous record's last block (0: none)
-  bool bad = false, err = false;
-  if (i0 && i0 < n) {
-    const ulonglong2 p = __ldg(acc + i0 - 1);
-    const unsigned long long poff = p.x, plen = (uint32_t)p.y;
-    if (!plen || poff > arena || plen > arena - poff) bad = true;   // conservative: fall back
-    else prev_end = ((poff + plen - 1) >> lg) + 1ull;
-  }
-  uint32_t lo[kExpIPT], cnt[kExpIPT];
-  uint32_t tot_b = 0, tot_w = 0, wmask = 0;
-#pragma unroll
-  for (int q = 0; q < kExpIPT; ++q) {
-    const unsigned long long off = r[q].x, len = (uint32_t)r[q].y;
-    lo[q] = 0u;
-    cnt[q] = 0u;
-    if (off > arena || len > arena - off) {
-      err = true;
-    } else if (len) {
-      const unsigned long long l = off >> lg, h = ((off + len - 1) >> lg) + 1ull;
-      if (l < prev_end) bad = true;   // not ascending / shares a block with its predecessor
-      prev_end = h;
-      lo[q] = (uint32_t)l;
-      cnt[q] = (uint32_t)(h - l);
-      if ((uint32_t)(r[q].y >> 32) & 2u) {   // UM_ACC_WRITE (include/um.h)
-        wmask |= 1u << q;
-        tot_w += cnt[q];
-      }
-      tot_b += cnt[q];
-    } else if (i0 + q < n) {
-      bad = true;   // an empty record inside the batch: its successor's check would need
-                    // the record before it (rare: fall back)
-    }
-  }
-  if (__syncthreads_or(err) && threadIdx.x == 0) T.ctl->iv_err = 1u;
-  if (__syncthreads_or(bad) && threadIdx.x == 0) T.ctl->iv_unsorted = 1u;
-  unsigned long long tot;
-  // packed 31-bit counts: a sorted batch lists at most nblocks < 2^31 blocks (an unsorted
-  // one may wrap: its list is discarded)
-  const unsigned long long pre = block_excl_scan<kExpTPB>(pack2(tot_b & 0x7fffffffu, tot_w & 0x7fffffffu), tot, s_sc);
-  if (threadIdx.x < 32) {
-    const unsigned long long ex = lookback_warp(T, tile, tot);
-    if (threadIdx.x == 0) s_excl = ex;
-  }
-  __syncthreads();
-  uint32_t P = unpackA(s_excl) + unpackA(pre);
-  // an unsorted tile writes nothing (the host discards the list); neither does a tile
-  // whose range would pass the list's end (possible only after an unsorted tile)
-  const unsigned long long tend = (unsigned long long)unpackA(s_excl) + unpackA(tot);
-  if (!__syncthreads_or(bad) && tend <= T.nblocks) {
-#pragma unroll
-    for (int q = 0; q < kExpIPT; ++q) {
-      const uint32_t wbit = ((wmask >> q) & 1u) << 31;
-      for (uint32_t x = 0; x < cnt[q]; ++x) T.dlo[P + x] = (lo[q] + x) | wbit;
-      P += cnt[q];
-    }
-  }
-  if (tile == ntiles - 1 && threadIdx.x == 0) {
-    const unsigned long long all = s_excl + tot;
-    T.ctl->iv_d = unpackA(all);
-    T.ctl->iv_m = unpackB(all);
-  }
-  scan_finish(T, ntiles);
-}
-
 constexpr int kMarkIPT = 8;   // consecutive records per thread, all loads in flight
 
 // Each thread takes kMarkIPT CONSECUTIVE records: in a sorted fault batch they fall in
@@ -2947,13 +2864,6 @@ cudaError_t launch_mark_acc(const Tables& T, const void* acc, uint32_t n, uint32
   unsigned grid = ceil_div(n, 256 * kMarkIPT);
   if (grid > (unsigned)g_nsm * 8) grid = g_nsm * 8;
   cudaError_t e = launch_pdl(k_mark_acc, dim3(grid), dim3(256), 0, s, T, (const ulonglong2*)acc, n, lg);
-  if (e) return e;
-  return cudaGetLastError();
-}
-
-cudaError_t launch_expand(const Tables& T, const void* acc, uint32_t n, uint32_t lg, cudaStream_t s) {
-  unsigned nt = n ? ceil_div(n, kExpTile) : 1;
-  cudaError_t e = launch_pdl(k_expand, dim3(nt), dim3(kExpTPB), 0, s, T, (const ulonglong2*)acc, n, lg);
   if (e) return e;
   return cudaGetLastError();
 }
