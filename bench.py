@@ -803,6 +803,31 @@ def state_runs(torch, um, mem, budget, arena_bytes):
                 "classify = the LIST classify of touch_2^21_random (same list); host_api_us = the whole "
                 "API call on an idle device (intake launch, block-count read-back, classify and zero-fill "
                 "enqueue), against touch_2^21_random's host_api_us (host scan of the records)"}
+    # the same bytes through torch's own copy kernel, timed the same way (events around
+    # one launch, cold L2): what a plain streaming pass of that size reaches on this GPU
+    dev = mem.frames.device
+    scrub = torch.empty(512 * MiB, dtype=torch.uint8, device=dev)
+    for op in ("touch_2^21_random", "discard_2^21", "touch_2^21_pressure", "touch_2^21_device_records"):
+        by = state[op]["algorithmic_bytes"]
+        x = torch.empty(by // 2, dtype=torch.uint8, device=dev)
+        y = torch.empty_like(x)
+        ts = []
+        for _ in range(11):
+            scrub.add_(1)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            y.copy_(x)
+            e1.record()
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        cu = statistics.median(ts[1:])
+        state[op]["copy_same_bytes"] = {"ms": cu, "gbs": by / (cu / 1e3) / 1e9,
+                                        "op_time_over_copy_time": state[op]["ms"] / cu}
+        del x, y
+    del scrub
+    state["copy_same_bytes_note"] = ("torch copy kernel moving each op's algorithmic bytes (half read, half "
+                                     "written), CUDA events around one launch, cold L2: the rate a plain "
+                                     "streaming pass of that size reaches with this timing")
     return state
 
 
