@@ -1496,272 +1496,6 @@ __global__ void __launch_bounds__(kVaTPB, 2) k_victims_apply(Tables T, int evict
 }
 
 // ------------------------------------------------------------------------------------
-// K3 (wide, fused): the same victim rule as k_victims_scan + k_victims_apply in ONE
-// persistent launch (UM_VS_FUSED=1, A/B).  Each tile learns its exclusive candidate
-// prefix by decoupled look-back over the tiles before it (tickets hand tiles out in
-// index order and every grid CTA is resident, so every predecessor publishes), and
-// reclaims its own victims prefix + rank < k at once -- no scratch list, no one-CTA
-// finalize, no second launch.  The tile holding the k-th candidate records itself; tiles
-// wholly before it min-reduce their first kept live entry per ring; the last CTA to
-// finish moves the ring heads, publishes n_vict and the frame bookkeeping, and clears
-// the look-back status of the tiles handed out.
-// ------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kVsTPB, 3) k_victims_fused(Tables T, uint32_t seq, int evict_mode, uint32_t want,
-                                                             int npar) {
-  pdl_enter();
-  constexpr int NW = kVsTPB / 32;
-  __shared__ uint32_t s_off[kVsIPT * NW + 1];
-  __shared__ unsigned long long s_dh, s_ld, s_uh, s_lu, s_mk[2], s_pre;
-  __shared__ uint32_t s_k, s_nn, s_f0, s_tile, s_skip;
-  __shared__ int s_last;
-  __shared__ uint32_t s_cnt[8];
-  Ctl* c = T.ctl;
-  if (threadIdx.x == 0) {
-    s_dh = c->disc_head;
-    s_ld = c->disc_tail - c->disc_head;
-    s_uh = c->used_head;
-    s_lu = c->used_tail - c->used_head;
-    const uint32_t f0 = (uint32_t)c->free_top;
-    const uint32_t nn = evict_mode ? want : c->need_cnt[npar];
-    s_k = nn > f0 ? nn - f0 : 0u;
-    s_nn = nn;
-    s_f0 = f0;
-    if (blockIdx.x == 0 && !evict_mode) {
-      c->n_need = nn;
-      c->need_cnt[npar ^ 1] = 0;
-    }
-  }
-  __syncthreads();
-  const uint32_t k = s_k;
-  const unsigned long long L = s_ld + s_lu;
-  const uint32_t ntiles = k ? (uint32_t)((L + kVsTile - 1) / kVsTile) : 0u;
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const unsigned lt = lanemask_lt();
-  const unsigned me = 1u << lane;
-  const int f0 = (int)s_f0;
-  uint32_t nG = 0, nAv = 0, nGL = 0;
-  if (threadIdx.x == 0) {
-    s_tile = blockIdx.x;
-    s_skip = 0;
-  }
-  while (k) {
-    __syncthreads();
-    const uint32_t tile = s_tile, snap = s_skip;
-    __syncthreads();
-    if (tile >= ntiles || snap >= k) break;   // (a skipped ticket: later tickets skip too)
-    if (threadIdx.x == 0) s_mk[0] = s_mk[1] = ~0ull;
-    const unsigned long long tbase = (unsigned long long)tile * kVsTile;
-    uint32_t bb[kVsIPT], kk[kVsIPT], wv[kVsIPT];
-    uint8_t ssv[kVsIPT];
-    unsigned bC[kVsIPT], bL[kVsIPT];
-#pragma unroll
-    for (int q = 0; q < kVsIPT; ++q) {
-      const unsigned long long idx = tbase + q * kVsTPB + threadIdx.x;
-      unsigned long long e = ~0ull;
-      if (idx < L) {
-        const bool disc = idx < s_ld;
-        const unsigned long long pos = disc ? s_dh + idx : s_uh + (idx - s_ld);
-        e = (disc ? T.disc_ring : T.used_ring)[pos & T.cap_mask];
-      }
-      bb[q] = (uint32_t)e;
-      kk[q] = (uint32_t)(e >> 32);
-    }
-#pragma unroll
-    for (int q = 0; q < kVsIPT; ++q) wv[q] = bb[q] != UM_NONE ? T.sk[bb[q]] : 0u;
-#pragma unroll
-    for (int q = 0; q < kVsIPT; ++q) {
-      const unsigned long long idx = tbase + q * kVsTPB + threadIdx.x;
-      ssv[q] = st_of(wv[q]);
-      const bool live = bb[q] != UM_NONE && (idx < s_ld ? (ssv[q] == ST_GE || ssv[q] == ST_GL) : ssv[q] == ST_G) &&
-                        key_of(wv[q]) == kk[q];
-      wv[q] = live ? T.pin[bb[q]] : UM_NONE;
-      bL[q] = __ballot_sync(FULL, live);
-    }
-#pragma unroll
-    for (int q = 0; q < kVsIPT; ++q) bC[q] = __ballot_sync(FULL, wv[q] < T.pfloor);
-    const uint32_t cnt = ordered_offsets<kVsTPB, kVsIPT>(bC, bC, s_off) & 0xffffu;
-    unsigned long long mk0 = ~0ull, mk1 = ~0ull;
-#pragma unroll
-    for (int q = 0; q < kVsIPT; ++q) {
-      if (!(bC[q] & me) && (bL[q] & me)) {
-        const unsigned long long idx = tbase + q * kVsTPB + threadIdx.x;
-        if (idx < s_ld) mk0 = min(mk0, idx);
-        else mk1 = min(mk1, idx);
-      }
-    }
-    if (mk0 != ~0ull) atomicMin(&s_mk[0], mk0);
-    if (mk1 != ~0ull) atomicMin(&s_mk[1], mk1);
-    // the tile's count goes into the running total now (pacing, skip snapshots), its
-    // exclusive prefix comes from the look-back
-    if (threadIdx.x == 0 && cnt) atomicAdd(&c->vs_combo, (unsigned long long)cnt << 32);
-    if (threadIdx.x < 32) {
-      const unsigned long long ex = lookback_warp(T, tile, (unsigned long long)cnt);
-      if (threadIdx.x == 0) s_pre = ex;
-    }
-    __syncthreads();
-    const unsigned long long prefix = s_pre;
-    const uint32_t take = prefix >= k ? 0u : (uint32_t)min((unsigned long long)cnt, k - prefix);
-    if (threadIdx.x == 0) {
-      if (prefix < k && prefix + cnt >= k) c->reach_tile = tile;   // exactly one tile
-      if (prefix + cnt < k) {                                        // wholly before it
-        if (s_mk[0] != ~0ull) atomicMin(&c->minkeep[0], s_mk[0]);
-        if (s_mk[1] != ~0ull) atomicMin(&c->minkeep[1], s_mk[1]);
-      }
-    }
-    if (take) {
-      // reclaim this tile's victims: candidate of rank r < take is victim prefix + r
-#pragma unroll
-      for (int q = 0; q < kVsIPT; ++q) {
-        const uint32_t r = (s_off[q * NW + w] & 0xffffu) + __popc(bC[q] & lt);
-        const bool vic = ((bC[q] & me) != 0) && r < take;
-        const uint32_t j = (uint32_t)prefix + r;
-        const uint32_t v = bb[q];
-        const uint8_t ss = ssv[q];
-        uint32_t fr = UM_NONE, hf = UM_NONE;
-        uint8_t nk = 0xff;
-        if (vic) {
-          fr = T.frame_of[v];
-          if (!evict_mode) nk = T.needk[(uint32_t)f0 + j];
-        }
-        if (vic && ss == ST_G && nk == ST_H) hf = T.needhf[(uint32_t)f0 + j];   // fused swap (R5)
-        const bool isG = vic && ss == ST_G;
-        const unsigned bA = __ballot_sync(FULL, isG && hf == UM_NONE);
-        const unsigned bD = __ballot_sync(FULL, evict_mode && isG);
-        int hb = 0;
-        uint32_t hav = 0, db = 0;
-        if (lane == 0) {
-          const uint32_t tA = __popc(bA), tD = __popc(bD);
-          if (tA) {
-            const int old = atomicSub(&c->hfree_top, (int)tA);
-            const int avail = old < 0 ? 0 : (old < (int)tA ? old : (int)tA);
-            if (avail < (int)tA) {
-              atomicAdd(&c->hfree_top, (int)tA - avail);
-              atomicExch(&c->err, 2u);   // host-frame pool exhausted -> UM_ENOMEM
-            }
-            hb = old;
-            hav = (uint32_t)avail;
-          }
-          if (tD) db = atomicAdd(&c->n_d2h, tD);
-        }
-        hb = __shfl_sync(FULL, hb, 0);
-        hav = __shfl_sync(FULL, hav, 0);
-        db = __shfl_sync(FULL, db, 0);
-        if ((bA >> lane) & 1u) {
-          const uint32_t ra = __popc(bA & lt);
-          hf = ra < hav ? T.hfree_stack[hb - 1 - (int)ra] : UM_NONE;
-        }
-        if (vic) {
-          T.victim[j] = v;
-          T.vframe[j] = fr;
-          T.vkind[j] = ss;
-          T.vhf[j] = hf;
-          T.sk[v] = mk_sk(isG ? ST_H : ST_HD, 0);
-          if (T.phz) T.phz[v] = 0u;
-          T.map[v] = UM_NONE;
-          T.frame_of[v] = UM_NONE;
-          T.hframe[v] = hf;
-          nG += isG;
-          nAv += !isG;
-          nGL += ss == ST_GL;
-          if (evict_mode) {
-            T.free_stack[f0 + j] = fr;
-            if (isG) {
-              const uint32_t d = db + __popc(bD & lt);
-              T.d2h_frame[d] = fr;
-              T.d2h_hf[d] = hf;
-              d2h_listed(T, seq, v, d, ss);
-            }
-          }
-        }
-      }
-    }
-    // next tile: paced tickets, as in k_victims_scan
-    if (threadIdx.x == 0) {
-      unsigned long long v = *(volatile unsigned long long*)&c->vs_combo;
-      unsigned int fin = atomicAdd(&c->vs_fin, 1u) + 1u;
-      unsigned long long nxt;
-      while (true) {
-        const unsigned long long tot = v >> 32;
-        const unsigned int issued = (unsigned int)min((unsigned long long)ntiles, (unsigned long long)gridDim.x + (uint32_t)v);
-        const unsigned int inflight = issued > fin ? issued - fin : 0u;
-        if (tot >= k || issued >= ntiles && inflight == 0) {
-          nxt = v | 0xffffffffull;
-          break;
-        }
-        if (!inflight || tot + (unsigned long long)inflight * tot / fin < k) {
-          nxt = atomicAdd(&c->vs_combo, 1ull);
-          break;
-        }
-        __nanosleep(128);
-        v = *(volatile unsigned long long*)&c->vs_combo;
-        fin = *(volatile unsigned int*)&c->vs_fin;
-      }
-      s_tile = (uint32_t)nxt == 0xffffffffu ? ntiles : gridDim.x + (uint32_t)nxt;
-      s_skip = (uint32_t)(nxt >> 32);
-    }
-  }
-  uint32_t cnt3[3] = {nG, nAv, nGL};
-  const int slots[3] = {S_D2H, S_D2H_AV, S_UNMAPS};
-  const long long mul[3] = {(long long)T.B, (long long)T.B, 1};
-  block_counts_to<3>(T, cnt3, s_cnt, slots, mul);
-  // completion: the last CTA publishes the launch's results and cleans up
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    s_last = atomicAdd(&c->scan_done, 1u) == gridDim.x - 1;
-  }
-  __syncthreads();
-  if (!s_last) return;
-  __threadfence();
-  const unsigned long long vc = *(volatile unsigned long long*)&c->vs_combo;
-  const uint32_t handed = (uint32_t)min((unsigned long long)ntiles, (unsigned long long)gridDim.x + (uint32_t)vc);
-  for (uint32_t i = threadIdx.x; i < handed; i += blockDim.x) T.tile_status[i] = 0ull;
-  if (threadIdx.x == 0) {
-    if (k == 0) {
-      c->n_vict = 0;
-      c->f0 = s_f0;
-      if (evict_mode) {
-        c->free_top = f0;
-      } else {
-        c->free_top = f0 - (int)min(s_f0, s_nn);
-        c->used_tail += c->n_rekey;
-      }
-    } else {
-      const uint32_t found = (uint32_t)min((unsigned long long)k, vc >> 32);
-      unsigned long long kd = *(volatile unsigned long long*)&c->minkeep[0];
-      unsigned long long ku = *(volatile unsigned long long*)&c->minkeep[1];
-      const uint32_t reach = *(volatile uint32_t*)&c->reach_tile;
-      if (reach != ~0u) {
-        const unsigned long long bound = (unsigned long long)reach * kVsTile;
-        if (bound < s_ld) {
-          kd = min(kd, bound);
-          ku = min(ku, s_ld);   // USED not reached: its head stays
-        } else {
-          ku = min(ku, bound);
-        }
-      }
-      c->disc_head = kd != ~0ull ? s_dh + kd : c->disc_tail;
-      c->used_head = ku != ~0ull ? s_uh + (ku - s_ld) : c->used_tail;
-      c->n_vict = found;
-      stat_add(T, S_EVICT, found);
-      c->f0 = s_f0;
-      if (evict_mode) {
-        c->free_top = f0 + (int)found;
-      } else {
-        c->free_top = f0 - (int)min(s_f0, s_nn);
-        c->used_tail += c->n_rekey;
-      }
-    }
-    c->scan_done = 0;
-    c->vs_combo = 0;
-    c->vs_fin = 0;
-    c->minkeep[0] = c->minkeep[1] = ~0ull;
-    c->reach_tile = ~0u;
-  }
-  __threadfence();
-}
-
-// ------------------------------------------------------------------------------------
 // K4/K5/K6: the transfer engine.  One elected thread per CTA drives a kXferStages-deep
 // ring of TMA bulk copies (cp.async.bulk, mbarrier complete_tx) through shared memory.
 // Work unit = one kXferChunk slice of one frame.  Fused swap per unit: the victim's
@@ -2860,8 +2594,6 @@ static bool g_pdl = true;     // UM_PDL=0 disables programmatic dependent launch
 static int g_dir_occ = 8;     // resident k_directive CTAs per SM (persistent grid)
 static int g_dir_minb = 6;    // k_directive CTAs/SM the registers allow: 6 (40 regs); UM_DIR_MINB=7/8 (36/32 regs: one wave for 2^21 blocks) for A/B
 static int g_vs_ctas = 0;     // UM_VS_CTAS=n caps the victim scan grid at n CTAs (test hook: small tables then take tiles by ticket and skip past the k-th candidate)
-static int g_vs_fused = 0;    // UM_VS_FUSED=1: fused wide victim scan + reclaim (k_victims_fused), A/B
-static int g_vfused_occ = 1;  // resident k_victims_fused CTAs per SM
 static int g_vs_prefetch = 0; // UM_VS_PREFETCH=1: the wide victim scan fetches its next ticket a tile ahead (A/B on B200: 79 vs 73 us pressured touch -- the earlier snapshot reads more tiles past the k-th candidate)
 
 cudaError_t setup_kernels() {
@@ -2873,7 +2605,6 @@ cudaError_t setup_kernels() {
   if (const char* v = getenv("UM_PDL")) g_pdl = atoi(v) != 0;
   if (const char* v = getenv("UM_VS_PREFETCH")) g_vs_prefetch = atoi(v) != 0;
   if (const char* v = getenv("UM_VS_CTAS")) g_vs_ctas = atoi(v) > 0 ? atoi(v) : 0;
-  if (const char* v = getenv("UM_VS_FUSED")) g_vs_fused = atoi(v) != 0;
   if (const char* v = getenv("UM_CLS_TPB")) g_cls_tpb = atoi(v) == 512 ? 512 : 256;
   // Optionally one L1/shared carveout for every paging kernel (k_service needs 144 KB of
   // shared memory; a carveout change between consecutive kernels can force an SM drain).
@@ -2896,9 +2627,6 @@ cudaError_t setup_kernels() {
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_vscan_occ, k_victims_scan, kVsTPB, 0);
   if (e) return e;
   if (g_vscan_occ < 1) g_vscan_occ = 1;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_vfused_occ, k_victims_fused, kVsTPB, 0);
-  if (e) return e;
-  if (g_vfused_occ < 1) g_vfused_occ = 1;
   if (const char* v = getenv("UM_DIR_MINB")) g_dir_minb = std::min(8, std::max(6, atoi(v)));
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
       &g_dir_occ,
@@ -2977,13 +2705,6 @@ cudaError_t launch_victims_wide(const Tables& T, uint32_t seq, int evict_mode, u
   // persistent scan grid: never more CTAs than can be resident (tiles are taken from a
   // ticket in order and a tile may wait on its predecessors' status)
   unsigned nt = ceil_div(scan_bound ? scan_bound : 1, kVsTile);
-  if (g_vs_fused) {
-    const unsigned capf = g_vs_ctas ? (unsigned)g_vs_ctas : (unsigned)(g_nsm * g_vfused_occ);
-    cudaError_t lf = launch_pdl(k_victims_fused, dim3(nt < capf ? nt : capf), dim3(kVsTPB), 0, s, T, seq, evict_mode,
-                                want, npar);
-    if (lf) return lf;
-    return cudaGetLastError();
-  }
   const unsigned cap = g_vs_ctas ? (unsigned)g_vs_ctas : (unsigned)(g_nsm * g_vscan_occ);
   cudaError_t le__ = launch_pdl(k_victims_scan, dim3(nt < cap ? nt : cap), dim3(kVsTPB), 0, s, T, seq, evict_mode, want, npar, g_vs_prefetch);
   if (le__) return le__;
