@@ -725,7 +725,6 @@ def state_dev_records(torch, um, mem, budget, arena_bytes, seed=0, block=64 * 10
     import numpy as np
     import tracegen as tg
     B = block
-    nb = arena_bytes // B
     n = 1 << 21
     acc = tg.gen_state_micro(seed, block_bytes=B, arena_bytes=arena_bytes, budget_bytes=budget, n=n).acc[:n]
     dacc = torch.from_numpy(acc.view(np.uint8).reshape(-1)).to(mem.frames.device)
