@@ -665,3 +665,13 @@ def test_dev_records_edge_cases():
         assert e.value.status == um.UM_EINVAL
     finally:
         a.close()
+
+
+def test_c3_full_size_reserve():
+    """Proactive eviction (R12) at the bench's full size and launch configuration: C3 at
+    1.5x of the 170 GiB budget, 2 MiB blocks, reserve 128 frames (the bench's
+    proactive-eviction leg), two iterations, bit-exact against the oracle with reserve."""
+    t = _full_size_trace()
+    pool = t.arena_bytes - t.budget_bytes + (2 << 30)
+    g = _gpu(t, "eager", host_pool_bytes=pool, reserve=128)
+    assert_parity(t, "eager", g, reserve=128)
