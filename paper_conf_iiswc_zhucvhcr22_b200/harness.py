@@ -19,7 +19,7 @@ def mode_flags(mode: str) -> int:
 
 
 def make_arena(trace, mode: str, *, flags: int = um.UM_F_APP_STAMP | um.UM_F_CHECK, host_pool_bytes=None,
-               device: int = 0, mem=None, page_bytes: int = 0, reserve_blocks: int = 0) -> um.Arena:
+               device: int | None = None, mem=None, page_bytes: int = 0, reserve_blocks: int = 0) -> um.Arena:
     """page_bytes < block_bytes: a two-level arena (chunks of block_bytes, pages of
     page_bytes).  reserve_blocks > 0: proactive eviction (R12)."""
     return um.Arena(trace.block_bytes, trace.arena_bytes, trace.budget_bytes, flags=flags | mode_flags(mode),
@@ -41,10 +41,12 @@ def iteration_bounds(trace) -> list:
     return [(i * per, (i + 1) * per) for i in range(it)]
 
 
-def _dev_records(trace, device: int = 0) -> int:
+def _dev_records(trace, device: int | None = None) -> int:
     """The trace's access records copied once into device memory (the GPU's fault buffer
     analogue for um_touch_batch_dev); returns its device address."""
     import torch
+    if device is None:
+        device = torch.cuda.current_device()
     key = f"_acc_dev{device}"
     t = trace.meta.get(key)
     if t is None:

@@ -247,8 +247,10 @@ class Memory:
     (pinned host memory in chunks of <= 1 GiB, allocated from `threads` threads)."""
 
     def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, host_pool_bytes=None,
-                 host_chunk_bytes=None, device: int = 0, threads: int = 1, page_bytes: int = 0):
+                 host_chunk_bytes=None, device: int | None = None, threads: int = 1, page_bytes: int = 0):
         import torch
+        if device is None:   # the caller's current device (one process per GPU under torchrun)
+            device = torch.cuda.current_device()
         self.B = block_bytes
         self.page_bytes = page_bytes
         self.nframes = budget_bytes // block_bytes
@@ -293,7 +295,7 @@ class Arena:
     """A libum arena over `Memory` (allocated here unless `mem` is given)."""
 
     def __init__(self, block_bytes: int, arena_bytes: int, budget_bytes: int, *, flags: int = 0,
-                 host_pool_bytes: int | None = None, host_chunk_bytes: int | None = None, device: int = 0,
+                 host_pool_bytes: int | None = None, host_chunk_bytes: int | None = None, device: int | None = None,
                  mem: Memory | None = None, page_bytes: int = 0, reserve_blocks: int = 0):
         self.B = block_bytes
         self.nblocks = arena_bytes // block_bytes
